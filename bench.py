@@ -1,0 +1,331 @@
+#!/usr/bin/env python
+"""Benchmark of the hot path: batched decision-tree-ensemble prediction (Tahoe, EuroSys '21).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config 2]
+    python -m torch.distributed.run --nnodes=1 --nproc-per-node N --master-addr 127.0.0.1 \
+        --master-port P bench.py --gpus N ...
+
+Workload (BASELINE.json configs[1], the config the metric is quoted on and that fits one GPU):
+C2, a Higgs-shaped binary forest of 500 random post-pruned trees (depth <= 8, 28 attributes) over
+1M synthetic samples per GPU.  A step = one tahoe_predict of the whole batch (all §8(a) rows:
+traversal, combine, finalize).  N > 1: every rank predicts its own 1M rows (sample sharding, weak
+scaling, no data-path collective).  Rank 0 prints one JSON line.
+
+--impl reference: the CPU oracle (oracle/, the "reference arm" of this tier) timed on the box's
+host cores on a bounded sample of the same workload per step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+
+METRIC = "samples/sec per forest"
+UNIT = "samples/s"
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return dict(hbm_gbs=float(d["hbm_gbs"]), sm_max_mhz=float(d.get("sm_max_mhz", 1965.0)),
+                    source="measured (MEASURED_PEAKS.json)")
+    return dict(hbm_gbs=6650.0, sm_max_mhz=1965.0, source="fallback (B200_PROFILING.md)")
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+        self.thread = None
+
+    def start(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 7:
+                self.rows.append(parts)
+
+    def stop(self) -> dict | None:
+        if not self.proc:
+            return None
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[j] for r in self.rows for j in range(4) if r[3 + j] == "Active"})
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(sm)}
+
+
+def build_workload(cfg, rank: int, n: int):
+    f = gen.make_forest(cfg, leaf_mode="normal")
+    X = gen.make_rows(cfg, n, row0=rank * n)
+    return f, X
+
+
+def oracle_rate(f, X, target_s: float, max_rows: int):
+    """Oracle (as it stands) on a bounded sample of X: returns (rows/s, rows, seconds, visits)."""
+    import oracle
+    probe = min(2000, X.shape[0])
+    t = time.perf_counter()
+    oracle.predict(f, X[:probe])
+    dt = max(time.perf_counter() - t, 1e-6)
+    rows = int(min(max_rows, X.shape[0], max(probe, probe / dt * target_s)))
+    idx = gen.subsample(4242, X.shape[0], rows)
+    t = time.perf_counter()
+    r = oracle.predict(f, X, rows=idx)
+    dt = time.perf_counter() - t
+    return rows / dt, rows, dt, float(r["visits"].mean())
+
+
+def run_reference(args, cfg):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import oracle
+    n = cfg.n_samples
+    f, X = build_workload(cfg, 0, min(n, 200_000))
+    cores = oracle.n_threads()
+    rate0, _, _, _ = oracle_rate(f, X, 1.0, 20000)
+    rows = int(min(X.shape[0], max(1000, rate0 * 4.0)))   # ~4 s of oracle work per step
+    idx = gen.subsample(99, X.shape[0], rows)
+    for _ in range(args.warmup):
+        oracle.predict(f, X, rows=idx[: max(1, rows // 8)])
+    times = []
+    for _ in range(args.steps):
+        t = time.perf_counter()
+        oracle.predict(f, X, rows=idx)
+        times.append(time.perf_counter() - t)
+    ms = 1000.0 * statistics.mean(times)
+    value = rows / (ms / 1000.0)
+    sample = f"{rows} seeded rows per step of the {cfg.name} workload (of {n} per GPU)"
+    line = dict(metric=METRIC, value=value, unit=UNIT, n_gpus=args.gpus, steps=args.steps,
+                warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="weak",
+                vs_baseline=None, dtype="f32", data="synthetic", impl="reference",
+                config=_config(cfg, n, None),
+                cpu_baseline=dict(value=value, unit=UNIT, cores=cores, kind="oracle",
+                                  sample=sample),
+                e2e=dict(value=value, unit=UNIT, h2d_bytes_per_step=0, d2h_bytes_per_step=0))
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def _config(cfg, n, stats):
+    c = {"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
+                     f"{cfg.n_features} features, {n} samples per GPU (BASELINE configs[{cfg.cid - 1}])",
+         "n_per_gpu": n, "n_trees": cfg.n_trees, "n_features": cfg.n_features,
+         "max_depth": cfg.max_depth, "agg": "binary margin + class",
+         "parallelism": "sample-sharded (no collective)",
+         "l2": "256 MiB L2 flush between timed steps (inputs 112 MB < L2), outside the events"}
+    if stats:
+        c.update({k: stats[k] for k in ("nodes", "leaves", "n_slices", "slots_max", "lockstep_eff",
+                                        "expected_visits_per_sample", "sliced_bytes") if k in stats})
+    return c
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--strategy", type=int, default=-1)
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    cfg = gen.CONFIGS[args.config]
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_eurosys_xiedlll21_b200 import tahoe as T
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    T.load(build_if_missing=(rank == 0 and world == 1))
+    args.warmup = max(args.warmup, 3)
+    n = cfg.n_samples
+    f, X = build_workload(cfg, rank, n)
+    t0 = time.perf_counter()
+    F = T.Forest(f, device=local)
+    F.layout(gen.make_calibration(cfg))
+    layout_s = time.perf_counter() - t0
+    stats = F.stats()
+    strategy = args.strategy if args.strategy >= 0 else F.select_strategy(n, cfg.n_features)
+    Xd = torch.from_numpy(X).to(dev)
+    out = torch.empty((n, F.n_out), dtype=torch.float32, device=dev)
+    cls = torch.empty(n, dtype=torch.int32, device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+           torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    for e in ev:
+        for x in e:
+            x.record(stream)
+    torch.cuda.synchronize()
+
+    def step(e=None):
+        if e is None:
+            F.predict(Xd, out=out, out_class=cls, force_strategy=strategy)
+        else:
+            e[0].record(stream)
+            F.predict(Xd, out=out, out_class=cls, force_strategy=strategy,
+                      ev_main_begin=e[2], ev_main_end=e[3])
+            e[1].record(stream)
+
+    for _ in range(args.warmup):
+        step()
+        flush.zero_()
+    sampler = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    time.sleep(0.2)
+    wall0 = time.perf_counter()
+    for k in range(args.steps):
+        step(ev[k])
+        flush.zero_()   # L2 flush between timed steps (outside the step events)
+    torch.cuda.synchronize()
+    wall = time.perf_counter() - wall0
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    step_ms = [e[0].elapsed_time(e[1]) for e in ev]
+    kern_ms = [e[2].elapsed_time(e[3]) for e in ev]
+    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    ms_per_step = float(tot[0]) / args.steps
+    kern_avg_ms = float(tot[1]) / args.steps
+    value = world * n / (ms_per_step / 1000.0)
+
+    # ---- end to end through the public API with HOST buffers (pinned), copies inside
+    Xh = torch.from_numpy(X).pin_memory()
+    oh = torch.empty((n, F.n_out), dtype=torch.float32).pin_memory()
+    ch = torch.empty(n, dtype=torch.int32).pin_memory()
+    for _ in range(2):
+        F.predict_host(Xh, oh, ch)
+    torch.cuda.synchronize()
+    e2e_ms = []
+    for _ in range(max(3, min(args.steps, 10))):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        F.predict_host(Xh, oh, ch)
+        b.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms.append(a.elapsed_time(b))
+    e2e_t = torch.tensor([statistics.mean(e2e_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_value = world * n / (float(e2e_t[0]) / 1000.0)
+
+    if rank != 0:
+        if world > 1:
+            dist.barrier()
+            dist.destroy_process_group()
+        return 0
+
+    peaks = _peaks()
+    # algorithmic bytes (HBM roofline the metric asks for): sample row read + outputs written
+    hbm_bytes = n * (cfg.n_features * 4 + F.n_out * 4 + 4)
+    hbm_gbs = hbm_bytes / (ms_per_step / 1000.0) / 1e9
+    # dominant kernel roofline: shared-memory LSU pipe: per node visit
+    # 8 B node + 4 B attribute, per leaf 8 B; peak 128 B/clk/SM x SMs x max SM clock
+    cpu = None
+    visits = stats["expected_visits_per_sample"]
+    if not args.no_cpu and world == 1:
+        rate, rows, secs, vis = oracle_rate(f, X, 12.0, 1_000_000)
+        import oracle
+        cpu = dict(value=rate, unit=UNIT, cores=oracle.n_threads(), kind="oracle",
+                   sample=f"{rows} seeded rows of this workload ({secs:.1f} s of oracle work)")
+        visits = vis
+    smem_bytes_per_sample = visits * 12.0 + cfg.n_trees * 8.0
+    n_sms = stats["num_sms"]
+    smem_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
+    achieved = n * smem_bytes_per_sample / (kern_avg_ms / 1000.0) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(f"C{cfg.cid}", {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    launches_per_step = 1 if strategy == T.STRATEGY_DIRECT and F.n_out == 1 else (
+        1 + (1 if (strategy != T.STRATEGY_DIRECT and stats["n_slices"] > 1) or F.n_out > 1 else 0))
+    line = dict(
+        metric=METRIC, value=value, unit=UNIT, n_gpus=world, steps=args.steps, warmup=args.warmup,
+        ms_per_step=ms_per_step, higher_is_better=True, scaling="weak", vs_baseline=None,
+        dtype="f32", accum="f64", data="synthetic", impl="ours",
+        config=_config(cfg, n, stats),
+        strategy={0: "direct", 1: "sliced"}.get(strategy, str(strategy)),
+        roofline=dict(bound="alu", pipe="shared-memory LSU, 128 B/clk/SM (DESIGN.md Roofline)",
+                      kernel="k_sliced" if strategy == 1 else "k_direct",
+                      achieved=achieved, peak=smem_peak, unit="GB/s", frac=achieved / smem_peak,
+                      traffic=traffic, kernel_ms=kern_avg_ms,
+                      units_per_launch=f"{n} samples x {smem_bytes_per_sample:.0f} B "
+                                       f"({visits:.0f} visits x 12 B + {cfg.n_trees} leaves x 8 B)",
+                      peak_source=f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz"),
+        hbm=dict(achieved=hbm_gbs, peak=peaks["hbm_gbs"], unit="GB/s",
+                 frac=hbm_gbs / peaks["hbm_gbs"], bytes_per_step=hbm_bytes,
+                 peak_source=peaks["source"]),
+        cpu_baseline=cpu,
+        e2e=dict(value=e2e_value, unit=UNIT, h2d_bytes_per_step=n * cfg.n_features * 4,
+                 d2h_bytes_per_step=n * (F.n_out * 4 + 4)),
+        gpu_launches=launches_per_step * args.steps,
+        clocks=clocks, wall_s=wall, layout_s=layout_s)
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

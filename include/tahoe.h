@@ -1,0 +1,228 @@
+/*
+ * include/tahoe.h — C ABI of the B200-native Tahoe forest-inference engine (libtahoe.so).
+ *
+ * The path (BASELINE.json north_star): for every (sample, tree) pair walk
+ * root -> leaf by the node test "x_j < b_i", then combine the
+ * per-tree leaf values per sample.  The calls follow the paper's Algorithm 1
+ * (P:1360-1419): an online CPU step that rearranges nodes and trees once per forest
+ * (tahoe_forest_layout, lines 5-7) and an online GPU step per batch that picks a strategy with a
+ * cost model and launches it (tahoe_predict, lines 8-15).
+ *
+ * Conventions
+ *  - Every symbol is extern "C"; no C++ exception crosses the boundary.  Every call returns a
+ *    tahoe_status; tahoe_last_error() gives a thread-local message for the last failure.
+ *  - Node arrays use GLOBAL node indices: tree t's root is root[t]; children index the same arrays.
+ *  - X is row-major float32, n rows x d columns; sample i's attribute j is X[i*d + j].
+ *  - Device pointers are raw CUDA device pointers on the forest's device; `stream` is a
+ *    cudaStream_t (NULL = legacy default stream).  All GPU work is enqueued asynchronously; device
+ *    faults surface at the caller's next synchronisation.
+ *  - Results never depend on the layout: leaf ids are the caller's node ids and sums are fp64
+ *    (reading Z17); with dyadic leaf values every output is bit-identical across layouts.
+ *  - There is no CPU fallback: prediction runs only in this library's sm_100a kernels.
+ */
+#ifndef TAHOE_H
+#define TAHOE_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tahoe_forest tahoe_forest;   /* opaque; owns its host and device images */
+typedef struct CUstream_st* tahoe_stream;   /* == cudaStream_t */
+
+typedef enum {
+  TAHOE_OK = 0,
+  TAHOE_E_INVAL = 1,        /* invalid argument or invalid forest                          */
+  TAHOE_E_NOMEM = 2,        /* host or device allocation failed                            */
+  TAHOE_E_CUDA = 3,         /* CUDA runtime error (launch, copy, no device)                */
+  TAHOE_E_UNSUPPORTED = 4,  /* valid input outside what the encoding supports              */
+  TAHOE_E_STATE = 5         /* call not allowed in this handle state (e.g. host-only)     */
+} tahoe_status;
+
+/* How per-tree leaf values v(i,t) are combined per sample (north star; reading Z14). */
+typedef enum {
+  TAHOE_AGG_SUM = 0,        /* out[i]     = base + sum_t v(i,t)                                 */
+  TAHOE_AGG_AVERAGE = 1,    /* out[i]     = base + (sum_t v(i,t)) / T        (fp64 divide)      */
+  TAHOE_AGG_BINARY = 2,     /* out[i]     = base + sum_t v(i,t); class = out > 0 (fp64; 0 -> 0)  */
+  TAHOE_AGG_CLASS_SUM = 3,  /* out[i*C+c] = base + sum_{t: class(t)=c} v(i,t); class = argmax,
+                               ties -> lowest c                                               */
+  TAHOE_AGG_VOTE = 4        /* out[i*C+c] = #{t : v(i,t) == c}; class = argmax, ties -> lowest */
+} tahoe_agg;
+
+/* Strategies (Algorithm 1 line 15, re-targeted to B200). */
+typedef enum {
+  TAHOE_STRATEGY_AUTO = -1,   /* cost model (Algorithm 1 lines 8-13)                          */
+  TAHOE_STRATEGY_DIRECT = 0,  /* lane = sample; forest image in HBM/L2 (paper's "direct")     */
+  TAHOE_STRATEGY_SLICED = 1   /* lane = tree; forest slices resident in shared memory, sample
+                                 tiles staged by TMA ("shared forest" / "splitting shared
+                                 forest")                                        */
+} tahoe_strategy;
+
+/*
+ * tahoe_forest_build — validate and copy a forest, encode it with the default layout (input tree
+ * order, left child first), upload it to `device`.  Passage: P:181-192 (binary trees, node =
+ * attribute index + threshold), P:397-399 (default path D).
+ *
+ *  n_trees, root[n_trees]      global index of each tree's root
+ *  n_nodes                     length of the node arrays
+ *  feature[n_nodes]            attribute index; < 0 marks a leaf
+ *  threshold[n_nodes]          internal node: go LEFT iff x[feature] < threshold (IEEE fp32)
+ *  left/right[n_nodes]         children (ignored for leaves)
+ *  leaf_value[n_nodes]         leaf value (VOTE: the class id, an integer in [0, n_classes))
+ *  default_left[n_nodes]|NULL  NaN goes left iff 1; NULL => NaN follows the comparison (right)
+ *  tree_class[n_trees]|NULL    class of each tree for CLASS_SUM; NULL => t % n_classes
+ *  n_features                  attributes per sample the forest may address (feature < it)
+ *  n_classes                   1 for SUM/AVERAGE/BINARY; C >= 1 for CLASS_SUM/VOTE
+ *  device                      CUDA device ordinal, or -1 for a HOST-ONLY handle (layout and
+ *                              introspection only; prediction returns TAHOE_E_STATE)
+ * Ownership: every array is copied; the caller keeps its buffers.  *out is owned by the caller
+ * and released with tahoe_forest_free.
+ * Errors: E_INVAL on n_trees < 1, n_classes < 1, a feature outside [0, n_features), a child
+ * outside [0, n_nodes), a node reachable twice (shared or cyclic), a NaN threshold, tree_class
+ * out of range, VOTE leaves that are not integers in [0, n_classes), NULL required pointers.
+ * Unreachable nodes are ignored.  E_CUDA if `device` is not usable.
+ */
+tahoe_status tahoe_forest_build(int32_t n_trees, const int32_t* root, int32_t n_nodes,
+                                const int32_t* feature, const float* threshold,
+                                const int32_t* left, const int32_t* right,
+                                const float* leaf_value, const uint8_t* default_left,
+                                const int32_t* tree_class, int32_t n_features, int32_t n_classes,
+                                tahoe_agg agg, float base_score, int32_t device,
+                                tahoe_forest** out);
+
+/* Layout options; zero fields take the paper's defaults T_nodes=4, L_hash=128, M=64.
+ * node_reorder / tree_group: 1 = on (default), 0 = off (ablation switches, EX8).            */
+typedef struct {
+  int32_t t_nodes, l_hash, m_chunks;
+  int32_t node_reorder, tree_group;
+  int32_t _reserved;
+  uint64_t seed;
+} tahoe_layout_opts;
+
+/*
+ * tahoe_forest_layout — Algorithm 1 lines 5-7 on the host: count how many of the
+ * n_calib calibration rows take each edge (edge / node probability), put the more
+ * probable child of every node next to it (probability-based node rearrangement),
+ * order trees by SimHash/LSH similarity and deal them into balanced work units, then
+ * re-encode and re-upload.  X_calib_host: HOST pointer, n_calib x d row-major float32.
+ * opts may be NULL (defaults).  Mutates the handle: must not overlap predictions on it.
+ * Results of later predictions are unchanged bit for bit (leaf ids, classes; sums are fp64).
+ */
+tahoe_status tahoe_forest_layout(tahoe_forest* f, const float* X_calib_host, int64_t n_calib,
+                                 int32_t d, const tahoe_layout_opts* opts);
+
+/*
+ * tahoe_predict — Algorithm 1 lines 8-15 per batch: cost model, launch.  X: DEVICE pointer
+ * n x d row-major float32 (d >= largest attribute index used by the forest + 1; extra columns are
+ * ignored); out: DEVICE float32 n x n_out (n_out = tahoe_forest_n_outputs).  n == 0 is a no-op.
+ * Returns E_INVAL on a too-small d or NULL pointers with n > 0, E_STATE on a host-only handle,
+ * E_CUDA on launch failure.
+ * X and out are borrowed and must stay valid until the work enqueued on `stream` completes.
+ * Concurrent predictions on one handle from several threads/streams are allowed.
+ */
+tahoe_status tahoe_predict(const tahoe_forest* f, const float* X, int64_t n, int32_t d,
+                           float* out, tahoe_stream stream);
+
+typedef struct {
+  int32_t* out_class;         /* DEVICE int32[n] (BINARY / CLASS_SUM / VOTE), or NULL           */
+  int32_t* out_leaf;          /* DEVICE int32[n*T]: leaf reached in tree t (caller's node id),
+                                 caller's tree order, or NULL                                  */
+  uint64_t* out_fingerprint;  /* DEVICE uint64[n]: sum_t mix64(((u64)t << 32) | leaf) mod 2^64,
+                                 mix64 = splitmix64 finaliser, or NULL                         */
+  int32_t force_strategy;     /* tahoe_strategy; -1 = cost model                                */
+  int32_t _reserved;
+  void* ev_main_begin;        /* cudaEvent_t or NULL: recorded on `stream` right before / after  */
+  void* ev_main_end;          /*   the main traversal kernel (bench-side kernel timing)          */
+} tahoe_predict_opts;
+
+/* tahoe_predict with optional class / leaf / fingerprint outputs and a forced strategy. */
+tahoe_status tahoe_predict_ex(const tahoe_forest* f, const float* X, int64_t n, int32_t d,
+                              float* out, const tahoe_predict_opts* opts, tahoe_stream stream);
+
+/*
+ * tahoe_predict_host — the end-to-end call with HOST buffers: X_host (n x d float32), out_host
+ * (n x n_out float32) and class_host (int32[n] or NULL) are host pointers (pinned memory gives
+ * overlapped copies).  The batch is cut into chunks; host->device copies, prediction and
+ * device->host copies of consecutive chunks overlap on internal streams; `stream` is made to
+ * wait for all of it, so events recorded on `stream` bracket the whole transfer + compute.
+ * The host buffers must stay valid until `stream` reaches that point.
+ */
+tahoe_status tahoe_predict_host(const tahoe_forest* f, const float* X_host, int64_t n, int32_t d,
+                                float* out_host, int32_t* class_host, tahoe_stream stream);
+
+/* ---------------- tree sharding (multi-GPU) ---------------- */
+
+/* Sub-forest of the trees assigned to `rank` of `world` (balanced by expected visits per tree,
+ * deterministic), encoded and uploaded to `device` (-1 = host-only).  The shard keeps the full
+ * forest's layout decisions.  Caller frees *shard. */
+tahoe_status tahoe_forest_shard(const tahoe_forest* f, int32_t rank, int32_t world,
+                                int32_t device, tahoe_forest** shard);
+
+/* Raw fp64 sums of the shard's trees, DEVICE partial[n * n_out] (no base, no average, no argmax;
+ * VOTE: vote counts).  Summing the partials of all shards (e.g. NCCL reduce) and finalising with
+ * the full forest reproduces tahoe_predict. */
+tahoe_status tahoe_predict_partial(const tahoe_forest* shard, const float* X, int64_t n, int32_t d,
+                                   double* partial, tahoe_stream stream);
+
+/* out[n * n_out] (+ out_class[n] or NULL) from summed raw partials, using the FULL forest's
+ * aggregation, base score and tree count. */
+tahoe_status tahoe_finalize(const tahoe_forest* full, const double* partial, int64_t n,
+                            float* out, int32_t* out_class, tahoe_stream stream);
+
+/* ---------------- queries ---------------- */
+int32_t tahoe_forest_n_outputs(const tahoe_forest* f);   /* 1 or n_classes; -1 on NULL        */
+int32_t tahoe_forest_n_trees(const tahoe_forest* f);
+/* JSON object with realised forest and layout statistics (nodes, leaves, depths, expected
+ * visits per sample, encoded bytes, slices, chosen strategy for a batch size, ...). */
+tahoe_status tahoe_forest_stats(const tahoe_forest* f, char* buf, int64_t buf_len);
+/* Strategy the cost model picks for a batch of n rows of width d (Algorithm 1 lines 8-13). */
+int32_t tahoe_select_strategy(const tahoe_forest* f, int64_t n, int32_t d);
+void tahoe_forest_free(tahoe_forest* f);                  /* synchronise in-flight work first  */
+const char* tahoe_last_error(void);                       /* thread-local, never NULL          */
+
+/* ---------------- layout introspection (host-only; used by tests, no GPU needed) ----------- */
+
+/* Per ORIGINAL node: calibration visit count and hot_is_left (1 = left child stays next to the
+ * node); per tree: expected nodes read per sample; the similarity tree order.  Any pointer may be
+ * NULL.  Arrays: count[n_nodes], hot_left[n_nodes], exp_reads[n_trees], order[n_trees]. */
+tahoe_status tahoe_forest_layout_info(const tahoe_forest* f, uint64_t* count, uint8_t* hot_left,
+                                      double* exp_reads, int32_t* order);
+
+/* Tokens of tree t (reading Z6): windows of t_nodes caller node ids (-1 padded), each with the
+ * node probability of its last node; ordered by last node in hot-first preorder.  Writes at most
+ * cap tokens and sets *n_tokens to the total. */
+tahoe_status tahoe_tree_tokens(const tahoe_forest* f, int32_t t, int32_t t_nodes,
+                               int32_t* token_nodes, double* weights, int32_t cap,
+                               int32_t* n_tokens);
+
+/* The L_hash-bit SimHash of tree t: checksum[l_hash] and normalised bits[l_hash]. */
+tahoe_status tahoe_tree_simhash(const tahoe_forest* f, int32_t t, int32_t t_nodes, int32_t l_hash,
+                                double* checksum, uint8_t* bits);
+
+/* Pure SimHash of given +-1 strings (n_str x l_hash int8) and weights. */
+tahoe_status tahoe_simhash(const int8_t* strings, const double* weights, int32_t n_str,
+                           int32_t l_hash, double* checksum, uint8_t* bits);
+
+/* LSH: bits[n_trees x l_hash] -> collisions[n_trees x n_trees] (or NULL) and the
+ * greedy similarity order[n_trees] (reading Z11). */
+tahoe_status tahoe_lsh_order(const uint8_t* bits, int32_t n_trees, int32_t l_hash,
+                             int32_t m_chunks, int32_t* collisions, int32_t* order);
+
+/* SHA1 digest (FIPS 180-4) used by tokenisation. */
+tahoe_status tahoe_sha1(const uint8_t* msg, int64_t len, uint8_t digest[20]);
+
+/* Export of the encoded SLICED image for host-side decoding in tests:
+ *   header[0..7] = {n_slices, slots_max, feature_bits, n_trees, n_classes, 0, 0, 0}
+ *   slice_info[n_slices*4] = {slots, class, n_trees_in_slice, 0}
+ *   col_len[n_slices*32], nodes[n_slices*slots_max*32] (uint2 as uint32 pairs),
+ *   leaf_meta[n_slices*slots_max*32*2] = {caller tree index, caller node id} at leaf slots.
+ * Any array pointer may be NULL (then only header is filled). */
+tahoe_status tahoe_forest_export_sliced(const tahoe_forest* f, int32_t* header,
+                                        int32_t* slice_info, int32_t* col_len, uint32_t* nodes,
+                                        int32_t* leaf_meta);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TAHOE_H */

@@ -1,0 +1,646 @@
+// capi.cpp — the extern "C" boundary of libtahoe.so (include/tahoe.h), Algorithm 1's online
+// steps: layout on the host once per forest, strategy choice + launch per batch.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <sstream>
+#include <string>
+
+#include "internal.hpp"
+
+namespace tahoe {
+
+static thread_local std::string g_err;
+
+tahoe_status fail(tahoe_status st, const std::string& msg) {
+  g_err = msg;
+  return st;
+}
+
+static tahoe_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(TAHOE_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+// Restores the caller's current device on scope exit (torch owns the thread's device state).
+struct DeviceGuard {
+  int prev = -1;
+  bool ok = true;
+  explicit DeviceGuard(int dev) {
+    if (dev < 0) return;
+    cudaGetDevice(&prev);
+    if (prev != dev) ok = cudaSetDevice(dev) == cudaSuccess;
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+constexpr int32_t kDefaultMaxSmem = 232448;  // sharedMemPerBlockOptin on sm_100 (227 KB)
+constexpr int32_t kBarrierBytes = 64;
+
+// Rows of a sample tile staged in shared memory for a row width of d floats (0 = read rows from
+// global memory): 64 rows (2 per warp) when two buffers fit in 48 KB, else 32 rows within 64 KB.
+static int32_t tile_rows_for(int32_t d) {
+  const int64_t row = (int64_t)d * 4;
+  if (2 * 64 * row <= 48 * 1024) return 64;
+  if (2 * 32 * row <= 64 * 1024) return 32;
+  return 0;
+}
+
+static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
+  const int32_t R = tile_rows_for(n_features);
+  const int64_t reserve = (int64_t)2 * R * n_features * 4 + kBarrierBytes;
+  return (int32_t)std::max<int64_t>(0, (max_smem - reserve) / 256);
+}
+
+static void free_device(tahoe_forest* f) {
+  if (f->device < 0) return;
+  DeviceGuard g(f->device);
+  cudaFree((void*)f->dd.nodes);
+  cudaFree((void*)f->dd.root);
+  cudaFree((void*)f->dd.cls);
+  cudaFree((void*)f->dd.tree_orig);
+  cudaFree((void*)f->ds.nodes);
+  cudaFree((void*)f->ds.col_len);
+  cudaFree((void*)f->ds.slots);
+  cudaFree((void*)f->ds.leaf_meta);
+  cudaFree(f->d_class_ptr);
+  cudaFree(f->d_class_parts);
+  f->dd = DevDirect();
+  f->ds = DevSliced();
+  f->d_class_ptr = f->d_class_parts = nullptr;
+}
+
+template <class T>
+static tahoe_status upload(const std::vector<T>& v, const T** dst) {
+  if (v.empty()) { *dst = nullptr; return TAHOE_OK; }
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, v.size() * sizeof(T));
+  if (e != cudaSuccess) return fail(TAHOE_E_NOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+  e = cudaMemcpy(p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) { cudaFree(p); return cuda_fail(e, "cudaMemcpy"); }
+  *dst = static_cast<const T*>(p);
+  return TAHOE_OK;
+}
+
+// encode both images with the current layout state and (re)upload them (Algorithm 1 line 7)
+static tahoe_status encode_and_upload(tahoe_forest* f) {
+  tahoe_status st = encode_direct(f->host, f->di);
+  if (st != TAHOE_OK) return st;
+  st = encode_sliced(f->host, f->slot_budget, f->sl);
+  if (st != TAHOE_OK) return st;
+  if (f->device < 0) return TAHOE_OK;
+  DeviceGuard g(f->device);
+  if (!g.ok) return fail(TAHOE_E_CUDA, "cannot select device");
+  free_device(f);
+  if ((st = upload(f->di.nodes, &f->dd.nodes)) != TAHOE_OK) return st;
+  if ((st = upload(f->di.root, &f->dd.root)) != TAHOE_OK) return st;
+  if ((st = upload(f->di.cls, &f->dd.cls)) != TAHOE_OK) return st;
+  if ((st = upload(f->di.tree_orig, &f->dd.tree_orig)) != TAHOE_OK) return st;
+  f->dd.n_slots = (int32_t)f->di.root.size();
+  f->dd.fbits = f->di.fbits;
+  f->dd.n_nodes = (int64_t)f->di.nodes.size() / 2;
+  if (f->sl.valid) {
+    if ((st = upload(f->sl.nodes, &f->ds.nodes)) != TAHOE_OK) return st;
+    if ((st = upload(f->sl.col_len, &f->ds.col_len)) != TAHOE_OK) return st;
+    if ((st = upload(f->sl.slots, &f->ds.slots)) != TAHOE_OK) return st;
+    if ((st = upload(f->sl.leaf_meta, &f->ds.leaf_meta)) != TAHOE_OK) return st;
+    const int32_t* cp = nullptr;
+    const int32_t* cq = nullptr;
+    if ((st = upload(f->sl.class_ptr, &cp)) != TAHOE_OK) return st;
+    if ((st = upload(f->sl.class_parts, &cq)) != TAHOE_OK) return st;
+    f->d_class_ptr = const_cast<int32_t*>(cp);
+    f->d_class_parts = const_cast<int32_t*>(cq);
+    f->ds.n_slices = f->sl.n_slices;
+    f->ds.slots_max = f->sl.slots_max;
+    f->ds.fbits = f->sl.fbits;
+  }
+  return TAHOE_OK;
+}
+
+static tahoe_status init_handle(tahoe_forest* f, int32_t device) {
+  f->device = device;
+  f->num_sms = 148;
+  f->max_smem = kDefaultMaxSmem;
+  if (device >= 0) {
+    int cnt = 0;
+    cudaError_t e = cudaGetDeviceCount(&cnt);
+    if (e != cudaSuccess || device >= cnt) return fail(TAHOE_E_CUDA, "no such CUDA device");
+    int v = 0;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device) == cudaSuccess) f->num_sms = v;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, device) == cudaSuccess) f->max_smem = v;
+  }
+  f->slot_budget = slot_budget_for(f->max_smem, f->host.n_features);
+  return TAHOE_OK;
+}
+
+static PlanStats plan_stats(const tahoe_forest* f) {
+  PlanStats st;
+  for (double v : f->host.exp_reads) st.V += v;
+  st.sliced_ok = f->sl.valid;
+  st.sliced_eff = f->sl.eff;
+  st.n_slices = f->sl.n_slices;
+  return st;
+}
+
+static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t forced) {
+  if (forced < 0) {
+    const char* env = std::getenv("TAHOE_FORCE_STRATEGY");
+    if (env && *env) forced = std::atoi(env);
+  }
+  if (forced == TAHOE_STRATEGY_DIRECT) return TAHOE_STRATEGY_DIRECT;
+  if (forced == TAHOE_STRATEGY_SLICED) return f->sl.valid ? TAHOE_STRATEGY_SLICED : -2;
+  return select_strategy(plan_stats(f), n, d, f->host.agg);
+}
+
+static SlicedPlan sliced_plan(const tahoe_forest* f, int32_t d) {
+  SlicedPlan p;
+  p.forest_smem = f->sl.slots_max * 256;
+  const int64_t left = (int64_t)f->max_smem - p.forest_smem - kBarrierBytes;
+  int32_t R = tile_rows_for(d);
+  while (R >= 32 && 2LL * R * d * 4 > left) R -= 32;
+  p.rows_in_smem = R >= 32;
+  p.tile_rows = p.rows_in_smem ? R : 128;
+  p.smem_bytes = p.forest_smem + (p.rows_in_smem ? 2 * R * d * 4 : 0) + kBarrierBytes;
+  const int32_t ns = f->sl.n_slices;
+  if (ns <= f->num_sms) {
+    p.cps = std::max(1, f->num_sms / ns);
+    p.grid = ns * p.cps;
+  } else {
+    p.cps = 1;
+    p.grid = f->num_sms;
+  }
+  p.block = 1024;
+  return p;
+}
+
+// One batch on the device.  mode 0: final outputs; mode 1: raw fp64 partial [n x n_out].
+static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_t d, float* out,
+                        int32_t* out_class, int32_t* out_leaf, uint64_t* out_fp, double* raw_user,
+                        int32_t forced, cudaStream_t st, void* ev_b = nullptr, void* ev_e = nullptr) {
+  const Forest& H = f->host;
+  const int32_t C = H.n_out();
+  const int32_t strat = choose(f, n, d, forced);
+  if (strat == -2) return fail(TAHOE_E_UNSUPPORTED, "sliced strategy unavailable: " + f->sl.why_invalid);
+  cudaError_t e;
+  if (out_fp && (e = cudaMemsetAsync(out_fp, 0, (size_t)n * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
+  OutArgs o;
+  o.out = out;
+  o.out_class = out_class;
+  o.out_leaf = out_leaf;
+  o.out_fp = out_fp;
+  o.agg = H.agg;
+  o.base = H.base;
+  o.n_trees_full = H.n_trees_full;
+  o.n_classes = C;
+  o.T_leaf = H.n_trees_full;
+  FinalizeArgs fa;
+  fa.n_classes = C;
+  fa.agg = H.agg;
+  fa.base = H.base;
+  fa.n_trees_full = H.n_trees_full;
+  fa.n = n;
+  fa.out = out;
+  fa.out_class = out_class;
+  fa.raw_out = raw_user;
+  const bool scalar = C == 1 && H.agg != TAHOE_AGG_VOTE;
+  if (strat == TAHOE_STRATEGY_DIRECT) {
+    if (scalar && !raw_user) {
+      if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+      int rc = launch_direct(f->dd, X, n, d, o, true, f->num_sms, st);
+      if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+      if (rc) return cuda_fail((cudaError_t)rc, "direct kernel");
+      return TAHOE_OK;
+    }
+    double* raw = raw_user;
+    if (!raw && (e = cudaMallocAsync((void**)&raw, (size_t)n * C * 8, st)) != cudaSuccess)
+      return fail(TAHOE_E_NOMEM, "cudaMallocAsync partial");
+    if ((e = cudaMemsetAsync(raw, 0, (size_t)n * C * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
+    o.raw = raw;
+    if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+    int rc = launch_direct(f->dd, X, n, d, o, false, f->num_sms, st);
+    if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+    if (rc) return cuda_fail((cudaError_t)rc, "direct kernel");
+    if (!raw_user) {
+      fa.partial = raw;
+      fa.part_stride = 1;
+      fa.row_stride = C;
+      rc = launch_finalize(fa, st);
+      cudaFreeAsync(raw, st);
+      if (rc) return cuda_fail((cudaError_t)rc, "finalize kernel");
+    }
+    return TAHOE_OK;
+  }
+  // sliced
+  const SlicedPlan plan = sliced_plan(f, d);
+  const bool fused = scalar && !raw_user && f->sl.n_slices == 1;
+  double* part = nullptr;
+  if (!fused) {
+    if ((e = cudaMallocAsync((void**)&part, (size_t)f->sl.n_slices * n * 8, st)) != cudaSuccess)
+      return fail(TAHOE_E_NOMEM, "cudaMallocAsync partial");
+    o.raw = part;
+  }
+  if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+  int rc = launch_sliced(f->ds, plan, X, n, d, o, fused, st);
+  if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+  if (rc) { if (part) cudaFreeAsync(part, st); return cuda_fail((cudaError_t)rc, "sliced kernel"); }
+  if (!fused) {
+    fa.partial = part;
+    fa.part_stride = n;
+    fa.row_stride = 1;
+    fa.class_ptr = f->d_class_ptr;
+    fa.class_parts = f->d_class_parts;
+    rc = launch_finalize(fa, st);
+    cudaFreeAsync(part, st);
+    if (rc) return cuda_fail((cudaError_t)rc, "finalize kernel");
+  }
+  return TAHOE_OK;
+}
+
+static tahoe_status check_predict(const tahoe_forest* f, const float* X, int64_t n, int32_t d,
+                                  const void* out) {
+  if (!f) return fail(TAHOE_E_INVAL, "NULL forest");
+  if (n < 0) return fail(TAHOE_E_INVAL, "n < 0");
+  if (f->device < 0) return fail(TAHOE_E_STATE, "host-only forest handle (device = -1)");
+  if (n == 0) return TAHOE_OK;
+  if (!X || !out) return fail(TAHOE_E_INVAL, "NULL X or output pointer");
+  if (d < f->host.max_feature + 1 || d < 1)
+    return fail(TAHOE_E_INVAL, "d = " + std::to_string(d) + " < largest attribute index + 1 (" +
+                                   std::to_string(f->host.max_feature + 1) + ")");
+  return TAHOE_OK;
+}
+
+}  // namespace tahoe
+
+using namespace tahoe;
+
+#define TAHOE_GUARD_BEGIN try {
+#define TAHOE_GUARD_END                                                         \
+  }                                                                             \
+  catch (const std::bad_alloc&) { return fail(TAHOE_E_NOMEM, "host allocation failed"); } \
+  catch (const std::exception& ex) { return fail(TAHOE_E_INVAL, ex.what()); }  \
+  catch (...) { return fail(TAHOE_E_INVAL, "unknown exception"); }
+
+extern "C" {
+
+__attribute__((visibility("default"))) const char* tahoe_last_error(void) { return g_err.c_str(); }
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_build(
+    int32_t n_trees, const int32_t* root, int32_t n_nodes, const int32_t* feature,
+    const float* threshold, const int32_t* left, const int32_t* right, const float* leaf_value,
+    const uint8_t* default_left, const int32_t* tree_class, int32_t n_features, int32_t n_classes,
+    tahoe_agg agg, float base_score, int32_t device, tahoe_forest** out) {
+  TAHOE_GUARD_BEGIN
+  if (!out) return fail(TAHOE_E_INVAL, "NULL out");
+  *out = nullptr;
+  tahoe_forest* f = new tahoe_forest();
+  tahoe_status st = build_forest(f->host, n_trees, root, n_nodes, feature, threshold, left, right,
+                                 leaf_value, default_left, tree_class, n_features, n_classes,
+                                 (int32_t)agg, base_score);
+  if (st == TAHOE_OK) st = init_handle(f, device);
+  if (st == TAHOE_OK) st = encode_and_upload(f);
+  if (st != TAHOE_OK) { free_device(f); delete f; return st; }
+  *out = f;
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_layout(
+    tahoe_forest* f, const float* X_calib_host, int64_t n_calib, int32_t d,
+    const tahoe_layout_opts* opts) {
+  TAHOE_GUARD_BEGIN
+  if (!f) return fail(TAHOE_E_INVAL, "NULL forest");
+  if (n_calib < 0 || (n_calib > 0 && !X_calib_host)) return fail(TAHOE_E_INVAL, "bad calibration set");
+  if (n_calib > 0 && d < f->host.max_feature + 1) return fail(TAHOE_E_INVAL, "calibration d too small");
+  tahoe_layout_opts o{};
+  if (opts) o = *opts;
+  else { o.node_reorder = 1; o.tree_group = 1; }
+  if (o.t_nodes <= 0) o.t_nodes = 4;
+  if (o.l_hash <= 0) o.l_hash = 128;
+  if (o.m_chunks <= 0) o.m_chunks = 64;
+  if (o.m_chunks > o.l_hash) return fail(TAHOE_E_INVAL, "m_chunks > l_hash");
+  Forest& F = f->host;
+  F.opts = o;
+  if (n_calib > 0) calibrate(F, X_calib_host, n_calib, d);
+  reorder_nodes(F, o.node_reorder != 0);
+  order_trees(F);
+  return encode_and_upload(f);
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_predict_ex(
+    const tahoe_forest* f, const float* X, int64_t n, int32_t d, float* out,
+    const tahoe_predict_opts* opts, tahoe_stream stream) {
+  TAHOE_GUARD_BEGIN
+  tahoe_status st = check_predict(f, X, n, d, out);
+  if (st != TAHOE_OK || n == 0) return st;
+  DeviceGuard g(f->device);
+  tahoe_predict_opts o{};
+  o.force_strategy = -1;
+  if (opts) o = *opts;
+  return run(f, X, n, d, out, o.out_class, o.out_leaf, o.out_fingerprint, nullptr, o.force_strategy,
+             reinterpret_cast<cudaStream_t>(stream), o.ev_main_begin, o.ev_main_end);
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_predict(
+    const tahoe_forest* f, const float* X, int64_t n, int32_t d, float* out, tahoe_stream stream) {
+  return tahoe_predict_ex(f, X, n, d, out, nullptr, stream);
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
+    const tahoe_forest* f, const float* X_host, int64_t n, int32_t d, float* out_host,
+    int32_t* class_host, tahoe_stream stream) {
+  TAHOE_GUARD_BEGIN
+  tahoe_status st = check_predict(f, X_host, n, d, out_host);
+  if (st != TAHOE_OK || n == 0) return st;
+  DeviceGuard g(f->device);
+  cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
+  const int32_t C = f->host.n_out();
+  const int64_t chunk = std::min<int64_t>(n, std::max<int64_t>(65536, (n + 7) / 8));
+  const int64_t nchunks = (n + chunk - 1) / chunk;
+  cudaStream_t s_in, s_cmp, s_out;
+  cudaStreamCreateWithFlags(&s_in, cudaStreamNonBlocking);
+  cudaStreamCreateWithFlags(&s_cmp, cudaStreamNonBlocking);
+  cudaStreamCreateWithFlags(&s_out, cudaStreamNonBlocking);
+  cudaEvent_t ev_start, ev_in[2], ev_cmp[2], ev_out[2];
+  cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming);
+  for (int b = 0; b < 2; b++) {
+    cudaEventCreateWithFlags(&ev_in[b], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_cmp[b], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&ev_out[b], cudaEventDisableTiming);
+  }
+  float* dX = nullptr;
+  float* dO = nullptr;
+  int32_t* dC = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&dX, (size_t)2 * chunk * d * 4, user);
+  if (e == cudaSuccess) e = cudaMallocAsync((void**)&dO, (size_t)2 * chunk * C * 4, user);
+  if (e == cudaSuccess && class_host) e = cudaMallocAsync((void**)&dC, (size_t)2 * chunk * 4, user);
+  cudaEventRecord(ev_start, user);
+  cudaStreamWaitEvent(s_in, ev_start, 0);
+  cudaStreamWaitEvent(s_cmp, ev_start, 0);
+  cudaStreamWaitEvent(s_out, ev_start, 0);
+  for (int64_t c = 0; c < nchunks && e == cudaSuccess && st == TAHOE_OK; c++) {
+    const int b = (int)(c & 1);
+    const int64_t r0 = c * chunk, nr = std::min(chunk, n - r0);
+    float* xb = dX + (size_t)b * chunk * d;
+    float* ob = dO + (size_t)b * chunk * C;
+    int32_t* cb = dC ? dC + (size_t)b * chunk : nullptr;
+    if (c >= 2) cudaStreamWaitEvent(s_in, ev_cmp[b], 0);     // X buffer consumed by chunk c-2
+    e = cudaMemcpyAsync(xb, X_host + r0 * d, (size_t)nr * d * 4, cudaMemcpyHostToDevice, s_in);
+    cudaEventRecord(ev_in[b], s_in);
+    cudaStreamWaitEvent(s_cmp, ev_in[b], 0);
+    if (c >= 2) cudaStreamWaitEvent(s_cmp, ev_out[b], 0);    // out buffer drained by chunk c-2
+    if (e == cudaSuccess)
+      st = run(f, xb, nr, d, ob, cb, nullptr, nullptr, nullptr, -1, s_cmp);
+    cudaEventRecord(ev_cmp[b], s_cmp);
+    cudaStreamWaitEvent(s_out, ev_cmp[b], 0);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(out_host + r0 * C, ob, (size_t)nr * C * 4, cudaMemcpyDeviceToHost, s_out);
+    if (e == cudaSuccess && cb) e = cudaMemcpyAsync(class_host + r0, cb, (size_t)nr * 4, cudaMemcpyDeviceToHost, s_out);
+    cudaEventRecord(ev_out[b], s_out);
+  }
+  cudaEventRecord(ev_in[0], s_in);
+  cudaEventRecord(ev_cmp[0], s_cmp);
+  cudaEventRecord(ev_out[0], s_out);
+  cudaStreamWaitEvent(user, ev_in[0], 0);
+  cudaStreamWaitEvent(user, ev_cmp[0], 0);
+  cudaStreamWaitEvent(user, ev_out[0], 0);
+  if (dX) cudaFreeAsync(dX, user);
+  if (dO) cudaFreeAsync(dO, user);
+  if (dC) cudaFreeAsync(dC, user);
+  cudaEventDestroy(ev_start);
+  for (int b = 0; b < 2; b++) { cudaEventDestroy(ev_in[b]); cudaEventDestroy(ev_cmp[b]); cudaEventDestroy(ev_out[b]); }
+  cudaStreamDestroy(s_in);
+  cudaStreamDestroy(s_cmp);
+  cudaStreamDestroy(s_out);
+  if (st != TAHOE_OK) return st;
+  if (e != cudaSuccess) return cuda_fail(e, "tahoe_predict_host");
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_shard(
+    const tahoe_forest* f, int32_t rank, int32_t world, int32_t device, tahoe_forest** shard) {
+  TAHOE_GUARD_BEGIN
+  if (!f || !shard) return fail(TAHOE_E_INVAL, "NULL argument");
+  if (world < 1 || rank < 0 || rank >= world) return fail(TAHOE_E_INVAL, "bad rank/world");
+  *shard = nullptr;
+  tahoe_forest* s = new tahoe_forest();
+  s->host = make_shard(f->host, rank, world);
+  if (s->host.n_trees == 0) { delete s; return fail(TAHOE_E_INVAL, "shard has no trees (world > n_trees)"); }
+  tahoe_status st = init_handle(s, device);
+  if (st == TAHOE_OK) st = encode_and_upload(s);
+  if (st != TAHOE_OK) { free_device(s); delete s; return st; }
+  *shard = s;
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_predict_partial(
+    const tahoe_forest* shard, const float* X, int64_t n, int32_t d, double* partial,
+    tahoe_stream stream) {
+  TAHOE_GUARD_BEGIN
+  tahoe_status st = check_predict(shard, X, n, d, partial);
+  if (st != TAHOE_OK || n == 0) return st;
+  DeviceGuard g(shard->device);
+  return run(shard, X, n, d, nullptr, nullptr, nullptr, nullptr, partial, -1,
+             reinterpret_cast<cudaStream_t>(stream));
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_finalize(
+    const tahoe_forest* full, const double* partial, int64_t n, float* out, int32_t* out_class,
+    tahoe_stream stream) {
+  TAHOE_GUARD_BEGIN
+  if (!full) return fail(TAHOE_E_INVAL, "NULL forest");
+  if (n < 0) return fail(TAHOE_E_INVAL, "n < 0");
+  if (full->device < 0) return fail(TAHOE_E_STATE, "host-only forest handle");
+  if (n == 0) return TAHOE_OK;
+  if (!partial || !out) return fail(TAHOE_E_INVAL, "NULL pointer");
+  DeviceGuard g(full->device);
+  const Forest& H = full->host;
+  FinalizeArgs fa;
+  fa.partial = partial;
+  fa.part_stride = 1;
+  fa.row_stride = H.n_out();
+  fa.n_classes = H.n_out();
+  fa.agg = H.agg;
+  fa.base = H.base;
+  fa.n_trees_full = H.n_trees_full;
+  fa.n = n;
+  fa.out = out;
+  fa.out_class = out_class;
+  int rc = launch_finalize(fa, reinterpret_cast<cudaStream_t>(stream));
+  if (rc) return cuda_fail((cudaError_t)rc, "finalize kernel");
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) int32_t tahoe_forest_n_outputs(const tahoe_forest* f) {
+  return f ? f->host.n_out() : -1;
+}
+__attribute__((visibility("default"))) int32_t tahoe_forest_n_trees(const tahoe_forest* f) {
+  return f ? f->host.n_trees : -1;
+}
+
+__attribute__((visibility("default"))) int32_t tahoe_select_strategy(const tahoe_forest* f,
+                                                                     int64_t n, int32_t d) {
+  if (!f) return -1;
+  return choose(f, n, d, -1);
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tahoe_forest* f,
+                                                                       char* buf, int64_t len) {
+  TAHOE_GUARD_BEGIN
+  if (!f || !buf || len <= 0) return fail(TAHOE_E_INVAL, "bad argument");
+  const Forest& H = f->host;
+  int64_t leaves = 0;
+  int32_t maxd = 0;
+  for (size_t k = 0; k < H.feat.size(); k++) {
+    leaves += H.feat[k] < 0;
+    maxd = std::max(maxd, H.depth[k]);
+  }
+  double V = 0;
+  for (double v : H.exp_reads) V += v;
+  std::ostringstream js;
+  js.precision(6);
+  js << "{\"n_trees\":" << H.n_trees << ",\"n_trees_full\":" << H.n_trees_full
+     << ",\"nodes\":" << H.feat.size() << ",\"leaves\":" << leaves << ",\"max_depth\":" << maxd
+     << ",\"n_features\":" << H.n_features << ",\"n_classes\":" << H.n_classes
+     << ",\"agg\":" << H.agg << ",\"calibrated\":" << (H.calibrated ? "true" : "false")
+     << ",\"n_calib\":" << H.n_cal << ",\"expected_node_reads_per_sample\":" << V
+     << ",\"expected_visits_per_sample\":" << (V - H.n_trees)
+     << ",\"feature_bits\":" << f->di.fbits << ",\"direct_bytes\":" << f->di.bytes()
+     << ",\"bytes_fixed_index\":" << (int64_t)H.feat.size() * 12
+     << ",\"sliced_valid\":" << (f->sl.valid ? "true" : "false")
+     << ",\"sliced_why\":\"" << f->sl.why_invalid << "\""
+     << ",\"n_slices\":" << f->sl.n_slices << ",\"slots_max\":" << f->sl.slots_max
+     << ",\"slot_budget\":" << f->slot_budget << ",\"sliced_bytes\":" << f->sl.bytes()
+     << ",\"lockstep_eff\":" << f->sl.eff << ",\"trees_per_lane\":" << f->sl.trees_per_lane
+     << ",\"num_sms\":" << f->num_sms << ",\"max_smem\":" << f->max_smem << "}";
+  std::string s = js.str();
+  if ((int64_t)s.size() + 1 > len) return fail(TAHOE_E_INVAL, "buffer too small");
+  std::memcpy(buf, s.c_str(), s.size() + 1);
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) void tahoe_forest_free(tahoe_forest* f) {
+  if (!f) return;
+  free_device(f);
+  delete f;
+}
+
+// ------------------------------------------------------------------ introspection
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_layout_info(
+    const tahoe_forest* f, uint64_t* count, uint8_t* hot_left, double* exp_reads, int32_t* order) {
+  TAHOE_GUARD_BEGIN
+  if (!f) return fail(TAHOE_E_INVAL, "NULL forest");
+  const Forest& H = f->host;
+  if (count) std::fill(count, count + H.n_nodes_user, 0);
+  if (hot_left) std::fill(hot_left, hot_left + H.n_nodes_user, 1);
+  for (size_t k = 0; k < H.feat.size(); k++) {
+    if (count) count[H.orig[k]] = H.count[k];
+    if (hot_left) hot_left[H.orig[k]] = H.hot_left[k];
+  }
+  if (exp_reads) for (int32_t t = 0; t < H.n_trees; t++) exp_reads[t] = H.exp_reads[t];
+  if (order) for (int32_t i = 0; i < H.n_trees; i++) order[i] = H.tree_orig[H.order[i]];
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_tree_tokens(
+    const tahoe_forest* f, int32_t t, int32_t t_nodes, int32_t* token_nodes, double* weights,
+    int32_t cap, int32_t* n_tokens) {
+  TAHOE_GUARD_BEGIN
+  if (!f || t < 0 || t >= f->host.n_trees || t_nodes < 1 || !n_tokens) return fail(TAHOE_E_INVAL, "bad argument");
+  std::vector<int32_t> tok;
+  std::vector<double> w;
+  tree_tokens(f->host, t, t_nodes, tok, w);
+  *n_tokens = (int32_t)w.size();
+  for (int32_t i = 0; i < std::min<int32_t>(cap, (int32_t)w.size()); i++) {
+    for (int32_t j = 0; j < t_nodes; j++) {
+      int32_t k = tok[(size_t)i * t_nodes + j];
+      if (token_nodes) token_nodes[(size_t)i * t_nodes + j] = k < 0 ? -1 : f->host.orig[k];
+    }
+    if (weights) weights[i] = w[i];
+  }
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_tree_simhash(
+    const tahoe_forest* f, int32_t t, int32_t t_nodes, int32_t l_hash, double* checksum, uint8_t* bits) {
+  TAHOE_GUARD_BEGIN
+  if (!f || t < 0 || t >= f->host.n_trees || t_nodes < 1 || l_hash < 1) return fail(TAHOE_E_INVAL, "bad argument");
+  std::vector<double> cs;
+  std::vector<uint8_t> b;
+  tree_simhash(f->host, t, t_nodes, l_hash, cs, b);
+  if (checksum) std::copy(cs.begin(), cs.end(), checksum);
+  if (bits) std::copy(b.begin(), b.end(), bits);
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_simhash(
+    const int8_t* strings, const double* weights, int32_t n_str, int32_t l_hash, double* checksum,
+    uint8_t* bits) {
+  TAHOE_GUARD_BEGIN
+  if (!strings || !weights || !checksum || !bits || n_str < 0 || l_hash < 1) return fail(TAHOE_E_INVAL, "bad argument");
+  simhash(strings, weights, n_str, l_hash, checksum, bits);
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_lsh_order(
+    const uint8_t* bits, int32_t n_trees, int32_t l_hash, int32_t m_chunks, int32_t* collisions,
+    int32_t* order) {
+  TAHOE_GUARD_BEGIN
+  if (!bits || n_trees < 1 || l_hash < 1 || m_chunks < 1 || m_chunks > l_hash || !order)
+    return fail(TAHOE_E_INVAL, "bad argument");
+  std::vector<uint8_t> b(bits, bits + (size_t)n_trees * l_hash);
+  std::vector<uint16_t> col;
+  std::vector<int32_t> ord = lsh_order(b, n_trees, l_hash, m_chunks, &col);
+  std::copy(ord.begin(), ord.end(), order);
+  if (collisions) for (size_t i = 0; i < col.size(); i++) collisions[i] = col[i];
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_sha1(const uint8_t* msg, int64_t len,
+                                                               uint8_t digest[20]) {
+  if ((!msg && len > 0) || len < 0 || !digest) return fail(TAHOE_E_INVAL, "bad argument");
+  sha1(msg, (size_t)len, digest);
+  return TAHOE_OK;
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_export_sliced(
+    const tahoe_forest* f, int32_t* header, int32_t* slice_info, int32_t* col_len, uint32_t* nodes,
+    int32_t* leaf_meta) {
+  TAHOE_GUARD_BEGIN
+  if (!f || !header) return fail(TAHOE_E_INVAL, "bad argument");
+  const SlicedImage& S = f->sl;
+  int32_t h[8] = {S.valid ? S.n_slices : 0, S.slots_max, S.fbits, f->host.n_trees, f->host.n_classes, 0, 0, 0};
+  std::copy(h, h + 8, header);
+  if (!S.valid) return TAHOE_OK;
+  if (slice_info)
+    for (int32_t s = 0; s < S.n_slices; s++) {
+      slice_info[4 * s] = S.slots[s];
+      slice_info[4 * s + 1] = S.cls[s];
+      slice_info[4 * s + 2] = S.ntrees[s];
+      slice_info[4 * s + 3] = 0;
+    }
+  if (col_len) std::copy(S.col_len.begin(), S.col_len.end(), col_len);
+  if (nodes) std::copy(S.nodes.begin(), S.nodes.end(), nodes);
+  if (leaf_meta) std::copy(S.leaf_meta.begin(), S.leaf_meta.end(), leaf_meta);
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+}  // extern "C"

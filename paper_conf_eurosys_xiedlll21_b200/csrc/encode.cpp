@@ -1,0 +1,232 @@
+// encode.cpp — the adaptive forest format re-targeted to B200.
+//
+// Work units: the trees of one class, in similarity order, are cut into SLICES whose
+// nodes fit one CTA's shared memory; inside a slice each tree is dealt to one of 32 LANE COLUMNS
+// ("assigned to threads in a round-robin way, such that loads are roughly balanced"),
+// with a longest-processing-time alternative when it balances expected work better (reading Z12).
+// A lane column holds its trees back to back, each in hot-first preorder, so the hot
+// child of every node is the next slot.  Slot s of lane l lives at word pair (32*s + l): a warp
+// whose lanes read 32 different slots hits 32 different bank pairs.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+
+#include "internal.hpp"
+
+namespace tahoe {
+
+static uint32_t f2u(float f) { uint32_t u; std::memcpy(&u, &f, 4); return u; }
+
+// ------------------------------------------------------------------ direct image
+tahoe_status encode_direct(const Forest& F, DirectImage& D) {
+  D = DirectImage();
+  D.fbits = feature_bits(F.n_features);
+  const uint32_t off_lim = 1u << (kOffsetTop - D.fbits);
+  D.nodes.assign(F.feat.size() * 2, 0);
+  int64_t base = 0;
+  std::vector<int64_t> slot(F.feat.size());
+  for (int32_t t : F.order) {
+    std::vector<int32_t> pre = hot_preorder(F, t);
+    for (size_t i = 0; i < pre.size(); i++) slot[pre[i]] = base + (int64_t)i;
+    D.root.push_back((int32_t)base);
+    D.cls.push_back(F.tclass[t]);
+    D.tree_orig.push_back(F.tree_orig[t]);
+    for (size_t i = 0; i < pre.size(); i++) {
+      const int32_t k = pre[i];
+      const int64_t s = base + (int64_t)i;
+      uint32_t y;
+      if (F.feat[k] < 0) {
+        y = kLeafBit | (uint32_t)F.orig[k];
+        D.nodes[2 * s] = f2u(F.val[k]);
+      } else {
+        const int32_t hot = F.hot_left[k] ? F.lc[k] : F.rc[k];
+        const int32_t cold = F.hot_left[k] ? F.rc[k] : F.lc[k];
+        if (slot[hot] != s + 1) return fail(TAHOE_E_INVAL, "internal: hot child not adjacent");
+        const int64_t delta = slot[cold] - s;
+        if (delta <= 0 || (uint64_t)delta >= off_lim)
+          return fail(TAHOE_E_UNSUPPORTED, "tree too large for the node encoding (cold offset " +
+                                                std::to_string(delta) + ")");
+        y = (F.dl[k] ? kDefaultLeftBit : 0u) | (F.hot_left[k] ? kHotLeftBit : 0u) |
+            ((uint32_t)delta << D.fbits) | (uint32_t)F.feat[k];
+        D.nodes[2 * s] = f2u(F.thr[k]);
+      }
+      D.nodes[2 * s + 1] = y;
+    }
+    base += (int64_t)pre.size();
+  }
+  return TAHOE_OK;
+}
+
+// ------------------------------------------------------------------ sliced image
+struct Pack {
+  std::vector<std::vector<int32_t>> lanes = std::vector<std::vector<int32_t>>(32);
+  int32_t max_len = 0;
+  double max_work = 0, sum_work = 0;
+};
+
+static void pack_stats(const Forest& F, Pack& P) {
+  P.max_len = 0; P.max_work = 0; P.sum_work = 0;
+  for (auto& L : P.lanes) {
+    int32_t len = 0; double w = 0;
+    for (int32_t t : L) { len += F.tree_size(t); w += F.exp_reads[t]; }
+    P.max_len = std::max(P.max_len, len);
+    P.max_work = std::max(P.max_work, w);
+    P.sum_work += w;
+  }
+}
+
+static bool pack_round_robin(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
+  P = Pack();
+  for (size_t j = 0; j < trees.size(); j++) P.lanes[j % 32].push_back(trees[j]);
+  pack_stats(F, P);
+  return P.max_len <= cap;
+}
+
+static bool pack_lpt(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
+  P = Pack();
+  std::vector<int32_t> ts(trees);
+  std::stable_sort(ts.begin(), ts.end(), [&](int32_t a, int32_t b) {
+    if (F.exp_reads[a] != F.exp_reads[b]) return F.exp_reads[a] > F.exp_reads[b];
+    return F.tree_size(a) > F.tree_size(b);
+  });
+  std::vector<double> w(32, 0.0);
+  std::vector<int32_t> len(32, 0);
+  for (int32_t t : ts) {
+    int32_t best = -1;
+    for (int32_t l = 0; l < 32; l++) {
+      if (len[l] + F.tree_size(t) > cap) continue;
+      if (best < 0 || w[l] < w[best] || (w[l] == w[best] && len[l] < len[best])) best = l;
+    }
+    if (best < 0) return false;
+    P.lanes[best].push_back(t);
+    w[best] += F.exp_reads[t];
+    len[best] += F.tree_size(t);
+  }
+  pack_stats(F, P);
+  return true;
+}
+
+static bool pack_best(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
+  Pack a, b;
+  bool ra = pack_round_robin(F, trees, cap, a);
+  bool rb = pack_lpt(F, trees, cap, b);
+  if (!ra && !rb) return false;
+  if (ra && (!rb || a.max_work <= b.max_work * 1.000001)) P = a; else P = b;
+  return true;
+}
+
+tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
+  S = SlicedImage();
+  S.fbits = feature_bits(F.n_features);
+  if (F.agg == TAHOE_AGG_VOTE) { S.why_invalid = "VOTE runs on the direct strategy"; return TAHOE_OK; }
+  if (cap < 1) { S.why_invalid = "no shared memory budget"; return TAHOE_OK; }
+  for (int32_t t = 0; t < F.n_trees; t++)
+    if (F.tree_size(t) > cap) { S.why_invalid = "a tree exceeds one lane column of shared memory"; return TAHOE_OK; }
+
+  std::vector<std::vector<int32_t>> groups(F.n_classes);
+  for (int32_t t : F.order) groups[F.tclass[t]].push_back(t);
+  std::vector<Pack> packs;
+  for (int32_t c = 0; c < F.n_classes; c++) {
+    const auto& G = groups[c];
+    if (G.empty()) continue;
+    int64_t total = 0;
+    for (int32_t t : G) total += F.tree_size(t);
+    int32_t k = (int32_t)std::max<int64_t>(1, (int64_t)std::ceil((double)total / (32.0 * cap * 0.97)));
+    for (;; k++) {
+      if (k > (int32_t)G.size()) { S.why_invalid = "cannot pack trees into slices"; return TAHOE_OK; }
+      // k contiguous chunks of balanced node counts (each non-empty)
+      std::vector<size_t> cut((size_t)k + 1, 0);
+      cut[k] = G.size();
+      {
+        size_t pos = 0;
+        int64_t acc = 0;
+        for (int32_t j = 1; j < k; j++) {
+          const int64_t target = total * j / k;
+          while (pos < G.size() && acc < target) acc += F.tree_size(G[pos++]);
+          cut[j] = std::min(std::max(pos, cut[j - 1] + 1), G.size() - (size_t)(k - j));
+          pos = cut[j];
+          acc = 0;
+          for (size_t q = 0; q < pos; q++) acc += F.tree_size(G[q]);
+        }
+      }
+      std::vector<Pack> ps;
+      bool ok = true;
+      for (int32_t j = 0; j < k && ok; j++) {
+        std::vector<int32_t> chunk(G.begin() + cut[j], G.begin() + cut[j + 1]);
+        Pack P;
+        if (!pack_best(F, chunk, cap, P)) ok = false;
+        else { ps.push_back(P); S.cls.push_back(c); S.ntrees.push_back((int32_t)chunk.size()); }
+      }
+      if (ok) { packs.insert(packs.end(), ps.begin(), ps.end()); break; }
+      S.cls.resize(packs.size());
+      S.ntrees.resize(packs.size());
+    }
+  }
+  S.n_slices = (int32_t)packs.size();
+  S.slots_max = 0;
+  double work = 0, padded = 0;
+  for (auto& P : packs) {
+    S.slots_max = std::max(S.slots_max, P.max_len);
+    work += P.sum_work;
+    padded += 32.0 * P.max_work;
+  }
+  S.eff = padded > 0 ? work / padded : 0;
+  S.trees_per_lane = (double)F.n_trees / (32.0 * std::max(1, S.n_slices));
+  const uint32_t off_lim = 1u << (kOffsetTop - S.fbits);
+  const size_t per_slice = (size_t)S.slots_max * 32;
+  S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
+  S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
+  S.col_len.assign((size_t)S.n_slices * 32, 0);
+  S.slots.assign(S.n_slices, 0);
+  std::vector<int32_t> slot(F.feat.size(), -1);
+  for (int32_t s = 0; s < S.n_slices; s++) {
+    const Pack& P = packs[s];
+    S.slots[s] = P.max_len;
+    for (int32_t l = 0; l < 32; l++) {
+      int32_t pos = 0;
+      const auto& L = P.lanes[l];
+      for (size_t ti = 0; ti < L.size(); ti++) {
+        const int32_t t = L[ti];
+        std::vector<int32_t> pre = hot_preorder(F, t);
+        for (size_t i = 0; i < pre.size(); i++) slot[pre[i]] = pos + (int32_t)i;
+        const int32_t next_root = pos + (int32_t)pre.size();
+        for (size_t i = 0; i < pre.size(); i++) {
+          const int32_t k = pre[i];
+          const int32_t sl = pos + (int32_t)i;
+          const size_t w = ((size_t)s * per_slice + (size_t)sl * 32 + l);
+          uint32_t y;
+          if (F.feat[k] < 0) {
+            y = kLeafBit | (uint32_t)(next_root - sl);
+            S.nodes[2 * w] = f2u(F.val[k]);
+            S.leaf_meta[2 * w] = F.tree_orig[t];
+            S.leaf_meta[2 * w + 1] = F.orig[k];
+          } else {
+            const int32_t hot = F.hot_left[k] ? F.lc[k] : F.rc[k];
+            const int32_t cold = F.hot_left[k] ? F.rc[k] : F.lc[k];
+            if (slot[hot] != sl + 1) return fail(TAHOE_E_INVAL, "internal: hot child not adjacent");
+            const int32_t delta = slot[cold] - sl;
+            if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "cold offset overflow");
+            y = (F.dl[k] ? kDefaultLeftBit : 0u) | (F.hot_left[k] ? kHotLeftBit : 0u) |
+                ((uint32_t)delta << S.fbits) | (uint32_t)F.feat[k];
+            S.nodes[2 * w] = f2u(F.thr[k]);
+          }
+          S.nodes[2 * w + 1] = y;
+        }
+        pos = next_root;
+      }
+      S.col_len[(size_t)s * 32 + l] = pos;
+    }
+  }
+  // class -> slices (in slice order: the fixed fp64 summation order of the finalize step)
+  S.class_ptr.assign(F.n_classes + 1, 0);
+  for (int32_t s = 0; s < S.n_slices; s++) S.class_ptr[S.cls[s] + 1]++;
+  for (int32_t c = 0; c < F.n_classes; c++) S.class_ptr[c + 1] += S.class_ptr[c];
+  S.class_parts.assign(S.n_slices, 0);
+  std::vector<int32_t> fillp(S.class_ptr.begin(), S.class_ptr.end() - 1);
+  for (int32_t s = 0; s < S.n_slices; s++) S.class_parts[fillp[S.cls[s]]++] = s;
+  S.valid = true;
+  return TAHOE_OK;
+}
+
+}  // namespace tahoe

@@ -1,0 +1,126 @@
+// internal.hpp — host-side model of a forest, its layout state and its encoded images.
+// Everything here is product code (libtahoe.so); nothing is shared with oracle/.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "tahoe.h"
+#include "kernels.hpp"
+
+namespace tahoe {
+
+// Set the thread-local error message and return the status.
+tahoe_status fail(tahoe_status st, const std::string& msg);
+
+// Forest in compact form: every tree's reachable nodes, tree-local DFS order (left first),
+// concatenated.  Child indices are compact (global within this struct).  P:181-192.
+struct Forest {
+  int32_t n_trees = 0;
+  int32_t n_trees_full = 0;     // tree count of the full forest (AVERAGE divides by it; shards)
+  int32_t n_nodes_user = 0;     // length of the caller's arrays
+  int32_t n_features = 0;
+  int32_t n_classes = 1;
+  int32_t agg = 0;
+  float base = 0.0f;
+  int32_t max_feature = -1;     // largest attribute index used by an internal node
+
+  std::vector<int32_t> node_base;   // [T+1]
+  std::vector<int32_t> feat;        // -1 = leaf
+  std::vector<float> thr;
+  std::vector<int32_t> lc, rc;      // compact children
+  std::vector<float> val;
+  std::vector<uint8_t> dl;          // default_left (NaN goes left)
+  std::vector<int32_t> orig;        // caller node id
+  std::vector<int32_t> depth;       // node depth (root 0)
+  std::vector<int32_t> tclass;      // per tree
+  std::vector<int32_t> tree_orig;   // caller tree index
+
+  // ---- layout state (tahoe_forest_layout) ----
+  bool calibrated = false;
+  int64_t n_cal = 0;
+  std::vector<uint64_t> count;      // calibration visits per compact node
+  std::vector<uint8_t> hot_left;    // 1 = left child is the hot child
+  std::vector<double> exp_reads;    // per tree: expected nodes read per sample (incl. leaf)
+  std::vector<int32_t> order;       // tree order (class-major, similarity order within class)
+  tahoe_layout_opts opts{};
+
+  int32_t n_out() const { return (agg == TAHOE_AGG_CLASS_SUM || agg == TAHOE_AGG_VOTE) ? n_classes : 1; }
+  int32_t tree_size(int32_t t) const { return node_base[t + 1] - node_base[t]; }
+};
+
+// Build + validate from the caller's arrays (tahoe_forest_build's checks).
+tahoe_status build_forest(Forest& F, int32_t n_trees, const int32_t* root, int32_t n_nodes,
+                          const int32_t* feature, const float* threshold, const int32_t* left,
+                          const int32_t* right, const float* leaf_value,
+                          const uint8_t* default_left, const int32_t* tree_class,
+                          int32_t n_features, int32_t n_classes, int32_t agg, float base);
+void default_layout(Forest& F);
+Forest make_shard(const Forest& F, int32_t rank, int32_t world);
+
+// ---- layout steps (layout.cpp) ----
+void calibrate(Forest& F, const float* X, int64_t n, int32_t d);
+void reorder_nodes(Forest& F, bool enable);
+std::vector<int32_t> hot_preorder(const Forest& F, int32_t t);   // compact ids, hot child first
+void tree_tokens(const Forest& F, int32_t t, int32_t t_nodes, std::vector<int32_t>& tok_nodes,
+                 std::vector<double>& weights);
+void tree_simhash(const Forest& F, int32_t t, int32_t t_nodes, int32_t l_hash,
+                  std::vector<double>& checksum, std::vector<uint8_t>& bits);
+void sha1(const uint8_t* msg, size_t len, uint8_t out[20]);
+void simhash(const int8_t* strings, const double* w, int32_t n, int32_t l, double* cs, uint8_t* bits);
+std::vector<int32_t> lsh_order(const std::vector<uint8_t>& bits, int32_t n_trees, int32_t l_hash,
+                               int32_t m_chunks, std::vector<uint16_t>* collisions);
+void order_trees(Forest& F);
+
+// ---- encoded images (encode.cpp) ----
+struct SlicedImage {
+  bool valid = false;
+  std::string why_invalid;
+  int32_t n_slices = 0, slots_max = 0, fbits = 0;
+  std::vector<int32_t> slots, cls, ntrees;       // per slice
+  std::vector<int32_t> col_len;                  // [ns*32]
+  std::vector<uint32_t> nodes;                   // [ns*slots_max*32*2]
+  std::vector<int32_t> leaf_meta;                // [ns*slots_max*32*2] {tree, node}
+  std::vector<int32_t> class_ptr, class_parts;   // class -> slices (CSR)
+  double eff = 0.0;                              // est. lockstep efficiency (mean/max column)
+  double trees_per_lane = 0.0;
+  int64_t bytes() const { return (int64_t)nodes.size() * 4; }
+};
+
+struct DirectImage {
+  int32_t fbits = 0;
+  std::vector<uint32_t> nodes;        // [N*2]
+  std::vector<int32_t> root, cls, tree_orig;
+  int64_t bytes() const { return (int64_t)nodes.size() * 4; }
+};
+
+int32_t feature_bits(int32_t n_features);
+tahoe_status encode_direct(const Forest& F, DirectImage& D);
+tahoe_status encode_sliced(const Forest& F, int32_t slot_budget, SlicedImage& S);
+
+// Cost model (costmodel.cpp) — Algorithm 1 lines 8-13 re-targeted.
+struct PlanStats {
+  double V = 0;            // expected nodes read per sample (sum over trees)
+  double sliced_eff = 0;   // lockstep efficiency of the sliced packing
+  int32_t n_slices = 0;
+  bool sliced_ok = false;
+};
+int32_t select_strategy(const PlanStats& st, int64_t n, int32_t d, int32_t agg);
+
+}  // namespace tahoe
+
+// The opaque handle.
+struct tahoe_forest {
+  tahoe::Forest host;
+  tahoe::DirectImage di;
+  tahoe::SlicedImage sl;
+  int32_t device = -1;
+  int32_t slot_budget = 0;       // slot rows of 32 nodes that fit the per-CTA forest smem budget
+  int32_t num_sms = 0;
+  int32_t max_smem = 0;
+  // device copies
+  tahoe::DevDirect dd{};
+  tahoe::DevSliced ds{};
+  int32_t* d_class_ptr = nullptr;   // sliced class CSR
+  int32_t* d_class_parts = nullptr;
+};

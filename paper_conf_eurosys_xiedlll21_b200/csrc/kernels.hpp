@@ -1,0 +1,84 @@
+// kernels.hpp — device images and launch arguments shared by the host code and kernels.cu.
+// Plain structs of raw pointers and sizes (no CUDA types), so host .cpp files compile with g++.
+#pragma once
+#include <cstdint>
+
+namespace tahoe {
+
+// ------------------------------------------------------------------ node word encoding
+// 8-byte node {x, y} (variable-length attribute index P:1006-1015):
+//   internal: x = fp32 threshold bits;
+//             y = [31] 0 | [30] default_left | [29] hot_is_left | [28:F] cold delta | [F-1:0] feature
+//   leaf:     x = fp32 leaf value bits;
+//             y = [31] 1 | [30:0] sliced image: slot delta to the lane's next tree root
+//                                 direct image: caller node id
+// The hot child (the more probable one) is always the next node/slot (+1); the cold
+// child is at +cold delta.  F = feature_bits(n_features).
+constexpr uint32_t kLeafBit = 0x80000000u;
+constexpr uint32_t kDefaultLeftBit = 0x40000000u;
+constexpr uint32_t kHotLeftBit = 0x20000000u;
+constexpr int kOffsetTop = 29;   // cold delta occupies bits [28:F]
+
+struct DevDirect {
+  const uint32_t* nodes = nullptr;   // uint2 per node
+  const int32_t* root = nullptr;     // per tree slot (class-major order)
+  const int32_t* cls = nullptr;      // per tree slot
+  const int32_t* tree_orig = nullptr;
+  int32_t n_slots = 0;
+  int32_t fbits = 0;
+  int64_t n_nodes = 0;
+};
+
+struct DevSliced {
+  const uint32_t* nodes = nullptr;   // [ns][slots_max][32] uint2
+  const int32_t* col_len = nullptr;  // [ns][32]
+  const int32_t* slots = nullptr;    // [ns]
+  const int32_t* leaf_meta = nullptr;// [ns][slots_max][32] int2 {caller tree, caller node}
+  int32_t n_slices = 0;
+  int32_t slots_max = 0;
+  int32_t fbits = 0;
+};
+
+struct OutArgs {
+  float* out = nullptr;          // final scores (fused finalize) or nullptr
+  int32_t* out_class = nullptr;
+  int32_t* out_leaf = nullptr;   // [n][T_leaf] caller tree order
+  uint64_t* out_fp = nullptr;    // fingerprint (atomic u64 adds; zeroed by the launcher)
+  double* raw = nullptr;         // fp64 parts (layout chosen by the strategy)
+  int32_t agg = 0;
+  float base = 0.0f;
+  int32_t n_trees_full = 1;      // AVERAGE divisor
+  int32_t n_classes = 1;
+  int32_t T_leaf = 0;            // row stride of out_leaf
+};
+
+struct FinalizeArgs {
+  const double* partial = nullptr;
+  int64_t part_stride = 0;       // element stride between parts
+  int64_t row_stride = 0;        // element stride between samples
+  const int32_t* class_ptr = nullptr;    // device CSR class -> parts, or nullptr: part c == class c
+  const int32_t* class_parts = nullptr;
+  int32_t n_classes = 1;
+  int32_t agg = 0;
+  float base = 0.0f;
+  int32_t n_trees_full = 1;
+  int64_t n = 0;
+  float* out = nullptr;          // FINAL mode
+  int32_t* out_class = nullptr;
+  double* raw_out = nullptr;     // RAW mode (n x C fp64, no base) if non-null
+};
+
+// Launchers (kernels.cu).  Return a cudaError_t value as int (0 = success).
+struct SlicedPlan {
+  int32_t grid = 0, block = 1024, tile_rows = 0, cps = 1;
+  int32_t smem_bytes = 0, forest_smem = 0;
+  bool rows_in_smem = true;
+};
+int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
+                  bool fused, int32_t num_sms, void* stream);
+int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
+                  int32_t d, const OutArgs& o, bool fused, void* stream);
+int launch_finalize(const FinalizeArgs& a, void* stream);
+int set_sliced_smem_limit(int32_t bytes);
+
+}  // namespace tahoe

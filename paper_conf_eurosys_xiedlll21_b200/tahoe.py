@@ -1,0 +1,385 @@
+"""Thin Python binding of libtahoe.so (include/tahoe.h): argument marshalling only.
+
+Functions carry the C ABI names (``tahoe_forest_build``, ``tahoe_forest_layout``,
+``tahoe_predict`` ...).  Every step of prediction runs in the library's sm_100a kernels; PyTorch is
+used only for device memory and streams.  There is no CPU fallback: if the shared library is
+missing, importing this module raises.
+
+``Forest`` is a small convenience wrapper that owns a handle and accepts torch tensors / numpy
+arrays.
+"""
+from __future__ import annotations
+
+import ctypes
+import json
+import os
+
+import numpy as np
+
+from . import build as _build
+
+_lib = None
+
+TAHOE_OK, TAHOE_E_INVAL, TAHOE_E_NOMEM, TAHOE_E_CUDA, TAHOE_E_UNSUPPORTED, TAHOE_E_STATE = range(6)
+AGG_SUM, AGG_AVERAGE, AGG_BINARY, AGG_CLASS_SUM, AGG_VOTE = range(5)
+STRATEGY_AUTO, STRATEGY_DIRECT, STRATEGY_SLICED = -1, 0, 1
+
+
+class TahoeError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"tahoe status {status}: {msg}")
+        self.status = status
+
+
+class LayoutOpts(ctypes.Structure):
+    _fields_ = [("t_nodes", ctypes.c_int32), ("l_hash", ctypes.c_int32),
+                ("m_chunks", ctypes.c_int32), ("node_reorder", ctypes.c_int32),
+                ("tree_group", ctypes.c_int32), ("_reserved", ctypes.c_int32),
+                ("seed", ctypes.c_uint64)]
+
+
+class PredictOpts(ctypes.Structure):
+    _fields_ = [("out_class", ctypes.c_void_p), ("out_leaf", ctypes.c_void_p),
+                ("out_fingerprint", ctypes.c_void_p), ("force_strategy", ctypes.c_int32),
+                ("_reserved", ctypes.c_int32), ("ev_main_begin", ctypes.c_void_p),
+                ("ev_main_end", ctypes.c_void_p)]
+
+
+SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_predict_ex",
+           "tahoe_predict_host", "tahoe_forest_shard", "tahoe_predict_partial", "tahoe_finalize",
+           "tahoe_forest_n_outputs", "tahoe_forest_n_trees", "tahoe_forest_stats",
+           "tahoe_select_strategy", "tahoe_forest_free", "tahoe_last_error",
+           "tahoe_forest_layout_info", "tahoe_tree_tokens", "tahoe_tree_simhash", "tahoe_simhash",
+           "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced")
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def load(build_if_missing: bool = True):
+    """Load libtahoe.so (building it with nvcc if missing/stale and allowed)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = _build.LIB
+    if build_if_missing:
+        path = _build.build()
+    if not os.path.exists(path):
+        raise ImportError(f"libtahoe.so not found at {path}: run __graft_entry__.build()")
+    L = ctypes.CDLL(path)
+    P, i32, i64, f32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_float
+    st = ctypes.c_int
+    sig = {
+        "tahoe_forest_build": (st, [i32, P, i32, P, P, P, P, P, P, P, i32, i32, i32, f32, i32, P]),
+        "tahoe_forest_layout": (st, [P, P, i64, i32, P]),
+        "tahoe_predict": (st, [P, P, i64, i32, P, P]),
+        "tahoe_predict_ex": (st, [P, P, i64, i32, P, P, P]),
+        "tahoe_predict_host": (st, [P, P, i64, i32, P, P, P]),
+        "tahoe_forest_shard": (st, [P, i32, i32, i32, P]),
+        "tahoe_predict_partial": (st, [P, P, i64, i32, P, P]),
+        "tahoe_finalize": (st, [P, P, i64, P, P, P]),
+        "tahoe_forest_n_outputs": (i32, [P]),
+        "tahoe_forest_n_trees": (i32, [P]),
+        "tahoe_forest_stats": (st, [P, P, i64]),
+        "tahoe_select_strategy": (i32, [P, i64, i32]),
+        "tahoe_forest_free": (None, [P]),
+        "tahoe_last_error": (ctypes.c_char_p, []),
+        "tahoe_forest_layout_info": (st, [P, P, P, P, P]),
+        "tahoe_tree_tokens": (st, [P, i32, i32, P, P, i32, P]),
+        "tahoe_tree_simhash": (st, [P, i32, i32, i32, P, P]),
+        "tahoe_simhash": (st, [P, P, i32, i32, P, P]),
+        "tahoe_lsh_order": (st, [P, i32, i32, i32, P, P]),
+        "tahoe_sha1": (st, [P, i64, P]),
+        "tahoe_forest_export_sliced": (st, [P, P, P, P, P, P]),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(L, name)
+        fn.restype = res
+        fn.argtypes = args
+    _lib = L
+    return L
+
+
+def _check(status: int):
+    if status != TAHOE_OK:
+        raise TahoeError(status, load().tahoe_last_error().decode())
+
+
+def _np_ptr(a):
+    return None if a is None else ctypes.c_void_p(a.ctypes.data)
+
+
+def _dev_ptr(t):
+    """Raw pointer of a torch tensor (device or host) or None."""
+    if t is None:
+        return None
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+# ----------------------------------------------------------------------- C ABI names
+def tahoe_forest_build(arrays: dict, n_features: int, n_classes: int = 1, agg: int = AGG_SUM,
+                       base_score: float = 0.0, device: int = 0) -> ctypes.c_void_p:
+    L = load()
+    a = {k: np.ascontiguousarray(arrays[k]) for k in
+         ("root", "feature", "threshold", "left", "right", "leaf_value")}
+    a["root"] = a["root"].astype(np.int32, copy=False)
+    for k in ("feature", "left", "right"):
+        a[k] = a[k].astype(np.int32, copy=False)
+    for k in ("threshold", "leaf_value"):
+        a[k] = a[k].astype(np.float32, copy=False)
+    dl = arrays.get("default_left")
+    dl = None if dl is None else np.ascontiguousarray(dl, dtype=np.uint8)
+    tc = arrays.get("tree_class")
+    tc = None if tc is None else np.ascontiguousarray(tc, dtype=np.int32)
+    h = ctypes.c_void_p()
+    _check(L.tahoe_forest_build(len(a["root"]), _np_ptr(a["root"]), len(a["feature"]),
+                                _np_ptr(a["feature"]), _np_ptr(a["threshold"]), _np_ptr(a["left"]),
+                                _np_ptr(a["right"]), _np_ptr(a["leaf_value"]), _np_ptr(dl),
+                                _np_ptr(tc), int(n_features), int(n_classes), int(agg),
+                                float(base_score), int(device), ctypes.byref(h)))
+    return h
+
+
+def tahoe_forest_layout(h, X_calib: np.ndarray, opts: LayoutOpts | None = None):
+    X = np.ascontiguousarray(X_calib, dtype=np.float32)
+    _check(load().tahoe_forest_layout(h, _np_ptr(X), X.shape[0], X.shape[1],
+                                      None if opts is None else ctypes.byref(opts)))
+
+
+def tahoe_predict(h, X, n: int, d: int, out, stream=None):
+    _check(load().tahoe_predict(h, _dev_ptr(X), n, d, _dev_ptr(out), _stream_ptr(stream)))
+
+
+def tahoe_predict_ex(h, X, n: int, d: int, out, out_class=None, out_leaf=None,
+                     out_fingerprint=None, force_strategy: int = -1, stream=None,
+                     ev_main_begin=None, ev_main_end=None):
+    """ev_main_begin / ev_main_end: optional torch.cuda.Event (timing enabled, already recorded
+    once) recorded around the main traversal kernel on ``stream``."""
+    o = PredictOpts(_dev_ptr(out_class), _dev_ptr(out_leaf), _dev_ptr(out_fingerprint),
+                    int(force_strategy), 0,
+                    None if ev_main_begin is None else ctypes.c_void_p(ev_main_begin.cuda_event),
+                    None if ev_main_end is None else ctypes.c_void_p(ev_main_end.cuda_event))
+    _check(load().tahoe_predict_ex(h, _dev_ptr(X), n, d, _dev_ptr(out), ctypes.byref(o),
+                                   _stream_ptr(stream)))
+
+
+def tahoe_predict_host(h, X_host, n: int, d: int, out_host, class_host=None, stream=None):
+    _check(load().tahoe_predict_host(h, _dev_ptr(X_host), n, d, _dev_ptr(out_host),
+                                     _dev_ptr(class_host), _stream_ptr(stream)))
+
+
+def tahoe_forest_shard(h, rank: int, world: int, device: int):
+    s = ctypes.c_void_p()
+    _check(load().tahoe_forest_shard(h, rank, world, device, ctypes.byref(s)))
+    return s
+
+
+def tahoe_predict_partial(shard, X, n: int, d: int, partial, stream=None):
+    _check(load().tahoe_predict_partial(shard, _dev_ptr(X), n, d, _dev_ptr(partial),
+                                        _stream_ptr(stream)))
+
+
+def tahoe_finalize(h, partial, n: int, out, out_class=None, stream=None):
+    _check(load().tahoe_finalize(h, _dev_ptr(partial), n, _dev_ptr(out), _dev_ptr(out_class),
+                                 _stream_ptr(stream)))
+
+
+def tahoe_forest_n_outputs(h) -> int:
+    return int(load().tahoe_forest_n_outputs(h))
+
+
+def tahoe_forest_n_trees(h) -> int:
+    return int(load().tahoe_forest_n_trees(h))
+
+
+def tahoe_forest_stats(h) -> dict:
+    buf = ctypes.create_string_buffer(8192)
+    _check(load().tahoe_forest_stats(h, buf, len(buf)))
+    return json.loads(buf.value.decode())
+
+
+def tahoe_select_strategy(h, n: int, d: int) -> int:
+    return int(load().tahoe_select_strategy(h, n, d))
+
+
+def tahoe_forest_free(h):
+    if h:
+        load().tahoe_forest_free(h)
+
+
+def tahoe_last_error() -> str:
+    return load().tahoe_last_error().decode()
+
+
+def tahoe_forest_layout_info(h, n_nodes: int, n_trees: int) -> dict:
+    cnt = np.zeros(n_nodes, np.uint64)
+    hot = np.zeros(n_nodes, np.uint8)
+    er = np.zeros(n_trees, np.float64)
+    order = np.zeros(n_trees, np.int32)
+    _check(load().tahoe_forest_layout_info(h, _np_ptr(cnt), _np_ptr(hot), _np_ptr(er),
+                                           _np_ptr(order)))
+    return dict(count=cnt, hot_left=hot, exp_reads=er, order=order)
+
+
+def tahoe_tree_tokens(h, t: int, t_nodes: int):
+    n = ctypes.c_int32()
+    _check(load().tahoe_tree_tokens(h, t, t_nodes, None, None, 0, ctypes.byref(n)))
+    tok = np.zeros((n.value, t_nodes), np.int32)
+    w = np.zeros(n.value, np.float64)
+    _check(load().tahoe_tree_tokens(h, t, t_nodes, _np_ptr(tok), _np_ptr(w), n.value,
+                                    ctypes.byref(n)))
+    return tok, w
+
+
+def tahoe_tree_simhash(h, t: int, t_nodes: int = 4, l_hash: int = 128):
+    cs = np.zeros(l_hash, np.float64)
+    bits = np.zeros(l_hash, np.uint8)
+    _check(load().tahoe_tree_simhash(h, t, t_nodes, l_hash, _np_ptr(cs), _np_ptr(bits)))
+    return cs, bits
+
+
+def tahoe_simhash(strings: np.ndarray, weights: np.ndarray):
+    s = np.ascontiguousarray(strings, dtype=np.int8)
+    w = np.ascontiguousarray(weights, dtype=np.float64)
+    cs = np.zeros(s.shape[1], np.float64)
+    bits = np.zeros(s.shape[1], np.uint8)
+    _check(load().tahoe_simhash(_np_ptr(s), _np_ptr(w), s.shape[0], s.shape[1], _np_ptr(cs),
+                                _np_ptr(bits)))
+    return cs, bits
+
+
+def tahoe_lsh_order(bits: np.ndarray, m_chunks: int):
+    b = np.ascontiguousarray(bits, dtype=np.uint8)
+    T, L = b.shape
+    col = np.zeros((T, T), np.int32)
+    order = np.zeros(T, np.int32)
+    _check(load().tahoe_lsh_order(_np_ptr(b), T, L, m_chunks, _np_ptr(col), _np_ptr(order)))
+    return col, order
+
+
+def tahoe_sha1(msg: bytes) -> bytes:
+    buf = (ctypes.c_uint8 * max(1, len(msg))).from_buffer_copy(msg or b"\0")
+    out = (ctypes.c_uint8 * 20)()
+    _check(load().tahoe_sha1(buf, len(msg), out))
+    return bytes(out)
+
+
+def tahoe_forest_export_sliced(h) -> dict | None:
+    L = load()
+    hdr = np.zeros(8, np.int32)
+    _check(L.tahoe_forest_export_sliced(h, _np_ptr(hdr), None, None, None, None))
+    ns, smax = int(hdr[0]), int(hdr[1])
+    if ns == 0:
+        return None
+    info = np.zeros((ns, 4), np.int32)
+    col = np.zeros((ns, 32), np.int32)
+    nodes = np.zeros((ns, smax, 32, 2), np.uint32)
+    meta = np.zeros((ns, smax, 32, 2), np.int32)
+    _check(L.tahoe_forest_export_sliced(h, _np_ptr(hdr), _np_ptr(info), _np_ptr(col),
+                                        _np_ptr(nodes), _np_ptr(meta)))
+    return dict(n_slices=ns, slots_max=smax, feature_bits=int(hdr[2]), n_trees=int(hdr[3]),
+                n_classes=int(hdr[4]), slice_info=info, col_len=col, nodes=nodes, leaf_meta=meta)
+
+
+# ----------------------------------------------------------------------- convenience wrapper
+class Forest:
+    """Owns a tahoe_forest handle.  ``arrays`` are the user-level node arrays (as produced by
+    gen.make_forest)."""
+
+    def __init__(self, arrays: dict, n_features: int | None = None, n_classes: int | None = None,
+                 agg: int | None = None, base_score: float = 0.0, device: int = 0):
+        self.n_features = int(arrays.get("n_features") if n_features is None else n_features)
+        self.n_classes = int(arrays.get("n_classes", 1) if n_classes is None else n_classes)
+        self.agg = int(arrays.get("agg", AGG_SUM) if agg is None else agg)
+        self.device = device
+        self.n_nodes = len(arrays["feature"])
+        self.handle = tahoe_forest_build(arrays, self.n_features, self.n_classes, self.agg,
+                                         base_score, device)
+        self.n_trees = tahoe_forest_n_trees(self.handle)
+        self.n_out = tahoe_forest_n_outputs(self.handle)
+
+    @classmethod
+    def _wrap(cls, handle, like: "Forest", device: int):
+        f = cls.__new__(cls)
+        f.n_features, f.n_classes, f.agg = like.n_features, like.n_classes, like.agg
+        f.device, f.n_nodes, f.handle = device, like.n_nodes, handle
+        f.n_trees = tahoe_forest_n_trees(handle)
+        f.n_out = tahoe_forest_n_outputs(handle)
+        return f
+
+    def layout(self, X_calib: np.ndarray, **kw):
+        opts = None
+        if kw:
+            opts = LayoutOpts(kw.get("t_nodes", 0), kw.get("l_hash", 0), kw.get("m_chunks", 0),
+                              kw.get("node_reorder", 1), kw.get("tree_group", 1), 0,
+                              kw.get("seed", 0))
+        tahoe_forest_layout(self.handle, X_calib, opts)
+        return self
+
+    def stats(self) -> dict:
+        return tahoe_forest_stats(self.handle)
+
+    def select_strategy(self, n: int, d: int) -> int:
+        return tahoe_select_strategy(self.handle, n, d)
+
+    def predict(self, X, out=None, out_class=None, out_leaf=None, out_fingerprint=None,
+                force_strategy: int = -1, stream=None, ev_main_begin=None, ev_main_end=None):
+        """X: torch tensor on the forest's device (n x d float32).  Returns ``out``."""
+        import torch
+        n, d = X.shape
+        if out is None:
+            out = torch.empty((n, self.n_out), dtype=torch.float32, device=X.device)
+        if (out_class is None and out_leaf is None and out_fingerprint is None
+                and force_strategy < 0 and ev_main_begin is None):
+            tahoe_predict(self.handle, X, n, d, out, stream)
+        else:
+            tahoe_predict_ex(self.handle, X, n, d, out, out_class, out_leaf, out_fingerprint,
+                             force_strategy, stream, ev_main_begin, ev_main_end)
+        return out
+
+    def predict_host(self, X_host, out_host, class_host=None, stream=None):
+        n, d = X_host.shape
+        tahoe_predict_host(self.handle, X_host, n, d, out_host, class_host, stream)
+        return out_host
+
+    def shard(self, rank: int, world: int, device: int | None = None) -> "Forest":
+        dev = self.device if device is None else device
+        return Forest._wrap(tahoe_forest_shard(self.handle, rank, world, dev), self, dev)
+
+    def predict_partial(self, X, partial=None, stream=None):
+        import torch
+        n, d = X.shape
+        if partial is None:
+            partial = torch.empty((n, self.n_out), dtype=torch.float64, device=X.device)
+        tahoe_predict_partial(self.handle, X, n, d, partial, stream)
+        return partial
+
+    def finalize(self, partial, out=None, out_class=None, stream=None):
+        import torch
+        n = partial.shape[0]
+        if out is None:
+            out = torch.empty((n, self.n_out), dtype=torch.float32, device=partial.device)
+        tahoe_finalize(self.handle, partial, n, out, out_class, stream)
+        return out
+
+    def export_sliced(self):
+        return tahoe_forest_export_sliced(self.handle)
+
+    def close(self):
+        if getattr(self, "handle", None):
+            tahoe_forest_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

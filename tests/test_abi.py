@@ -1,0 +1,251 @@
+"""C-ABI tests that need no GPU: the library loads and exports every symbol include/tahoe.h
+declares; tahoe_forest_build's validation codes; host-only handles; and the layout introspection
+hooks against the layout oracle (Fig. 1 / Fig. 3 of the paper)."""
+import ctypes
+import hashlib
+import json
+import os
+import re
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from oracle import layout_oracle as lo
+from paper_conf_eurosys_xiedlll21_b200 import tahoe as T
+from tlib import GOLDEN, ROOT
+
+
+def test_library_exports_every_header_symbol():
+    hdr = open(os.path.join(ROOT, "include", "tahoe.h")).read()
+    names = set(re.findall(r"\b(tahoe_[a-z0-9_]+)\s*\(", hdr))
+    assert len(names) >= 20
+    L = T.load()
+    for nm in sorted(names):
+        assert hasattr(L, nm), nm
+    assert names == set(T.SYMBOLS)
+
+
+def _stump_arrays():
+    return dict(root=np.array([0], np.int32), feature=np.array([0, -1, -1], np.int32),
+                threshold=np.array([0.5, 0, 0], np.float32), left=np.array([1, -1, -1], np.int32),
+                right=np.array([2, -1, -1], np.int32),
+                leaf_value=np.array([0, 1.0, 2.0], np.float32))
+
+
+def _build(arrs, n_features=1, n_classes=1, agg=T.AGG_SUM):
+    return T.tahoe_forest_build(arrs, n_features, n_classes, agg, 0.0, -1)
+
+
+def test_build_ok_and_host_only_predict_is_state_error():
+    h = _build(_stump_arrays())
+    assert T.tahoe_forest_n_outputs(h) == 1 and T.tahoe_forest_n_trees(h) == 1
+    L = T.load()
+    st = L.tahoe_predict(h, ctypes.c_void_p(16), 1, 1, ctypes.c_void_p(16), None)
+    assert st == T.TAHOE_E_STATE
+    assert L.tahoe_predict(h, None, 0, 1, None, None) == T.TAHOE_E_STATE
+    T.tahoe_forest_free(h)
+
+
+@pytest.mark.parametrize("mutate,msg", [
+    (lambda a: a.update(feature=np.array([3, -1, -1], np.int32)), "n_features"),
+    (lambda a: a.update(left=np.array([7, -1, -1], np.int32)), "out of range"),
+    (lambda a: a.update(left=np.array([2, -1, -1], np.int32)), "reachable twice"),
+    (lambda a: a.update(left=np.array([0, -1, -1], np.int32)), "reachable twice"),
+    (lambda a: a.update(threshold=np.array([np.nan, 0, 0], np.float32)), "NaN threshold"),
+    (lambda a: a.update(root=np.array([5], np.int32)), "out of range"),
+])
+def test_build_validation_errors(mutate, msg):
+    a = _stump_arrays()
+    mutate(a)
+    with pytest.raises(T.TahoeError) as e:
+        _build(a)
+    assert e.value.status == T.TAHOE_E_INVAL and msg in str(e.value)
+
+
+def test_build_vote_and_class_validation():
+    a = _stump_arrays()
+    with pytest.raises(T.TahoeError) as e:
+        _build(dict(a, leaf_value=np.array([0, 0.5, 1], np.float32)), n_classes=2, agg=T.AGG_VOTE)
+    assert e.value.status == T.TAHOE_E_INVAL
+    with pytest.raises(T.TahoeError):
+        _build(dict(a, tree_class=np.array([3], np.int32)), n_classes=2, agg=T.AGG_CLASS_SUM)
+    with pytest.raises(T.TahoeError):
+        T.tahoe_forest_build(a, 1, 0, T.AGG_SUM, 0.0, -1)
+    h = _build(dict(a, leaf_value=np.array([0, 1, 0], np.float32)), n_classes=2, agg=T.AGG_VOTE)
+    assert T.tahoe_forest_n_outputs(h) == 2
+    T.tahoe_forest_free(h)
+
+
+def test_unreachable_nodes_ignored():
+    a = _stump_arrays()
+    a = {k: np.concatenate([v, v[:1]]) if k != "root" else v for k, v in a.items()}
+    a["left"][3] = 99  # garbage in an unreachable node
+    h = _build(a)
+    assert T.tahoe_forest_stats(h)["nodes"] == 3
+    T.tahoe_forest_free(h)
+
+
+def test_sha1_matches_hashlib():
+    for m in [b"", b"abc", bytes(range(200)), b"\x00" * 64, b"tahoe" * 33]:
+        assert T.tahoe_sha1(m) == hashlib.sha1(m).digest()
+
+
+def test_product_simhash_and_lsh_reproduce_fig3():
+    g = json.load(open(os.path.join(GOLDEN, "fig3_simhash.json")))
+    cs, bits = T.tahoe_simhash(np.array(g["strings"]), np.array(g["weights"]))
+    assert np.allclose(cs, g["checksum"], atol=1e-12) and bits.tolist() == g["normalized"]
+    reps = np.array([g["reps"][k] for k in ("T1", "T2", "T3")], np.uint8)
+    col, order = T.tahoe_lsh_order(reps, g["m_chunks"])
+    assert col[0, 1] == 0 and col[1, 2] == 2 and col[0, 2] == 1
+    assert ["T1", "T2", "T3"][order[0]] == "T2" and list(order) == [1, 2, 0]
+
+
+def test_product_lsh_order_equals_oracle_random():
+    rng = np.random.default_rng(4)
+    for T_ in (5, 17, 60):
+        bits = (rng.random((T_, 32)) < 0.5).astype(np.uint8)
+        col, order = T.tahoe_lsh_order(bits, 8)
+        ocol = lo.lsh_collisions(bits, 8)
+        assert np.array_equal(col, ocol)
+        assert list(order) == lo.lsh_order(ocol)
+
+
+def _fig1_product_forest():
+    """Fig. 1's three trees with one attribute per internal node, and 100 calibration rows that
+    reproduce the edge counts of tests/golden/fig1_reorg.json."""
+    g = json.load(open(os.path.join(GOLDEN, "fig1_reorg.json")))
+    names = ["V11", "V12", "V13", "V14", "V15", "V16", "V17", "V21", "V22", "V23", "V24", "V25",
+             "V31", "V32", "V33", "V34", "V35"]
+    idx = {n: i for i, n in enumerate(names)}
+    feat_of = {"V11": 0, "V12": 1, "V13": 2, "V21": 7, "V23": 8, "V31": 9, "V32": 10}
+    adj = {}
+    for t in g["trees"]:
+        adj.update({k: v for k, v in t.items() if k != "_root"})
+    N = len(names)
+    a = dict(root=np.array([0, 7, 12], np.int32), feature=np.full(N, -1, np.int32),
+             threshold=np.zeros(N, np.float32), left=np.full(N, -1, np.int32),
+             right=np.full(N, -1, np.int32), leaf_value=np.arange(N, dtype=np.float32) / 4)
+    for n, (l, r) in adj.items():
+        a["feature"][idx[n]] = feat_of[n]
+        a["threshold"][idx[n]] = 0.5
+        a["left"][idx[n]] = idx[l]
+        a["right"][idx[n]] = idx[r]
+    X = np.ones((100, 11), np.float32)
+    X[:80, 0] = 0; X[:48, 1] = 0; X[80:86, 2] = 0
+    X[:30, 7] = 0; X[30:50, 8] = 0; X[:, 9] = 0; X[:, 10] = 0
+    return g, names, idx, a, X
+
+
+def test_product_layout_matches_fig1_fig3_and_oracle():
+    g, names, idx, a, X = _fig1_product_forest()
+    h = T.tahoe_forest_build(a, 11, 1, T.AGG_SUM, 0.0, -1)
+    T.tahoe_forest_layout(h, X)
+    info = T.tahoe_forest_layout_info(h, len(names), 3)
+    cnt = oracle.node_counts(a, X)
+    assert np.array_equal(info["count"], cnt)
+    for e, c in g["edge_counts_after_training"].items():
+        assert info["count"][idx[e.split("->")[1]]] == c
+    assert np.array_equal(info["hot_left"], lo.hot_is_left(a, cnt))
+    assert info["hot_left"][idx["V21"]] == 0 and info["hot_left"][idx["V13"]] == 0
+    g3 = json.load(open(os.path.join(GOLDEN, "fig3_simhash.json")))
+    tok, w = T.tahoe_tree_tokens(h, 0, 2)
+    assert [[names[k] for k in t] for t in tok] == g3["tree1_tokens_tnodes2"]
+    assert w.tolist() == g3["weights"]
+    # expected node reads per tree = sum of node probabilities
+    assert info["exp_reads"][0] == pytest.approx(1 + 0.8 + 0.2 + 0.48 + 0.32 + 0.06 + 0.14)
+    T.tahoe_forest_free(h)
+
+
+def test_product_tokens_simhash_equal_oracle_on_generated_forest():
+    f = gen.make_forest(2, n_trees=12)
+    Xc = gen.make_calibration(2, 3000)
+    h = T.tahoe_forest_build(f, f["n_features"], 1, f["agg"], 0.0, -1)
+    T.tahoe_forest_layout(h, Xc)
+    info = T.tahoe_forest_layout_info(h, len(f["feature"]), 12)
+    cnt = oracle.node_counts(f, Xc)
+    assert np.array_equal(info["count"], cnt)
+    hl = lo.hot_is_left(f, cnt)
+    assert np.array_equal(info["hot_left"], hl)
+    npb = cnt / len(Xc)
+    for t in range(12):
+        tok, w = T.tahoe_tree_tokens(h, t, 4)
+        otok = lo.tokens(f, t, 4, hl)
+        assert [tuple(int(k) for k in row if k >= 0) for row in tok] == otok
+        assert np.array_equal(w, np.array([npb[tk[-1]] for tk in otok]))
+        cs, bits = T.tahoe_tree_simhash(h, t, 4, 128)
+        S = np.stack([lo.token_bits(lo.token_bytes(f, tk), 128).astype(np.int64) * 2 - 1
+                      for tk in otok])
+        ocs = np.zeros(128)
+        for i in range(len(otok)):      # sequential sum in token order
+            ocs = ocs + npb[otok[i][-1]] * S[i]
+        assert np.allclose(cs, ocs, rtol=0, atol=1e-12)
+        assert np.array_equal(bits, (ocs >= 0).astype(np.uint8))
+    T.tahoe_forest_free(h)
+
+
+def decode_sliced(img, X, n_trees, n_classes):
+    """Walk the exported SLICED image on the host (test-side decoder, independent of the
+    product): returns leaf[n, T] (caller node ids) and per-class fp64 sums in slice order."""
+    n = X.shape[0]
+    F = img["feature_bits"]
+    leaf = np.full((n, n_trees), -1, np.int64)
+    sums = np.zeros((n, n_classes))
+    for s in range(img["n_slices"]):
+        c = img["slice_info"][s, 1]
+        for lane in range(32):
+            end = img["col_len"][s, lane]
+            for i in range(n):
+                k = 0
+                while k < end:
+                    x, y = (int(v) for v in img["nodes"][s, k, lane])
+                    if y & 0x80000000:
+                        t, node = img["leaf_meta"][s, k, lane]
+                        leaf[i, t] = node
+                        sums[i, c] += float(np.uint32(x).view(np.float32))
+                        k += y & 0x7FFFFFFF
+                    else:
+                        thr = float(np.uint32(x).view(np.float32))
+                        v = X[i, y & ((1 << F) - 1)]
+                        go_left = bool((y >> 30) & 1) if np.isnan(v) else bool(v < thr)
+                        hot = go_left == bool((y >> 29) & 1)
+                        k += 1 if hot else (y >> F) & ((1 << (29 - F)) - 1)
+    return leaf, sums
+
+
+@pytest.mark.parametrize("cid,ntrees,nrows", [(1, None, 200), (2, 60, 60), (3, 70, 40)])
+def test_sliced_image_decodes_to_oracle(cid, ntrees, nrows):
+    f = gen.make_forest(cid, n_trees=ntrees)
+    X = gen.make_rows(cid, nrows)
+    X[::7, 1] = np.nan
+    h = T.tahoe_forest_build(f, f["n_features"], f["n_classes"], f["agg"], 0.0, -1)
+    for layout in (False, True):
+        if layout:
+            T.tahoe_forest_layout(h, gen.make_calibration(cid, 2000))
+        img = T.tahoe_forest_export_sliced(h)
+        assert img is not None
+        leaf, sums = decode_sliced(img, X, len(f["root"]), f["n_classes"])
+        r = oracle.predict(f, X, want_leaf=True)
+        assert np.array_equal(leaf, r["leaf"])
+        if f["agg"] == oracle.AGG_CLASS_SUM:
+            assert np.array_equal(sums, r["raw"])      # dyadic leaves: exact in any order
+        else:
+            assert np.array_equal(sums[:, 0], r["raw"][:, 0])
+    T.tahoe_forest_free(h)
+
+
+def test_shards_partition_trees():
+    f = gen.make_forest(2, n_trees=50)
+    h = T.tahoe_forest_build(f, 28, 1, T.AGG_BINARY, 0.0, -1)
+    T.tahoe_forest_layout(h, gen.make_calibration(2, 1000))
+    seen = []
+    for r in range(4):
+        s = T.tahoe_forest_shard(h, r, 4, -1)
+        info = T.tahoe_forest_layout_info(s, len(f["feature"]), T.tahoe_forest_n_trees(s))
+        seen += list(info["order"])
+        st = T.tahoe_forest_stats(s)
+        assert st["n_trees_full"] == 50
+        T.tahoe_forest_free(s)
+    assert sorted(seen) == list(range(50))
+    T.tahoe_forest_free(h)

@@ -1,0 +1,206 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Bars (BASELINE.json north_star):
+  * leaf ids (caller node ids, n x T) and fingerprints: bit-exact;
+  * classes: bit-exact (dyadic runs) / exact wherever the fp64 decision margin exceeds the fp64
+    rounding bound (random-leaf runs);
+  * scores: bit-exact with dyadic leaves; |gpu - ref| <= max(1e-5 |ref|, 1e-6) with N(0, 0.1) leaves.
+Every strategy is forced in turn; sizes span many tiles and a ragged tail.
+"""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_eurosys_xiedlll21_b200 import tahoe as T  # noqa: E402
+
+STRATS = [T.STRATEGY_DIRECT, T.STRATEGY_SLICED]
+
+
+def _gpu_run(F, X, strategy, want_leaf=True):
+    dev = torch.device("cuda", 0)
+    Xd = torch.from_numpy(X).to(dev)
+    n = X.shape[0]
+    out = torch.empty((n, F.n_out), dtype=torch.float32, device=dev)
+    cls = torch.full((n,), -7, dtype=torch.int32, device=dev)
+    leaf = torch.full((n, F.n_trees), -7, dtype=torch.int32, device=dev) if want_leaf else None
+    fp = torch.empty(n, dtype=torch.int64, device=dev) if want_leaf else None
+    F.predict(Xd, out=out, out_class=cls, out_leaf=leaf, out_fingerprint=fp, force_strategy=strategy)
+    torch.cuda.synchronize()
+    res = dict(out=out.cpu().numpy(), cls=cls.cpu().numpy())
+    if want_leaf:
+        res["leaf"] = leaf.cpu().numpy()
+        res["fp"] = fp.cpu().numpy().view(np.uint64)
+    return res
+
+
+def _check(res, ref, agg, exact, want_leaf=True):
+    if want_leaf:
+        assert np.array_equal(res["leaf"], ref["leaf"]), "leaf ids differ"
+        assert np.array_equal(res["fp"], ref["fp"]), "fingerprints differ"
+    if exact:
+        assert np.array_equal(res["out"], ref["out"]), "dyadic scores must be bit-exact"
+        if agg in (oracle.AGG_BINARY, oracle.AGG_CLASS_SUM, oracle.AGG_VOTE):
+            assert np.array_equal(res["cls"], ref["cls"])
+    else:
+        tol = np.maximum(1e-5 * np.abs(ref["out"]), 1e-6)
+        assert (np.abs(res["out"] - ref["out"]) <= tol).all(), \
+            f"max err {np.abs(res['out'] - ref['out']).max()}"
+        if agg == oracle.AGG_BINARY:
+            sure = np.abs(ref["raw"][:, 0]) > 1e-9
+            assert np.array_equal(res["cls"][sure], ref["cls"][sure])
+        elif agg == oracle.AGG_CLASS_SUM:
+            srt = np.sort(ref["raw"], axis=1)
+            sure = (srt[:, -1] - srt[:, -2]) > 1e-9
+            assert np.array_equal(res["cls"][sure], ref["cls"][sure])
+
+
+CASES = [  # (config, n_trees override, n rows, leaf mode)
+    (1, None, 1000, "dyadic"),
+    (1, None, 1000, "normal"),
+    (2, None, 20011, "dyadic"),
+    (2, None, 6007, "normal"),
+    (3, None, 8009, "dyadic"),
+    (4, 200, 3001, "dyadic"),
+]
+
+
+@pytest.mark.parametrize("cid,ntrees,n,mode", CASES)
+@pytest.mark.parametrize("layout", [False, True])
+def test_parity_configs(cid, ntrees, n, mode, layout):
+    f = gen.make_forest(cid, n_trees=ntrees, leaf_mode=mode)
+    X = gen.make_rows(cid, n)
+    F = T.Forest(f, device=0)
+    if layout:
+        F.layout(gen.make_calibration(cid, 4096))
+    ref = oracle.predict(f, X, want_leaf=True)
+    for s in STRATS:
+        if s == T.STRATEGY_SLICED and not F.stats()["sliced_valid"]:
+            continue
+        _check(_gpu_run(F, X, s), ref, f["agg"], mode == "dyadic")
+
+
+def test_parity_c4_full_forest_subsample():
+    f = gen.make_forest(4)
+    X = gen.make_rows(4, 2003)
+    F = T.Forest(f, device=0).layout(gen.make_calibration(4, 4096))
+    ref = oracle.predict(f, X, want_leaf=True)
+    for s in STRATS:
+        _check(_gpu_run(F, X, s), ref, f["agg"], True)
+
+
+def test_parity_c5_subsample_direct_and_shards():
+    f = gen.make_forest(5, n_trees=600)
+    X = gen.make_rows(5, 1500)
+    F = T.Forest(f, device=0).layout(gen.make_calibration(5, 8192))
+    ref = oracle.predict(f, X, want_leaf=True)
+    _check(_gpu_run(F, X, -1), ref, f["agg"], True)
+    # fake multi-rank tree sharding on one GPU: sum of shard partials -> finalize == full
+    dev = torch.device("cuda", 0)
+    Xd = torch.from_numpy(X).to(dev)
+    tot = torch.zeros((X.shape[0], 1), dtype=torch.float64, device=dev)
+    for r in range(4):
+        S = F.shard(r, 4)
+        tot += S.predict_partial(Xd)
+    out = F.finalize(tot)
+    assert np.array_equal(out.cpu().numpy(), ref["out"])
+
+
+def test_edge_cases_nan_misaligned_wide_d_and_tiny_batches():
+    f = gen.make_forest(2, n_trees=64)
+    F = T.Forest(f, device=0).layout(gen.make_calibration(2, 2048))
+    X = gen.make_rows(2, 4099)
+    X[::5, 3] = np.nan
+    X[::11, :] = np.nan
+    ref = oracle.predict(f, X, want_leaf=True)
+    for s in STRATS:
+        _check(_gpu_run(F, X, s), ref, f["agg"], True)
+    # misaligned X (offset by one float => no TMA) and wider rows than the forest needs
+    dev = torch.device("cuda", 0)
+    Xw = np.concatenate([X, np.full((X.shape[0], 5), 9.0, np.float32)], axis=1)
+    buf = torch.empty(Xw.size + 1, dtype=torch.float32, device=dev)
+    buf[1:] = torch.from_numpy(Xw.ravel()).to(dev)
+    Xm = buf[1:].view(Xw.shape)
+    for s in STRATS:
+        out = torch.empty((X.shape[0], 1), dtype=torch.float32, device=dev)
+        F.predict(Xm, out=out, force_strategy=s)
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy(), ref["out"])
+    for n in (0, 1, 31, 33, 64, 65):
+        for s in STRATS:
+            Xd = torch.from_numpy(X[:n].copy()).to(dev)
+            out = torch.full((n, 1), -1.0, dtype=torch.float32, device=dev)
+            F.predict(Xd, out=out, force_strategy=s)
+            torch.cuda.synchronize()
+            assert np.array_equal(out.cpu().numpy(), ref["out"][:n])
+
+
+def test_aggregations_average_base_vote():
+    from test_oracle_pins import random_forest
+    rng = np.random.default_rng(21)
+    f = random_forest(rng, 45, 6, 5)
+    X = rng.normal(size=(3001, 5)).astype(np.float32)
+    for agg, base in ((oracle.AGG_AVERAGE, 0.625), (oracle.AGG_SUM, -2.0), (oracle.AGG_BINARY, 0.25)):
+        F = T.Forest(f, n_features=5, n_classes=1, agg=agg, base_score=base, device=0)
+        ref = oracle.predict(f, X, agg=agg, base_score=base, want_leaf=True)
+        for s in STRATS:
+            _check(_gpu_run(F, X, s), ref, agg, True)
+    C = 4
+    fv = random_forest(rng, 40, 5, 5, n_classes=C, vote=True)
+    F = T.Forest(fv, n_features=5, n_classes=C, agg=oracle.AGG_VOTE, device=0)
+    ref = oracle.predict(fv, X, agg=oracle.AGG_VOTE, n_classes=C, want_leaf=True)
+    _check(_gpu_run(F, X, -1), ref, oracle.AGG_VOTE, True)
+
+
+def test_layout_never_changes_results():
+    f = gen.make_forest(3, n_trees=140)
+    X = gen.make_rows(3, 3000)
+    ref = oracle.predict(f, X, want_leaf=True)
+    F = T.Forest(f, device=0)
+    outs = []
+    for kw in (dict(), dict(node_reorder=0, tree_group=0), dict(node_reorder=1, tree_group=0),
+               dict(t_nodes=2, l_hash=64, m_chunks=16)):
+        F.layout(gen.make_calibration(3, 3000), **kw)
+        for s in STRATS:
+            r = _gpu_run(F, X, s)
+            _check(r, ref, f["agg"], True)
+            outs.append(r["out"])
+    assert all(np.array_equal(o, outs[0]) for o in outs)
+
+
+def test_predict_host_end_to_end():
+    f = gen.make_forest(2, n_trees=100)
+    F = T.Forest(f, device=0).layout(gen.make_calibration(2, 2048))
+    X = gen.make_rows(2, 300_001)
+    Xh = torch.from_numpy(X).pin_memory()
+    out = torch.empty((X.shape[0], 1), dtype=torch.float32).pin_memory()
+    cls = torch.empty(X.shape[0], dtype=torch.int32).pin_memory()
+    F.predict_host(Xh, out, cls)
+    torch.cuda.synchronize()
+    idx = gen.subsample(5, X.shape[0], 3000)
+    ref = oracle.predict(f, X, rows=idx)
+    assert np.array_equal(out.numpy()[idx], ref["out"])
+    assert np.array_equal(cls.numpy()[idx], ref["cls"])
+
+
+def test_full_size_c2_sampled_rows_in_bench_configuration():
+    """BASELINE.json C2 at full size (1M rows) in the launch configuration bench.py times;
+    sampled outputs checked one by one against the oracle."""
+    cfg = gen.CONFIGS[2]
+    f = gen.make_forest(2, leaf_mode="normal")
+    F = T.Forest(f, device=0).layout(gen.make_calibration(2))
+    X = gen.make_rows(2, cfg.n_samples)
+    dev = torch.device("cuda", 0)
+    Xd = torch.from_numpy(X).to(dev)
+    out = torch.empty((cfg.n_samples, 1), dtype=torch.float32, device=dev)
+    cls = torch.empty(cfg.n_samples, dtype=torch.int32, device=dev)
+    F.predict(Xd, out=out, out_class=cls)
+    torch.cuda.synchronize()
+    idx = gen.subsample(77, cfg.n_samples, 4000)
+    ref = oracle.predict(f, X, rows=idx)
+    res = dict(out=out.cpu().numpy()[idx], cls=cls.cpu().numpy()[idx])
+    _check(res, ref, f["agg"], False, want_leaf=False)

@@ -41,22 +41,14 @@ struct DeviceGuard {
   }
 };
 
-constexpr int32_t kDefaultMaxSmem = 232448;  // sharedMemPerBlockOptin on sm_100 (227 KB)
-constexpr int32_t kBarrierBytes = 64;
+constexpr int32_t kDefaultMaxSmem = kMaxSmemOptin;
 
-// Rows of a sample tile staged in shared memory for a row width of d floats (0 = read rows from
-// global memory): 64 rows (2 per warp) when two buffers fit in 48 KB, else 32 rows within 64 KB.
-static int32_t tile_rows_for(int32_t d) {
-  const int64_t row = (int64_t)d * 4;
-  if (2 * 64 * row <= 48 * 1024) return 64;
-  if (2 * 32 * row <= 64 * 1024) return 32;
-  return 0;
-}
-
+// Slot rows (32 nodes each) of the per-CTA forest slice: the opt-in shared memory minus the
+// sample-tile ring for rows of n_features attributes (none when rows stay in global memory).
 static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
-  const int32_t R = tile_rows_for(n_features);
-  const int64_t reserve = (int64_t)2 * R * n_features * 4 + kBarrierBytes;
-  return (int32_t)std::max<int64_t>(0, (max_smem - reserve) / 256);
+  const int32_t fb = feature_bits(n_features + 1);
+  const int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb));
+  return (int32_t)std::max<int64_t>(0, (max_smem - ring - kSlicedBarrierBytes) / 256);
 }
 
 static void free_device(tahoe_forest* f) {
@@ -162,12 +154,11 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
 static SlicedPlan sliced_plan(const tahoe_forest* f, int32_t d) {
   SlicedPlan p;
   p.forest_smem = f->sl.slots_max * 256;
-  const int64_t left = (int64_t)f->max_smem - p.forest_smem - kBarrierBytes;
-  int32_t R = tile_rows_for(d);
-  while (R >= 32 && 2LL * R * d * 4 > left) R -= 32;
-  p.rows_in_smem = R >= 32;
-  p.tile_rows = p.rows_in_smem ? R : 128;
-  p.smem_bytes = p.forest_smem + (p.rows_in_smem ? 2 * R * d * 4 : 0) + kBarrierBytes;
+  const int64_t ring = sliced_ring_bytes(d, f->sl.fbits);
+  p.rows_in_smem = ring >= 0 && p.forest_smem + ring + kSlicedBarrierBytes <= f->max_smem;
+  p.tile_rows = kSlicedTileRows;
+  p.buf_floats = p.rows_in_smem ? sliced_buf_floats(d, f->sl.fbits) : 0;
+  p.smem_bytes = p.forest_smem + (p.rows_in_smem ? (int32_t)ring : 0) + kSlicedBarrierBytes;
   const int32_t ns = f->sl.n_slices;
   if (ns <= f->num_sms) {
     p.cps = std::max(1, f->num_sms / ns);

@@ -118,7 +118,8 @@ static bool pack_best(const Forest& F, const std::vector<int32_t>& trees, int32_
 
 tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   S = SlicedImage();
-  S.fbits = feature_bits(F.n_features);
+  S.fbits = feature_bits(F.n_features + 1);   // all-ones attribute field marks a leaf
+  cap -= 1;                                    // one terminal slot per lane column
   if (F.agg == TAHOE_AGG_VOTE) { S.why_invalid = "VOTE runs on the direct strategy"; return TAHOE_OK; }
   if (cap < 1) { S.why_invalid = "no shared memory budget"; return TAHOE_OK; }
   for (int32_t t = 0; t < F.n_trees; t++)
@@ -167,19 +168,25 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   S.slots_max = 0;
   double work = 0, padded = 0;
   for (auto& P : packs) {
+    P.max_len += 1;  // terminal slot
     S.slots_max = std::max(S.slots_max, P.max_len);
     work += P.sum_work;
     padded += 32.0 * P.max_work;
   }
   S.eff = padded > 0 ? work / padded : 0;
   S.trees_per_lane = (double)F.n_trees / (32.0 * std::max(1, S.n_slices));
-  const uint32_t off_lim = 1u << (kOffsetTop - S.fbits);
+  // Sliced node words (kernels.hpp "sliced encoding"): left child first, right child at +off,
+  // leaves carry the all-ones attribute field and the delta to the lane's next tree root; one
+  // self-looping terminal leaf (value 0.0, delta 0) closes every lane column.
+  const uint32_t fmask = (1u << S.fbits) - 1u;
+  const uint32_t off_lim = 1u << (31 - S.fbits - 8);   // offsets are stored in bytes (x256)
   const size_t per_slice = (size_t)S.slots_max * 32;
   S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
   S.col_len.assign((size_t)S.n_slices * 32, 0);
   S.slots.assign(S.n_slices, 0);
   std::vector<int32_t> slot(F.feat.size(), -1);
+  std::vector<int32_t> pre, st;
   for (int32_t s = 0; s < S.n_slices; s++) {
     const Pack& P = packs[s];
     S.slots[s] = P.max_len;
@@ -188,7 +195,13 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
       const auto& L = P.lanes[l];
       for (size_t ti = 0; ti < L.size(); ti++) {
         const int32_t t = L[ti];
-        std::vector<int32_t> pre = hot_preorder(F, t);
+        pre.clear();
+        st.assign(1, F.node_base[t]);
+        while (!st.empty()) {  // preorder, left child first
+          int32_t k = st.back(); st.pop_back();
+          pre.push_back(k);
+          if (F.feat[k] >= 0) { st.push_back(F.rc[k]); st.push_back(F.lc[k]); }
+        }
         for (size_t i = 0; i < pre.size(); i++) slot[pre[i]] = pos + (int32_t)i;
         const int32_t next_root = pos + (int32_t)pre.size();
         for (size_t i = 0; i < pre.size(); i++) {
@@ -197,24 +210,25 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
           const size_t w = ((size_t)s * per_slice + (size_t)sl * 32 + l);
           uint32_t y;
           if (F.feat[k] < 0) {
-            y = kLeafBit | (uint32_t)(next_root - sl);
+            y = ((uint32_t)(next_root - sl) << (S.fbits + 9)) | fmask;
             S.nodes[2 * w] = f2u(F.val[k]);
             S.leaf_meta[2 * w] = F.tree_orig[t];
             S.leaf_meta[2 * w + 1] = F.orig[k];
           } else {
-            const int32_t hot = F.hot_left[k] ? F.lc[k] : F.rc[k];
-            const int32_t cold = F.hot_left[k] ? F.rc[k] : F.lc[k];
-            if (slot[hot] != sl + 1) return fail(TAHOE_E_INVAL, "internal: hot child not adjacent");
-            const int32_t delta = slot[cold] - sl;
-            if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "cold offset overflow");
-            y = (F.dl[k] ? kDefaultLeftBit : 0u) | (F.hot_left[k] ? kHotLeftBit : 0u) |
-                ((uint32_t)delta << S.fbits) | (uint32_t)F.feat[k];
+            if (slot[F.lc[k]] != sl + 1) return fail(TAHOE_E_INVAL, "internal: left child not adjacent");
+            const int32_t delta = slot[F.rc[k]] - sl;   // in slots; stored as bytes
+            if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "right offset overflow");
+            y = ((uint32_t)delta << (S.fbits + 9)) | ((F.dl[k] ? 1u : 0u) << S.fbits) | (uint32_t)F.feat[k];
             S.nodes[2 * w] = f2u(F.thr[k]);
           }
           S.nodes[2 * w + 1] = y;
         }
         pos = next_root;
       }
+      // terminal self-loop
+      const size_t w = ((size_t)s * per_slice + (size_t)pos * 32 + l);
+      S.nodes[2 * w] = 0u;
+      S.nodes[2 * w + 1] = fmask;
       S.col_len[(size_t)s * 32 + l] = pos;
     }
   }

@@ -15,6 +15,7 @@
 //              fixed-order finalize kernel combines; a single-slice forest finalizes in-kernel.
 //  k_finalize — fixed-order fp64 sum of parts per class, base / average / argmax, RN to fp32.
 #include <cuda_runtime.h>
+#include <atomic>
 #include <cstdint>
 
 #include "kernels.hpp"
@@ -153,6 +154,12 @@ __global__ void __launch_bounds__(256) k_direct(const DirectKArgs a) {
 }
 
 // ------------------------------------------------------------------ sliced strategy
+// Sliced node words (encode.cpp): x = threshold (internal) or leaf value;
+//   internal y = off_bytes << (F+1) | default_left << F | attribute   (left child = next slot)
+//   leaf     y = next_root_bytes << (F+1) | (2^F - 1)                  (all-ones attribute field)
+// Offsets are byte distances between slots (slot = 32 lanes x 8 B = 256 B).  Every lane column
+// ends with a self-looping leaf of value 0.0, so a lane that has finished its trees can keep
+// stepping without effect.  Slot s of lane l is the word pair 32*s + l.
 struct SlicedKArgs {
   DevSliced img;
   const float* X;
@@ -161,108 +168,198 @@ struct SlicedKArgs {
   int32_t tile_rows;
   int32_t cps;           // CTAs per slice (single-pass)
   int32_t forest_smem;   // bytes reserved for the slice
-  int32_t tile_floats;   // floats per tile buffer
-  int32_t tma_ok;        // X is 16-byte aligned and tile_rows*d*4 % 16 == 0
+  int32_t buf_floats;    // floats per ring buffer (tile + leaf-read pad, multiple of 4)
+  int32_t x_aligned;     // X is 16-byte aligned (TMA bulk copies allowed)
   OutArgs o;
 };
+
+constexpr int kRing = 4;   // sample-tile ring depth (3 tiles in flight while one is consumed)
+
+// One step of one lane: read the node at shared address p, test "x_j < b_i", move to
+// the left child (+256 B) or the right child (+off); a leaf adds its value (fp64, reading Z17)
+// and jumps to the lane's next tree root.  NAN_AWARE: NaN takes the default path.
+template <bool NAN_AWARE>
+__device__ __forceinline__ void sliced_step(uint32_t& p, uint32_t rowaddr, uint32_t fmask,
+                                            uint32_t sh, double& acc) {
+  uint32_t x, y;
+  float v;
+  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+  const uint32_t f = y & fmask;
+  asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(rowaddr + (f << 2)));
+  bool go_left = v < __uint_as_float(x);
+  if (NAN_AWARE) go_left = go_left || ((v != v) && ((y >> (sh - 1)) & 1u));
+  const bool leaf = f == fmask;
+  p += (go_left && !leaf) ? 256u : (y >> sh);
+  // internal nodes add +0.0, which leaves an fp64 sum that started at +0.0 unchanged
+  const uint32_t xv = leaf ? x : 0u;
+  double dv;
+  asm("cvt.f64.f32 %0, %1;" : "=d"(dv) : "f"(__uint_as_float(xv)));
+  acc += dv;
+}
+
+template <bool LEAF, bool NAN_AWARE>
+__device__ __forceinline__ double walk_columns(uint32_t p, uint32_t pe, uint32_t rowaddr,
+                                               uint32_t fmask, uint32_t sh, uint32_t sbase,
+                                               const SlicedKArgs& a,
+                                               const int32_t* __restrict__ leaf_meta, int64_t i,
+                                               uint64_t& fp) {
+  double acc = 0.0;
+  if (!LEAF) {
+    // two steps per exit test; a finished lane idles on its terminal self-loop
+    while (p != pe) {
+      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, acc);
+      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, acc);
+    }
+  } else {
+    while (p != pe) {
+      const uint32_t lp = p;
+      uint32_t yy;
+      asm("ld.shared.u32 %0, [%1];" : "=r"(yy) : "r"(lp + 4));
+      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, acc);
+      if ((yy & fmask) == fmask) {
+        const uint32_t slot_word = (lp - sbase) >> 3;
+        const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * slot_word]);
+        a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
+        fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
+      }
+    }
+  }
+  return acc;
+}
+
+// Rows too wide to stage (e.g. 2000 attributes) are read from global memory through L1; this walk
+// is always NaN-aware and clamps the attribute index of leaves to stay inside the row.
+template <bool LEAF>
+__device__ __forceinline__ double walk_columns_global(uint32_t p, uint32_t pe,
+                                                      const float* __restrict__ row,
+                                                      uint32_t fmask, uint32_t sh, uint32_t sbase,
+                                                      const SlicedKArgs& a,
+                                                      const int32_t* __restrict__ leaf_meta,
+                                                      int64_t i, uint64_t& fp) {
+  double acc = 0.0;
+  while (p != pe) {
+    uint32_t x, y;
+    asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+    const uint32_t f = y & fmask;
+    const bool leaf = f == fmask;
+    const float v = __ldg(&row[leaf ? 0u : f]);
+    const bool go_left = (v < __uint_as_float(x)) || ((v != v) && ((y >> (sh - 1)) & 1u));
+    const uint32_t delta = (go_left && !leaf) ? 256u : (y >> sh);
+    if (leaf) {
+      acc += (double)__uint_as_float(x);
+      if (LEAF && delta) {
+        const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * ((p - sbase) >> 3)]);
+        a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
+        fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
+      }
+    }
+    p += delta;
+  }
+  return acc;
+}
 
 template <bool LEAF, bool FUSED, bool ROWS_SMEM>
 __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
   extern __shared__ __align__(128) unsigned char smem[];
-  uint2* s_nodes = reinterpret_cast<uint2*>(smem);
-  float* s_tile = reinterpret_cast<float*>(smem + a.forest_smem);
-  uint64_t* s_bar = reinterpret_cast<uint64_t*>(
-      smem + a.forest_smem + (ROWS_SMEM ? 2 * (size_t)a.tile_floats * sizeof(float) : 0));
+  float* s_ring = reinterpret_cast<float*>(smem + a.forest_smem);
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(
+      smem + a.forest_smem + (ROWS_SMEM ? (size_t)kRing * a.buf_floats * sizeof(float) : 0));
+  uint64_t* s_forest = s_full + kRing;
+  int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int nwarps = blockDim.x >> 5;
-  const int fbits = a.img.fbits;
-  const uint32_t fmask = (1u << fbits) - 1u;
-  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const uint32_t F = (uint32_t)a.img.fbits;
+  const uint32_t fmask = (1u << F) - 1u;
+  const uint32_t sh = F + 1;  // offsets (bytes) sit above the default-left bit
   const int32_t ns = a.img.n_slices;
   const int32_t G = gridDim.x;
   const bool multipass = ns > G;
   const int64_t R = a.tile_rows;
   const int64_t ntiles = (a.n + R - 1) / R;
-  const size_t tile_bytes_full = (size_t)R * a.d * sizeof(float);
 
   if (threadIdx.x == 0) {
-    mbar_init(&s_bar[0], 1);
-    mbar_init(&s_bar[1], 1);
-    mbar_init(&s_bar[2], 1);
+    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; }
+    mbar_init(s_forest, 1);
     fence_mbar_init();
   }
   __syncthreads();
-  uint32_t ph_forest = 0, ph0 = 0, ph1 = 0;
 
-  auto tile_tma = [&](int64_t tile) -> bool {
-    return ROWS_SMEM && a.tma_ok && (tile + 1) * R <= a.n;
-  };
-  auto issue_tile = [&](int64_t tile, int buf) {  // thread 0 only
-    fence_proxy_async_smem();
-    mbar_expect_tx(&s_bar[1 + buf], (uint32_t)tile_bytes_full);
-    bulk_g2s_big(s_tile + (size_t)buf * a.tile_floats, a.X + tile * R * a.d,
-                 (uint32_t)tile_bytes_full, &s_bar[1 + buf]);
+  // a6: stage tile `tile` into ring buffer b; called by one whole warp
+  auto issue_tile = [&](int64_t tile, int b) {
+    const int64_t r0 = tile * R;
+    const int64_t nr = (a.n - r0) < R ? (a.n - r0) : R;
+    const uint32_t bytes = (uint32_t)(nr * a.d * sizeof(float));
+    float* dst = s_ring + (size_t)b * a.buf_floats;
+    const float* src = a.X + r0 * a.d;
+    if (a.x_aligned) {
+      if (lane == 0) {
+        const uint32_t body = bytes & ~15u;
+        for (uint32_t q = body / 4; q < bytes / 4; q++) dst[q] = __ldg(&src[q]);  // <= 3 floats
+        fence_proxy_async_smem();
+        mbar_expect_tx(&s_full[b], body);
+        if (body) bulk_g2s_big(dst, src, body, &s_full[b]);
+      }
+    } else {  // misaligned X: the warp copies the tile itself
+      const uint32_t cnt = bytes / 4;
+      for (uint32_t q = lane; q < cnt; q += 32) dst[q] = __ldg(&src[q]);
+      __threadfence_block();
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_full[b])) : "memory");
+      }
+    }
+    __syncwarp();
   };
 
+  uint32_t g = 0;  // tiles this CTA has consumed so far (identical in every warp)
+  uint32_t ph_forest = 0;
   for (int32_t sl = multipass ? (int32_t)blockIdx.x : (int32_t)blockIdx.x % ns; sl < ns;
        sl += multipass ? G : ns) {
     const int64_t t0 = multipass ? 0 : blockIdx.x / ns;
     const int64_t ts = multipass ? 1 : a.cps;
-    // stage the slice (a7): one bulk copy of slots*32*8 bytes
-    if (threadIdx.x == 0) {
-      const uint32_t bytes = (uint32_t)a.img.slots[sl] * 256u;
-      fence_proxy_async_smem();
-      mbar_expect_tx(&s_bar[0], bytes);
-      bulk_g2s_big(s_nodes, a.img.nodes + (size_t)sl * a.img.slots_max * 64, bytes, &s_bar[0]);
-      if (t0 < ntiles && tile_tma(t0)) issue_tile(t0, 0);
+    const int64_t my_tiles = t0 < ntiles ? (ntiles - t0 + ts - 1) / ts : 0;
+    if (warp == 0) {
+      if (lane == 0) {  // a7: the slice, one bulk copy of slots*32*8 bytes
+        const uint32_t bytes = (uint32_t)a.img.slots[sl] * 256u;
+        fence_proxy_async_smem();
+        mbar_expect_tx(s_forest, bytes);
+        bulk_g2s_big(smem, a.img.nodes + (size_t)sl * a.img.slots_max * 64, bytes, s_forest);
+      }
+      if (ROWS_SMEM)
+        for (int64_t k = 0; k < kRing && k < my_tiles; k++) issue_tile(t0 + k * ts, (int)((g + k) % kRing));
     }
-    const uint32_t end = (uint32_t)a.img.col_len[sl * 32 + lane];
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t p0 = sbase + (uint32_t)lane * 8u;
+    const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * 32 + lane] * 32u + (uint32_t)lane) * 8u;
     const int32_t* __restrict__ leaf_meta = a.img.leaf_meta + (size_t)sl * a.img.slots_max * 64;
-    mbar_wait(&s_bar[0], ph_forest);
-    ph_forest ^= 1;
+    mbar_wait(s_forest, ph_forest);
+    ph_forest ^= 1u;
 
-    int64_t it = 0;
-    for (int64_t tile = t0; tile < ntiles; tile += ts, ++it) {
-      const int buf = (int)(it & 1);
+    for (int64_t it = 0; it < my_tiles; it++, g++) {
+      const int b = (int)(g % kRing);
+      const int64_t tile = t0 + it * ts;
       const int64_t r0 = tile * R;
       const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-      const float* tbuf = s_tile + (size_t)buf * a.tile_floats;
-      if (ROWS_SMEM) {
-        const int64_t nxt = tile + ts;
-        if (threadIdx.x == 0 && nxt < ntiles && tile_tma(nxt)) issue_tile(nxt, buf ^ 1);
-        if (tile_tma(tile)) {
-          if (buf == 0) { mbar_wait(&s_bar[1], ph0); ph0 ^= 1; }
-          else { mbar_wait(&s_bar[2], ph1); ph1 ^= 1; }
-        } else {  // ragged or unaligned tile: cooperative copy (a6 fallback)
-          float* dst = s_tile + (size_t)buf * a.tile_floats;
-          const float* src = a.X + r0 * a.d;
-          const int64_t cnt = (int64_t)nr * a.d;
-          for (int64_t q = threadIdx.x; q < cnt; q += blockDim.x) dst[q] = __ldg(&src[q]);
-          __syncthreads();
-        }
-      }
+      const float* tbuf = s_ring + (size_t)b * a.buf_floats;
+      if (ROWS_SMEM) mbar_wait(&s_full[b], (g / kRing) & 1u);
       for (int r = warp; r < nr; r += nwarps) {
         const int64_t i = r0 + r;
-        const float* __restrict__ row = ROWS_SMEM ? tbuf + (size_t)r * a.d : a.X + i * a.d;
-        double acc = 0.0;
         uint64_t fp = 0;
-        uint32_t s = 0;
-        // a8: each lane walks the trees of its column for sample i; leaves jump to the next root
-        while (s < end) {
-          const uint2 nd = s_nodes[s * 32 + lane];
-          if ((int32_t)nd.y < 0) {
-            acc += (double)__uint_as_float(nd.x);
-            if (LEAF) {
-              const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * (s * 32 + lane)]);
-              a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
-              fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
-            }
-            s += nd.y & 0x7fffffffu;
-          } else {
-            const float v = ROWS_SMEM ? row[nd.y & fmask] : __ldg(&row[nd.y & fmask]);
-            s += step(nd.x, nd.y, v, fbits, offmask);
-          }
+        double acc;
+        if (ROWS_SMEM) {
+          const float* row = tbuf + (size_t)r * a.d;
+          bool has_nan = false;
+          for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
+          const uint32_t rowaddr = smem_u32(row);
+          if (__any_sync(0xffffffffu, has_nan))
+            acc = walk_columns<LEAF, true>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
+          else
+            acc = walk_columns<LEAF, false>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
+        } else {
+          // wide rows stay in global memory (L1-cached); the leaf attribute read is clamped
+          const float* row = a.X + i * a.d;
+          acc = walk_columns_global<LEAF>(p0, pe, row, fmask, sh, sbase, a, leaf_meta, i, fp);
         }
         // a9: fp64 butterfly over the 32 lane sums (lane 0's order is fixed)
 #pragma unroll
@@ -278,9 +375,20 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
             atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
         }
       }
-      __syncthreads();  // the tile buffer is free for the next prefetch
+      if (ROWS_SMEM) {
+        // release buffer b; the last warp out refills it with the tile kRing ahead
+        __syncwarp();
+        int last = 0;
+        if (lane == 0) {
+          __threadfence_block();
+          last = atomicAdd(&s_cnt[b], 1) == nwarps - 1;
+          if (last) atomicExch(&s_cnt[b], 0);
+        }
+        last = __shfl_sync(0xffffffffu, last, 0);
+        if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+      }
     }
-    __syncthreads();  // the slice buffer is free for the next slice (multi-pass)
+    __syncthreads();  // every warp is done with this slice (multi-pass reload)
   }
 }
 
@@ -343,8 +451,15 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
 template <bool L, bool F, bool R>
 static cudaError_t sliced_one(const SlicedKArgs& a, const SlicedPlan& p, cudaStream_t st) {
   auto kern = k_sliced<L, F, R>;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
-  if (e != cudaSuccess) return e;
+  // raise the dynamic shared-memory limit once per process and device (not per launch)
+  static std::atomic<int> configured[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64 && configured[dev].load() < p.smem_bytes) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+    if (e != cudaSuccess) return e;
+    configured[dev].store(kMaxSmemOptin);
+  }
   kern<<<p.grid, p.block, p.smem_bytes, st>>>(a);
   return cudaGetLastError();
 }
@@ -359,9 +474,9 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
   a.tile_rows = plan.tile_rows;
   a.cps = plan.cps;
   a.forest_smem = plan.forest_smem;
-  a.tile_floats = plan.tile_rows * d;
-  a.tma_ok = ((reinterpret_cast<uintptr_t>(X) & 15) == 0) &&
-             (((int64_t)plan.tile_rows * d * 4) % 16 == 0);
+  a.buf_floats = plan.buf_floats;
+  a.x_aligned = ((reinterpret_cast<uintptr_t>(X) & 15) == 0) &&
+                (((int64_t)plan.tile_rows * d * 4) % 16 == 0);
   a.o = o;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;

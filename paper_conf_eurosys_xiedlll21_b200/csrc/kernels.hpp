@@ -69,9 +69,25 @@ struct FinalizeArgs {
 };
 
 // Launchers (kernels.cu).  Return a cudaError_t value as int (0 = success).
+constexpr int32_t kMaxSmemOptin = 232448;   // sharedMemPerBlockOptin on sm_100 (227 KB)
+constexpr int32_t kSlicedRing = 4;          // sample-tile ring depth of k_sliced
+constexpr int32_t kSlicedTileRows = 32;     // rows per tile (one per warp of a 1024-thread CTA)
+constexpr int32_t kSlicedBarrierBytes = 128;
+
+// Floats per ring buffer: a tile of rows plus the pad a leaf's all-ones attribute read touches.
+inline int32_t sliced_buf_floats(int32_t d, int32_t fbits) {
+  int64_t f = (int64_t)kSlicedTileRows * d + (1 << fbits);
+  return (int32_t)((f + 3) & ~3LL);
+}
+// Shared memory of the sample-tile ring, or -1 when rows are too wide to stage (> 64 KB).
+inline int64_t sliced_ring_bytes(int32_t d, int32_t fbits) {
+  int64_t b = (int64_t)kSlicedRing * sliced_buf_floats(d, fbits) * 4;
+  return b <= 64 * 1024 ? b : -1;
+}
+
 struct SlicedPlan {
   int32_t grid = 0, block = 1024, tile_rows = 0, cps = 1;
-  int32_t smem_bytes = 0, forest_smem = 0;
+  int32_t smem_bytes = 0, forest_smem = 0, buf_floats = 0;
   bool rows_in_smem = true;
 };
 int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,

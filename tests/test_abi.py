@@ -187,30 +187,35 @@ def test_product_tokens_simhash_equal_oracle_on_generated_forest():
 
 def decode_sliced(img, X, n_trees, n_classes):
     """Walk the exported SLICED image on the host (test-side decoder, independent of the
-    product): returns leaf[n, T] (caller node ids) and per-class fp64 sums in slice order."""
+    product's kernels): returns leaf[n, T] (caller node ids) and per-class fp64 sums.
+    Node words: internal y = off_bytes << (F+1) | default_left << F | attribute (left child next);
+    leaf y = next_root_bytes << (F+1) | (2^F - 1); slot = 256 bytes."""
     n = X.shape[0]
     F = img["feature_bits"]
+    fmask = (1 << F) - 1
     leaf = np.full((n, n_trees), -1, np.int64)
     sums = np.zeros((n, n_classes))
     for s in range(img["n_slices"]):
         c = img["slice_info"][s, 1]
         for lane in range(32):
             end = img["col_len"][s, lane]
+            x_t, y_t = img["nodes"][s, end, lane]
+            assert y_t == fmask and x_t == 0, "terminal self-loop closes the column"
             for i in range(n):
                 k = 0
                 while k < end:
                     x, y = (int(v) for v in img["nodes"][s, k, lane])
-                    if y & 0x80000000:
+                    if (y & fmask) == fmask:
                         t, node = img["leaf_meta"][s, k, lane]
                         leaf[i, t] = node
                         sums[i, c] += float(np.uint32(x).view(np.float32))
-                        k += y & 0x7FFFFFFF
+                        k += (y >> (F + 1)) // 256
                     else:
                         thr = float(np.uint32(x).view(np.float32))
-                        v = X[i, y & ((1 << F) - 1)]
-                        go_left = bool((y >> 30) & 1) if np.isnan(v) else bool(v < thr)
-                        hot = go_left == bool((y >> 29) & 1)
-                        k += 1 if hot else (y >> F) & ((1 << (29 - F)) - 1)
+                        v = X[i, y & fmask]
+                        go_left = bool((y >> F) & 1) if np.isnan(v) else bool(v < thr)
+                        k += 1 if go_left else (y >> (F + 1)) // 256
+                assert k == end
     return leaf, sums
 
 

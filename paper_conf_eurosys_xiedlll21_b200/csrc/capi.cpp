@@ -7,6 +7,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <sstream>
 #include <string>
@@ -42,6 +43,32 @@ struct DeviceGuard {
 };
 
 constexpr int32_t kDefaultMaxSmem = kMaxSmemOptin;
+
+// Stream-ordered scratch (fp64 partials) comes from a library-owned pool per device that keeps
+// its memory across synchronisations (release threshold = max), so a predict call never waits
+// for the driver to map fresh pages.
+static cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
+  static std::mutex mu;
+  static cudaMemPool_t pools[64] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaMallocAsync(p, bytes, st);
+  {
+    std::lock_guard<std::mutex> g(mu);
+    if (!pools[dev]) {
+      cudaMemPoolProps props = {};
+      props.allocType = cudaMemAllocationTypePinned;
+      props.location.type = cudaMemLocationTypeDevice;
+      props.location.id = dev;
+      e = cudaMemPoolCreate(&pools[dev], &props);
+      if (e != cudaSuccess) { pools[dev] = nullptr; return cudaMallocAsync(p, bytes, st); }
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pools[dev], cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  return cudaMallocFromPoolAsync(p, bytes, pools[dev], st);
+}
 
 // Slot rows (32 nodes each) of the per-CTA forest slice: the opt-in shared memory minus the
 // sample-tile ring for rows of n_features attributes (none when rows stay in global memory).
@@ -210,7 +237,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       return TAHOE_OK;
     }
     double* raw = raw_user;
-    if (!raw && (e = cudaMallocAsync((void**)&raw, (size_t)n * C * 8, st)) != cudaSuccess)
+    if (!raw && (e = scratch_alloc((void**)&raw, (size_t)n * C * 8, st)) != cudaSuccess)
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync partial");
     if ((e = cudaMemsetAsync(raw, 0, (size_t)n * C * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
     o.raw = raw;
@@ -233,7 +260,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   const bool fused = scalar && !raw_user && f->sl.n_slices == 1;
   double* part = nullptr;
   if (!fused) {
-    if ((e = cudaMallocAsync((void**)&part, (size_t)f->sl.n_slices * n * 8, st)) != cudaSuccess)
+    if ((e = scratch_alloc((void**)&part, (size_t)f->sl.n_slices * n * 8, st)) != cudaSuccess)
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync partial");
     o.raw = part;
   }
@@ -370,9 +397,9 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   float* dX = nullptr;
   float* dO = nullptr;
   int32_t* dC = nullptr;
-  cudaError_t e = cudaMallocAsync((void**)&dX, (size_t)2 * chunk * d * 4, user);
-  if (e == cudaSuccess) e = cudaMallocAsync((void**)&dO, (size_t)2 * chunk * C * 4, user);
-  if (e == cudaSuccess && class_host) e = cudaMallocAsync((void**)&dC, (size_t)2 * chunk * 4, user);
+  cudaError_t e = scratch_alloc((void**)&dX, (size_t)2 * chunk * d * 4, user);
+  if (e == cudaSuccess) e = scratch_alloc((void**)&dO, (size_t)2 * chunk * C * 4, user);
+  if (e == cudaSuccess && class_host) e = scratch_alloc((void**)&dC, (size_t)2 * chunk * 4, user);
   cudaEventRecord(ev_start, user);
   cudaStreamWaitEvent(s_in, ev_start, 0);
   cudaStreamWaitEvent(s_cmp, ev_start, 0);

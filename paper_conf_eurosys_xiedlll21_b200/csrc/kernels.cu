@@ -173,14 +173,14 @@ struct SlicedKArgs {
   OutArgs o;
 };
 
-constexpr int kRing = 4;   // sample-tile ring depth (3 tiles in flight while one is consumed)
+constexpr int kRing = kSlicedRing;  // sample-tile ring depth
 
 // One step of one lane: read the node at shared address p, test "x_j < b_i", move to
 // the left child (+256 B) or the right child (+off); a leaf adds its value (fp64, reading Z17)
 // and jumps to the lane's next tree root.  NAN_AWARE: NaN takes the default path.
 template <bool NAN_AWARE>
 __device__ __forceinline__ void sliced_step(uint32_t& p, uint32_t rowaddr, uint32_t fmask,
-                                            uint32_t sh, double& acc) {
+                                            uint32_t sh, uint32_t shmul, double& acc) {
   uint32_t x, y;
   float v;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
@@ -189,12 +189,30 @@ __device__ __forceinline__ void sliced_step(uint32_t& p, uint32_t rowaddr, uint3
   bool go_left = v < __uint_as_float(x);
   if (NAN_AWARE) go_left = go_left || ((v != v) && ((y >> (sh - 1)) & 1u));
   const bool leaf = f == fmask;
-  p += (go_left && !leaf) ? 256u : (y >> sh);
+  // y >> sh computed as a high multiply: IMAD.HI runs on the FMA pipe, relieving the ALU pipe
+  p += (go_left && !leaf) ? 256u : __umulhi(y, shmul);
   // internal nodes add +0.0, which leaves an fp64 sum that started at +0.0 unchanged
   const uint32_t xv = leaf ? x : 0u;
   double dv;
   asm("cvt.f64.f32 %0, %1;" : "=d"(dv) : "f"(__uint_as_float(xv)));
   acc += dv;
+}
+
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_columns2(uint32_t pA, uint32_t pB, uint32_t pe,
+                                              uint32_t rowA, uint32_t rowB, uint32_t fmask,
+                                              uint32_t sh, uint32_t shmul, double& accA,
+                                              double& accB) {
+  // two independent samples per lane (ILP): while one chain waits on shared memory the other
+  // issues; a chain that reached its terminal self-loop steps harmlessly
+  accA = 0.0;
+  accB = 0.0;
+  while ((pA != pe) | (pB != pe)) {
+    sliced_step<NAN_AWARE>(pA, rowA, fmask, sh, shmul, accA);
+    sliced_step<NAN_AWARE>(pB, rowB, fmask, sh, shmul, accB);
+    sliced_step<NAN_AWARE>(pA, rowA, fmask, sh, shmul, accA);
+    sliced_step<NAN_AWARE>(pB, rowB, fmask, sh, shmul, accB);
+  }
 }
 
 template <bool LEAF, bool NAN_AWARE>
@@ -207,15 +225,15 @@ __device__ __forceinline__ double walk_columns(uint32_t p, uint32_t pe, uint32_t
   if (!LEAF) {
     // two steps per exit test; a finished lane idles on its terminal self-loop
     while (p != pe) {
-      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, acc);
-      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, acc);
+      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, 1u << (32 - sh), acc);
+      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, 1u << (32 - sh), acc);
     }
   } else {
     while (p != pe) {
       const uint32_t lp = p;
       uint32_t yy;
       asm("ld.shared.u32 %0, [%1];" : "=r"(yy) : "r"(lp + 4));
-      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, acc);
+      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, 1u << (32 - sh), acc);
       if ((yy & fmask) == fmask) {
         const uint32_t slot_word = (lp - sbase) >> 3;
         const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * slot_word]);
@@ -272,6 +290,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
   const uint32_t F = (uint32_t)a.img.fbits;
   const uint32_t fmask = (1u << F) - 1u;
   const uint32_t sh = F + 1;  // offsets (bytes) sit above the default-left bit
+  const uint32_t shmul = 1u << (32 - sh);
   const int32_t ns = a.img.n_slices;
   const int32_t G = gridDim.x;
   const bool multipass = ns > G;
@@ -343,24 +362,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
       const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
       const float* tbuf = s_ring + (size_t)b * a.buf_floats;
       if (ROWS_SMEM) mbar_wait(&s_full[b], (g / kRing) & 1u);
-      for (int r = warp; r < nr; r += nwarps) {
-        const int64_t i = r0 + r;
-        uint64_t fp = 0;
-        double acc;
-        if (ROWS_SMEM) {
-          const float* row = tbuf + (size_t)r * a.d;
-          bool has_nan = false;
-          for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
-          const uint32_t rowaddr = smem_u32(row);
-          if (__any_sync(0xffffffffu, has_nan))
-            acc = walk_columns<LEAF, true>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
-          else
-            acc = walk_columns<LEAF, false>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
-        } else {
-          // wide rows stay in global memory (L1-cached); the leaf attribute read is clamped
-          const float* row = a.X + i * a.d;
-          acc = walk_columns_global<LEAF>(p0, pe, row, fmask, sh, sbase, a, leaf_meta, i, fp);
-        }
+      auto finish_row = [&](double acc, uint64_t fp, int64_t i) {
         // a9: fp64 butterfly over the 32 lane sums (lane 0's order is fixed)
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
@@ -373,6 +375,46 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
           else a.o.raw[(size_t)sl * a.n + i] = acc;
           if (LEAF && a.o.out_fp)
             atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
+        }
+      };
+      if (ROWS_SMEM && !LEAF) {
+        // rows r and r + nwarps of the tile walk together (two chains per lane)
+        for (int r = warp; r < nr; r += 2 * nwarps) {
+          const int r2 = r + nwarps;
+          const bool two = r2 < nr;
+          const float* rowA = tbuf + (size_t)r * a.d;
+          const float* rowB = tbuf + (size_t)(two ? r2 : r) * a.d;
+          bool has_nan = false;
+          for (int j = lane; j < a.d; j += 32) has_nan |= (rowA[j] != rowA[j]) | (rowB[j] != rowB[j]);
+          double accA, accB;
+          const uint32_t pB = two ? p0 : pe;
+          if (__any_sync(0xffffffffu, has_nan))
+            walk_columns2<true>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), fmask, sh, shmul, accA, accB);
+          else
+            walk_columns2<false>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), fmask, sh, shmul, accA, accB);
+          finish_row(accA, 0, r0 + r);
+          if (two) finish_row(accB, 0, r0 + r2);
+        }
+      } else {
+        for (int r = warp; r < nr; r += nwarps) {
+          const int64_t i = r0 + r;
+          uint64_t fp = 0;
+          double acc;
+          if (ROWS_SMEM) {
+            const float* row = tbuf + (size_t)r * a.d;
+            bool has_nan = false;
+            for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
+            const uint32_t rowaddr = smem_u32(row);
+            if (__any_sync(0xffffffffu, has_nan))
+              acc = walk_columns<LEAF, true>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
+            else
+              acc = walk_columns<LEAF, false>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
+          } else {
+            // wide rows stay in global memory (L1-cached); the leaf attribute read is clamped
+            const float* row = a.X + i * a.d;
+            acc = walk_columns_global<LEAF>(p0, pe, row, fmask, sh, sbase, a, leaf_meta, i, fp);
+          }
+          finish_row(acc, fp, i);
         }
       }
       if (ROWS_SMEM) {

@@ -70,8 +70,8 @@ struct FinalizeArgs {
 
 // Launchers (kernels.cu).  Return a cudaError_t value as int (0 = success).
 constexpr int32_t kMaxSmemOptin = 232448;   // sharedMemPerBlockOptin on sm_100 (227 KB)
-constexpr int32_t kSlicedRing = 4;          // sample-tile ring depth of k_sliced
-constexpr int32_t kSlicedTileRows = 32;     // rows per tile (one per warp of a 1024-thread CTA)
+constexpr int32_t kSlicedRing = 3;          // sample-tile ring depth of k_sliced
+constexpr int32_t kSlicedTileRows = 64;     // rows per tile (two per warp of a 1024-thread CTA)
 constexpr int32_t kSlicedBarrierBytes = 128;
 
 // Floats per ring buffer: a tile of rows plus the pad a leaf's all-ones attribute read touches.

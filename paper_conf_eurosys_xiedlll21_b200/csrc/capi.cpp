@@ -74,8 +74,10 @@ static cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
 // sample-tile ring for rows of n_features attributes (none when rows stay in global memory).
 static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
   const int32_t fb = feature_bits(n_features + 1);
-  const int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb));
-  return (int32_t)std::max<int64_t>(0, (max_smem - ring - kSlicedBarrierBytes) / 256);
+  const bool padded = n_features % 4 == 0;   // predict with d == n_features takes the 2-D TMA path
+  const int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb, padded));
+  // the slice region is rounded up to 1 KB so the ring's row bases stay aligned
+  return (int32_t)std::max<int64_t>(0, ((max_smem - ring - kSlicedBarrierBytes) & ~1023LL) / 256);
 }
 
 static void free_device(tahoe_forest* f) {
@@ -178,14 +180,21 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
   return select_strategy(plan_stats(f), n, d, f->host.agg);
 }
 
-static SlicedPlan sliced_plan(const tahoe_forest* f, int32_t d) {
+static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int32_t d) {
   SlicedPlan p;
-  p.forest_smem = f->sl.slots_max * 256;
-  const int64_t ring = sliced_ring_bytes(d, f->sl.fbits);
-  p.rows_in_smem = ring >= 0 && p.forest_smem + ring + kSlicedBarrierBytes <= f->max_smem;
+  p.forest_smem = ((f->sl.slots_max * 256) + 1023) & ~1023;
+  const int32_t fb = f->sl.fbits;
+  const int64_t room = (int64_t)f->max_smem - p.forest_smem - kSlicedBarrierBytes;
+  const int64_t ring_p = padded_rows_possible(X, d) ? sliced_ring_bytes(d, fb, true) : -1;
+  const int64_t ring_d = sliced_ring_bytes(d, fb, false);
+  int64_t ring = 0;
+  if (ring_p >= 0 && ring_p <= room) { p.rows = 2; ring = ring_p; }
+  else if (ring_d >= 0 && ring_d <= room) { p.rows = 1; ring = ring_d; }
+  else p.rows = 0;
   p.tile_rows = kSlicedTileRows;
-  p.buf_floats = p.rows_in_smem ? sliced_buf_floats(d, f->sl.fbits) : 0;
-  p.smem_bytes = p.forest_smem + (p.rows_in_smem ? (int32_t)ring : 0) + kSlicedBarrierBytes;
+  p.buf_floats = p.rows ? sliced_buf_floats(d, fb, p.rows == 2) : 0;
+  p.row_stride = sliced_row_stride(d, fb, p.rows == 2);
+  p.smem_bytes = p.forest_smem + (int32_t)ring + kSlicedBarrierBytes;
   const int32_t ns = f->sl.n_slices;
   if (ns <= f->num_sms) {
     p.cps = std::max(1, f->num_sms / ns);
@@ -256,7 +265,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
     return TAHOE_OK;
   }
   // sliced
-  const SlicedPlan plan = sliced_plan(f, d);
+  const SlicedPlan plan = sliced_plan(f, X, d);
   const bool fused = scalar && !raw_user && f->sl.n_slices == 1;
   double* part = nullptr;
   if (!fused) {

@@ -65,11 +65,18 @@ struct Pack {
   double max_work = 0, sum_work = 0;
 };
 
+// Slots a tree occupies in a lane column: a single-leaf tree is encoded as a 3-node stump (an
+// internal root whose two children are copies of the leaf) so that every tree starts with an
+// internal node — two consecutive steps of a lane then never both meet a nonzero leaf.
+static int32_t enc_size(const Forest& F, int32_t t) {
+  return F.tree_size(t) == 1 ? 3 : F.tree_size(t);
+}
+
 static void pack_stats(const Forest& F, Pack& P) {
   P.max_len = 0; P.max_work = 0; P.sum_work = 0;
   for (auto& L : P.lanes) {
     int32_t len = 0; double w = 0;
-    for (int32_t t : L) { len += F.tree_size(t); w += F.exp_reads[t]; }
+    for (int32_t t : L) { len += enc_size(F, t); w += F.exp_reads[t]; }
     P.max_len = std::max(P.max_len, len);
     P.max_work = std::max(P.max_work, w);
     P.sum_work += w;
@@ -88,20 +95,20 @@ static bool pack_lpt(const Forest& F, const std::vector<int32_t>& trees, int32_t
   std::vector<int32_t> ts(trees);
   std::stable_sort(ts.begin(), ts.end(), [&](int32_t a, int32_t b) {
     if (F.exp_reads[a] != F.exp_reads[b]) return F.exp_reads[a] > F.exp_reads[b];
-    return F.tree_size(a) > F.tree_size(b);
+    return enc_size(F, a) > enc_size(F, b);
   });
   std::vector<double> w(32, 0.0);
   std::vector<int32_t> len(32, 0);
   for (int32_t t : ts) {
     int32_t best = -1;
     for (int32_t l = 0; l < 32; l++) {
-      if (len[l] + F.tree_size(t) > cap) continue;
+      if (len[l] + enc_size(F, t) > cap) continue;
       if (best < 0 || w[l] < w[best] || (w[l] == w[best] && len[l] < len[best])) best = l;
     }
     if (best < 0) return false;
     P.lanes[best].push_back(t);
     w[best] += F.exp_reads[t];
-    len[best] += F.tree_size(t);
+    len[best] += enc_size(F, t);
   }
   pack_stats(F, P);
   return true;
@@ -123,7 +130,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   if (F.agg == TAHOE_AGG_VOTE) { S.why_invalid = "VOTE runs on the direct strategy"; return TAHOE_OK; }
   if (cap < 1) { S.why_invalid = "no shared memory budget"; return TAHOE_OK; }
   for (int32_t t = 0; t < F.n_trees; t++)
-    if (F.tree_size(t) > cap) { S.why_invalid = "a tree exceeds one lane column of shared memory"; return TAHOE_OK; }
+    if (enc_size(F, t) > cap) { S.why_invalid = "a tree exceeds one lane column of shared memory"; return TAHOE_OK; }
 
   std::vector<std::vector<int32_t>> groups(F.n_classes);
   for (int32_t t : F.order) groups[F.tclass[t]].push_back(t);
@@ -132,7 +139,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
     const auto& G = groups[c];
     if (G.empty()) continue;
     int64_t total = 0;
-    for (int32_t t : G) total += F.tree_size(t);
+    for (int32_t t : G) total += enc_size(F, t);
     int32_t k = (int32_t)std::max<int64_t>(1, (int64_t)std::ceil((double)total / (32.0 * cap * 0.97)));
     for (;; k++) {
       if (k > (int32_t)G.size()) { S.why_invalid = "cannot pack trees into slices"; return TAHOE_OK; }
@@ -144,11 +151,11 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
         int64_t acc = 0;
         for (int32_t j = 1; j < k; j++) {
           const int64_t target = total * j / k;
-          while (pos < G.size() && acc < target) acc += F.tree_size(G[pos++]);
+          while (pos < G.size() && acc < target) acc += enc_size(F, G[pos++]);
           cut[j] = std::min(std::max(pos, cut[j - 1] + 1), G.size() - (size_t)(k - j));
           pos = cut[j];
           acc = 0;
-          for (size_t q = 0; q < pos; q++) acc += F.tree_size(G[q]);
+          for (size_t q = 0; q < pos; q++) acc += enc_size(F, G[q]);
         }
       }
       std::vector<Pack> ps;
@@ -179,7 +186,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   // leaves carry the all-ones attribute field and the delta to the lane's next tree root; one
   // self-looping terminal leaf (value 0.0, delta 0) closes every lane column.
   const uint32_t fmask = (1u << S.fbits) - 1u;
-  const uint32_t off_lim = 1u << (31 - S.fbits - 8);   // offsets are stored in bytes (x256)
+  const uint32_t off_lim = 1u << (32 - (S.fbits + 3) - 8);   // offsets stored in bytes (x256)
   const size_t per_slice = (size_t)S.slots_max * 32;
   S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
@@ -195,6 +202,21 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
       const auto& L = P.lanes[l];
       for (size_t ti = 0; ti < L.size(); ti++) {
         const int32_t t = L[ti];
+        if (F.tree_size(t) == 1) {  // 3-node stump: root (attribute 0, +2 slots right) + 2 leaves
+          const int32_t k = F.node_base[t];
+          const uint32_t ynode = (2u * 256u) << (S.fbits + 3);
+          const uint32_t yleaf1 = (2u * 256u) << (S.fbits + 3) | (fmask << 2);
+          const uint32_t yleaf2 = (1u * 256u) << (S.fbits + 3) | (fmask << 2);
+          const uint32_t ys[3] = {ynode, yleaf1, yleaf2};
+          for (int32_t q = 0; q < 3; q++) {
+            const size_t w = ((size_t)s * per_slice + (size_t)(pos + q) * 32 + l);
+            S.nodes[2 * w] = q == 0 ? 0u : f2u(F.val[k]);
+            S.nodes[2 * w + 1] = ys[q];
+            if (q > 0) { S.leaf_meta[2 * w] = F.tree_orig[t]; S.leaf_meta[2 * w + 1] = F.orig[k]; }
+          }
+          pos += 3;
+          continue;
+        }
         pre.clear();
         st.assign(1, F.node_base[t]);
         while (!st.empty()) {  // preorder, left child first
@@ -210,7 +232,8 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
           const size_t w = ((size_t)s * per_slice + (size_t)sl * 32 + l);
           uint32_t y;
           if (F.feat[k] < 0) {
-            y = ((uint32_t)(next_root - sl) << (S.fbits + 9)) | fmask;
+            if ((uint32_t)(next_root - sl) >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "leaf offset overflow");
+            y = ((uint32_t)(next_root - sl) << (S.fbits + 11)) | (fmask << 2);
             S.nodes[2 * w] = f2u(F.val[k]);
             S.leaf_meta[2 * w] = F.tree_orig[t];
             S.leaf_meta[2 * w + 1] = F.orig[k];
@@ -218,7 +241,8 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
             if (slot[F.lc[k]] != sl + 1) return fail(TAHOE_E_INVAL, "internal: left child not adjacent");
             const int32_t delta = slot[F.rc[k]] - sl;   // in slots; stored as bytes
             if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "right offset overflow");
-            y = ((uint32_t)delta << (S.fbits + 9)) | ((F.dl[k] ? 1u : 0u) << S.fbits) | (uint32_t)F.feat[k];
+            y = ((uint32_t)delta << (S.fbits + 11)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 2)) |
+                ((uint32_t)F.feat[k] << 2);
             S.nodes[2 * w] = f2u(F.thr[k]);
           }
           S.nodes[2 * w + 1] = y;
@@ -228,7 +252,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
       // terminal self-loop
       const size_t w = ((size_t)s * per_slice + (size_t)pos * 32 + l);
       S.nodes[2 * w] = 0u;
-      S.nodes[2 * w + 1] = fmask;
+      S.nodes[2 * w + 1] = fmask << 2;
       S.col_len[(size_t)s * 32 + l] = pos;
     }
   }

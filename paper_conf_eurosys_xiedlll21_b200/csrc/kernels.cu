@@ -14,6 +14,7 @@
 //              32 fp64 lane sums with a shuffle butterfly.  Slices write fp64 partials that a
 //              fixed-order finalize kernel combines; a single-slice forest finalizes in-kernel.
 //  k_finalize — fixed-order fp64 sum of parts per class, base / average / argmax, RN to fp32.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <atomic>
 #include <cstdint>
@@ -155,114 +156,137 @@ __global__ void __launch_bounds__(256) k_direct(const DirectKArgs a) {
 
 // ------------------------------------------------------------------ sliced strategy
 // Sliced node words (encode.cpp): x = threshold (internal) or leaf value;
-//   internal y = off_bytes << (F+1) | default_left << F | attribute   (left child = next slot)
-//   leaf     y = next_root_bytes << (F+1) | (2^F - 1)                  (all-ones attribute field)
-// Offsets are byte distances between slots (slot = 32 lanes x 8 B = 256 B).  Every lane column
-// ends with a self-looping leaf of value 0.0, so a lane that has finished its trees can keep
-// stepping without effect.  Slot s of lane l is the word pair 32*s + l.
-struct SlicedKArgs {
+//   internal y = off_bytes << (F+3) | default_left << (F+2) | attribute << 2   (left child next)
+//   leaf     y = next_root_bytes << (F+3) | (2^F - 1) << 2            (all-ones attribute field)
+// Offsets are byte distances between slots (slot = 32 lanes x 8 B = 256 B).  The attribute is
+// stored as a byte offset, and staged rows sit at a power-of-two stride >= 2^F floats, so the
+// attribute's shared address is one LOP3: (y & amask) | row_base; a leaf is the one address
+// row_base | amask.  Every lane column ends with a self-looping leaf of value 0.0, so a lane that
+// has finished its trees keeps stepping harmlessly.  Slot s of lane l is the word pair 32*s + l.
+struct alignas(64) SlicedKArgs {
+  CUtensorMap tmap;      // PADDED rows: X as a 2-D tensor [n][d], box [row_stride][tile_rows]
   DevSliced img;
   const float* X;
   int64_t n;
   int32_t d;
   int32_t tile_rows;
   int32_t cps;           // CTAs per slice (single-pass)
-  int32_t forest_smem;   // bytes reserved for the slice
-  int32_t buf_floats;    // floats per ring buffer (tile + leaf-read pad, multiple of 4)
-  int32_t x_aligned;     // X is 16-byte aligned (TMA bulk copies allowed)
+  int32_t forest_smem;   // bytes reserved for the slice (multiple of 1024)
+  int32_t row_stride;    // floats between staged rows (PADDED: multiple of 2^F; DENSE: d)
+  int32_t buf_floats;    // floats per ring buffer
+  int32_t x_aligned;     // DENSE rows: X 16-byte aligned (one 1-D bulk copy per tile)
   OutArgs o;
 };
 
+// Row staging layouts of k_sliced (SlicedPlan::rows)
+constexpr int kRowsGlobal = 0;  // rows read from global memory (too wide to stage)
+constexpr int kRowsDense = 1;   // rows at stride d, one 1-D bulk copy per tile
+constexpr int kRowsPadded = 2;  // rows at stride 2^F*k via one 2-D tensor TMA per tile
+
 constexpr int kRing = kSlicedRing;  // sample-tile ring depth
 
+struct StepConsts {
+  uint32_t amask;   // attribute byte-offset mask (2^F - 1) << 2
+  uint32_t dlbit;   // default-left bit
+  uint32_t shmul;   // 2^(32 - (F+3)): y >> (F+3) == umulhi(y, shmul)
+};
+
 // One step of one lane: read the node at shared address p, test "x_j < b_i", move to
-// the left child (+256 B) or the right child (+off); a leaf adds its value (fp64, reading Z17)
-// and jumps to the lane's next tree root.  NAN_AWARE: NaN takes the default path.
-template <bool NAN_AWARE>
-__device__ __forceinline__ void sliced_step(uint32_t& p, uint32_t rowaddr, uint32_t fmask,
-                                            uint32_t sh, uint32_t shmul, double& acc) {
+// the left child (+256 B) or the right child (+off); return the leaf value met (0.0f at internal
+// nodes).  A leaf jumps to the lane's next tree root.  NAN_AWARE: NaN takes the node's default
+// path.
+template <bool NAN_AWARE, bool PADDED>
+__device__ __forceinline__ float sliced_step_v(uint32_t& p, uint32_t rowaddr, uint32_t leafaddr,
+                                               const StepConsts& k) {
   uint32_t x, y;
   float v;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
-  const uint32_t f = y & fmask;
-  asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(rowaddr + (f << 2)));
+  // PADDED: row bases are aligned to the attribute field, so OR == ADD and the leaf is the one
+  // address row | amask; DENSE: add, and test the attribute field itself
+  const uint32_t off = y & k.amask;
+  const uint32_t addr = PADDED ? ((y & k.amask) | rowaddr) : (rowaddr + off);
+  asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr));
   bool go_left = v < __uint_as_float(x);
-  if (NAN_AWARE) go_left = go_left || ((v != v) && ((y >> (sh - 1)) & 1u));
-  const bool leaf = f == fmask;
-  // y >> sh computed as a high multiply: IMAD.HI runs on the FMA pipe, relieving the ALU pipe
-  p += (go_left && !leaf) ? 256u : __umulhi(y, shmul);
-  // internal nodes add +0.0, which leaves an fp64 sum that started at +0.0 unchanged
-  const uint32_t xv = leaf ? x : 0u;
+  if (NAN_AWARE) go_left = go_left || ((v != v) && (y & k.dlbit));
+  const bool leaf = PADDED ? (addr == leafaddr) : (off == k.amask);
+  // y >> (F+3) as a high multiply: IMAD.HI runs on the FMA pipe, relieving the ALU pipe
+  p += (go_left && !leaf) ? 256u : __umulhi(y, k.shmul);
+  return __uint_as_float(leaf ? x : 0u);
+}
+
+// fp32 sum of two consecutive step values of one chain, then ONE fp64 add: exact, because two
+// consecutive steps never both meet a nonzero leaf (every tree has an internal root in the sliced
+// encoding, and the terminal leaf is 0.0), so the fp32 add is x + 0 = x.  Internal nodes add
+// +0.0, which leaves an fp64 sum that started at +0.0 unchanged.
+__device__ __forceinline__ void add_pair(double& acc, float v1, float v2) {
   double dv;
-  asm("cvt.f64.f32 %0, %1;" : "=d"(dv) : "f"(__uint_as_float(xv)));
+  asm("cvt.f64.f32 %0, %1;" : "=d"(dv) : "f"(__fadd_rn(v1, v2)));
   acc += dv;
 }
 
-template <bool NAN_AWARE>
+template <bool NAN_AWARE, bool PADDED>
 __device__ __forceinline__ void walk_columns2(uint32_t pA, uint32_t pB, uint32_t pe,
-                                              uint32_t rowA, uint32_t rowB, uint32_t fmask,
-                                              uint32_t sh, uint32_t shmul, double& accA,
-                                              double& accB) {
+                                              uint32_t rowA, uint32_t rowB, const StepConsts& k,
+                                              double& accA, double& accB) {
   // two independent samples per lane (ILP): while one chain waits on shared memory the other
   // issues; a chain that reached its terminal self-loop steps harmlessly
+  const uint32_t leafA = rowA | k.amask, leafB = rowB | k.amask;
   accA = 0.0;
   accB = 0.0;
   while ((pA != pe) | (pB != pe)) {
-    sliced_step<NAN_AWARE>(pA, rowA, fmask, sh, shmul, accA);
-    sliced_step<NAN_AWARE>(pB, rowB, fmask, sh, shmul, accB);
-    sliced_step<NAN_AWARE>(pA, rowA, fmask, sh, shmul, accA);
-    sliced_step<NAN_AWARE>(pB, rowB, fmask, sh, shmul, accB);
+    const float a1 = sliced_step_v<NAN_AWARE, PADDED>(pA, rowA, leafA, k);
+    const float b1 = sliced_step_v<NAN_AWARE, PADDED>(pB, rowB, leafB, k);
+    const float a2 = sliced_step_v<NAN_AWARE, PADDED>(pA, rowA, leafA, k);
+    const float b2 = sliced_step_v<NAN_AWARE, PADDED>(pB, rowB, leafB, k);
+    add_pair(accA, a1, a2);
+    add_pair(accB, b1, b2);
   }
 }
 
-template <bool LEAF, bool NAN_AWARE>
-__device__ __forceinline__ double walk_columns(uint32_t p, uint32_t pe, uint32_t rowaddr,
-                                               uint32_t fmask, uint32_t sh, uint32_t sbase,
-                                               const SlicedKArgs& a,
-                                               const int32_t* __restrict__ leaf_meta, int64_t i,
-                                               uint64_t& fp) {
+// One chain with the per-leaf diagnostics (caller leaf ids, fingerprint).
+template <bool NAN_AWARE, bool PADDED>
+__device__ __forceinline__ double walk_columns_leaf(uint32_t p, uint32_t pe, uint32_t rowaddr,
+                                                    const StepConsts& k, uint32_t sbase,
+                                                    const SlicedKArgs& a,
+                                                    const int32_t* __restrict__ leaf_meta,
+                                                    int64_t i, uint64_t& fp) {
+  const uint32_t leafaddr = rowaddr | k.amask;
   double acc = 0.0;
-  if (!LEAF) {
-    // two steps per exit test; a finished lane idles on its terminal self-loop
-    while (p != pe) {
-      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, 1u << (32 - sh), acc);
-      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, 1u << (32 - sh), acc);
-    }
-  } else {
-    while (p != pe) {
-      const uint32_t lp = p;
-      uint32_t yy;
-      asm("ld.shared.u32 %0, [%1];" : "=r"(yy) : "r"(lp + 4));
-      sliced_step<NAN_AWARE>(p, rowaddr, fmask, sh, 1u << (32 - sh), acc);
-      if ((yy & fmask) == fmask) {
-        const uint32_t slot_word = (lp - sbase) >> 3;
-        const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * slot_word]);
-        a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
-        fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
-      }
+  while (p != pe) {
+    const uint32_t lp = p;
+    uint32_t yy;
+    asm("ld.shared.u32 %0, [%1];" : "=r"(yy) : "r"(lp + 4));
+    const float v = sliced_step_v<NAN_AWARE, PADDED>(p, rowaddr, leafaddr, k);
+    add_pair(acc, v, 0.0f);
+    if ((yy & k.amask) == k.amask) {
+      const uint32_t slot_word = (lp - sbase) >> 3;
+      const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * slot_word]);
+      a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
+      fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
     }
   }
   return acc;
 }
 
 // Rows too wide to stage (e.g. 2000 attributes) are read from global memory through L1; this walk
-// is always NaN-aware and clamps the attribute index of leaves to stay inside the row.
+// is always NaN-aware and never reads past the row for a leaf.
 template <bool LEAF>
 __device__ __forceinline__ double walk_columns_global(uint32_t p, uint32_t pe,
                                                       const float* __restrict__ row,
-                                                      uint32_t fmask, uint32_t sh, uint32_t sbase,
+                                                      const StepConsts& k, uint32_t sbase,
                                                       const SlicedKArgs& a,
                                                       const int32_t* __restrict__ leaf_meta,
                                                       int64_t i, uint64_t& fp) {
   double acc = 0.0;
+  const char* rowb = reinterpret_cast<const char*>(row);
   while (p != pe) {
     uint32_t x, y;
     asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
-    const uint32_t f = y & fmask;
-    const bool leaf = f == fmask;
-    const float v = __ldg(&row[leaf ? 0u : f]);
-    const bool go_left = (v < __uint_as_float(x)) || ((v != v) && ((y >> (sh - 1)) & 1u));
-    const uint32_t delta = (go_left && !leaf) ? 256u : (y >> sh);
+    const uint32_t off = y & k.amask;
+    const bool leaf = off == k.amask;
+    const float v = __ldg(reinterpret_cast<const float*>(rowb + (leaf ? 0u : off)));
+    const bool go_left = (v < __uint_as_float(x)) || ((v != v) && (y & k.dlbit));
+    const uint32_t delta = (go_left && !leaf) ? 256u : __umulhi(y, k.shmul);
     if (leaf) {
       acc += (double)__uint_as_float(x);
       if (LEAF && delta) {
@@ -276,9 +300,11 @@ __device__ __forceinline__ double walk_columns_global(uint32_t p, uint32_t pe,
   return acc;
 }
 
-template <bool LEAF, bool FUSED, bool ROWS_SMEM>
-__global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
-  extern __shared__ __align__(128) unsigned char smem[];
+template <bool LEAF, bool FUSED, int ROWS>
+__global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ SlicedKArgs a) {
+  constexpr bool ROWS_SMEM = ROWS != kRowsGlobal;
+  constexpr bool PADDED = ROWS == kRowsPadded;
+  extern __shared__ __align__(1024) unsigned char smem[];
   float* s_ring = reinterpret_cast<float*>(smem + a.forest_smem);
   uint64_t* s_full = reinterpret_cast<uint64_t*>(
       smem + a.forest_smem + (ROWS_SMEM ? (size_t)kRing * a.buf_floats * sizeof(float) : 0));
@@ -288,14 +314,16 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
   const int warp = threadIdx.x >> 5;
   const int nwarps = blockDim.x >> 5;
   const uint32_t F = (uint32_t)a.img.fbits;
-  const uint32_t fmask = (1u << F) - 1u;
-  const uint32_t sh = F + 1;  // offsets (bytes) sit above the default-left bit
-  const uint32_t shmul = 1u << (32 - sh);
+  StepConsts k;
+  k.amask = ((1u << F) - 1u) << 2;
+  k.dlbit = 1u << (F + 2);
+  k.shmul = 1u << (32 - (F + 3));
   const int32_t ns = a.img.n_slices;
   const int32_t G = gridDim.x;
   const bool multipass = ns > G;
   const int64_t R = a.tile_rows;
   const int64_t ntiles = (a.n + R - 1) / R;
+  const int rs = a.row_stride;
 
   if (threadIdx.x == 0) {
     for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; }
@@ -307,25 +335,38 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
   // a6: stage tile `tile` into ring buffer b; called by one whole warp
   auto issue_tile = [&](int64_t tile, int b) {
     const int64_t r0 = tile * R;
-    const int64_t nr = (a.n - r0) < R ? (a.n - r0) : R;
-    const uint32_t bytes = (uint32_t)(nr * a.d * sizeof(float));
     float* dst = s_ring + (size_t)b * a.buf_floats;
-    const float* src = a.X + r0 * a.d;
-    if (a.x_aligned) {
+    if (PADDED) {
+      // one 2-D tensor copy: box [row_stride][R] at (0, r0); columns >= d and rows >= n are
+      // zero-filled by the TMA unit and still counted in the transaction bytes
       if (lane == 0) {
-        const uint32_t body = bytes & ~15u;
-        for (uint32_t q = body / 4; q < bytes / 4; q++) dst[q] = __ldg(&src[q]);  // <= 3 floats
         fence_proxy_async_smem();
-        mbar_expect_tx(&s_full[b], body);
-        if (body) bulk_g2s_big(dst, src, body, &s_full[b]);
+        mbar_expect_tx(&s_full[b], (uint32_t)(R * rs * sizeof(float)));
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+            " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_u32(dst)),
+            "l"(reinterpret_cast<uint64_t>(&a.tmap)), "r"(0), "r"((int32_t)r0), "r"(smem_u32(&s_full[b]))
+            : "memory");
       }
-    } else {  // misaligned X: the warp copies the tile itself
-      const uint32_t cnt = bytes / 4;
-      for (uint32_t q = lane; q < cnt; q += 32) dst[q] = __ldg(&src[q]);
-      __threadfence_block();
-      __syncwarp();
-      if (lane == 0) {
-        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_full[b])) : "memory");
+    } else {
+      const int64_t nr = (a.n - r0) < R ? (a.n - r0) : R;
+      const uint32_t bytes = (uint32_t)(nr * a.d * sizeof(float));
+      const float* src = a.X + r0 * a.d;
+      if (a.x_aligned) {
+        if (lane == 0) {
+          const uint32_t body = bytes & ~15u;
+          for (uint32_t q = body / 4; q < bytes / 4; q++) dst[q] = __ldg(&src[q]);  // <= 3 floats
+          fence_proxy_async_smem();
+          mbar_expect_tx(&s_full[b], body);
+          if (body) bulk_g2s_big(dst, src, body, &s_full[b]);
+        }
+      } else {  // misaligned X: the warp copies the tile itself
+        const uint32_t cnt = bytes / 4;
+        for (uint32_t q = lane; q < cnt; q += 32) dst[q] = __ldg(&src[q]);
+        __threadfence_block();
+        __syncwarp();
+        if (lane == 0)
+          asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_full[b])) : "memory");
       }
     }
     __syncwarp();
@@ -346,7 +387,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
         bulk_g2s_big(smem, a.img.nodes + (size_t)sl * a.img.slots_max * 64, bytes, s_forest);
       }
       if (ROWS_SMEM)
-        for (int64_t k = 0; k < kRing && k < my_tiles; k++) issue_tile(t0 + k * ts, (int)((g + k) % kRing));
+        for (int64_t q = 0; q < kRing && q < my_tiles; q++) issue_tile(t0 + q * ts, (int)((g + q) % kRing));
     }
     const uint32_t sbase = smem_u32(smem);
     const uint32_t p0 = sbase + (uint32_t)lane * 8u;
@@ -382,16 +423,16 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
         for (int r = warp; r < nr; r += 2 * nwarps) {
           const int r2 = r + nwarps;
           const bool two = r2 < nr;
-          const float* rowA = tbuf + (size_t)r * a.d;
-          const float* rowB = tbuf + (size_t)(two ? r2 : r) * a.d;
+          const float* rowA = tbuf + (size_t)r * rs;
+          const float* rowB = tbuf + (size_t)(two ? r2 : r) * rs;
           bool has_nan = false;
           for (int j = lane; j < a.d; j += 32) has_nan |= (rowA[j] != rowA[j]) | (rowB[j] != rowB[j]);
           double accA, accB;
           const uint32_t pB = two ? p0 : pe;
           if (__any_sync(0xffffffffu, has_nan))
-            walk_columns2<true>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), fmask, sh, shmul, accA, accB);
+            walk_columns2<true, PADDED>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
           else
-            walk_columns2<false>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), fmask, sh, shmul, accA, accB);
+            walk_columns2<false, PADDED>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
           finish_row(accA, 0, r0 + r);
           if (two) finish_row(accB, 0, r0 + r2);
         }
@@ -401,18 +442,16 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const SlicedKArgs a) {
           uint64_t fp = 0;
           double acc;
           if (ROWS_SMEM) {
-            const float* row = tbuf + (size_t)r * a.d;
+            const float* row = tbuf + (size_t)r * rs;
             bool has_nan = false;
             for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
-            const uint32_t rowaddr = smem_u32(row);
             if (__any_sync(0xffffffffu, has_nan))
-              acc = walk_columns<LEAF, true>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
+              acc = walk_columns_leaf<true, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
             else
-              acc = walk_columns<LEAF, false>(p0, pe, rowaddr, fmask, sh, sbase, a, leaf_meta, i, fp);
+              acc = walk_columns_leaf<false, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
           } else {
-            // wide rows stay in global memory (L1-cached); the leaf attribute read is clamped
             const float* row = a.X + i * a.d;
-            acc = walk_columns_global<LEAF>(p0, pe, row, fmask, sh, sbase, a, leaf_meta, i, fp);
+            acc = walk_columns_global<LEAF>(p0, pe, row, k, sbase, a, leaf_meta, i, fp);
           }
           finish_row(acc, fp, i);
         }
@@ -490,7 +529,7 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
   return (int)cudaGetLastError();
 }
 
-template <bool L, bool F, bool R>
+template <bool L, bool F, int R>
 static cudaError_t sliced_one(const SlicedKArgs& a, const SlicedPlan& p, cudaStream_t st) {
   auto kern = k_sliced<L, F, R>;
   // raise the dynamic shared-memory limit once per process and device (not per launch)
@@ -506,6 +545,34 @@ static cudaError_t sliced_one(const SlicedKArgs& a, const SlicedPlan& p, cudaStr
   return cudaGetLastError();
 }
 
+template <bool L, bool F>
+static cudaError_t sliced_rows(const SlicedKArgs& a, const SlicedPlan& p, cudaStream_t st) {
+  if (p.rows == kRowsPadded) return sliced_one<L, F, kRowsPadded>(a, p, st);
+  if (p.rows == kRowsDense) return sliced_one<L, F, kRowsDense>(a, p, st);
+  return sliced_one<L, F, kRowsGlobal>(a, p, st);
+}
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda needed)
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_tiled_fn() {
+  static EncodeTiledFn fn = [] {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (EncodeTiledFn) nullptr;
+    return reinterpret_cast<EncodeTiledFn>(ptr);
+  }();
+  return fn;
+}
+
+bool padded_rows_possible(const float* X, int32_t d) {
+  return ((reinterpret_cast<uintptr_t>(X) & 15) == 0) && (d % 4 == 0) && encode_tiled_fn() != nullptr;
+}
+
 int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                   int32_t d, const OutArgs& o, bool fused, void* stream) {
   SlicedKArgs a{};
@@ -517,19 +584,27 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
   a.cps = plan.cps;
   a.forest_smem = plan.forest_smem;
   a.buf_floats = plan.buf_floats;
+  a.row_stride = plan.row_stride;
   a.x_aligned = ((reinterpret_cast<uintptr_t>(X) & 15) == 0) &&
                 (((int64_t)plan.tile_rows * d * 4) % 16 == 0);
   a.o = o;
+  if (plan.rows == kRowsPadded) {
+    EncodeTiledFn enc = encode_tiled_fn();
+    if (!enc) return (int)cudaErrorNotSupported;
+    const cuuint64_t gdim[2] = {(cuuint64_t)d, (cuuint64_t)n};
+    const cuuint64_t gstride[1] = {(cuuint64_t)d * 4};
+    const cuuint32_t box[2] = {(cuuint32_t)plan.row_stride, (cuuint32_t)plan.tile_rows};
+    const cuuint32_t estride[2] = {1, 1};
+    CUresult r = enc(&a.tmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(X), gdim, gstride,
+                     box, estride, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return (int)cudaErrorInvalidValue;
+  }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
   cudaError_t e;
-  if (plan.rows_in_smem) {
-    if (leaf) e = fused ? sliced_one<true, true, true>(a, plan, st) : sliced_one<true, false, true>(a, plan, st);
-    else e = fused ? sliced_one<false, true, true>(a, plan, st) : sliced_one<false, false, true>(a, plan, st);
-  } else {
-    if (leaf) e = fused ? sliced_one<true, true, false>(a, plan, st) : sliced_one<true, false, false>(a, plan, st);
-    else e = fused ? sliced_one<false, true, false>(a, plan, st) : sliced_one<false, false, false>(a, plan, st);
-  }
+  if (leaf) e = fused ? sliced_rows<true, true>(a, plan, st) : sliced_rows<true, false>(a, plan, st);
+  else e = fused ? sliced_rows<false, true>(a, plan, st) : sliced_rows<false, false>(a, plan, st);
   return (int)e;
 }
 

@@ -74,21 +74,31 @@ constexpr int32_t kSlicedRing = 3;          // sample-tile ring depth of k_slice
 constexpr int32_t kSlicedTileRows = 64;     // rows per tile (two per warp of a 1024-thread CTA)
 constexpr int32_t kSlicedBarrierBytes = 128;
 
-// Floats per ring buffer: a tile of rows plus the pad a leaf's all-ones attribute read touches.
-inline int32_t sliced_buf_floats(int32_t d, int32_t fbits) {
-  int64_t f = (int64_t)kSlicedTileRows * d + (1 << fbits);
-  return (int32_t)((f + 3) & ~3LL);
+// PADDED staging: rows at a stride that is a multiple of 2^fbits floats (>= d, >= 4), so that row
+// bases are aligned to the attribute byte-offset field and a leaf's all-ones attribute stays
+// inside the row.  DENSE staging: rows at stride d plus a tail pad for the last row's leaf read.
+inline int32_t sliced_row_stride(int32_t d, int32_t fbits, bool padded) {
+  if (!padded) return d;
+  int32_t q = 1 << fbits;
+  if (q < 4) q = 4;
+  return ((d + q - 1) / q) * q;
+}
+inline int32_t sliced_buf_floats(int32_t d, int32_t fbits, bool padded) {
+  if (padded) return kSlicedTileRows * sliced_row_stride(d, fbits, true);
+  const int64_t f = (int64_t)kSlicedTileRows * d + (1 << fbits);
+  return (int32_t)((f + 255) & ~255LL);  // keep every buffer 1 KB aligned
 }
 // Shared memory of the sample-tile ring, or -1 when rows are too wide to stage (> 64 KB).
-inline int64_t sliced_ring_bytes(int32_t d, int32_t fbits) {
-  int64_t b = (int64_t)kSlicedRing * sliced_buf_floats(d, fbits) * 4;
+inline int64_t sliced_ring_bytes(int32_t d, int32_t fbits, bool padded) {
+  int64_t b = (int64_t)kSlicedRing * sliced_buf_floats(d, fbits, padded) * 4;
   return b <= 64 * 1024 ? b : -1;
 }
+bool padded_rows_possible(const float* X, int32_t d);  // kernels.cu
 
 struct SlicedPlan {
   int32_t grid = 0, block = 1024, tile_rows = 0, cps = 1;
-  int32_t smem_bytes = 0, forest_smem = 0, buf_floats = 0;
-  bool rows_in_smem = true;
+  int32_t smem_bytes = 0, forest_smem = 0, buf_floats = 0, row_stride = 0;
+  int32_t rows = 0;  // 0 global, 1 dense, 2 padded (kernels.cu kRows*)
 };
 int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                   bool fused, int32_t num_sms, void* stream);

@@ -188,8 +188,8 @@ def test_product_tokens_simhash_equal_oracle_on_generated_forest():
 def decode_sliced(img, X, n_trees, n_classes):
     """Walk the exported SLICED image on the host (test-side decoder, independent of the
     product's kernels): returns leaf[n, T] (caller node ids) and per-class fp64 sums.
-    Node words: internal y = off_bytes << (F+1) | default_left << F | attribute (left child next);
-    leaf y = next_root_bytes << (F+1) | (2^F - 1); slot = 256 bytes."""
+    Node words: internal y = off_bytes << (F+3) | default_left << (F+2) | attribute << 2 (left
+    child next); leaf y = next_root_bytes << (F+3) | (2^F - 1) << 2; slot = 256 bytes."""
     n = X.shape[0]
     F = img["feature_bits"]
     fmask = (1 << F) - 1
@@ -200,21 +200,21 @@ def decode_sliced(img, X, n_trees, n_classes):
         for lane in range(32):
             end = img["col_len"][s, lane]
             x_t, y_t = img["nodes"][s, end, lane]
-            assert y_t == fmask and x_t == 0, "terminal self-loop closes the column"
+            assert y_t == fmask << 2 and x_t == 0, "terminal self-loop closes the column"
             for i in range(n):
                 k = 0
                 while k < end:
                     x, y = (int(v) for v in img["nodes"][s, k, lane])
-                    if (y & fmask) == fmask:
+                    if ((y >> 2) & fmask) == fmask:
                         t, node = img["leaf_meta"][s, k, lane]
                         leaf[i, t] = node
                         sums[i, c] += float(np.uint32(x).view(np.float32))
-                        k += (y >> (F + 1)) // 256
+                        k += (y >> (F + 3)) // 256
                     else:
                         thr = float(np.uint32(x).view(np.float32))
-                        v = X[i, y & fmask]
-                        go_left = bool((y >> F) & 1) if np.isnan(v) else bool(v < thr)
-                        k += 1 if go_left else (y >> (F + 1)) // 256
+                        v = X[i, (y >> 2) & fmask]
+                        go_left = bool((y >> (F + 2)) & 1) if np.isnan(v) else bool(v < thr)
+                        k += 1 if go_left else (y >> (F + 3)) // 256
                 assert k == end
     return leaf, sums
 

@@ -204,3 +204,26 @@ def test_full_size_c2_sampled_rows_in_bench_configuration():
     ref = oracle.predict(f, X, rows=idx)
     res = dict(out=out.cpu().numpy()[idx], cls=cls.cpu().numpy()[idx])
     _check(res, ref, f["agg"], False, want_leaf=False)
+
+
+def test_single_leaf_trees_and_stumps():
+    """Trees whose root is a leaf (encoded as a 3-node stump in the sliced image) mixed with
+    ordinary trees: consecutive nonzero leaves must still be summed exactly."""
+    from test_oracle_pins import random_forest
+    rng = np.random.default_rng(8)
+    base = random_forest(rng, 40, 4, 6)
+    nn = len(base["feature"])
+    k = 25
+    f = {kk: np.concatenate([base[kk], v]).astype(base[kk].dtype) for kk, v in dict(
+        feature=np.full(k, -1), threshold=np.zeros(k), left=np.full(k, -1), right=np.full(k, -1),
+        leaf_value=(rng.integers(-256, 257, size=k) / 256.0),
+        default_left=np.zeros(k)).items()}
+    order = rng.permutation(40 + k)
+    roots = np.concatenate([base["root"], np.arange(nn, nn + k, dtype=np.int32)])[order]
+    f["root"] = roots.astype(np.int32)
+    f["tree_class"] = np.zeros(len(roots), np.int32)
+    X = rng.normal(size=(2049, 6)).astype(np.float32)
+    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
+    F = T.Forest(f, n_features=6, n_classes=1, agg=oracle.AGG_SUM, device=0)
+    for s in STRATS:
+        _check(_gpu_run(F, X, s), ref, oracle.AGG_SUM, True)

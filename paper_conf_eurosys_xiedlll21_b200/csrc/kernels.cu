@@ -16,7 +16,9 @@
 //  k_finalize — fixed-order fp64 sum of parts per class, base / average / argmax, RN to fp32.
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <algorithm>
 #include <atomic>
+#include <cstdlib>
 #include <cstdint>
 
 #include "kernels.hpp"
@@ -151,6 +153,104 @@ __global__ void __launch_bounds__(256) k_direct(const DirectKArgs a) {
     else if (!vote) a.o.raw[i * C + cls] = acc;
     if (LEAF && a.o.out_fp) atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]),
                                      (unsigned long long)fp);
+  }
+}
+
+// Direct strategy with staged rows: a CTA copies a tile of BLOCK rows into shared memory (odd
+// row stride, so lanes reading different rows at random attributes spread over the banks), then
+// each thread walks every tree for its row.  The tree loop is warp-uniform: the lanes of a warp
+// stay in the same tree, so with hot-child-next ordering their node loads fall on few
+// L1 lines ("nodes that tend to be accessed at the same time ... contiguous").
+template <bool LEAF, bool FUSED, int BLOCK, bool LOCKSTEP>
+__global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int32_t rs) {
+  extern __shared__ __align__(16) float s_rows[];
+  const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(a.img.nodes);
+  const int fbits = a.img.fbits;
+  const uint32_t fmask = (1u << fbits) - 1u;
+  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const int32_t C = a.o.n_classes;
+  const bool vote = a.o.agg == TAHOE_AGG_VOTE;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t ntiles = (a.n + BLOCK - 1) / BLOCK;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * BLOCK;
+    const int nr = (int)((a.n - r0) < BLOCK ? (a.n - r0) : BLOCK);
+    __syncthreads();
+    for (int r = warp; r < nr; r += BLOCK / 32) {
+      const float* src = a.X + (r0 + r) * a.d;
+      for (int c = lane; c < a.d; c += 32) s_rows[r * rs + c] = __ldg(&src[c]);
+    }
+    __syncthreads();
+    const bool active = threadIdx.x < nr;
+    const int64_t i = r0 + threadIdx.x;
+    const float* row = s_rows + threadIdx.x * rs;
+    double acc = 0.0;
+    uint64_t fp = 0;
+    int32_t cls = __ldg(&a.img.cls[0]);
+    if (LOCKSTEP) {
+      for (int32_t t = 0; t < a.img.n_slots; t++) {
+        uint32_t k = (uint32_t)__ldg(&a.img.root[t]);
+        if (!FUSED) {
+          const int32_t c2 = __ldg(&a.img.cls[t]);
+          if (c2 != cls) {
+            if (active && !vote) a.o.raw[i * C + cls] = acc;
+            acc = 0.0;
+            cls = c2;
+          }
+        }
+        if (!active) continue;
+        uint2 nd = __ldg(&nodes[k]);
+        while ((int32_t)nd.y >= 0) {
+          k += step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask);
+          nd = __ldg(&nodes[k]);
+        }
+        const float v = __uint_as_float(nd.x);
+        if (vote) a.o.raw[i * C + (int32_t)v] += 1.0;
+        else acc += (double)v;
+        if (LEAF) {
+          const int32_t tree = __ldg(&a.img.tree_orig[t]);
+          const uint32_t leaf = nd.y & 0x7fffffffu;
+          a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
+          fp += mix64(((uint64_t)(uint32_t)tree << 32) | leaf);
+        }
+      }
+    } else if (active) {
+      // free-running: each thread moves to its next tree as soon as it reaches a leaf
+      int32_t t = 0;
+      uint32_t k = (uint32_t)__ldg(&a.img.root[0]);
+      for (;;) {
+        const uint2 nd = __ldg(&nodes[k]);
+        if ((int32_t)nd.y < 0) {
+          const float v = __uint_as_float(nd.x);
+          if (vote) a.o.raw[i * C + (int32_t)v] += 1.0;
+          else acc += (double)v;
+          if (LEAF) {
+            const int32_t tree = __ldg(&a.img.tree_orig[t]);
+            const uint32_t leaf = nd.y & 0x7fffffffu;
+            a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
+            fp += mix64(((uint64_t)(uint32_t)tree << 32) | leaf);
+          }
+          if (++t == a.img.n_slots) break;
+          k = (uint32_t)__ldg(&a.img.root[t]);
+          if (!FUSED) {
+            const int32_t c2 = __ldg(&a.img.cls[t]);
+            if (c2 != cls) {
+              if (!vote) a.o.raw[i * C + cls] = acc;
+              acc = 0.0;
+              cls = c2;
+            }
+          }
+        } else {
+          k += step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask);
+        }
+      }
+    }
+    if (active) {
+      if (FUSED) write_scalar(a.o, i, acc);
+      else if (!vote) a.o.raw[i * C + cls] = acc;
+      if (LEAF && a.o.out_fp)
+        atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
+    }
   }
 }
 
@@ -512,13 +612,52 @@ static int grid_for(int64_t n, int block, int num_sms, int per_sm) {
   return (int)(g < 1 ? 1 : g);
 }
 
+template <bool L, bool F, int B, bool LS>
+static cudaError_t direct_tiled_one(const DirectKArgs& a, int32_t rs, int32_t num_sms,
+                                    cudaStream_t st) {
+  auto kern = k_direct_tiled<L, F, B, LS>;
+  const int smem = B * rs * 4;
+  static std::atomic<int> configured[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64 && configured[dev].load() < smem) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+    if (e != cudaSuccess) return e;
+    configured[dev].store(kMaxSmemOptin);
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, B, smem);
+  if (per_sm < 1) per_sm = 1;
+  const int64_t ntiles = (a.n + B - 1) / B;
+  const int grid = (int)std::min<int64_t>(ntiles, (int64_t)num_sms * per_sm);
+  kern<<<grid, B, smem, st>>>(a, rs);
+  return cudaGetLastError();
+}
+
 int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                   bool fused, int32_t num_sms, void* stream) {
   DirectKArgs a{img, X, n, d, o};
-  const int block = 256;
-  const int grid = grid_for(n, block, num_sms, 8);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
+  // 0 = rows read from global memory; 1 = staged rows, warp-lockstep over trees;
+  // 2 = staged rows, free-running over trees
+  const char* env = std::getenv("TAHOE_DIRECT_VARIANT");
+  int variant = env ? std::atoi(env) : 0;
+  if (d > 256) variant = 0;  // 128 staged rows must fit shared memory
+  if (variant == 1 || variant == 2) {
+    const int32_t rs = d | 1;  // odd stride: lanes on different rows spread over the banks
+    cudaError_t e;
+    if (variant == 1) {
+      if (leaf) e = fused ? direct_tiled_one<true, true, 128, true>(a, rs, num_sms, st) : direct_tiled_one<true, false, 128, true>(a, rs, num_sms, st);
+      else e = fused ? direct_tiled_one<false, true, 128, true>(a, rs, num_sms, st) : direct_tiled_one<false, false, 128, true>(a, rs, num_sms, st);
+    } else {
+      if (leaf) e = fused ? direct_tiled_one<true, true, 128, false>(a, rs, num_sms, st) : direct_tiled_one<true, false, 128, false>(a, rs, num_sms, st);
+      else e = fused ? direct_tiled_one<false, true, 128, false>(a, rs, num_sms, st) : direct_tiled_one<false, false, 128, false>(a, rs, num_sms, st);
+    }
+    return (int)e;
+  }
+  const int block = 256;
+  const int grid = grid_for(n, block, num_sms, 8);
   if (leaf) {
     if (fused) k_direct<true, true><<<grid, block, 0, st>>>(a);
     else k_direct<true, false><<<grid, block, 0, st>>>(a);

@@ -178,6 +178,10 @@ int32_t tahoe_forest_n_trees(const tahoe_forest* f);
 tahoe_status tahoe_forest_stats(const tahoe_forest* f, char* buf, int64_t buf_len);
 /* Strategy the cost model picks for a batch of n rows of width d (Algorithm 1 lines 8-13). */
 int32_t tahoe_select_strategy(const tahoe_forest* f, int64_t n, int32_t d);
+/* The cost model's predicted time (microseconds) of `strategy` for a batch of n rows; +inf when the
+ * strategy is unavailable for this forest, -1 on NULL.  Constants: costmodel_b200.json next to the
+ * library (fitted by scripts/fit_costmodel.py) or $TAHOE_COSTMODEL. */
+double tahoe_predict_cost_us(const tahoe_forest* f, int32_t strategy, int64_t n);
 void tahoe_forest_free(tahoe_forest* f);                  /* synchronise in-flight work first  */
 const char* tahoe_last_error(void);                       /* thread-local, never NULL          */
 

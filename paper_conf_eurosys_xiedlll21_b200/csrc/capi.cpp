@@ -4,6 +4,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <climits>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -161,12 +162,21 @@ static tahoe_status init_handle(tahoe_forest* f, int32_t device) {
   return TAHOE_OK;
 }
 
-static PlanStats plan_stats(const tahoe_forest* f) {
+static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   PlanStats st;
+  if (d < 0) d = f->host.n_features;
+  st.wide_rows = d > 256;
+  if (f->sl.valid) {
+    const int64_t room = (int64_t)f->max_smem - (((f->sl.slots_max * 256) + 1023) & ~1023) - kSlicedBarrierBytes;
+    const int64_t ring = std::min<int64_t>(sliced_ring_bytes(d, f->sl.fbits, false) < 0 ? INT64_MAX : sliced_ring_bytes(d, f->sl.fbits, false),
+                                           sliced_ring_bytes(d, f->sl.fbits, true) < 0 ? INT64_MAX : sliced_ring_bytes(d, f->sl.fbits, true));
+    st.rows_global = ring > room;
+  }
   for (double v : f->host.exp_reads) st.V += v;
   st.sliced_ok = f->sl.valid;
-  st.sliced_eff = f->sl.eff;
+  st.sliced_eff = f->sl.eff_sim;
   st.n_slices = f->sl.n_slices;
+  st.num_sms = f->num_sms;
   return st;
 }
 
@@ -177,7 +187,7 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
   }
   if (forced == TAHOE_STRATEGY_DIRECT) return TAHOE_STRATEGY_DIRECT;
   if (forced == TAHOE_STRATEGY_SLICED) return f->sl.valid ? TAHOE_STRATEGY_SLICED : -2;
-  return select_strategy(plan_stats(f), n, d, f->host.agg);
+  return select_strategy(plan_stats(f, d), n, d, f->host.agg);
 }
 
 static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int32_t d) {
@@ -354,7 +364,15 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_layout(
   if (o.m_chunks > o.l_hash) return fail(TAHOE_E_INVAL, "m_chunks > l_hash");
   Forest& F = f->host;
   F.opts = o;
-  if (n_calib > 0) calibrate(F, X_calib_host, n_calib, d);
+  if (n_calib > 0) {
+    calibrate(F, X_calib_host, n_calib, d);
+    // keep an evenly spaced subsample of the calibration rows for the lockstep simulation
+    const int64_t m = std::min<int64_t>(n_calib, 512);
+    F.dsim = d;
+    F.Xsim.resize((size_t)m * d);
+    for (int64_t r = 0; r < m; r++)
+      std::memcpy(&F.Xsim[(size_t)r * d], X_calib_host + (r * n_calib / m) * d, (size_t)d * 4);
+  }
   reorder_nodes(F, o.node_reorder != 0);
   order_trees(F);
   return encode_and_upload(f);
@@ -522,6 +540,12 @@ __attribute__((visibility("default"))) int32_t tahoe_select_strategy(const tahoe
   return choose(f, n, d, -1);
 }
 
+__attribute__((visibility("default"))) double tahoe_predict_cost_us(const tahoe_forest* f,
+                                                                   int32_t strategy, int64_t n) {
+  if (!f) return -1.0;
+  return predict_us(plan_stats(f), strategy, n);
+}
+
 __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tahoe_forest* f,
                                                                        char* buf, int64_t len) {
   TAHOE_GUARD_BEGIN
@@ -549,7 +573,9 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"sliced_why\":\"" << f->sl.why_invalid << "\""
      << ",\"n_slices\":" << f->sl.n_slices << ",\"slots_max\":" << f->sl.slots_max
      << ",\"slot_budget\":" << f->slot_budget << ",\"sliced_bytes\":" << f->sl.bytes()
-     << ",\"lockstep_eff\":" << f->sl.eff << ",\"trees_per_lane\":" << f->sl.trees_per_lane
+     << ",\"lockstep_eff\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim
+     << ",\"trees_per_lane\":" << f->sl.trees_per_lane << ",\"cost_fitted\":"
+     << (cost_params().fitted ? "true" : "false")
      << ",\"num_sms\":" << f->num_sms << ",\"max_smem\":" << f->max_smem << "}";
   std::string s = js.str();
   if ((int64_t)s.size() + 1 > len) return fail(TAHOE_E_INVAL, "buffer too small");

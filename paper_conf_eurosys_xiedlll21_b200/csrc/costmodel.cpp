@@ -1,37 +1,98 @@
 // costmodel.cpp — per-batch strategy choice (Algorithm 1 lines 8-13; Eq. 1-7
 // reconstructed in SURVEY Appendix A), re-targeted to the two B200 strategies.
 //
-// Per-sample time (Eq. 1: T = T_SMEM + T_GMEM + T_B_REDU + T_G_REDU) becomes
-//   direct : V * c_gmem_visit                                   (T_GMEM: nodes + attributes from
-//                                                                 L1/L2, no reduction)
-//   sliced : V * c_smem_visit / eff  + P * (c_reduce + 4 d / BW) (T_SMEM of a lockstep warp at
-//                                                                 packing efficiency eff, plus one
-//                                                                 warp reduction and one row read
-//                                                                 per slice P: T_B_REDU + T_G_REDU)
-// V = expected node reads per sample (calibrated E[path]+1 summed over trees, reading Z16).
-// Constants are in units of one conflict-free shared-memory node visit; they can be overridden by
-// TAHOE_COST_GMEM / TAHOE_COST_REDUCE / TAHOE_COST_ROWBYTE (fitted on the chip).
+// Eq. 1 (T = T_SMEM + T_GMEM + T_B_REDU + T_G_REDU) becomes, per batch of n rows:
+//   sliced : T = a_s + b_s * U_s * (rows in global memory ? g_s : 1),
+//            U_s = ceil(tiles / cps) * 64 * V / (slices * eff)
+//            the node reads of the busiest CTA (T_SMEM at the simulated lockstep efficiency eff);
+//            a_s absorbs launch, slice staging and the fixed-order slice reduction (T_G_REDU);
+//   direct : T = a_d + (d > 256 ? g_d : 1) * max(l_d * V, b_d * V * n / SMs)
+//            one thread per sample: latency-bound below a full GPU of threads (l_d per visit),
+//            L1/L2-throughput-bound above it (T_GMEM).
+// V = expected node reads per sample (calibrated E[path] + 1 leaf read, summed over trees,
+// reading Z16).  The constants are fitted on the chip by scripts/fit_costmodel.py and read from
+// costmodel_b200.json next to libtahoe.so (or $TAHOE_COSTMODEL); defaults are round-1 B200
+// measurements.
+#include <dlfcn.h>
+
+#include <cmath>
+#include <cstdio>
 #include <cstdlib>
+#include <cstring>
+#include <string>
 
 #include "internal.hpp"
 
 namespace tahoe {
 
-static double env_or(const char* name, double dflt) {
-  const char* v = std::getenv(name);
-  return (v && *v) ? std::atof(v) : dflt;
+static bool read_key(const std::string& js, const char* key, double* v) {
+  const std::string k = std::string("\"") + key + "\"";
+  size_t p = js.find(k);
+  if (p == std::string::npos) return false;
+  p = js.find(':', p);
+  if (p == std::string::npos) return false;
+  return std::sscanf(js.c_str() + p + 1, "%lf", v) == 1;
+}
+
+static std::string lib_dir() {
+  Dl_info info;
+  if (dladdr(reinterpret_cast<void*>(&cost_params), &info) && info.dli_fname) {
+    std::string s(info.dli_fname);
+    size_t k = s.rfind('/');
+    if (k != std::string::npos) return s.substr(0, k);
+  }
+  return ".";
+}
+
+const CostParams& cost_params() {
+  static CostParams P = [] {
+    CostParams c;
+    const char* env = std::getenv("TAHOE_COSTMODEL");
+    std::string path = env && *env ? std::string(env) : lib_dir() + "/costmodel_b200.json";
+    FILE* fp = std::fopen(path.c_str(), "rb");
+    if (!fp) return c;
+    std::string js;
+    char buf[4096];
+    size_t k;
+    while ((k = std::fread(buf, 1, sizeof(buf), fp)) > 0) js.append(buf, k);
+    std::fclose(fp);
+    double v;
+    bool all = true;
+    all &= read_key(js, "a_s", &v); if (all) c.a_s = v;
+    all &= read_key(js, "b_s", &v); if (all) c.b_s = v;
+    all &= read_key(js, "a_d", &v); if (all) c.a_d = v;
+    all &= read_key(js, "l_d", &v); if (all) c.l_d = v;
+    all &= read_key(js, "b_d", &v); if (all) c.b_d = v;
+    if (read_key(js, "g_s", &v)) c.g_s = v;
+    if (read_key(js, "g_d", &v)) c.g_d = v;
+    c.fitted = all;
+    return c;
+  }();
+  return P;
+}
+
+double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
+  const CostParams& c = cost_params();
+  if (strategy == TAHOE_STRATEGY_SLICED) {
+    if (!st.sliced_ok || st.n_slices < 1) return INFINITY;
+    const int64_t tiles = (n + 63) / 64;
+    const int64_t cps = st.n_slices <= st.num_sms ? std::max(1, st.num_sms / st.n_slices) : 1;
+    const double passes = st.n_slices <= st.num_sms ? 1.0 : std::ceil((double)st.n_slices / st.num_sms);
+    const double eff = st.sliced_eff > 0.05 ? st.sliced_eff : 0.05;
+    const double U = (double)((tiles + cps - 1) / cps) * 64.0 * st.V / (st.n_slices * eff) * passes;
+    return c.a_s + c.b_s * U * (st.rows_global ? c.g_s : 1.0);
+  }
+  const double sms = st.num_sms > 0 ? st.num_sms : 148;
+  const double g = st.wide_rows ? c.g_d : 1.0;
+  return c.a_d + g * std::max(c.l_d * st.V, c.b_d * st.V * (double)n / sms);
 }
 
 int32_t select_strategy(const PlanStats& st, int64_t n, int32_t d, int32_t agg) {
+  (void)d;
   if (agg == TAHOE_AGG_VOTE || !st.sliced_ok) return TAHOE_STRATEGY_DIRECT;
-  const double c_gmem = env_or("TAHOE_COST_GMEM", 4.0);
-  const double c_reduce = env_or("TAHOE_COST_REDUCE", 24.0);
-  const double c_rowbyte = env_or("TAHOE_COST_ROWBYTE", 0.02);
-  const double eff = st.sliced_eff > 0.05 ? st.sliced_eff : 0.05;
-  const double t_direct = st.V * c_gmem;
-  const double t_sliced = st.V / eff + st.n_slices * (c_reduce + c_rowbyte * 4.0 * d);
-  (void)n;
-  return t_sliced <= t_direct ? TAHOE_STRATEGY_SLICED : TAHOE_STRATEGY_DIRECT;
+  return predict_us(st, TAHOE_STRATEGY_SLICED, n) <= predict_us(st, TAHOE_STRATEGY_DIRECT, n)
+             ? TAHOE_STRATEGY_SLICED
+             : TAHOE_STRATEGY_DIRECT;
 }
 
 }  // namespace tahoe

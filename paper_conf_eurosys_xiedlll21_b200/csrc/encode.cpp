@@ -181,6 +181,42 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
     padded += 32.0 * P.max_work;
   }
   S.eff = padded > 0 ? work / padded : 0;
+  // Simulated lockstep efficiency of k_sliced (two rows per warp, two steps per exit test) on the
+  // kept calibration rows: useful node reads / lane-steps issued.  Falls back to 0.75 x expected.
+  S.eff_sim = S.eff * 0.75;
+  if (!F.Xsim.empty()) {
+    const int64_t m = (int64_t)F.Xsim.size() / F.dsim;
+    std::vector<int32_t> reads((size_t)m * F.n_trees);
+    for (int64_t r = 0; r < m; r++) {
+      const float* x = &F.Xsim[(size_t)r * F.dsim];
+      for (int32_t t = 0; t < F.n_trees; t++) {
+        int32_t k = F.node_base[t], c = 1;
+        while (F.feat[k] >= 0) {
+          const float v = x[F.feat[k]];
+          const bool left = std::isnan(v) ? F.dl[k] != 0 : v < F.thr[k];
+          k = left ? F.lc[k] : F.rc[k];
+          c++;
+        }
+        reads[(size_t)r * F.n_trees + t] = (F.tree_size(t) == 1) ? 2 : c;
+      }
+    }
+    double useful = 0, issued = 0;
+    std::vector<double> W(32);
+    for (auto& P : packs) {
+      for (int64_t r = 0; r + 1 < m; r += 2) {
+        double mx = 0;
+        for (int64_t q = r; q < r + 2; q++)
+          for (int32_t l = 0; l < 32; l++) {
+            double w = 0;
+            for (int32_t t : P.lanes[l]) w += reads[(size_t)q * F.n_trees + t];
+            useful += w;
+            mx = std::max(mx, w);
+          }
+        issued += 64.0 * 2.0 * std::ceil(mx / 2.0);
+      }
+    }
+    if (issued > 0) S.eff_sim = useful / issued;
+  }
   S.trees_per_lane = (double)F.n_trees / (32.0 * std::max(1, S.n_slices));
   // Sliced node words (kernels.hpp "sliced encoding"): left child first, right child at +off,
   // leaves carry the all-ones attribute field and the delta to the lane's next tree root; one

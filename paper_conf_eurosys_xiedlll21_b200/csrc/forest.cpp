@@ -151,6 +151,8 @@ Forest make_shard(const Forest& F, int32_t rank, int32_t world) {
   S.calibrated = F.calibrated;
   S.n_cal = F.n_cal;
   S.opts = F.opts;
+  S.Xsim = F.Xsim;
+  S.dsim = F.dsim;
   S.node_base.assign(1, 0);
   std::vector<int32_t> newidx((size_t)F.n_trees, -1);
   for (int32_t t = 0; t < F.n_trees; t++) {

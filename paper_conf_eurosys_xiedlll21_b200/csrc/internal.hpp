@@ -43,6 +43,8 @@ struct Forest {
   std::vector<uint8_t> hot_left;    // 1 = left child is the hot child
   std::vector<double> exp_reads;    // per tree: expected nodes read per sample (incl. leaf)
   std::vector<int32_t> order;       // tree order (class-major, similarity order within class)
+  std::vector<float> Xsim;          // <= 512 calibration rows kept to simulate lockstep efficiency
+  int32_t dsim = 0;
   tahoe_layout_opts opts{};
 
   int32_t n_out() const { return (agg == TAHOE_AGG_CLASS_SUM || agg == TAHOE_AGG_VOTE) ? n_classes : 1; }
@@ -83,6 +85,7 @@ struct SlicedImage {
   std::vector<int32_t> leaf_meta;                // [ns*slots_max*32*2] {tree, node}
   std::vector<int32_t> class_ptr, class_parts;   // class -> slices (CSR)
   double eff = 0.0;                              // est. lockstep efficiency (mean/max column)
+  double eff_sim = 0.0;                          // simulated 2-chain lockstep efficiency
   double trees_per_lane = 0.0;
   int64_t bytes() const { return (int64_t)nodes.size() * 4; }
 };
@@ -101,11 +104,25 @@ tahoe_status encode_sliced(const Forest& F, int32_t slot_budget, SlicedImage& S)
 // Cost model (costmodel.cpp) — Algorithm 1 lines 8-13 re-targeted.
 struct PlanStats {
   double V = 0;            // expected nodes read per sample (sum over trees)
-  double sliced_eff = 0;   // lockstep efficiency of the sliced packing
+  double sliced_eff = 0;   // simulated lockstep efficiency of the sliced packing
   int32_t n_slices = 0;
+  int32_t num_sms = 148;
   bool sliced_ok = false;
+  bool rows_global = false;  // sliced rows too wide to stage in shared memory
+  bool wide_rows = false;    // d > 256: direct reads attributes from rows far apart in memory
 };
+// Fitted per-platform constants (costmodel_b200.json, scripts/fit_costmodel.py), microseconds.
+struct CostParams {
+  double a_s = 22.3, b_s = 9.5e-5;           // sliced: launch + slice staging; per work unit
+  double g_s = 4.0;                          // sliced: slowdown when rows stay in global memory
+  double a_d = 11.8, l_d = 0.34, b_d = 6.3e-4; // direct: launch; per-visit latency; per unit
+  double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
+  bool fitted = false;
+};
+const CostParams& cost_params();
+double predict_us(const PlanStats& st, int32_t strategy, int64_t n);
 int32_t select_strategy(const PlanStats& st, int64_t n, int32_t d, int32_t agg);
+PlanStats plan_stats_for(const struct ::tahoe_forest* f, int32_t d);
 
 }  // namespace tahoe
 

@@ -48,7 +48,7 @@ class PredictOpts(ctypes.Structure):
 SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_predict_ex",
            "tahoe_predict_host", "tahoe_forest_shard", "tahoe_predict_partial", "tahoe_finalize",
            "tahoe_forest_n_outputs", "tahoe_forest_n_trees", "tahoe_forest_stats",
-           "tahoe_select_strategy", "tahoe_forest_free", "tahoe_last_error",
+           "tahoe_select_strategy", "tahoe_predict_cost_us", "tahoe_forest_free", "tahoe_last_error",
            "tahoe_forest_layout_info", "tahoe_tree_tokens", "tahoe_tree_simhash", "tahoe_simhash",
            "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced")
 
@@ -83,6 +83,7 @@ def load(build_if_missing: bool = True):
         "tahoe_forest_n_trees": (i32, [P]),
         "tahoe_forest_stats": (st, [P, P, i64]),
         "tahoe_select_strategy": (i32, [P, i64, i32]),
+        "tahoe_predict_cost_us": (ctypes.c_double, [P, i32, i64]),
         "tahoe_forest_free": (None, [P]),
         "tahoe_last_error": (ctypes.c_char_p, []),
         "tahoe_forest_layout_info": (st, [P, P, P, P, P]),
@@ -210,6 +211,10 @@ def tahoe_select_strategy(h, n: int, d: int) -> int:
     return int(load().tahoe_select_strategy(h, n, d))
 
 
+def tahoe_predict_cost_us(h, strategy: int, n: int) -> float:
+    return float(load().tahoe_predict_cost_us(h, strategy, n))
+
+
 def tahoe_forest_free(h):
     if h:
         load().tahoe_forest_free(h)
@@ -329,6 +334,9 @@ class Forest:
 
     def select_strategy(self, n: int, d: int) -> int:
         return tahoe_select_strategy(self.handle, n, d)
+
+    def predict_cost_us(self, strategy: int, n: int) -> float:
+        return tahoe_predict_cost_us(self.handle, strategy, n)
 
     def predict(self, X, out=None, out_class=None, out_leaf=None, out_fingerprint=None,
                 force_strategy: int = -1, stream=None, ev_main_begin=None, ev_main_end=None):

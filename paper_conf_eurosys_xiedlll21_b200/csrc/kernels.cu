@@ -60,12 +60,14 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  // try_wait with a suspend-time hint: a waiting warp sleeps in hardware instead of re-issuing
+  // the probe (a plain try_wait loop spent a fifth of all issue slots on spinning)
   asm volatile(
       "{\n\t.reg .pred p;\n"
       "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
       "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
-      "r"(phase)
+      "r"(phase), "r"(20000u)
       : "memory");
 }
 // issue a (possibly > 64 KB) bulk copy in 64 KB pieces on one barrier; caller did expect_tx(total)
@@ -309,8 +311,11 @@ __device__ __forceinline__ float sliced_step_v(uint32_t& p, uint32_t rowaddr, ui
   bool go_left = v < __uint_as_float(x);
   if (NAN_AWARE) go_left = go_left || ((v != v) && (y & k.dlbit));
   const bool leaf = PADDED ? (addr == leafaddr) : (off == k.amask);
-  // y >> (F+3) as a high multiply: IMAD.HI runs on the FMA pipe, relieving the ALU pipe
-  p += (go_left && !leaf) ? 256u : __umulhi(y, k.shmul);
+  // both successors are ready before the compare resolves (y >> (F+3) as a high multiply on the
+  // FMA pipe), so the select is the only dependent step between the compare and the next load
+  const uint32_t p_right = p + __umulhi(y, k.shmul);
+  const uint32_t p_left = p + 256u;
+  p = (go_left && !leaf) ? p_left : p_right;
   return __uint_as_float(leaf ? x : 0u);
 }
 
@@ -410,6 +415,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
       smem + a.forest_smem + (ROWS_SMEM ? (size_t)kRing * a.buf_floats * sizeof(float) : 0));
   uint64_t* s_forest = s_full + kRing;
   int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
+  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int nwarps = blockDim.x >> 5;
@@ -427,6 +433,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
 
   if (threadIdx.x == 0) {
     for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; }
+    *s_next = 0ull;
     mbar_init(s_forest, 1);
     fence_mbar_init();
   }
@@ -496,80 +503,123 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
     mbar_wait(s_forest, ph_forest);
     ph_forest ^= 1u;
 
-    for (int64_t it = 0; it < my_tiles; it++, g++) {
-      const int b = (int)(g % kRing);
-      const int64_t tile = t0 + it * ts;
-      const int64_t r0 = tile * R;
-      const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-      const float* tbuf = s_ring + (size_t)b * a.buf_floats;
-      if (ROWS_SMEM) mbar_wait(&s_full[b], (g / kRing) & 1u);
-      auto finish_row = [&](double acc, uint64_t fp, int64_t i) {
-        // a9: fp64 butterfly over the 32 lane sums (lane 0's order is fixed)
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-        if (LEAF) {
-#pragma unroll
-          for (int o = 16; o > 0; o >>= 1) fp += __shfl_xor_sync(0xffffffffu, fp, o);
-        }
-        if (lane == 0) {
-          if (FUSED) write_scalar(a.o, i, acc);
-          else a.o.raw[(size_t)sl * a.n + i] = acc;
-          if (LEAF && a.o.out_fp)
-            atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
-        }
-      };
-      if (ROWS_SMEM && !LEAF) {
-        // rows r and r + nwarps of the tile walk together (two chains per lane)
-        for (int r = warp; r < nr; r += 2 * nwarps) {
-          const int r2 = r + nwarps;
+    if (ROWS_SMEM && !LEAF) {
+      // Dynamic schedule: warps grab row pairs (rows r and r + 32 of a 64-row tile) from a CTA
+      // counter, so a slow pair delays nobody; the warp finishing a tile's last pair refills that
+      // ring buffer with the tile kRing ahead.  At most 32 pairs are in flight, so no warp can run
+      // a full ring ahead of a buffer's refill.
+      constexpr int kPairs = kSlicedTileRows / 2;
+      const uint64_t total = (uint64_t)my_tiles * kPairs;
+      for (;;) {
+        unsigned long long q = 0;
+        if (lane == 0) q = atomicAdd(s_next, 1ull);
+        q = __shfl_sync(0xffffffffu, q, 0);
+        if (q >= total) break;
+        const int64_t it = (int64_t)(q / kPairs);
+        const int r = (int)(q % kPairs);
+        const uint32_t gt = g + (uint32_t)it;
+        const int b = (int)(gt % kRing);
+        const int64_t r0 = (t0 + it * ts) * R;
+        const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+        const float* tbuf = s_ring + (size_t)b * a.buf_floats;
+        mbar_wait(&s_full[b], (gt / kRing) & 1u);
+        if (r < nr) {
+          const int r2 = r + kPairs;
           const bool two = r2 < nr;
           const float* rowA = tbuf + (size_t)r * rs;
           const float* rowB = tbuf + (size_t)(two ? r2 : r) * rs;
           bool has_nan = false;
-          for (int j = lane; j < a.d; j += 32) has_nan |= (rowA[j] != rowA[j]) | (rowB[j] != rowB[j]);
+          if (lane < a.d) has_nan = (rowA[lane] != rowA[lane]) | (rowB[lane] != rowB[lane]);
+          for (int j = lane + 32; j < a.d; j += 32) has_nan |= (rowA[j] != rowA[j]) | (rowB[j] != rowB[j]);
           double accA, accB;
           const uint32_t pB = two ? p0 : pe;
           if (__any_sync(0xffffffffu, has_nan))
             walk_columns2<true, PADDED>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
           else
             walk_columns2<false, PADDED>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
-          finish_row(accA, 0, r0 + r);
-          if (two) finish_row(accB, 0, r0 + r2);
-        }
-      } else {
-        for (int r = warp; r < nr; r += nwarps) {
-          const int64_t i = r0 + r;
-          uint64_t fp = 0;
-          double acc;
-          if (ROWS_SMEM) {
-            const float* row = tbuf + (size_t)r * rs;
-            bool has_nan = false;
-            for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
-            if (__any_sync(0xffffffffu, has_nan))
-              acc = walk_columns_leaf<true, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
-            else
-              acc = walk_columns_leaf<false, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
-          } else {
-            const float* row = a.X + i * a.d;
-            acc = walk_columns_global<LEAF>(p0, pe, row, k, sbase, a, leaf_meta, i, fp);
+          // a9: one butterfly for both rows: after the first exchange lanes 0-15 hold row-A pair
+          // sums and lanes 16-31 row-B pair sums; four more steps finish both (fixed order)
+          const bool hi = lane & 16;
+          double v = (hi ? accB : accA) + __shfl_xor_sync(0xffffffffu, hi ? accA : accB, 16);
+#pragma unroll
+          for (int o = 8; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+          if ((lane & 15) == 0 && (!hi || two)) {
+            const int64_t i = r0 + (hi ? r2 : r);
+            if (FUSED) write_scalar(a.o, i, v);
+            else a.o.raw[(size_t)sl * a.n + i] = v;
           }
-          finish_row(acc, fp, i);
         }
-      }
-      if (ROWS_SMEM) {
-        // release buffer b; the last warp out refills it with the tile kRing ahead
         __syncwarp();
         int last = 0;
         if (lane == 0) {
           __threadfence_block();
-          last = atomicAdd(&s_cnt[b], 1) == nwarps - 1;
+          last = atomicAdd(&s_cnt[b], 1) == kPairs - 1;
           if (last) atomicExch(&s_cnt[b], 0);
         }
         last = __shfl_sync(0xffffffffu, last, 0);
         if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
       }
+      g += (uint32_t)my_tiles;
+    } else {
+      for (int64_t it = 0; it < my_tiles; it++, g++) {
+        const int b = (int)(g % kRing);
+        const int64_t tile = t0 + it * ts;
+        const int64_t r0 = tile * R;
+        const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+        const float* tbuf = s_ring + (size_t)b * a.buf_floats;
+        if (ROWS_SMEM) mbar_wait(&s_full[b], (g / kRing) & 1u);
+        auto finish_row = [&](double acc, uint64_t fp, int64_t i) {
+          // a9: fp64 butterfly over the 32 lane sums (lane 0's order is fixed)
+  #pragma unroll
+          for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+          if (LEAF) {
+  #pragma unroll
+            for (int o = 16; o > 0; o >>= 1) fp += __shfl_xor_sync(0xffffffffu, fp, o);
+          }
+          if (lane == 0) {
+            if (FUSED) write_scalar(a.o, i, acc);
+            else a.o.raw[(size_t)sl * a.n + i] = acc;
+            if (LEAF && a.o.out_fp)
+              atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
+          }
+        };
+        {
+          for (int r = warp; r < nr; r += nwarps) {
+            const int64_t i = r0 + r;
+            uint64_t fp = 0;
+            double acc;
+            if (ROWS_SMEM) {
+              const float* row = tbuf + (size_t)r * rs;
+              bool has_nan = false;
+              for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
+              if (__any_sync(0xffffffffu, has_nan))
+                acc = walk_columns_leaf<true, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
+              else
+                acc = walk_columns_leaf<false, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
+            } else {
+              const float* row = a.X + i * a.d;
+              acc = walk_columns_global<LEAF>(p0, pe, row, k, sbase, a, leaf_meta, i, fp);
+            }
+            finish_row(acc, fp, i);
+          }
+        }
+        if (ROWS_SMEM) {
+          // release buffer b; the last warp out refills it with the tile kRing ahead
+          __syncwarp();
+          int last = 0;
+          if (lane == 0) {
+            __threadfence_block();
+            last = atomicAdd(&s_cnt[b], 1) == nwarps - 1;
+            if (last) atomicExch(&s_cnt[b], 0);
+          }
+          last = __shfl_sync(0xffffffffu, last, 0);
+          if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+        }
+      }
     }
     __syncthreads();  // every warp is done with this slice (multi-pass reload)
+    if (threadIdx.x == 0) *s_next = 0ull;
+    __syncthreads();
   }
 }
 

@@ -159,6 +159,7 @@ static tahoe_status init_handle(tahoe_forest* f, int32_t device) {
     if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, device) == cudaSuccess) f->max_smem = v;
   }
   f->slot_budget = slot_budget_for(f->max_smem, f->host.n_features);
+  if (const char* e = std::getenv("TAHOE_SLOT_BUDGET")) f->slot_budget = std::atoi(e);  // experiments
   return TAHOE_OK;
 }
 

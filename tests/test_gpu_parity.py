@@ -227,3 +227,50 @@ def test_single_leaf_trees_and_stumps():
     F = T.Forest(f, n_features=6, n_classes=1, agg=oracle.AGG_SUM, device=0)
     for s in STRATS:
         _check(_gpu_run(F, X, s), ref, oracle.AGG_SUM, True)
+
+
+def _full_size_sampled(cid, n, n_trees=None, shard=None, k=3000, strategy=-1):
+    """BASELINE.json config at full size: predict all n rows on the GPU in the production launch
+    configuration, check a seeded sample of rows one by one against the oracle."""
+    cfg = gen.CONFIGS[cid]
+    f = gen.make_forest(cid, n_trees=n_trees, leaf_mode="normal")
+    F = T.Forest(f, device=0).layout(gen.make_calibration(cid, 16384))
+    X = gen.make_rows(cid, n)
+    dev = torch.device("cuda", 0)
+    Xd = torch.from_numpy(X).to(dev)
+    idx = gen.subsample(1000 + cid, n, k)
+    if shard is None:
+        out = torch.empty((n, F.n_out), dtype=torch.float32, device=dev)
+        cls = torch.empty(n, dtype=torch.int32, device=dev)
+        F.predict(Xd, out=out, out_class=cls, force_strategy=strategy)
+        torch.cuda.synchronize()
+        ref = oracle.predict(f, X, rows=idx)
+        res = dict(out=out.cpu().numpy()[idx], cls=cls.cpu().numpy()[idx])
+        _check(res, ref, f["agg"], False, want_leaf=False)
+    else:
+        # tree-sharded launch configuration (C5): rank `shard` of 8 computes its fp64 partials
+        r, world = shard
+        S = F.shard(r, world)
+        part = S.predict_partial(Xd)
+        torch.cuda.synchronize()
+        info = T.tahoe_forest_layout_info(S.handle, len(f["feature"]), S.n_trees)
+        trees = np.sort(info["order"])
+        sub = dict(f, root=f["root"][trees], tree_class=f["tree_class"][trees])
+        ref = oracle.predict(sub, X, rows=idx, agg=oracle.AGG_SUM, base_score=0.0)
+        got = part.cpu().numpy()[idx]
+        assert np.allclose(got, ref["raw"], rtol=1e-12, atol=1e-12)
+    del Xd
+
+
+def test_full_size_c3_sampled():
+    _full_size_sampled(3, gen.CONFIGS[3].n_samples)
+
+
+def test_full_size_c4_sampled():
+    _full_size_sampled(4, gen.CONFIGS[4].n_samples, k=1500)
+
+
+def test_full_size_c5_shard_sampled():
+    """C5 at full size: 4000 trees, 10M rows; one tree shard of 8 (the per-GPU work of the
+    tree-sharded launch), fp64 partials checked against the oracle on the shard's trees."""
+    _full_size_sampled(5, gen.CONFIGS[5].n_samples, shard=(3, 8), k=600)

@@ -149,6 +149,80 @@ def run_reference(args, cfg):
     return 0
 
 
+def run_tree_sharded(args, cfg):
+    """BASELINE C5 launch configuration: the forest's trees are split over the ranks
+    (tahoe_forest_shard), every rank predicts fp64 partials of its trees for ALL rows, one NCCL
+    reduce sums them on rank 0, which finalizes.  Strong scaling: total work is fixed."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_eurosys_xiedlll21_b200 import dist as D
+    from paper_conf_eurosys_xiedlll21_b200 import tahoe as T
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    T.load(build_if_missing=(rank == 0 and world == 1))
+    args.warmup = max(args.warmup, 3)
+    n = cfg.n_samples
+    f = gen.make_forest(cfg, leaf_mode="normal")
+    t0 = time.perf_counter()
+    full = T.Forest(f, device=-1).layout(gen.make_calibration(cfg))
+    S = full.shard(rank, world, device=local)
+    layout_s = time.perf_counter() - t0
+    Xd = torch.from_numpy(gen.make_rows(cfg, n)).to(dev)
+    part = torch.empty((n, S.n_out), dtype=torch.float64, device=dev)
+    out = torch.empty((n, S.n_out), dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        S.predict_partial(Xd, part)
+        if world > 1:
+            D.reduce_partials(part, dst=0)
+        if rank == 0:
+            S.finalize(part, out)   # the shard carries the full forest's aggregation and tree count
+
+    for _ in range(args.warmup):
+        step()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    sampler = ClockSampler(local)
+    sampler.start()
+    for e in ev:
+        e[0].record(stream)
+        step()
+        e[1].record(stream)
+    torch.cuda.synchronize()
+    clocks = sampler.stop()
+    ms = sum(a.elapsed_time(b) for a, b in ev) / args.steps
+    if world > 1:
+        ms = D.max_over_ranks(ms, device=dev)
+    if rank == 0:
+        st = S.stats()
+        line = dict(metric=METRIC, value=n / (ms / 1000.0), unit=UNIT, n_gpus=world, steps=args.steps,
+                    warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="strong",
+                    vs_baseline=None, dtype="f32", accum="f64", data="synthetic", impl="ours",
+                    config={"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
+                                        f"{cfg.n_features} features, {n} samples, tree-sharded over "
+                                        f"{world} GPU(s) + NCCL reduce of fp64 partials "
+                                        f"(BASELINE configs[{cfg.cid - 1}])",
+                            "n": n, "trees_per_shard": st["n_trees"],
+                            "parallelism": f"tree-sharded x{world}"},
+                    strategy="direct", roofline=None, cpu_baseline=None, e2e=None,
+                    gpu_launches=(2 if rank == 0 else 1) * args.steps, clocks=clocks,
+                    layout_s=layout_s)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
 def _config(cfg, n, stats):
     c = {"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
                      f"{cfg.n_features} features, {n} samples per GPU (BASELINE configs[{cfg.cid - 1}])",
@@ -171,10 +245,18 @@ def main():
     ap.add_argument("--config", type=int, default=2)
     ap.add_argument("--strategy", type=int, default=-1)
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--mode", default=None, choices=["sample", "tree"],
+                    help="sample sharding (default; C1-C4) or tree sharding (default for C5)")
+    ap.add_argument("--rows", type=int, default=None, help="override the config's row count")
     args = ap.parse_args()
     cfg = gen.CONFIGS[args.config]
+    if args.rows:
+        from dataclasses import replace
+        cfg = replace(cfg, n_samples=args.rows)
     if args.impl == "reference":
         return run_reference(args, cfg)
+    if (args.mode or ("tree" if cfg.cid == 5 else "sample")) == "tree":
+        return run_tree_sharded(args, cfg)
 
     import torch
     import torch.distributed as dist

@@ -113,6 +113,27 @@ tahoe_status tahoe_forest_layout(tahoe_forest* f, const float* X_calib_host, int
                                  int32_t d, const tahoe_layout_opts* opts);
 
 /*
+ * tahoe_count_visits — Algorithm 1 line 16, "Count edge probabilities during inference":
+ * for every row of X (DEVICE, n x d) and every tree, add 1 to counts[k] for each node k the row's
+ * path passes through (root and leaf included); k is the CALLER's node id.  counts: DEVICE
+ * uint32[n_nodes] (the build's array length), accumulated (zero it first), not thread-safe against
+ * concurrent layouts.  Edge probability (parent -> child) = counts[child] / counts[parent]
+ * (P:399-406).  Errors as tahoe_predict.
+ */
+tahoe_status tahoe_count_visits(const tahoe_forest* f, const float* X, int64_t n, int32_t d,
+                                uint32_t* counts, tahoe_stream stream);
+
+/*
+ * tahoe_forest_layout_counts — tahoe_forest_layout driven by visit counts measured elsewhere
+ * (e.g. tahoe_count_visits on live traffic; re-layout for incremental updates).
+ * counts: HOST uint64[n_nodes] by caller node id over n_calib rows.  X_sim_host (n_sim x d, may be
+ * NULL) feeds the lockstep-efficiency simulation of the cost model.
+ */
+tahoe_status tahoe_forest_layout_counts(tahoe_forest* f, const uint64_t* counts, int64_t n_calib,
+                                        const float* X_sim_host, int64_t n_sim, int32_t d,
+                                        const tahoe_layout_opts* opts);
+
+/*
  * tahoe_predict — Algorithm 1 lines 8-15 per batch: cost model, launch.  X: DEVICE pointer
  * n x d row-major float32 (d >= largest attribute index used by the forest + 1; extra columns are
  * ignored); out: DEVICE float32 n x n_out (n_out = tahoe_forest_n_outputs).  n == 0 is a no-op.

@@ -88,6 +88,7 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->dd.root);
   cudaFree((void*)f->dd.cls);
   cudaFree((void*)f->dd.tree_orig);
+  cudaFree((void*)f->dd.slot_orig);
   cudaFree((void*)f->ds.nodes);
   cudaFree((void*)f->ds.col_len);
   cudaFree((void*)f->ds.slots);
@@ -125,6 +126,7 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
   if ((st = upload(f->di.root, &f->dd.root)) != TAHOE_OK) return st;
   if ((st = upload(f->di.cls, &f->dd.cls)) != TAHOE_OK) return st;
   if ((st = upload(f->di.tree_orig, &f->dd.tree_orig)) != TAHOE_OK) return st;
+  if ((st = upload(f->di.slot_orig, &f->dd.slot_orig)) != TAHOE_OK) return st;
   f->dd.n_slots = (int32_t)f->di.root.size();
   f->dd.fbits = f->di.fbits;
   f->dd.n_nodes = (int64_t)f->di.nodes.size() / 2;
@@ -373,6 +375,57 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_layout(
     F.Xsim.resize((size_t)m * d);
     for (int64_t r = 0; r < m; r++)
       std::memcpy(&F.Xsim[(size_t)r * d], X_calib_host + (r * n_calib / m) * d, (size_t)d * 4);
+  }
+  reorder_nodes(F, o.node_reorder != 0);
+  order_trees(F);
+  return encode_and_upload(f);
+  TAHOE_GUARD_END
+}
+
+static tahoe_status layout_opts_fill(const tahoe_layout_opts* opts, tahoe_layout_opts* o) {
+  *o = tahoe_layout_opts{};
+  if (opts) *o = *opts;
+  else { o->node_reorder = 1; o->tree_group = 1; }
+  if (o->t_nodes <= 0) o->t_nodes = 4;
+  if (o->l_hash <= 0) o->l_hash = 128;
+  if (o->m_chunks <= 0) o->m_chunks = 64;
+  if (o->m_chunks > o->l_hash) return fail(TAHOE_E_INVAL, "m_chunks > l_hash");
+  return TAHOE_OK;
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_count_visits(
+    const tahoe_forest* f, const float* X, int64_t n, int32_t d, uint32_t* counts,
+    tahoe_stream stream) {
+  TAHOE_GUARD_BEGIN
+  tahoe_status st = check_predict(f, X, n, d, counts);
+  if (st != TAHOE_OK || n == 0) return st;
+  DeviceGuard g(f->device);
+  int rc = launch_count_visits(f->dd, X, n, d, counts, f->num_sms, reinterpret_cast<cudaStream_t>(stream));
+  if (rc) return cuda_fail((cudaError_t)rc, "visit-count kernel");
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_layout_counts(
+    tahoe_forest* f, const uint64_t* counts, int64_t n_calib, const float* X_sim_host,
+    int64_t n_sim, int32_t d, const tahoe_layout_opts* opts) {
+  TAHOE_GUARD_BEGIN
+  if (!f || !counts || n_calib < 1) return fail(TAHOE_E_INVAL, "bad argument");
+  if (n_sim > 0 && (!X_sim_host || d < f->host.max_feature + 1)) return fail(TAHOE_E_INVAL, "bad simulation rows");
+  tahoe_layout_opts o;
+  tahoe_status st = layout_opts_fill(opts, &o);
+  if (st != TAHOE_OK) return st;
+  Forest& F = f->host;
+  F.opts = o;
+  set_counts(F, counts, n_calib);
+  F.Xsim.clear();
+  F.dsim = 0;
+  if (n_sim > 0) {
+    const int64_t m = std::min<int64_t>(n_sim, 512);
+    F.dsim = d;
+    F.Xsim.resize((size_t)m * d);
+    for (int64_t r = 0; r < m; r++)
+      std::memcpy(&F.Xsim[(size_t)r * d], X_sim_host + (r * n_sim / m) * d, (size_t)d * 4);
   }
   reorder_nodes(F, o.node_reorder != 0);
   order_trees(F);

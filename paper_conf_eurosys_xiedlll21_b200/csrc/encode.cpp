@@ -24,6 +24,7 @@ tahoe_status encode_direct(const Forest& F, DirectImage& D) {
   D.fbits = feature_bits(F.n_features);
   const uint32_t off_lim = 1u << (kOffsetTop - D.fbits);
   D.nodes.assign(F.feat.size() * 2, 0);
+  D.slot_orig.assign(F.feat.size(), -1);
   int64_t base = 0;
   std::vector<int64_t> slot(F.feat.size());
   for (int32_t t : F.order) {
@@ -35,6 +36,7 @@ tahoe_status encode_direct(const Forest& F, DirectImage& D) {
     for (size_t i = 0; i < pre.size(); i++) {
       const int32_t k = pre[i];
       const int64_t s = base + (int64_t)i;
+      D.slot_orig[s] = F.orig[k];
       uint32_t y;
       if (F.feat[k] < 0) {
         y = kLeafBit | (uint32_t)F.orig[k];

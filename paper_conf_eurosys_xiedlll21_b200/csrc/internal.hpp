@@ -62,6 +62,7 @@ Forest make_shard(const Forest& F, int32_t rank, int32_t world);
 
 // ---- layout steps (layout.cpp) ----
 void calibrate(Forest& F, const float* X, int64_t n, int32_t d);
+void set_counts(Forest& F, const uint64_t* counts_by_caller_id, int64_t n_calib);
 void reorder_nodes(Forest& F, bool enable);
 std::vector<int32_t> hot_preorder(const Forest& F, int32_t t);   // compact ids, hot child first
 void tree_tokens(const Forest& F, int32_t t, int32_t t_nodes, std::vector<int32_t>& tok_nodes,
@@ -94,6 +95,7 @@ struct DirectImage {
   int32_t fbits = 0;
   std::vector<uint32_t> nodes;        // [N*2]
   std::vector<int32_t> root, cls, tree_orig;
+  std::vector<int32_t> slot_orig;     // caller node id per node slot
   int64_t bytes() const { return (int64_t)nodes.size() * 4; }
 };
 

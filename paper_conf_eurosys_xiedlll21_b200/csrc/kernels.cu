@@ -623,6 +623,51 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   }
 }
 
+static int grid_for(int64_t n, int block, int num_sms, int per_sm);
+
+// ------------------------------------------------------------------ visit counting
+// Algorithm 1 line 16 ("Count edge probabilities during inference"): every node a sample
+// passes through (leaves included) gets +1 on the counter of its caller node id.  Edge probability
+// of (parent -> child) = count[child] / count[parent].  Lanes meeting the same node in
+// the same step are aggregated into one atomic.
+__global__ void __launch_bounds__(256) k_count_visits(const DevDirect img, const float* X,
+                                                      int64_t n, int32_t d, uint32_t* counts) {
+  const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(img.nodes);
+  const int fbits = img.fbits;
+  const uint32_t fmask = (1u << fbits) - 1u;
+  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t n_pad = ((n + 31) / 32) * 32;  // whole warps iterate together
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_pad; i += stride) {
+    const bool active = i < n;
+    const float* __restrict__ x = X + (active ? i : 0) * d;
+    for (int32_t t = 0; t < img.n_slots; t++) {
+      uint32_t k = (uint32_t)__ldg(&img.root[t]);
+      bool going = active;
+      for (;;) {
+        const unsigned m = __ballot_sync(0xffffffffu, going);
+        if (!m) break;
+        if (going) {
+          const unsigned same = __match_any_sync(m, k);
+          if ((__ffs(same) - 1) == (int)(threadIdx.x & 31))
+            atomicAdd(&counts[__ldg(&img.slot_orig[k])], (uint32_t)__popc(same));
+          const uint2 nd = __ldg(&nodes[k]);
+          if ((int32_t)nd.y < 0) going = false;
+          else k += step(nd.x, nd.y, __ldg(&x[nd.y & fmask]), fbits, offmask);
+        }
+      }
+    }
+  }
+}
+
+int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t d,
+                        uint32_t* counts, int32_t num_sms, void* stream) {
+  const int block = 256;
+  k_count_visits<<<grid_for(n, block, num_sms, 8), block, 0, static_cast<cudaStream_t>(stream)>>>(
+      img, X, n, d, counts);
+  return (int)cudaGetLastError();
+}
+
 // ------------------------------------------------------------------ finalize
 __global__ void __launch_bounds__(256) k_finalize(const FinalizeArgs a) {
   const int32_t C = a.n_classes;

@@ -24,6 +24,7 @@ struct DevDirect {
   const int32_t* root = nullptr;     // per tree slot (class-major order)
   const int32_t* cls = nullptr;      // per tree slot
   const int32_t* tree_orig = nullptr;
+  const int32_t* slot_orig = nullptr; // caller node id of every node slot (visit counting)
   int32_t n_slots = 0;
   int32_t fbits = 0;
   int64_t n_nodes = 0;
@@ -105,6 +106,8 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
 int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                   int32_t d, const OutArgs& o, bool fused, void* stream);
 int launch_finalize(const FinalizeArgs& a, void* stream);
+int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t d,
+                        uint32_t* counts, int32_t num_sms, void* stream);
 int set_sliced_smem_limit(int32_t bytes);
 
 }  // namespace tahoe

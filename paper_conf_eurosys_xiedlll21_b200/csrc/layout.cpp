@@ -66,6 +66,20 @@ void calibrate(Forest& F, const float* X, int64_t n, int32_t d) {
   }
 }
 
+// Counts measured elsewhere (the GPU visit counter, Algorithm 1 line 16), indexed by caller node id.
+void set_counts(Forest& F, const uint64_t* counts, int64_t n) {
+  F.count.assign(F.feat.size(), 0);
+  for (size_t k = 0; k < F.feat.size(); k++) F.count[k] = counts[F.orig[k]];
+  F.n_cal = n;
+  F.calibrated = true;
+  F.exp_reads.assign(F.n_trees, 0.0);
+  for (int32_t t = 0; t < F.n_trees; t++) {
+    uint64_t s = 0;
+    for (int32_t k = F.node_base[t]; k < F.node_base[t + 1]; k++) s += F.count[k];
+    F.exp_reads[t] = n ? (double)s / (double)n : 0.0;
+  }
+}
+
 // ------------------------------------------------------ node rearrangement (Z5)
 void reorder_nodes(Forest& F, bool enable) {
   F.hot_left.assign(F.feat.size(), 1);

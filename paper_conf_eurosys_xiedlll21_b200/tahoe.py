@@ -50,7 +50,8 @@ SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_
            "tahoe_forest_n_outputs", "tahoe_forest_n_trees", "tahoe_forest_stats",
            "tahoe_select_strategy", "tahoe_predict_cost_us", "tahoe_forest_free", "tahoe_last_error",
            "tahoe_forest_layout_info", "tahoe_tree_tokens", "tahoe_tree_simhash", "tahoe_simhash",
-           "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced")
+           "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced", "tahoe_count_visits",
+           "tahoe_forest_layout_counts")
 
 
 def lib_path() -> str:
@@ -93,6 +94,8 @@ def load(build_if_missing: bool = True):
         "tahoe_lsh_order": (st, [P, i32, i32, i32, P, P]),
         "tahoe_sha1": (st, [P, i64, P]),
         "tahoe_forest_export_sliced": (st, [P, P, P, P, P, P]),
+        "tahoe_count_visits": (st, [P, P, i64, i32, P, P]),
+        "tahoe_forest_layout_counts": (st, [P, P, i64, P, i64, i32, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -153,6 +156,20 @@ def tahoe_forest_layout(h, X_calib: np.ndarray, opts: LayoutOpts | None = None):
     X = np.ascontiguousarray(X_calib, dtype=np.float32)
     _check(load().tahoe_forest_layout(h, _np_ptr(X), X.shape[0], X.shape[1],
                                       None if opts is None else ctypes.byref(opts)))
+
+
+def tahoe_count_visits(h, X, n: int, d: int, counts, stream=None):
+    _check(load().tahoe_count_visits(h, _dev_ptr(X), n, d, _dev_ptr(counts), _stream_ptr(stream)))
+
+
+def tahoe_forest_layout_counts(h, counts: np.ndarray, n_calib: int, X_sim: np.ndarray | None = None,
+                               opts: LayoutOpts | None = None):
+    c = np.ascontiguousarray(counts, dtype=np.uint64)
+    Xs = None if X_sim is None else np.ascontiguousarray(X_sim, dtype=np.float32)
+    _check(load().tahoe_forest_layout_counts(h, _np_ptr(c), n_calib, _np_ptr(Xs),
+                                             0 if Xs is None else Xs.shape[0],
+                                             0 if Xs is None else Xs.shape[1],
+                                             None if opts is None else ctypes.byref(opts)))
 
 
 def tahoe_predict(h, X, n: int, d: int, out, stream=None):
@@ -328,6 +345,23 @@ class Forest:
                               kw.get("seed", 0))
         tahoe_forest_layout(self.handle, X_calib, opts)
         return self
+
+    def layout_gpu(self, X_calib_dev, **kw):
+        """Layout from visit counts measured on the GPU (tahoe_count_visits) over the device rows
+        X_calib_dev; a host copy of up to 512 of them feeds the cost model's simulation."""
+        import torch
+        n, d = X_calib_dev.shape
+        cnt = torch.zeros(self.n_nodes, dtype=torch.int32, device=X_calib_dev.device)
+        tahoe_count_visits(self.handle, X_calib_dev, n, d, cnt)
+        counts = cnt.cpu().numpy().view(np.uint32).astype(np.uint64)
+        step = max(1, n // 512)
+        X_sim = X_calib_dev[::step][:512].cpu().numpy()
+        opts = None
+        if kw:
+            opts = LayoutOpts(kw.get("t_nodes", 0), kw.get("l_hash", 0), kw.get("m_chunks", 0),
+                              kw.get("node_reorder", 1), kw.get("tree_group", 1), 0, kw.get("seed", 0))
+        tahoe_forest_layout_counts(self.handle, counts, n, X_sim, opts)
+        return counts
 
     def stats(self) -> dict:
         return tahoe_forest_stats(self.handle)

@@ -254,3 +254,22 @@ def test_shards_partition_trees():
         T.tahoe_forest_free(s)
     assert sorted(seen) == list(range(50))
     T.tahoe_forest_free(h)
+
+
+def test_layout_from_counts_equals_layout_from_rows():
+    """tahoe_forest_layout_counts (counts measured elsewhere, Algorithm 1 line 16) gives the same
+    layout as calibrating on the rows themselves."""
+    f = gen.make_forest(2, n_trees=40)
+    Xc = gen.make_calibration(2, 2048)
+    a = T.tahoe_forest_build(f, 28, 1, T.AGG_BINARY, 0.0, -1)
+    b = T.tahoe_forest_build(f, 28, 1, T.AGG_BINARY, 0.0, -1)
+    T.tahoe_forest_layout(a, Xc)
+    T.tahoe_forest_layout_counts(b, oracle.node_counts(f, Xc), len(Xc), Xc)
+    ia = T.tahoe_forest_layout_info(a, len(f["feature"]), 40)
+    ib = T.tahoe_forest_layout_info(b, len(f["feature"]), 40)
+    for k in ("count", "hot_left", "exp_reads", "order"):
+        assert np.array_equal(ia[k], ib[k]), k
+    ea, eb = T.tahoe_forest_export_sliced(a), T.tahoe_forest_export_sliced(b)
+    assert np.array_equal(ea["nodes"], eb["nodes"])
+    T.tahoe_forest_free(a)
+    T.tahoe_forest_free(b)

@@ -274,3 +274,24 @@ def test_full_size_c5_shard_sampled():
     """C5 at full size: 4000 trees, 10M rows; one tree shard of 8 (the per-GPU work of the
     tree-sharded launch), fp64 partials checked against the oracle on the shard's trees."""
     _full_size_sampled(5, gen.CONFIGS[5].n_samples, shard=(3, 8), k=600)
+
+
+def test_gpu_visit_counts_equal_oracle_and_drive_layout():
+    """Algorithm 1 line 16: visit counts measured by the GPU equal the oracle's path counts, and a
+    layout driven by them equals the host-calibrated layout."""
+    f = gen.make_forest(3, n_trees=120)
+    Xc = gen.make_calibration(3, 5000)
+    Xc[::97, 5] = np.nan
+    F = T.Forest(f, device=0)
+    dev = torch.device("cuda", 0)
+    cnt = F.layout_gpu(torch.from_numpy(Xc).to(dev))
+    assert np.array_equal(cnt, oracle.node_counts(f, Xc))
+    G = T.Forest(f, device=0).layout(Xc)
+    ia = T.tahoe_forest_layout_info(F.handle, len(f["feature"]), F.n_trees)
+    ib = T.tahoe_forest_layout_info(G.handle, len(f["feature"]), G.n_trees)
+    for k in ("count", "hot_left", "order"):
+        assert np.array_equal(ia[k], ib[k]), k
+    X = gen.make_rows(3, 2000)
+    ref = oracle.predict(f, X, want_leaf=True)
+    for s in STRATS:
+        _check(_gpu_run(F, X, s), ref, f["agg"], True)

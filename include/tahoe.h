@@ -172,6 +172,14 @@ tahoe_status tahoe_predict_ex(const tahoe_forest* f, const float* X, int64_t n, 
 tahoe_status tahoe_predict_host(const tahoe_forest* f, const float* X_host, int64_t n, int32_t d,
                                 float* out_host, int32_t* class_host, tahoe_stream stream);
 
+/*
+ * tahoe_forest_l2_persist — low-latency serving (the paper's batch-100 workload,
+ * P:1714-1717): mark the forest image the strategy reads as an L2-persisting access-policy window
+ * on `stream` (hit_ratio in (0, 1]; 0 removes the window), so small batches do not re-fetch it
+ * from HBM between calls.  Mutates the stream's attributes and the device's persisting-L2 limit.
+ */
+tahoe_status tahoe_forest_l2_persist(const tahoe_forest* f, tahoe_stream stream, float hit_ratio);
+
 /* ---------------- tree sharding (multi-GPU) ---------------- */
 
 /* Sub-forest of the trees assigned to `rank` of `world` (balanced by expected visits per tree,

@@ -193,7 +193,7 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
   return select_strategy(plan_stats(f, d), n, d, f->host.agg);
 }
 
-static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int32_t d) {
+static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int64_t n, int32_t d) {
   SlicedPlan p;
   p.forest_smem = ((f->sl.slots_max * 256) + 1023) & ~1023;
   const int32_t fb = f->sl.fbits;
@@ -210,7 +210,10 @@ static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int32_t d) 
   p.smem_bytes = p.forest_smem + (int32_t)ring + kSlicedBarrierBytes;
   const int32_t ns = f->sl.n_slices;
   if (ns <= f->num_sms) {
-    p.cps = std::max(1, f->num_sms / ns);
+    // no more CTAs per slice than there are tiles: a small batch should not make 148 CTAs each
+    // stage a ~200 KB slice for nothing
+    const int64_t tiles = (n + p.tile_rows - 1) / p.tile_rows;
+    p.cps = (int32_t)std::max<int64_t>(1, std::min<int64_t>(f->num_sms / ns, tiles));
     p.grid = ns * p.cps;
   } else {
     p.cps = 1;
@@ -278,7 +281,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
     return TAHOE_OK;
   }
   // sliced
-  const SlicedPlan plan = sliced_plan(f, X, d);
+  const SlicedPlan plan = sliced_plan(f, X, n, d);
   const bool fused = scalar && !raw_user && f->sl.n_slices == 1;
   double* part = nullptr;
   if (!fused) {
@@ -430,6 +433,35 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_layout_counts(
   reorder_nodes(F, o.node_reorder != 0);
   order_trees(F);
   return encode_and_upload(f);
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_l2_persist(
+    const tahoe_forest* f, tahoe_stream stream, float hit_ratio) {
+  TAHOE_GUARD_BEGIN
+  if (!f) return fail(TAHOE_E_INVAL, "NULL forest");
+  if (f->device < 0) return fail(TAHOE_E_STATE, "host-only forest handle");
+  DeviceGuard g(f->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const void* base = f->sl.valid ? (const void*)f->ds.nodes : (const void*)f->dd.nodes;
+  size_t bytes = f->sl.valid ? (size_t)f->sl.bytes() : (size_t)f->di.bytes();
+  int max_persist = 0, max_window = 0;
+  cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, f->device);
+  cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, f->device);
+  cudaStreamAttrValue v = {};
+  if (hit_ratio > 0.0f && max_persist > 0 && max_window > 0) {
+    bytes = std::min(bytes, (size_t)max_window);
+    cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(bytes, (size_t)max_persist));
+    if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceSetLimit");
+    v.accessPolicyWindow.base_ptr = const_cast<void*>(base);
+    v.accessPolicyWindow.num_bytes = bytes;
+    v.accessPolicyWindow.hitRatio = std::min(1.0f, hit_ratio);
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+  }
+  cudaError_t e = cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaStreamSetAttribute");
+  return TAHOE_OK;
   TAHOE_GUARD_END
 }
 

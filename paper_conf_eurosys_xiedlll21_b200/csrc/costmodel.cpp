@@ -76,7 +76,9 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
   if (strategy == TAHOE_STRATEGY_SLICED) {
     if (!st.sliced_ok || st.n_slices < 1) return INFINITY;
     const int64_t tiles = (n + 63) / 64;
-    const int64_t cps = st.n_slices <= st.num_sms ? std::max(1, st.num_sms / st.n_slices) : 1;
+    const int64_t cps = st.n_slices <= st.num_sms
+                            ? std::max<int64_t>(1, std::min<int64_t>(st.num_sms / st.n_slices, tiles))
+                            : 1;
     const double passes = st.n_slices <= st.num_sms ? 1.0 : std::ceil((double)st.n_slices / st.num_sms);
     const double eff = st.sliced_eff > 0.05 ? st.sliced_eff : 0.05;
     const double U = (double)((tiles + cps - 1) / cps) * 64.0 * st.V / (st.n_slices * eff) * passes;

@@ -51,7 +51,7 @@ SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_
            "tahoe_select_strategy", "tahoe_predict_cost_us", "tahoe_forest_free", "tahoe_last_error",
            "tahoe_forest_layout_info", "tahoe_tree_tokens", "tahoe_tree_simhash", "tahoe_simhash",
            "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced", "tahoe_count_visits",
-           "tahoe_forest_layout_counts")
+           "tahoe_forest_layout_counts", "tahoe_forest_l2_persist")
 
 
 def lib_path() -> str:
@@ -95,6 +95,7 @@ def load(build_if_missing: bool = True):
         "tahoe_sha1": (st, [P, i64, P]),
         "tahoe_forest_export_sliced": (st, [P, P, P, P, P, P]),
         "tahoe_count_visits": (st, [P, P, i64, i32, P, P]),
+        "tahoe_forest_l2_persist": (st, [P, P, f32]),
         "tahoe_forest_layout_counts": (st, [P, P, i64, P, i64, i32, P]),
     }
     for name, (res, args) in sig.items():
@@ -156,6 +157,10 @@ def tahoe_forest_layout(h, X_calib: np.ndarray, opts: LayoutOpts | None = None):
     X = np.ascontiguousarray(X_calib, dtype=np.float32)
     _check(load().tahoe_forest_layout(h, _np_ptr(X), X.shape[0], X.shape[1],
                                       None if opts is None else ctypes.byref(opts)))
+
+
+def tahoe_forest_l2_persist(h, stream=None, hit_ratio: float = 1.0):
+    _check(load().tahoe_forest_l2_persist(h, _stream_ptr(stream), float(hit_ratio)))
 
 
 def tahoe_count_visits(h, X, n: int, d: int, counts, stream=None):

@@ -10,7 +10,9 @@
 #include <algorithm>
 #include <cmath>
 #include <cstring>
+#include <cstdlib>
 #include <numeric>
+#include <string>
 
 #include "internal.hpp"
 
@@ -116,8 +118,48 @@ static bool pack_lpt(const Forest& F, const std::vector<int32_t>& trees, int32_t
   return true;
 }
 
+// Rounds: the similarity-ordered trees are dealt 32 at a time, one per lane (similar trees walk in
+// different lanes at the same time, the paper's grouping + round-robin dealing), and
+// inside each round the heaviest remaining tree goes to the lane with the least work so far
+// (keeps the columns balanced like LPT).
+static bool pack_rounds(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
+  P = Pack();
+  std::vector<double> w(32, 0.0);
+  std::vector<int32_t> len(32, 0);
+  for (size_t r0 = 0; r0 < trees.size(); r0 += 32) {
+    std::vector<int32_t> round(trees.begin() + r0, trees.begin() + std::min(trees.size(), r0 + 32));
+    std::stable_sort(round.begin(), round.end(), [&](int32_t a, int32_t b) {
+      if (F.exp_reads[a] != F.exp_reads[b]) return F.exp_reads[a] > F.exp_reads[b];
+      return enc_size(F, a) > enc_size(F, b);
+    });
+    std::vector<int32_t> lanes(32);
+    std::iota(lanes.begin(), lanes.end(), 0);
+    std::stable_sort(lanes.begin(), lanes.end(), [&](int32_t a, int32_t b) {
+      if (w[a] != w[b]) return w[a] < w[b];
+      return len[a] < len[b];
+    });
+    std::vector<uint8_t> used(32, 0);
+    for (int32_t t : round) {
+      int32_t pick = -1;
+      for (int32_t l : lanes)
+        if (!used[l] && len[l] + enc_size(F, t) <= cap) { pick = l; break; }
+      if (pick < 0) return false;
+      used[pick] = 1;
+      P.lanes[pick].push_back(t);
+      w[pick] += F.exp_reads[t];
+      len[pick] += enc_size(F, t);
+    }
+  }
+  pack_stats(F, P);
+  return true;
+}
+
 static bool pack_best(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
   Pack a, b;
+  static const char* mode = std::getenv("TAHOE_PACK");   // experiments: "rr" or "lpt"
+  if (mode && std::string(mode) == "rr") return pack_round_robin(F, trees, cap, P);
+  if (mode && std::string(mode) == "lpt") return pack_lpt(F, trees, cap, P);
+  if (mode && std::string(mode) == "rounds") return pack_rounds(F, trees, cap, P);
   bool ra = pack_round_robin(F, trees, cap, a);
   bool rb = pack_lpt(F, trees, cap, b);
   if (!ra && !rb) return false;

@@ -432,7 +432,9 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   const int rs = a.row_stride;
 
   if (threadIdx.x == 0) {
-    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; }
+    // full barriers: one arrive.expect_tx per TMA fill, or 32 cp.async arrivals (misaligned X)
+    const uint32_t arrivals = (ROWS == kRowsDense && !a.x_aligned) ? 32u : 1u;
+    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], arrivals); s_cnt[b] = 0; }
     *s_next = 0ull;
     mbar_init(s_forest, 1);
     fence_mbar_init();
@@ -467,13 +469,15 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
           mbar_expect_tx(&s_full[b], body);
           if (body) bulk_g2s_big(dst, src, body, &s_full[b]);
         }
-      } else {  // misaligned X: the warp copies the tile itself
+      } else {
+        // misaligned X: 4-byte cp.async copies by the warp, each lane's completion counted on the
+        // buffer's mbarrier (initialised with 32 arrivals for this path)
         const uint32_t cnt = bytes / 4;
-        for (uint32_t q = lane; q < cnt; q += 32) dst[q] = __ldg(&src[q]);
-        __threadfence_block();
-        __syncwarp();
-        if (lane == 0)
-          asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_full[b])) : "memory");
+        for (uint32_t q = lane; q < cnt; q += 32)
+          asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst + q)), "l"(src + q)
+                       : "memory");
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&s_full[b]))
+                     : "memory");
       }
     }
     __syncwarp();
@@ -554,7 +558,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         if (lane == 0) {
           __threadfence_block();
           last = atomicAdd(&s_cnt[b], 1) == kPairs - 1;
-          if (last) atomicExch(&s_cnt[b], 0);
+          if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
         }
         last = __shfl_sync(0xffffffffu, last, 0);
         if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
@@ -610,7 +614,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
           if (lane == 0) {
             __threadfence_block();
             last = atomicAdd(&s_cnt[b], 1) == nwarps - 1;
-            if (last) atomicExch(&s_cnt[b], 0);
+            if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
           }
           last = __shfl_sync(0xffffffffu, last, 0);
           if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);

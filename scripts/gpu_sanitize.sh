@@ -1,0 +1,6 @@
+#!/bin/bash
+mkdir -p gpurun_out
+for tool in memcheck racecheck synccheck; do
+  timeout 900 compute-sanitizer --tool $tool --print-limit 20 --error-exitcode 9 python scripts/sanitize_case.py > gpurun_out/sanitize_$tool.log 2>&1
+  echo "$tool rc=$?"; tail -3 gpurun_out/sanitize_$tool.log
+done

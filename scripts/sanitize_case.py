@@ -1,0 +1,36 @@
+"""Small runs of every kernel variant for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import gen  # noqa: E402
+from paper_conf_eurosys_xiedlll21_b200 import tahoe as T  # noqa: E402
+
+dev = torch.device("cuda", 0)
+for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
+    f = gen.make_forest(cid, n_trees=ntrees)
+    F = T.Forest(f, device=0).layout(gen.make_calibration(cid, 2048))
+    X = gen.make_rows(cid, n)
+    X[::17, 1] = np.nan
+    Xd = torch.from_numpy(X).to(dev)
+    for s in (0, 1):
+        out = torch.empty((n, F.n_out), device=dev)
+        cls = torch.empty(n, dtype=torch.int32, device=dev)
+        leaf = torch.empty((n, F.n_trees), dtype=torch.int32, device=dev)
+        fp = torch.empty(n, dtype=torch.int64, device=dev)
+        F.predict(Xd, out=out, out_class=cls, force_strategy=s)
+        F.predict(Xd, out=out, out_class=cls, out_leaf=leaf, out_fingerprint=fp, force_strategy=s)
+    # misaligned X -> warp-copy staging path
+    buf = torch.empty(X.size + 1, device=dev)
+    buf[1:] = Xd.reshape(-1)
+    F.predict(buf[1:].view(X.shape), force_strategy=1)
+    cnt = torch.zeros(len(f["feature"]), dtype=torch.int32, device=dev)
+    T.tahoe_count_visits(F.handle, Xd, n, X.shape[1], cnt)
+    S = F.shard(0, 2)
+    S.predict_partial(Xd)
+torch.cuda.synchronize()
+print("sanitize case done")

@@ -245,11 +245,11 @@ tahoe_status tahoe_lsh_order(const uint8_t* bits, int32_t n_trees, int32_t l_has
 /* SHA1 digest (FIPS 180-4) used by tokenisation. */
 tahoe_status tahoe_sha1(const uint8_t* msg, int64_t len, uint8_t digest[20]);
 
-/* Export of the encoded SLICED image for host-side decoding in tests:
- *   header[0..7] = {n_slices, slots_max, feature_bits, n_trees, n_classes, 0, 0, 0}
+/* Export of the encoded SLICED image for host-side decoding in tests (C = lane columns = 16):
+ *   header[0..7] = {n_slices, slots_max, feature_bits, n_trees, n_classes, C, slot_bytes, 0}
  *   slice_info[n_slices*4] = {slots, class, n_trees_in_slice, 0}
- *   col_len[n_slices*32], nodes[n_slices*slots_max*32] (uint2 as uint32 pairs),
- *   leaf_meta[n_slices*slots_max*32*2] = {caller tree index, caller node id} at leaf slots.
+ *   col_len[n_slices*C], nodes[n_slices*slots_max*C] (uint2 as uint32 pairs),
+ *   leaf_meta[n_slices*slots_max*C*2] = {caller tree index, caller node id} at leaf slots.
  * Any array pointer may be NULL (then only header is filled). */
 tahoe_status tahoe_forest_export_sliced(const tahoe_forest* f, int32_t* header,
                                         int32_t* slice_info, int32_t* col_len, uint32_t* nodes,

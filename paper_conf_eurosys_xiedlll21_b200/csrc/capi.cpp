@@ -78,7 +78,7 @@ static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
   const bool padded = n_features % 4 == 0;   // predict with d == n_features takes the 2-D TMA path
   const int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb, padded));
   // the slice region is rounded up to 1 KB so the ring's row bases stay aligned
-  return (int32_t)std::max<int64_t>(0, ((max_smem - ring - kSlicedBarrierBytes) & ~1023LL) / 256);
+  return (int32_t)std::max<int64_t>(0, ((max_smem - ring - kSlicedBarrierBytes) & ~1023LL) / kSlotBytes);
 }
 
 static void free_device(tahoe_forest* f) {
@@ -170,7 +170,7 @@ static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   if (d < 0) d = f->host.n_features;
   st.wide_rows = d > 256;
   if (f->sl.valid) {
-    const int64_t room = (int64_t)f->max_smem - (((f->sl.slots_max * 256) + 1023) & ~1023) - kSlicedBarrierBytes;
+    const int64_t room = (int64_t)f->max_smem - (((f->sl.slots_max * kSlotBytes) + 1023) & ~1023) - kSlicedBarrierBytes;
     const int64_t ring = std::min<int64_t>(sliced_ring_bytes(d, f->sl.fbits, false) < 0 ? INT64_MAX : sliced_ring_bytes(d, f->sl.fbits, false),
                                            sliced_ring_bytes(d, f->sl.fbits, true) < 0 ? INT64_MAX : sliced_ring_bytes(d, f->sl.fbits, true));
     st.rows_global = ring > room;
@@ -195,7 +195,7 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
 
 static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int64_t n, int32_t d) {
   SlicedPlan p;
-  p.forest_smem = ((f->sl.slots_max * 256) + 1023) & ~1023;
+  p.forest_smem = ((f->sl.slots_max * kSlotBytes) + 1023) & ~1023;
   const int32_t fb = f->sl.fbits;
   const int64_t room = (int64_t)f->max_smem - p.forest_smem - kSlicedBarrierBytes;
   const int64_t ring_p = padded_rows_possible(X, d) ? sliced_ring_bytes(d, fb, true) : -1;
@@ -765,7 +765,8 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_export_sliced(
   TAHOE_GUARD_BEGIN
   if (!f || !header) return fail(TAHOE_E_INVAL, "bad argument");
   const SlicedImage& S = f->sl;
-  int32_t h[8] = {S.valid ? S.n_slices : 0, S.slots_max, S.fbits, f->host.n_trees, f->host.n_classes, 0, 0, 0};
+  int32_t h[8] = {S.valid ? S.n_slices : 0, S.slots_max, S.fbits, f->host.n_trees, f->host.n_classes,
+                  kSlicedCols, kSlotBytes, 0};
   std::copy(h, h + 8, header);
   if (!S.valid) return TAHOE_OK;
   if (slice_info)

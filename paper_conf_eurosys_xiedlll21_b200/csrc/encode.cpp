@@ -1,12 +1,13 @@
 // encode.cpp — the adaptive forest format re-targeted to B200.
 //
 // Work units: the trees of one class, in similarity order, are cut into SLICES whose
-// nodes fit one CTA's shared memory; inside a slice each tree is dealt to one of 32 LANE COLUMNS
+// nodes fit one CTA's shared memory; inside a slice each tree is dealt to one of 16 LANE COLUMNS
 // ("assigned to threads in a round-robin way, such that loads are roughly balanced"),
 // with a longest-processing-time alternative when it balances expected work better (reading Z12).
-// A lane column holds its trees back to back, each in hot-first preorder, so the hot
-// child of every node is the next slot.  Slot s of lane l lives at word pair (32*s + l): a warp
-// whose lanes read 32 different slots hits 32 different bank pairs.
+// A lane column holds its trees back to back, each in left-first preorder (reading R1), so the
+// left child of every node is the next slot.  Slot s of column c lives at word pair (16*s + c):
+// the two half-warps each walk all 16 columns (for different samples), and an 8-byte load of a
+// half-warp whose lanes sit at 16 different slots hits 16 different bank pairs.
 #include <algorithm>
 #include <cmath>
 #include <cstring>
@@ -64,7 +65,7 @@ tahoe_status encode_direct(const Forest& F, DirectImage& D) {
 
 // ------------------------------------------------------------------ sliced image
 struct Pack {
-  std::vector<std::vector<int32_t>> lanes = std::vector<std::vector<int32_t>>(32);
+  std::vector<std::vector<int32_t>> lanes = std::vector<std::vector<int32_t>>(kSlicedCols);
   int32_t max_len = 0;
   double max_work = 0, sum_work = 0;
 };
@@ -89,7 +90,7 @@ static void pack_stats(const Forest& F, Pack& P) {
 
 static bool pack_round_robin(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
   P = Pack();
-  for (size_t j = 0; j < trees.size(); j++) P.lanes[j % 32].push_back(trees[j]);
+  for (size_t j = 0; j < trees.size(); j++) P.lanes[j % kSlicedCols].push_back(trees[j]);
   pack_stats(F, P);
   return P.max_len <= cap;
 }
@@ -101,11 +102,11 @@ static bool pack_lpt(const Forest& F, const std::vector<int32_t>& trees, int32_t
     if (F.exp_reads[a] != F.exp_reads[b]) return F.exp_reads[a] > F.exp_reads[b];
     return enc_size(F, a) > enc_size(F, b);
   });
-  std::vector<double> w(32, 0.0);
-  std::vector<int32_t> len(32, 0);
+  std::vector<double> w(kSlicedCols, 0.0);
+  std::vector<int32_t> len(kSlicedCols, 0);
   for (int32_t t : ts) {
     int32_t best = -1;
-    for (int32_t l = 0; l < 32; l++) {
+    for (int32_t l = 0; l < kSlicedCols; l++) {
       if (len[l] + enc_size(F, t) > cap) continue;
       if (best < 0 || w[l] < w[best] || (w[l] == w[best] && len[l] < len[best])) best = l;
     }
@@ -118,27 +119,28 @@ static bool pack_lpt(const Forest& F, const std::vector<int32_t>& trees, int32_t
   return true;
 }
 
-// Rounds: the similarity-ordered trees are dealt 32 at a time, one per lane (similar trees walk in
+// Rounds: the similarity-ordered trees are dealt 16 at a time, one per lane (similar trees walk in
 // different lanes at the same time, the paper's grouping + round-robin dealing), and
 // inside each round the heaviest remaining tree goes to the lane with the least work so far
 // (keeps the columns balanced like LPT).
 static bool pack_rounds(const Forest& F, const std::vector<int32_t>& trees, int32_t cap, Pack& P) {
   P = Pack();
-  std::vector<double> w(32, 0.0);
-  std::vector<int32_t> len(32, 0);
-  for (size_t r0 = 0; r0 < trees.size(); r0 += 32) {
-    std::vector<int32_t> round(trees.begin() + r0, trees.begin() + std::min(trees.size(), r0 + 32));
+  const size_t C = kSlicedCols;
+  std::vector<double> w(C, 0.0);
+  std::vector<int32_t> len(C, 0);
+  for (size_t r0 = 0; r0 < trees.size(); r0 += C) {
+    std::vector<int32_t> round(trees.begin() + r0, trees.begin() + std::min(trees.size(), r0 + C));
     std::stable_sort(round.begin(), round.end(), [&](int32_t a, int32_t b) {
       if (F.exp_reads[a] != F.exp_reads[b]) return F.exp_reads[a] > F.exp_reads[b];
       return enc_size(F, a) > enc_size(F, b);
     });
-    std::vector<int32_t> lanes(32);
+    std::vector<int32_t> lanes(C);
     std::iota(lanes.begin(), lanes.end(), 0);
     std::stable_sort(lanes.begin(), lanes.end(), [&](int32_t a, int32_t b) {
       if (w[a] != w[b]) return w[a] < w[b];
       return len[a] < len[b];
     });
-    std::vector<uint8_t> used(32, 0);
+    std::vector<uint8_t> used(C, 0);
     for (int32_t t : round) {
       int32_t pick = -1;
       for (int32_t l : lanes)
@@ -184,7 +186,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
     if (G.empty()) continue;
     int64_t total = 0;
     for (int32_t t : G) total += enc_size(F, t);
-    int32_t k = (int32_t)std::max<int64_t>(1, (int64_t)std::ceil((double)total / (32.0 * cap * 0.97)));
+    int32_t k = (int32_t)std::max<int64_t>(1, (int64_t)std::ceil((double)total / ((double)kSlicedCols * cap * 0.97)));
     for (;; k++) {
       if (k > (int32_t)G.size()) { S.why_invalid = "cannot pack trees into slices"; return TAHOE_OK; }
       // k contiguous chunks of balanced node counts (each non-empty)
@@ -222,7 +224,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
     P.max_len += 1;  // terminal slot
     S.slots_max = std::max(S.slots_max, P.max_len);
     work += P.sum_work;
-    padded += 32.0 * P.max_work;
+    padded += (double)kSlicedCols * P.max_work;
   }
   S.eff = padded > 0 ? work / padded : 0;
   // Simulated lockstep efficiency of k_sliced (two rows per warp, two steps per exit test) on the
@@ -244,13 +246,14 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
         reads[(size_t)r * F.n_trees + t] = (F.tree_size(t) == 1) ? 2 : c;
       }
     }
+    // a warp walks 4 rows at once (2 per half-warp x 2 chains); its loop runs until the slowest
+    // of the 64 (row, column) walks ends, two steps per exit test
     double useful = 0, issued = 0;
-    std::vector<double> W(32);
     for (auto& P : packs) {
-      for (int64_t r = 0; r + 1 < m; r += 2) {
+      for (int64_t r = 0; r + 3 < m; r += 4) {
         double mx = 0;
-        for (int64_t q = r; q < r + 2; q++)
-          for (int32_t l = 0; l < 32; l++) {
+        for (int64_t q = r; q < r + 4; q++)
+          for (int32_t l = 0; l < kSlicedCols; l++) {
             double w = 0;
             for (int32_t t : P.lanes[l]) w += reads[(size_t)q * F.n_trees + t];
             useful += w;
@@ -261,35 +264,38 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
     }
     if (issued > 0) S.eff_sim = useful / issued;
   }
-  S.trees_per_lane = (double)F.n_trees / (32.0 * std::max(1, S.n_slices));
+  S.trees_per_lane = (double)F.n_trees / ((double)kSlicedCols * std::max(1, S.n_slices));
   // Sliced node words (kernels.hpp "sliced encoding"): left child first, right child at +off,
   // leaves carry the all-ones attribute field and the delta to the lane's next tree root; one
   // self-looping terminal leaf (value 0.0, delta 0) closes every lane column.
   const uint32_t fmask = (1u << S.fbits) - 1u;
-  const uint32_t off_lim = 1u << (32 - (S.fbits + 3) - 8);   // offsets stored in bytes (x256)
-  const size_t per_slice = (size_t)S.slots_max * 32;
+  const int32_t C = kSlicedCols;
+  const int32_t sb = 7;                                  // log2(kSlotBytes): offsets stored in bytes
+  static_assert(kSlotBytes == 128, "slot row is 128 bytes");
+  const uint32_t off_lim = 1u << (32 - (S.fbits + 3) - sb);
+  const size_t per_slice = (size_t)S.slots_max * C;
   S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
-  S.col_len.assign((size_t)S.n_slices * 32, 0);
+  S.col_len.assign((size_t)S.n_slices * C, 0);
   S.slots.assign(S.n_slices, 0);
   std::vector<int32_t> slot(F.feat.size(), -1);
   std::vector<int32_t> pre, st;
   for (int32_t s = 0; s < S.n_slices; s++) {
     const Pack& P = packs[s];
     S.slots[s] = P.max_len;
-    for (int32_t l = 0; l < 32; l++) {
+    for (int32_t l = 0; l < C; l++) {
       int32_t pos = 0;
       const auto& L = P.lanes[l];
       for (size_t ti = 0; ti < L.size(); ti++) {
         const int32_t t = L[ti];
         if (F.tree_size(t) == 1) {  // 3-node stump: root (attribute 0, +2 slots right) + 2 leaves
           const int32_t k = F.node_base[t];
-          const uint32_t ynode = (2u * 256u) << (S.fbits + 3);
-          const uint32_t yleaf1 = (2u * 256u) << (S.fbits + 3) | (fmask << 2);
-          const uint32_t yleaf2 = (1u * 256u) << (S.fbits + 3) | (fmask << 2);
+          const uint32_t ynode = (2u << sb) << (S.fbits + 3);
+          const uint32_t yleaf1 = (2u << sb) << (S.fbits + 3) | (fmask << 2);
+          const uint32_t yleaf2 = (1u << sb) << (S.fbits + 3) | (fmask << 2);
           const uint32_t ys[3] = {ynode, yleaf1, yleaf2};
           for (int32_t q = 0; q < 3; q++) {
-            const size_t w = ((size_t)s * per_slice + (size_t)(pos + q) * 32 + l);
+            const size_t w = ((size_t)s * per_slice + (size_t)(pos + q) * C + l);
             S.nodes[2 * w] = q == 0 ? 0u : f2u(F.val[k]);
             S.nodes[2 * w + 1] = ys[q];
             if (q > 0) { S.leaf_meta[2 * w] = F.tree_orig[t]; S.leaf_meta[2 * w + 1] = F.orig[k]; }
@@ -309,11 +315,11 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
         for (size_t i = 0; i < pre.size(); i++) {
           const int32_t k = pre[i];
           const int32_t sl = pos + (int32_t)i;
-          const size_t w = ((size_t)s * per_slice + (size_t)sl * 32 + l);
+          const size_t w = ((size_t)s * per_slice + (size_t)sl * C + l);
           uint32_t y;
           if (F.feat[k] < 0) {
             if ((uint32_t)(next_root - sl) >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "leaf offset overflow");
-            y = ((uint32_t)(next_root - sl) << (S.fbits + 11)) | (fmask << 2);
+            y = ((uint32_t)(next_root - sl) << (S.fbits + 3 + sb)) | (fmask << 2);
             S.nodes[2 * w] = f2u(F.val[k]);
             S.leaf_meta[2 * w] = F.tree_orig[t];
             S.leaf_meta[2 * w + 1] = F.orig[k];
@@ -321,7 +327,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
             if (slot[F.lc[k]] != sl + 1) return fail(TAHOE_E_INVAL, "internal: left child not adjacent");
             const int32_t delta = slot[F.rc[k]] - sl;   // in slots; stored as bytes
             if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "right offset overflow");
-            y = ((uint32_t)delta << (S.fbits + 11)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 2)) |
+            y = ((uint32_t)delta << (S.fbits + 3 + sb)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 2)) |
                 ((uint32_t)F.feat[k] << 2);
             S.nodes[2 * w] = f2u(F.thr[k]);
           }
@@ -330,10 +336,10 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
         pos = next_root;
       }
       // terminal self-loop
-      const size_t w = ((size_t)s * per_slice + (size_t)pos * 32 + l);
+      const size_t w = ((size_t)s * per_slice + (size_t)pos * C + l);
       S.nodes[2 * w] = 0u;
       S.nodes[2 * w + 1] = fmask << 2;
-      S.col_len[(size_t)s * 32 + l] = pos;
+      S.col_len[(size_t)s * C + l] = pos;
     }
   }
   // class -> slices (in slice order: the fixed fp64 summation order of the finalize step)

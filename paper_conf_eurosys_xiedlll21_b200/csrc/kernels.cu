@@ -260,11 +260,13 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
 // Sliced node words (encode.cpp): x = threshold (internal) or leaf value;
 //   internal y = off_bytes << (F+3) | default_left << (F+2) | attribute << 2   (left child next)
 //   leaf     y = next_root_bytes << (F+3) | (2^F - 1) << 2            (all-ones attribute field)
-// Offsets are byte distances between slots (slot = 32 lanes x 8 B = 256 B).  The attribute is
-// stored as a byte offset, and staged rows sit at a power-of-two stride >= 2^F floats, so the
-// attribute's shared address is one LOP3: (y & amask) | row_base; a leaf is the one address
-// row_base | amask.  Every lane column ends with a self-looping leaf of value 0.0, so a lane that
-// has finished its trees keeps stepping harmlessly.  Slot s of lane l is the word pair 32*s + l.
+// A slice has 16 lane columns; slot s of column c is the word pair 16*s + c, one slot row is
+// 16 x 8 B = 128 B and offsets are byte distances between slots.  Lane l walks column l & 15 for
+// the rows of its half-warp (l >> 4): an 8-byte load is served per half-warp, whose 16 lanes sit
+// in 16 different bank pairs.  The attribute is stored as a byte offset; staged rows sit at a
+// power-of-two stride >= 2^F floats, so its shared address is one LOP3: (y & amask) | row_base,
+// and a leaf is the one address row_base | amask.  Every lane column ends with a self-looping leaf
+// of value 0.0, so a lane that has finished its trees keeps stepping harmlessly.
 struct alignas(64) SlicedKArgs {
   CUtensorMap tmap;      // PADDED rows: X as a 2-D tensor [n][d], box [row_stride][tile_rows]
   DevSliced img;
@@ -294,9 +296,9 @@ struct StepConsts {
 };
 
 // One step of one lane: read the node at shared address p, test "x_j < b_i", move to
-// the left child (+256 B) or the right child (+off); return the leaf value met (0.0f at internal
-// nodes).  A leaf jumps to the lane's next tree root.  NAN_AWARE: NaN takes the node's default
-// path.
+// the left child (next slot row) or the right child (+off); return the leaf value met (0.0f at
+// internal nodes).  A leaf jumps to the lane's next tree root.  NAN_AWARE: NaN takes the node's
+// default path.
 template <bool NAN_AWARE, bool PADDED>
 __device__ __forceinline__ float sliced_step_v(uint32_t& p, uint32_t rowaddr, uint32_t leafaddr,
                                                const StepConsts& k) {
@@ -311,11 +313,8 @@ __device__ __forceinline__ float sliced_step_v(uint32_t& p, uint32_t rowaddr, ui
   bool go_left = v < __uint_as_float(x);
   if (NAN_AWARE) go_left = go_left || ((v != v) && (y & k.dlbit));
   const bool leaf = PADDED ? (addr == leafaddr) : (off == k.amask);
-  // both successors are ready before the compare resolves (y >> (F+3) as a high multiply on the
-  // FMA pipe), so the select is the only dependent step between the compare and the next load
-  const uint32_t p_right = p + __umulhi(y, k.shmul);
-  const uint32_t p_left = p + 256u;
-  p = (go_left && !leaf) ? p_left : p_right;
+  // y >> (F+3) as a high multiply: IMAD.HI runs on the FMA pipe, relieving the ALU pipe
+  p += (go_left && !leaf) ? (uint32_t)kSlotBytes : __umulhi(y, k.shmul);
   return __uint_as_float(leaf ? x : 0u);
 }
 
@@ -391,7 +390,7 @@ __device__ __forceinline__ double walk_columns_global(uint32_t p, uint32_t pe,
     const bool leaf = off == k.amask;
     const float v = __ldg(reinterpret_cast<const float*>(rowb + (leaf ? 0u : off)));
     const bool go_left = (v < __uint_as_float(x)) || ((v != v) && (y & k.dlbit));
-    const uint32_t delta = (go_left && !leaf) ? 256u : __umulhi(y, k.shmul);
+    const uint32_t delta = (go_left && !leaf) ? (uint32_t)kSlotBytes : __umulhi(y, k.shmul);
     if (leaf) {
       acc += (double)__uint_as_float(x);
       if (LEAF && delta) {
@@ -405,10 +404,43 @@ __device__ __forceinline__ double walk_columns_global(uint32_t p, uint32_t pe,
   return acc;
 }
 
+// Two chains over rows in global memory (always NaN-aware; a leaf reads the row's first float,
+// which is in bounds, and discards it).
+__device__ __forceinline__ float global_step_v(uint32_t& p, const char* __restrict__ row,
+                                               const StepConsts& k) {
+  uint32_t x, y;
+  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+  const uint32_t off = y & k.amask;
+  const bool leaf = off == k.amask;
+  const float v = __ldg(reinterpret_cast<const float*>(row + (leaf ? 0u : off)));
+  const bool go_left = (v < __uint_as_float(x)) || ((v != v) && (y & k.dlbit));
+  p += (go_left && !leaf) ? (uint32_t)kSlotBytes : __umulhi(y, k.shmul);
+  return __uint_as_float(leaf ? x : 0u);
+}
+
+__device__ __forceinline__ void walk_columns2_global(uint32_t pA, uint32_t pB, uint32_t pe,
+                                                     const float* rowA, const float* rowB,
+                                                     const StepConsts& k, double& accA,
+                                                     double& accB) {
+  const char* ra = reinterpret_cast<const char*>(rowA);
+  const char* rb = reinterpret_cast<const char*>(rowB);
+  accA = 0.0;
+  accB = 0.0;
+  while ((pA != pe) | (pB != pe)) {
+    const float a1 = global_step_v(pA, ra, k);
+    const float b1 = global_step_v(pB, rb, k);
+    const float a2 = global_step_v(pA, ra, k);
+    const float b2 = global_step_v(pB, rb, k);
+    add_pair(accA, a1, a2);
+    add_pair(accB, b1, b2);
+  }
+}
+
 template <bool LEAF, bool FUSED, int ROWS>
 __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ SlicedKArgs a) {
   constexpr bool ROWS_SMEM = ROWS != kRowsGlobal;
   constexpr bool PADDED = ROWS == kRowsPadded;
+  constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
   float* s_ring = reinterpret_cast<float*>(smem + a.forest_smem);
   uint64_t* s_full = reinterpret_cast<uint64_t*>(
@@ -419,6 +451,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int nwarps = blockDim.x >> 5;
+  const int col = lane & (C - 1);   // lane column walked by this lane
+  const int half = lane >> 4;       // half-warp: which rows of the work unit this lane walks
   const uint32_t F = (uint32_t)a.img.fbits;
   StepConsts k;
   k.amask = ((1u << F) - 1u) << 2;
@@ -483,6 +517,20 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
     __syncwarp();
   };
 
+  // release ring buffer b after one work unit; the warp finishing the tile's last unit refills it
+  // with the tile kRing ahead (acquire fence after observing the counter)
+  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts) {
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) {
+      __threadfence_block();
+      last = atomicAdd(&s_cnt[b], 1) == units - 1;
+      if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
+    }
+    last = __shfl_sync(0xffffffffu, last, 0);
+    if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+  };
+
   uint32_t g = 0;  // tiles this CTA has consumed so far (identical in every warp)
   uint32_t ph_forest = 0;
   for (int32_t sl = multipass ? (int32_t)blockIdx.x : (int32_t)blockIdx.x % ns; sl < ns;
@@ -491,80 +539,81 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
     const int64_t ts = multipass ? 1 : a.cps;
     const int64_t my_tiles = t0 < ntiles ? (ntiles - t0 + ts - 1) / ts : 0;
     if (warp == 0) {
-      if (lane == 0) {  // a7: the slice, one bulk copy of slots*32*8 bytes
-        const uint32_t bytes = (uint32_t)a.img.slots[sl] * 256u;
+      if (lane == 0) {  // a7: the slice, one bulk copy of slots x 128 bytes
+        const uint32_t bytes = (uint32_t)a.img.slots[sl] * (uint32_t)kSlotBytes;
         fence_proxy_async_smem();
         mbar_expect_tx(s_forest, bytes);
-        bulk_g2s_big(smem, a.img.nodes + (size_t)sl * a.img.slots_max * 64, bytes, s_forest);
+        bulk_g2s_big(smem, a.img.nodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
       if (ROWS_SMEM)
         for (int64_t q = 0; q < kRing && q < my_tiles; q++) issue_tile(t0 + q * ts, (int)((g + q) % kRing));
     }
     const uint32_t sbase = smem_u32(smem);
-    const uint32_t p0 = sbase + (uint32_t)lane * 8u;
-    const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * 32 + lane] * 32u + (uint32_t)lane) * 8u;
-    const int32_t* __restrict__ leaf_meta = a.img.leaf_meta + (size_t)sl * a.img.slots_max * 64;
+    const uint32_t p0 = sbase + (uint32_t)col * 8u;
+    const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+    const int32_t* __restrict__ leaf_meta = a.img.leaf_meta + (size_t)sl * a.img.slots_max * C * 2;
     mbar_wait(s_forest, ph_forest);
     ph_forest ^= 1u;
 
-    if (ROWS_SMEM && !LEAF) {
-      // Dynamic schedule: warps grab row pairs (rows r and r + 32 of a 64-row tile) from a CTA
-      // counter, so a slow pair delays nobody; the warp finishing a tile's last pair refills that
-      // ring buffer with the tile kRing ahead.  At most 32 pairs are in flight, so no warp can run
-      // a full ring ahead of a buffer's refill.
-      constexpr int kPairs = kSlicedTileRows / 2;
-      const uint64_t total = (uint64_t)my_tiles * kPairs;
+    if (!LEAF) {
+      // Dynamic schedule over work units of 4 rows {u, u+16, u+32, u+48} of a 64-row tile: half h
+      // of the warp walks rows u+16h (chain A) and u+32+16h (chain B).  Warps grab units from a CTA
+      // counter, so a slow unit delays nobody; at most 32 units are in flight, so no warp can run
+      // a full ring ahead of a buffer's refill.  Rows too wide to stage are read from global memory
+      // with the same schedule.
+      constexpr int kUnits = kSlicedTileRows / 4;
+      const uint64_t total = (uint64_t)my_tiles * kUnits;
       for (;;) {
         unsigned long long q = 0;
         if (lane == 0) q = atomicAdd(s_next, 1ull);
         q = __shfl_sync(0xffffffffu, q, 0);
         if (q >= total) break;
-        const int64_t it = (int64_t)(q / kPairs);
-        const int r = (int)(q % kPairs);
+        const int64_t it = (int64_t)(q / kUnits);
+        const int u = (int)(q % kUnits);
         const uint32_t gt = g + (uint32_t)it;
         const int b = (int)(gt % kRing);
         const int64_t r0 = (t0 + it * ts) * R;
         const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-        const float* tbuf = s_ring + (size_t)b * a.buf_floats;
-        mbar_wait(&s_full[b], (gt / kRing) & 1u);
-        if (r < nr) {
-          const int r2 = r + kPairs;
-          const bool two = r2 < nr;
-          const float* rowA = tbuf + (size_t)r * rs;
-          const float* rowB = tbuf + (size_t)(two ? r2 : r) * rs;
-          bool has_nan = false;
-          if (lane < a.d) has_nan = (rowA[lane] != rowA[lane]) | (rowB[lane] != rowB[lane]);
-          for (int j = lane + 32; j < a.d; j += 32) has_nan |= (rowA[j] != rowA[j]) | (rowB[j] != rowB[j]);
+        if (ROWS_SMEM) mbar_wait(&s_full[b], (gt / kRing) & 1u);
+        if (u < nr) {
+          const int rA = u + 16 * half, rB = rA + 32;
+          const bool okA = rA < nr, okB = rB < nr;
+          const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
           double accA, accB;
-          const uint32_t pB = two ? p0 : pe;
-          if (__any_sync(0xffffffffu, has_nan))
-            walk_columns2<true, PADDED>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
-          else
-            walk_columns2<false, PADDED>(p0, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
-          // a9: one butterfly for both rows: after the first exchange lanes 0-15 hold row-A pair
-          // sums and lanes 16-31 row-B pair sums; four more steps finish both (fixed order)
-          const bool hi = lane & 16;
-          double v = (hi ? accB : accA) + __shfl_xor_sync(0xffffffffu, hi ? accA : accB, 16);
+          if (ROWS_SMEM) {
+            const float* tbuf = s_ring + (size_t)b * a.buf_floats;
+            const float* rowA = tbuf + (size_t)(okA ? rA : u) * rs;
+            const float* rowB = tbuf + (size_t)(okB ? rB : u) * rs;
+            bool has_nan = false;
+            for (int j = col; j < a.d; j += C) has_nan |= (rowA[j] != rowA[j]) | (rowB[j] != rowB[j]);
+            if (__any_sync(0xffffffffu, has_nan))
+              walk_columns2<true, PADDED>(pA, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
+            else
+              walk_columns2<false, PADDED>(pA, pB, pe, smem_u32(rowA), smem_u32(rowB), k, accA, accB);
+          } else {
+            walk_columns2_global(pA, pB, pe, a.X + (r0 + (okA ? rA : u)) * a.d,
+                                 a.X + (r0 + (okB ? rB : u)) * a.d, k, accA, accB);
+          }
+          // a9: one butterfly for the four rows: after the first exchange (xor 8) lanes with bit 3
+          // clear hold chain-A pair sums and lanes with bit 3 set chain-B pair sums; three more
+          // steps finish all four (fixed order).  Lanes 0, 8, 16, 24 own rows u, u+32, u+16, u+48.
+          const bool b3 = lane & 8;
+          double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
 #pragma unroll
-          for (int o = 8; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-          if ((lane & 15) == 0 && (!hi || two)) {
-            const int64_t i = r0 + (hi ? r2 : r);
+          for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+          const int rr = b3 ? rB : rA;
+          if ((lane & 7) == 0 && (b3 ? okB : okA)) {
+            const int64_t i = r0 + rr;
             if (FUSED) write_scalar(a.o, i, v);
             else a.o.raw[(size_t)sl * a.n + i] = v;
           }
         }
-        __syncwarp();
-        int last = 0;
-        if (lane == 0) {
-          __threadfence_block();
-          last = atomicAdd(&s_cnt[b], 1) == kPairs - 1;
-          if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
-        }
-        last = __shfl_sync(0xffffffffu, last, 0);
-        if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+        if (ROWS_SMEM) release(b, kUnits, it, my_tiles, t0, ts);
       }
       g += (uint32_t)my_tiles;
     } else {
+      // static schedule (leaf / fingerprint diagnostics): warp w walks rows
+      // w (half 0) and w + 32 (half 1) of every tile, one chain per lane
       for (int64_t it = 0; it < my_tiles; it++, g++) {
         const int b = (int)(g % kRing);
         const int64_t tile = t0 + it * ts;
@@ -572,53 +621,40 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
         const float* tbuf = s_ring + (size_t)b * a.buf_floats;
         if (ROWS_SMEM) mbar_wait(&s_full[b], (g / kRing) & 1u);
-        auto finish_row = [&](double acc, uint64_t fp, int64_t i) {
-          // a9: fp64 butterfly over the 32 lane sums (lane 0's order is fixed)
-  #pragma unroll
-          for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-          if (LEAF) {
-  #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) fp += __shfl_xor_sync(0xffffffffu, fp, o);
+        for (int r = warp; r < (int)(R / 2); r += nwarps) {
+          const int rr = r + 32 * half;
+          const bool ok = rr < nr;
+          const int64_t i = r0 + (ok ? rr : 0);
+          uint64_t fp = 0;
+          double acc = 0.0;
+          if (ROWS_SMEM) {
+            const float* row = tbuf + (size_t)(ok ? rr : 0) * rs;
+            bool has_nan = false;
+            if (ok)
+              for (int j = col; j < a.d; j += C) has_nan |= row[j] != row[j];
+            const uint32_t p = ok ? p0 : pe;
+            if (__any_sync(0xffffffffu, has_nan))
+              acc = walk_columns_leaf<true, PADDED>(p, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
+            else
+              acc = walk_columns_leaf<false, PADDED>(p, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
+          } else if (ok) {
+            acc = walk_columns_global<LEAF>(p0, pe, a.X + i * a.d, k, sbase, a, leaf_meta, i, fp);
           }
-          if (lane == 0) {
+          // a9: butterfly within each half-warp (16 lane sums, fixed order); lanes 0 and 16 write
+#pragma unroll
+          for (int o = 8; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+          if (LEAF) {
+#pragma unroll
+            for (int o = 8; o > 0; o >>= 1) fp += __shfl_xor_sync(0xffffffffu, fp, o);
+          }
+          if (col == 0 && ok) {
             if (FUSED) write_scalar(a.o, i, acc);
             else a.o.raw[(size_t)sl * a.n + i] = acc;
             if (LEAF && a.o.out_fp)
               atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
           }
-        };
-        {
-          for (int r = warp; r < nr; r += nwarps) {
-            const int64_t i = r0 + r;
-            uint64_t fp = 0;
-            double acc;
-            if (ROWS_SMEM) {
-              const float* row = tbuf + (size_t)r * rs;
-              bool has_nan = false;
-              for (int j = lane; j < a.d; j += 32) has_nan |= row[j] != row[j];
-              if (__any_sync(0xffffffffu, has_nan))
-                acc = walk_columns_leaf<true, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
-              else
-                acc = walk_columns_leaf<false, PADDED>(p0, pe, smem_u32(row), k, sbase, a, leaf_meta, i, fp);
-            } else {
-              const float* row = a.X + i * a.d;
-              acc = walk_columns_global<LEAF>(p0, pe, row, k, sbase, a, leaf_meta, i, fp);
-            }
-            finish_row(acc, fp, i);
-          }
         }
-        if (ROWS_SMEM) {
-          // release buffer b; the last warp out refills it with the tile kRing ahead
-          __syncwarp();
-          int last = 0;
-          if (lane == 0) {
-            __threadfence_block();
-            last = atomicAdd(&s_cnt[b], 1) == nwarps - 1;
-            if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
-          }
-          last = __shfl_sync(0xffffffffu, last, 0);
-          if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
-        }
+        if (ROWS_SMEM) release(b, nwarps, it, my_tiles, t0, ts);
       }
     }
     __syncthreads();  // every warp is done with this slice (multi-pass reload)

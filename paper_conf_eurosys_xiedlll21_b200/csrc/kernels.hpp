@@ -71,6 +71,8 @@ struct FinalizeArgs {
 
 // Launchers (kernels.cu).  Return a cudaError_t value as int (0 = success).
 constexpr int32_t kMaxSmemOptin = 232448;   // sharedMemPerBlockOptin on sm_100 (227 KB)
+constexpr int32_t kSlicedCols = 16;         // lane columns per slice (one per half-warp lane)
+constexpr int32_t kSlotBytes = kSlicedCols * 8;  // one slot row: 16 columns x 8-byte nodes
 constexpr int32_t kSlicedRing = 3;          // sample-tile ring depth of k_sliced
 constexpr int32_t kSlicedTileRows = 64;     // rows per tile (two per warp of a 1024-thread CTA)
 constexpr int32_t kSlicedBarrierBytes = 128;

@@ -303,17 +303,18 @@ def tahoe_forest_export_sliced(h) -> dict | None:
     L = load()
     hdr = np.zeros(8, np.int32)
     _check(L.tahoe_forest_export_sliced(h, _np_ptr(hdr), None, None, None, None))
-    ns, smax = int(hdr[0]), int(hdr[1])
+    ns, smax, C = int(hdr[0]), int(hdr[1]), int(hdr[5])
     if ns == 0:
         return None
     info = np.zeros((ns, 4), np.int32)
-    col = np.zeros((ns, 32), np.int32)
-    nodes = np.zeros((ns, smax, 32, 2), np.uint32)
-    meta = np.zeros((ns, smax, 32, 2), np.int32)
+    col = np.zeros((ns, C), np.int32)
+    nodes = np.zeros((ns, smax, C, 2), np.uint32)
+    meta = np.zeros((ns, smax, C, 2), np.int32)
     _check(L.tahoe_forest_export_sliced(h, _np_ptr(hdr), _np_ptr(info), _np_ptr(col),
                                         _np_ptr(nodes), _np_ptr(meta)))
     return dict(n_slices=ns, slots_max=smax, feature_bits=int(hdr[2]), n_trees=int(hdr[3]),
-                n_classes=int(hdr[4]), slice_info=info, col_len=col, nodes=nodes, leaf_meta=meta)
+                n_classes=int(hdr[4]), cols=C, slot_bytes=int(hdr[6]), slice_info=info,
+                col_len=col, nodes=nodes, leaf_meta=meta)
 
 
 # ----------------------------------------------------------------------- convenience wrapper

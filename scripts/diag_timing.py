@@ -9,7 +9,9 @@ cid = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 n = int(sys.argv[2]) if len(sys.argv) > 2 else gen.CONFIGS[cid].n_samples
 f = gen.make_forest(cid, leaf_mode="normal")
 F = T.Forest(f, device=0).layout(gen.make_calibration(cid))
-print(json.dumps(F.stats()))
+st = F.stats()
+print(json.dumps(st))
+print(f"C{cid} slices={st['n_slices']} eff_sim={st['lockstep_eff_sim']:.3f} V={st['expected_node_reads_per_sample']:.1f}")
 X = torch.from_numpy(gen.make_rows(cid, n)).cuda()
 out = torch.empty((n, F.n_out), device="cuda")
 cls = torch.empty(n, dtype=torch.int32, device="cuda")

@@ -189,15 +189,16 @@ def decode_sliced(img, X, n_trees, n_classes):
     """Walk the exported SLICED image on the host (test-side decoder, independent of the
     product's kernels): returns leaf[n, T] (caller node ids) and per-class fp64 sums.
     Node words: internal y = off_bytes << (F+3) | default_left << (F+2) | attribute << 2 (left
-    child next); leaf y = next_root_bytes << (F+3) | (2^F - 1) << 2; slot = 256 bytes."""
+    child next); leaf y = next_root_bytes << (F+3) | (2^F - 1) << 2; slot rows of slot_bytes."""
     n = X.shape[0]
     F = img["feature_bits"]
     fmask = (1 << F) - 1
     leaf = np.full((n, n_trees), -1, np.int64)
     sums = np.zeros((n, n_classes))
+    sb = img["slot_bytes"]
     for s in range(img["n_slices"]):
         c = img["slice_info"][s, 1]
-        for lane in range(32):
+        for lane in range(img["cols"]):
             end = img["col_len"][s, lane]
             x_t, y_t = img["nodes"][s, end, lane]
             assert y_t == fmask << 2 and x_t == 0, "terminal self-loop closes the column"
@@ -209,12 +210,12 @@ def decode_sliced(img, X, n_trees, n_classes):
                         t, node = img["leaf_meta"][s, k, lane]
                         leaf[i, t] = node
                         sums[i, c] += float(np.uint32(x).view(np.float32))
-                        k += (y >> (F + 3)) // 256
+                        k += (y >> (F + 3)) // sb
                     else:
                         thr = float(np.uint32(x).view(np.float32))
                         v = X[i, (y >> 2) & fmask]
                         go_left = bool((y >> (F + 2)) & 1) if np.isnan(v) else bool(v < thr)
-                        k += 1 if go_left else (y >> (F + 3)) // 256
+                        k += 1 if go_left else (y >> (F + 3)) // sb
                 assert k == end
     return leaf, sums
 

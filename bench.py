@@ -151,8 +151,11 @@ def run_reference(args, cfg):
 
 def run_tree_sharded(args, cfg):
     """BASELINE C5 launch configuration: the forest's trees are split over the ranks
-    (tahoe_forest_shard), every rank predicts fp64 partials of its trees for ALL rows, one NCCL
-    reduce sums them on rank 0, which finalizes.  Strong scaling: total work is fixed."""
+    (tahoe_forest_shard), every rank predicts fp64 partials of its trees for ALL rows.
+    --reduce fused (default): the partials land in an NCCL symmetric window and one
+    kernel per rank sums the peers' partials of its row block over NVLink (LSA barrier, rank-order
+    fp64 sum) and finalises them (tahoe_predict_reduce).  --reduce nccl: one ncclReduce onto
+    rank 0, which finalises all rows.  Strong scaling: total work is fixed."""
     import torch
     import torch.distributed as dist
     from paper_conf_eurosys_xiedlll21_b200 import dist as D
@@ -173,11 +176,21 @@ def run_tree_sharded(args, cfg):
     S = full.shard(rank, world, device=local)
     layout_s = time.perf_counter() - t0
     Xd = torch.from_numpy(gen.make_rows(cfg, n)).to(dev)
-    part = torch.empty((n, S.n_out), dtype=torch.float64, device=dev)
-    out = torch.empty((n, S.n_out), dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
+    fused = args.reduce == "fused"
+    if fused:
+        os.environ.setdefault("NCCL_DEBUG", "WARN")   # keep stdout to the one JSON line
+        comm = D.init_comm(local)
+        lo, hi = T.tahoe_reduce_rows(n, world, rank, T.REDUCE_SCATTER)
+        out = torch.empty((hi - lo, S.n_out), dtype=torch.float32, device=dev)
+    else:
+        part = torch.empty((n, S.n_out), dtype=torch.float64, device=dev)
+        out = torch.empty((n, S.n_out), dtype=torch.float32, device=dev)
 
     def step():
+        if fused:
+            S.predict_reduce(comm, Xd, mode=T.REDUCE_SCATTER, out=out)
+            return
         S.predict_partial(Xd, part)
         if world > 1:
             D.reduce_partials(part, dst=0)
@@ -209,14 +222,19 @@ def run_tree_sharded(args, cfg):
                     vs_baseline=None, dtype="f32", accum="f64", data="synthetic", impl="ours",
                     config={"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
                                         f"{cfg.n_features} features, {n} samples, tree-sharded over "
-                                        f"{world} GPU(s) + NCCL reduce of fp64 partials "
-                                        f"(BASELINE configs[{cfg.cid - 1}])",
+                                        f"{world} GPU(s) + "
+                                        + ("fused NVLink reduce + finalize of fp64 partials "
+                                           if fused else "NCCL reduce of fp64 partials ")
+                                        + f"(BASELINE configs[{cfg.cid - 1}])",
                             "n": n, "trees_per_shard": st["n_trees"],
-                            "parallelism": f"tree-sharded x{world}"},
+                            "parallelism": f"tree-sharded x{world}",
+                            "reduce": "fused (NCCL device API, LSA)" if fused else "ncclReduce"},
                     strategy="direct", roofline=None, cpu_baseline=None, e2e=None,
-                    gpu_launches=(2 if rank == 0 else 1) * args.steps, clocks=clocks,
+                    gpu_launches=(2 if (fused or rank == 0) else 1) * args.steps, clocks=clocks,
                     layout_s=layout_s)
         print(json.dumps(line), flush=True)
+    if fused:
+        comm.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
@@ -248,6 +266,8 @@ def main():
     ap.add_argument("--mode", default=None, choices=["sample", "tree"],
                     help="sample sharding (default; C1-C4) or tree sharding (default for C5)")
     ap.add_argument("--rows", type=int, default=None, help="override the config's row count")
+    ap.add_argument("--reduce", default="fused", choices=["fused", "nccl"],
+                    help="tree mode: fused NVLink reduce + finalize kernel, or ncclReduce + finalize")
     args = ap.parse_args()
     cfg = gen.CONFIGS[args.config]
     if args.rows:

@@ -199,6 +199,57 @@ tahoe_status tahoe_predict_partial(const tahoe_forest* shard, const float* X, in
 tahoe_status tahoe_finalize(const tahoe_forest* full, const double* partial, int64_t n,
                             float* out, int32_t* out_class, tahoe_stream stream);
 
+/* ---------------- fused cross-GPU reduce (tree sharding over NVLink) ----------
+ * The paper scales the path over GPUs.  When the forest is split by trees
+ * (tahoe_forest_shard), every rank holds the SAME rows and computes the raw fp64 sums of its own
+ * trees; tahoe_predict_reduce writes them straight into an NCCL symmetric-memory window and ONE
+ * kernel then (1) meets the same CTA of every peer at an LSA barrier (NCCL device API), (2) loads
+ * the peers' partials of its rows over NVLink, sums them in rank order 0..world-1 (fixed order:
+ * identical bits on every rank that finalises a row) and applies the full forest's aggregation as
+ * tahoe_finalize does, (3) passes a second barrier before any rank may reuse its window.  No
+ * separate ncclReduce and no separate finalize launch.
+ *
+ * NCCL >= 2.28 (device API) is loaded at run time with dlopen: the copy already loaded in the
+ * process (torch's) is used, else $TAHOE_NCCL_LIB, else "libnccl.so.2" from the loader path.  The
+ * rest of libtahoe.so never needs NCCL; without it these calls return TAHOE_E_UNSUPPORTED.  All
+ * ranks must be load/store-reachable (one NVLink domain), else TAHOE_E_UNSUPPORTED at init. */
+typedef struct tahoe_comm tahoe_comm;
+#define TAHOE_COMM_ID_BYTES 128
+enum tahoe_reduce_mode {
+  TAHOE_REDUCE_SCATTER = 0,   /* rank r finalises rows [n*r/world, n*(r+1)/world)             */
+  TAHOE_REDUCE_ALL = 1        /* every rank finalises all n rows                               */
+};
+
+/* A fresh communicator id (ncclGetUniqueId) on one rank; the caller broadcasts the 128 bytes. */
+tahoe_status tahoe_comm_unique_id(uint8_t id[TAHOE_COMM_ID_BYTES]);
+
+/* Collective over `world` processes, one per GPU: ncclCommInitRank on `device`, plus a device
+ * communicator with one LSA barrier per SM.  *comm is owned by the caller (tahoe_comm_free). */
+tahoe_status tahoe_comm_init(const uint8_t id[TAHOE_COMM_ID_BYTES], int32_t world, int32_t rank,
+                             int32_t device, tahoe_comm** comm);
+void tahoe_comm_free(tahoe_comm* comm);   /* synchronises the device first; NULL is a no-op     */
+
+/* Rows [*lo, *hi) that `rank` finalises under `mode` (host arithmetic, no GPU). */
+tahoe_status tahoe_reduce_rows(int64_t n, int32_t world, int32_t rank, int32_t mode, int64_t* lo,
+                               int64_t* hi);
+
+/* Collective: every rank calls it with the same n, d and mode and its own shard of the forest
+ * (tahoe_forest_shard(full, rank, world, device)); a shard carries the full forest's aggregation,
+ * base score and tree count.  X: DEVICE [n x d] fp32, the same rows on every rank.  out: DEVICE [(hi-lo) x n_out] fp32 and out_class [(hi-lo)] (or NULL) for this rank's
+ * rows [lo, hi) (tahoe_reduce_rows).  Stream-ordered; the window grows (collectively) on the first
+ * call with a larger n, which synchronises the device. */
+tahoe_status tahoe_predict_reduce(const tahoe_forest* shard, tahoe_comm* comm, const float* X,
+                                  int64_t n, int32_t d, int32_t mode, float* out,
+                                  int32_t* out_class, tahoe_stream stream);
+
+/* The same fused sum + finalisation over caller-provided partials, with the aggregation of `full`
+ * (the full forest or any of its shards): partials is a HOST array of `world` DEVICE pointers to
+ * fp64 [n x n_out] partial sums (tahoe_predict_partial), each readable from full's device (same device, peer access or CUDA-IPC mappings); the caller orders the
+ * producers before this call.  out / out_class as in tahoe_predict_reduce.  world <= 64. */
+tahoe_status tahoe_reduce_partials(const tahoe_forest* full, const double* const* partials,
+                                   int32_t world, int32_t rank, int32_t mode, int64_t n,
+                                   float* out, int32_t* out_class, tahoe_stream stream);
+
 /* ---------------- queries ---------------- */
 int32_t tahoe_forest_n_outputs(const tahoe_forest* f);   /* 1 or n_classes; -1 on NULL        */
 int32_t tahoe_forest_n_trees(const tahoe_forest* f);

@@ -18,6 +18,20 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
+def nccl_include() -> str:
+    """Headers of the NCCL (>= 2.28, device API) that torch ships; the library is dlopen'ed at run
+    time, so only the headers are needed to build."""
+    try:
+        import nvidia.nccl as m  # type: ignore
+        for base in list(getattr(m, "__path__", [])):
+            inc = os.path.join(base, "include")
+            if os.path.exists(os.path.join(inc, "nccl_device.h")):
+                return inc
+    except ImportError:
+        pass
+    raise RuntimeError("NCCL >= 2.28 headers (nccl_device.h) not found (python package nvidia-nccl)")
+
+
 def sources() -> list[str]:
     return sorted(glob.glob(os.path.join(CSRC, "*.cpp")) + glob.glob(os.path.join(CSRC, "*.cu")))
 
@@ -35,8 +49,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-lineinfo", "-O3", "-std=c++17", "-shared", "-cudart", "static",
-           "-Xcompiler", "-fPIC,-fvisibility=hidden,-O3", "-I", INCLUDE, "-I", CSRC,
-           "-o", tmp, *sources(), "-lpthread"]
+           "-Xcompiler", "-fPIC,-fvisibility=hidden,-O3", "-I", nccl_include(), "-I", INCLUDE, "-I", CSRC,
+           "-o", tmp, *sources(), "-lpthread", "-ldl"]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -13,6 +13,10 @@ Two ways the path shards:
   finalizes with the full forest's aggregation (tahoe_finalize).  fp64 partials keep the result
   within the oracle tolerance whatever the reduction order; VOTE partials are exact counts.
 
+  With a tahoe Comm (init_comm) the reduce is fused instead: predict_tree_sharded_fused writes the
+  partials into an NCCL symmetric window and one kernel per rank sums the peers' partials over
+  NVLink in rank order and finalises its rows (tahoe_predict_reduce).
+
 The collective helpers take the partial producer as an argument so the same reduce logic runs in
 the GPU product path and in the CPU (gloo) tests.
 """
@@ -58,6 +62,41 @@ def predict_tree_sharded(full_forest, shard_forest, X: torch.Tensor, dst: int = 
     if dist.get_rank(group) == dst:
         return finalize_fn(partial), partial
     return None, partial
+
+
+def broadcast_comm_id(make_id: Callable[[], bytes], src: int = 0, group=None) -> bytes:
+    """One rank draws the 128-byte communicator id, every rank returns the same bytes."""
+    box = [make_id() if dist.get_rank(group) == src else None]
+    dist.broadcast_object_list(box, src=src, group=group)
+    uid = box[0]
+    if not isinstance(uid, (bytes, bytearray)) or len(uid) != 128:
+        raise RuntimeError("bad communicator id")
+    return bytes(uid)
+
+
+def init_comm(device: int, group=None):
+    """tahoe Comm over the ranks of `group` (one process per GPU, all in one NVLink domain); a
+    single process without torch.distributed gets a world-1 communicator."""
+    from . import tahoe as T
+    if not dist.is_available() or not dist.is_initialized():
+        return T.Comm(T.tahoe_comm_unique_id(), 1, 0, device)
+    uid = broadcast_comm_id(T.tahoe_comm_unique_id, group=group)
+    return T.Comm(uid, dist.get_world_size(group), dist.get_rank(group), device)
+
+
+def reduce_rows(n: int, world: int, rank: int, scatter: bool = True) -> tuple[int, int]:
+    """Rows a rank finalises in the fused reduce (== tahoe_reduce_rows; scatter=False: all)."""
+    return shard_rows(n, rank, world) if scatter else (0, n)
+
+
+def predict_tree_sharded_fused(shard_forest, comm, X: torch.Tensor, scatter: bool = True,
+                               out=None, out_class=None, stream=None):
+    """Tree-sharded prediction with the fused cross-GPU reduce: returns this rank's rows
+    [lo, hi) of the final output (scatter) or all rows (scatter=False)."""
+    from . import tahoe as T
+    mode = T.REDUCE_SCATTER if scatter else T.REDUCE_ALL
+    return shard_forest.predict_reduce(comm, X, mode=mode, out=out, out_class=out_class,
+                                       stream=stream)
 
 
 def max_over_ranks(value: float, device=None, group=None) -> float:

@@ -23,6 +23,8 @@ _lib = None
 TAHOE_OK, TAHOE_E_INVAL, TAHOE_E_NOMEM, TAHOE_E_CUDA, TAHOE_E_UNSUPPORTED, TAHOE_E_STATE = range(6)
 AGG_SUM, AGG_AVERAGE, AGG_BINARY, AGG_CLASS_SUM, AGG_VOTE = range(5)
 STRATEGY_AUTO, STRATEGY_DIRECT, STRATEGY_SLICED = -1, 0, 1
+REDUCE_SCATTER, REDUCE_ALL = 0, 1
+COMM_ID_BYTES = 128
 
 
 class TahoeError(RuntimeError):
@@ -51,7 +53,9 @@ SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_
            "tahoe_select_strategy", "tahoe_predict_cost_us", "tahoe_forest_free", "tahoe_last_error",
            "tahoe_forest_layout_info", "tahoe_tree_tokens", "tahoe_tree_simhash", "tahoe_simhash",
            "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced", "tahoe_count_visits",
-           "tahoe_forest_layout_counts", "tahoe_forest_l2_persist")
+           "tahoe_forest_layout_counts", "tahoe_forest_l2_persist", "tahoe_comm_unique_id",
+           "tahoe_comm_init", "tahoe_comm_free", "tahoe_reduce_rows", "tahoe_predict_reduce",
+           "tahoe_reduce_partials")
 
 
 def lib_path() -> str:
@@ -97,6 +101,12 @@ def load(build_if_missing: bool = True):
         "tahoe_count_visits": (st, [P, P, i64, i32, P, P]),
         "tahoe_forest_l2_persist": (st, [P, P, f32]),
         "tahoe_forest_layout_counts": (st, [P, P, i64, P, i64, i32, P]),
+        "tahoe_comm_unique_id": (st, [P]),
+        "tahoe_comm_init": (st, [P, i32, i32, i32, P]),
+        "tahoe_comm_free": (None, [P]),
+        "tahoe_reduce_rows": (st, [i64, i32, i32, i32, P, P]),
+        "tahoe_predict_reduce": (st, [P, P, P, i64, i32, i32, P, P, P]),
+        "tahoe_reduce_partials": (st, [P, P, i32, i32, i32, i64, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -213,6 +223,64 @@ def tahoe_predict_partial(shard, X, n: int, d: int, partial, stream=None):
 def tahoe_finalize(h, partial, n: int, out, out_class=None, stream=None):
     _check(load().tahoe_finalize(h, _dev_ptr(partial), n, _dev_ptr(out), _dev_ptr(out_class),
                                  _stream_ptr(stream)))
+
+
+def _nccl_hint():
+    """Point the library at torch's NCCL (>= 2.28) unless the caller chose one."""
+    if os.environ.get("TAHOE_NCCL_LIB"):
+        return
+    try:
+        import nvidia.nccl as m  # type: ignore
+        for base in list(getattr(m, "__path__", [])):
+            lib = os.path.join(base, "lib", "libnccl.so.2")
+            if os.path.exists(lib):
+                os.environ["TAHOE_NCCL_LIB"] = lib
+                return
+    except ImportError:
+        pass
+
+
+def tahoe_comm_unique_id() -> bytes:
+    _nccl_hint()
+    buf = (ctypes.c_uint8 * COMM_ID_BYTES)()
+    _check(load().tahoe_comm_unique_id(buf))
+    return bytes(buf)
+
+
+def tahoe_comm_init(uid: bytes, world: int, rank: int, device: int):
+    _nccl_hint()
+    if len(uid) != COMM_ID_BYTES:
+        raise ValueError("communicator id must be 128 bytes")
+    buf = (ctypes.c_uint8 * COMM_ID_BYTES).from_buffer_copy(uid)
+    c = ctypes.c_void_p()
+    _check(load().tahoe_comm_init(buf, world, rank, device, ctypes.byref(c)))
+    return c
+
+
+def tahoe_comm_free(c):
+    if c:
+        load().tahoe_comm_free(c)
+
+
+def tahoe_reduce_rows(n: int, world: int, rank: int, mode: int = REDUCE_SCATTER) -> tuple[int, int]:
+    lo, hi = ctypes.c_int64(), ctypes.c_int64()
+    _check(load().tahoe_reduce_rows(n, world, rank, mode, ctypes.byref(lo), ctypes.byref(hi)))
+    return lo.value, hi.value
+
+
+def tahoe_predict_reduce(shard, comm, X, n: int, d: int, mode: int, out, out_class=None,
+                         stream=None):
+    _check(load().tahoe_predict_reduce(shard, comm, _dev_ptr(X), n, d, mode, _dev_ptr(out),
+                                       _dev_ptr(out_class), _stream_ptr(stream)))
+
+
+def tahoe_reduce_partials(full, partials, world: int, rank: int, mode: int, n: int, out,
+                          out_class=None, stream=None):
+    """partials: sequence of `world` device tensors (or raw pointers) of fp64 [n x n_out]."""
+    arr = (ctypes.c_void_p * max(1, world))(
+        *[p if isinstance(p, int) else p.data_ptr() for p in partials])
+    _check(load().tahoe_reduce_partials(full, arr, world, rank, mode, n, _dev_ptr(out),
+                                        _dev_ptr(out_class), _stream_ptr(stream)))
 
 
 def tahoe_forest_n_outputs(h) -> int:
@@ -421,9 +489,54 @@ class Forest:
     def export_sliced(self):
         return tahoe_forest_export_sliced(self.handle)
 
+    def predict_reduce(self, comm: "Comm", X, mode: int = REDUCE_SCATTER, out=None,
+                       out_class=None, stream=None):
+        """Collective tree-sharded prediction with this shard (tahoe_predict_reduce): returns this
+        rank's rows [lo, hi) of the finalised output."""
+        import torch
+        n, d = X.shape
+        lo, hi = tahoe_reduce_rows(n, comm.world, comm.rank, mode)
+        if out is None:
+            out = torch.empty((hi - lo, self.n_out), dtype=torch.float32, device=X.device)
+        tahoe_predict_reduce(self.handle, comm.handle, X, n, d, mode, out, out_class, stream)
+        return out
+
+    def reduce_partials(self, partials, rank: int, mode: int = REDUCE_SCATTER, out=None,
+                        out_class=None, stream=None):
+        """Fixed-order sum + finalisation of per-shard partials resident on this device."""
+        import torch
+        n = partials[0].shape[0]
+        lo, hi = tahoe_reduce_rows(n, len(partials), rank, mode)
+        if out is None:
+            out = torch.empty((hi - lo, self.n_out), dtype=torch.float32, device=partials[0].device)
+        tahoe_reduce_partials(self.handle, partials, len(partials), rank, mode, n, out, out_class,
+                              stream)
+        return out
+
     def close(self):
         if getattr(self, "handle", None):
             tahoe_forest_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Comm:
+    """Owns a tahoe_comm (NCCL communicator + device communicator with LSA barriers).  Every rank
+    constructs it with the same 128-byte id (tahoe_comm_unique_id on one rank, broadcast by the
+    caller; dist.init_comm does both over torch.distributed)."""
+
+    def __init__(self, uid: bytes, world: int, rank: int, device: int):
+        self.world, self.rank, self.device = int(world), int(rank), int(device)
+        self.handle = tahoe_comm_init(uid, self.world, self.rank, self.device)
+
+    def close(self):
+        if getattr(self, "handle", None):
+            tahoe_comm_free(self.handle)
             self.handle = None
 
     def __del__(self):

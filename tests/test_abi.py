@@ -48,6 +48,34 @@ def test_build_ok_and_host_only_predict_is_state_error():
     T.tahoe_forest_free(h)
 
 
+def test_fused_reduce_host_validation():
+    """f4 boundary: row split, argument errors and host-only handles (no GPU needed)."""
+    L = T.load()
+    for n, w in ((0, 1), (1, 3), (10, 3), (1001, 8), (2**40 + 3, 7)):
+        cover = 0
+        prev = 0
+        for r in range(w):
+            lo, hi = T.tahoe_reduce_rows(n, w, r, T.REDUCE_SCATTER)
+            assert lo == prev and hi >= lo and hi - lo in (n // w, n // w + 1)
+            prev, cover = hi, cover + hi - lo
+        assert prev == n and cover == n
+    lo, hi = ctypes.c_int64(), ctypes.c_int64()
+    assert L.tahoe_reduce_rows(10, 2, 2, 0, ctypes.byref(lo), ctypes.byref(hi)) == T.TAHOE_E_INVAL
+    assert L.tahoe_reduce_rows(10, 0, 0, 0, ctypes.byref(lo), ctypes.byref(hi)) == T.TAHOE_E_INVAL
+    assert L.tahoe_reduce_rows(10, 2, 0, 7, ctypes.byref(lo), ctypes.byref(hi)) == T.TAHOE_E_INVAL
+    assert L.tahoe_reduce_rows(-1, 2, 0, 0, ctypes.byref(lo), ctypes.byref(hi)) == T.TAHOE_E_INVAL
+    h = _build(_stump_arrays())
+    arr = (ctypes.c_void_p * 1)(16)
+    assert L.tahoe_reduce_partials(h, arr, 1, 0, 0, 4, ctypes.c_void_p(16), None, None) == T.TAHOE_E_STATE
+    assert L.tahoe_predict_reduce(h, None, None, 4, 1, 0, None, None, None) == T.TAHOE_E_INVAL
+    c = ctypes.c_void_p()
+    buf = (ctypes.c_uint8 * 128)()
+    assert L.tahoe_comm_init(buf, 2, 2, 0, ctypes.byref(c)) == T.TAHOE_E_INVAL
+    assert L.tahoe_comm_init(None, 1, 0, 0, ctypes.byref(c)) == T.TAHOE_E_INVAL
+    L.tahoe_comm_free(None)
+    T.tahoe_forest_free(h)
+
+
 @pytest.mark.parametrize("mutate,msg", [
     (lambda a: a.update(feature=np.array([3, -1, -1], np.int32)), "n_features"),
     (lambda a: a.update(left=np.array([7, -1, -1], np.int32)), "out of range"),

@@ -3,7 +3,11 @@
 * sample sharding: the ranks' row ranges partition [0, n) (no collective on the data path);
 * tree sharding: the shards of tahoe_forest_shard (host-only handles here) partition the trees,
   and summing per-shard fp64 partials with the product's reduce_partials over gloo reproduces the
-  full forest's raw sums.  The per-shard partial producer in this CPU test is the oracle restricted
+  full forest's raw sums;
+* fused reduce (f4) host logic: the 128-byte communicator id drawn on rank 0 (ncclGetUniqueId via
+  tahoe_comm_unique_id) reaches every rank unchanged, tahoe_reduce_rows partitions the rows like
+  dist.shard_rows, and the rank-order sum of the gathered partials over a rank's rows (what
+  k_reduce_lsa computes over NVLink) equals the full forest's raw sums.  The per-shard partial producer in this CPU test is the oracle restricted
   to the shard's trees (test infrastructure); on GPUs it is tahoe_predict_partial (see
   tests/test_gpu_parity.py::test_parity_c5_subsample_direct_and_shards).
 """
@@ -79,6 +83,24 @@ def _worker(rank, world, port, q):
         if rank == 0:
             ref = oracle.predict(f, X, agg=oracle.AGG_CLASS_SUM)
             assert np.array_equal(out.numpy(), ref["raw"]), "dyadic partials sum exactly"
+        # fused reduce host logic
+        uid = D.broadcast_comm_id(T.tahoe_comm_unique_id)
+        ids = [None] * world
+        dist.all_gather_object(ids, uid)
+        assert all(u == ids[0] for u in ids) and len(uid) == T.COMM_ID_BYTES
+        for nn in (0, 1, 7, 300):
+            lo, hi = T.tahoe_reduce_rows(nn, world, rank, T.REDUCE_SCATTER)
+            assert (lo, hi) == D.reduce_rows(nn, world, rank) == D.shard_rows(nn, rank, world)
+            assert T.tahoe_reduce_rows(nn, world, rank, T.REDUCE_ALL) == (0, nn)
+        parts = [torch.zeros_like(part) for _ in range(world)]
+        dist.all_gather(parts, partial_fn(X))
+        lo, hi = T.tahoe_reduce_rows(X.shape[0], world, rank, T.REDUCE_SCATTER)
+        s = torch.zeros_like(parts[0][lo:hi])
+        for p in parts:          # rank order 0..world-1, as the kernel sums
+            s += p[lo:hi]
+        ref = oracle.predict(f, X, agg=oracle.AGG_CLASS_SUM)
+        assert np.array_equal(s.numpy(), ref["raw"][lo:hi])
+
         m = D.max_over_ranks(float(rank) + 0.5)
         assert m == world - 0.5
         T.tahoe_forest_free(sh)

@@ -113,9 +113,38 @@ static tahoe_status upload(const std::vector<T>& v, const T** dst) {
 }
 
 // encode both images with the current layout state and (re)upload them (Algorithm 1 line 7)
+// Direct image chunking (reading R4): B200's L2 is 126 MB; a direct image larger than
+// kDirectChunkMin is walked in chunks of whole trees of at most kDirectChunkBytes (one launch per
+// chunk, fp64 partials accumulated in chunk order), so the nodes every row visits come from L2
+// rather than HBM.  $TAHOE_DIRECT_CHUNK_KB overrides the chunk size (0 = never chunk).
+static void direct_chunks(tahoe_forest* f) {
+  int64_t chunk = (int64_t)20 << 20, min_total = (int64_t)64 << 20;
+  if (const char* e = std::getenv("TAHOE_DIRECT_CHUNK_KB")) {
+    chunk = (int64_t)std::atoll(e) << 10;
+    min_total = chunk;
+  }
+  const std::vector<int32_t>& root = f->di.root;
+  const int64_t N = (int64_t)f->di.nodes.size() / 2;
+  const int32_t T = (int32_t)root.size();
+  f->direct_chunks.assign(1, 0);
+  if (chunk > 0 && N * 8 > min_total) {
+    int64_t acc = 0;
+    for (int32_t t = 0; t < T; t++) {
+      const int64_t sz = (int64_t)((t + 1 < T ? root[t + 1] : N) - root[t]) * 8;
+      if (acc > 0 && acc + sz > chunk) {
+        f->direct_chunks.push_back(t);
+        acc = 0;
+      }
+      acc += sz;
+    }
+  }
+  f->direct_chunks.push_back(T);
+}
+
 static tahoe_status encode_and_upload(tahoe_forest* f) {
   tahoe_status st = encode_direct(f->host, f->di);
   if (st != TAHOE_OK) return st;
+  direct_chunks(f);
   st = encode_sliced(f->host, f->slot_budget, f->sl);
   if (st != TAHOE_OK) return st;
   if (f->device < 0) return TAHOE_OK;
@@ -254,7 +283,8 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   fa.raw_out = raw_user;
   const bool scalar = C == 1 && H.agg != TAHOE_AGG_VOTE;
   if (strat == TAHOE_STRATEGY_DIRECT) {
-    if (scalar && !raw_user) {
+    const size_t nchunks = f->direct_chunks.size() - 1;
+    if (scalar && !raw_user && nchunks == 1) {
       if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
       int rc = launch_direct(f->dd, X, n, d, o, true, f->num_sms, st);
       if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
@@ -267,7 +297,16 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
     if ((e = cudaMemsetAsync(raw, 0, (size_t)n * C * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
     o.raw = raw;
     if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
-    int rc = launch_direct(f->dd, X, n, d, o, false, f->num_sms, st);
+    int rc = 0;
+    for (size_t c = 0; c < nchunks && !rc; c++) {   // raw += each chunk's per-class sums
+      DevDirect dc = f->dd;
+      const int32_t s0 = f->direct_chunks[c], s1 = f->direct_chunks[c + 1];
+      dc.root += s0;
+      dc.cls += s0;
+      dc.tree_orig += s0;
+      dc.n_slots = s1 - s0;
+      rc = launch_direct(dc, X, n, d, o, false, f->num_sms, st);
+    }
     if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
     if (rc) return cuda_fail((cudaError_t)rc, "direct kernel");
     if (!raw_user) {
@@ -654,6 +693,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"n_calib\":" << H.n_cal << ",\"expected_node_reads_per_sample\":" << V
      << ",\"expected_visits_per_sample\":" << (V - H.n_trees)
      << ",\"feature_bits\":" << f->di.fbits << ",\"direct_bytes\":" << f->di.bytes()
+     << ",\"direct_chunks\":" << (f->direct_chunks.empty() ? 0 : f->direct_chunks.size() - 1)
      << ",\"bytes_fixed_index\":" << (int64_t)H.feat.size() * 12
      << ",\"sliced_valid\":" << (f->sl.valid ? "true" : "false")
      << ",\"sliced_why\":\"" << f->sl.why_invalid << "\""

@@ -136,6 +136,9 @@ struct tahoe_forest {
   int32_t device = -1;
   int32_t slot_budget = 0;       // slot rows of 32 nodes that fit the per-CTA forest smem budget
   int32_t num_sms = 0;
+  // direct strategy: tree-slot boundaries of L2-sized chunks (one launch per chunk when the direct
+  // image exceeds the L2 budget, so each chunk's nodes stay L2-resident while every row walks it)
+  std::vector<int32_t> direct_chunks;   // [0, s1, s2, ..., n_slots]
   int32_t max_smem = 0;
   // device copies
   tahoe::DevDirect dd{};

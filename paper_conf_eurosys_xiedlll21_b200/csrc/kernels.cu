@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(256) k_direct(const DirectKArgs a) {
         if (!FUSED) {
           const int32_t c2 = __ldg(&a.img.cls[t]);
           if (c2 != cls) {
-            if (!vote) a.o.raw[i * C + cls] = acc;
+            if (!vote) a.o.raw[i * C + cls] += acc;
             acc = 0.0;
             cls = c2;
           }
@@ -152,7 +152,7 @@ __global__ void __launch_bounds__(256) k_direct(const DirectKArgs a) {
       }
     }
     if (FUSED) write_scalar(a.o, i, acc);
-    else if (!vote) a.o.raw[i * C + cls] = acc;
+    else if (!vote) a.o.raw[i * C + cls] += acc;
     if (LEAF && a.o.out_fp) atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]),
                                      (unsigned long long)fp);
   }
@@ -195,7 +195,7 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
         if (!FUSED) {
           const int32_t c2 = __ldg(&a.img.cls[t]);
           if (c2 != cls) {
-            if (active && !vote) a.o.raw[i * C + cls] = acc;
+            if (active && !vote) a.o.raw[i * C + cls] += acc;
             acc = 0.0;
             cls = c2;
           }
@@ -237,7 +237,7 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
           if (!FUSED) {
             const int32_t c2 = __ldg(&a.img.cls[t]);
             if (c2 != cls) {
-              if (!vote) a.o.raw[i * C + cls] = acc;
+              if (!vote) a.o.raw[i * C + cls] += acc;
               acc = 0.0;
               cls = c2;
             }
@@ -249,7 +249,7 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
     }
     if (active) {
       if (FUSED) write_scalar(a.o, i, acc);
-      else if (!vote) a.o.raw[i * C + cls] = acc;
+      else if (!vote) a.o.raw[i * C + cls] += acc;
       if (LEAF && a.o.out_fp)
         atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
     }

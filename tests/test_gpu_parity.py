@@ -295,3 +295,21 @@ def test_gpu_visit_counts_equal_oracle_and_drive_layout():
     ref = oracle.predict(f, X, want_leaf=True)
     for s in STRATS:
         _check(_gpu_run(F, X, s), ref, f["agg"], True)
+
+
+def test_direct_chunked_image_parity(monkeypatch):
+    """Reading R4: a direct image walked in L2-sized chunks of trees (one launch per chunk, fp64
+    partials accumulated in chunk order) gives the same leaves, fingerprints, classes and dyadic
+    scores as the oracle; chunk size forced small through TAHOE_DIRECT_CHUNK_KB at build time."""
+    monkeypatch.setenv("TAHOE_DIRECT_CHUNK_KB", "64")
+    for cid, ntrees, nrows in ((3, 280, 2500), (5, 120, 700)):
+        f = gen.make_forest(cid, n_trees=ntrees)
+        F = T.Forest(f, device=0).layout(gen.make_calibration(cid, 4096))
+        assert F.stats()["direct_chunks"] > 1
+        X = gen.make_rows(cid, nrows)
+        X[::9, 2] = np.nan
+        ref = oracle.predict(f, X, want_leaf=True)
+        _check(_gpu_run(F, X, T.STRATEGY_DIRECT), ref, f["agg"], True)
+        res = _gpu_run(F, X, T.STRATEGY_DIRECT, want_leaf=False)   # fused-finalize path
+        _check(res, ref, f["agg"], True, want_leaf=False)
+        F.close()

@@ -155,7 +155,7 @@ def run_tree_sharded(args, cfg):
     --reduce fused (default): the partials land in an NCCL symmetric window and one
     kernel per rank sums the peers' partials of its row block over NVLink (LSA barrier, rank-order
     fp64 sum) and finalises them (tahoe_predict_reduce).  --reduce nccl: one ncclReduce onto
-    rank 0, which finalises all rows.  Strong scaling: total work is fixed."""
+    rank 0, which finalises all rows.  Strong scaling (total work fixed) unless --weak."""
     import torch
     import torch.distributed as dist
     from paper_conf_eurosys_xiedlll21_b200 import dist as D
@@ -169,13 +169,16 @@ def run_tree_sharded(args, cfg):
         dist.init_process_group("nccl", device_id=dev)
     T.load(build_if_missing=(rank == 0 and world == 1))
     args.warmup = max(args.warmup, 3)
-    n = cfg.n_samples
+    # --weak: the paper's weak-scaling setup, "duplicate the set N_G times": every
+    # GPU walks its 1/G of the trees over G copies of the rows, so per-GPU work stays fixed
+    reps = world if args.weak else 1
+    n = cfg.n_samples * reps
     f = gen.make_forest(cfg, leaf_mode="normal")
     t0 = time.perf_counter()
     full = T.Forest(f, device=-1).layout(gen.make_calibration(cfg))
     S = full.shard(rank, world, device=local)
     layout_s = time.perf_counter() - t0
-    Xd = torch.from_numpy(gen.make_rows(cfg, n)).to(dev)
+    Xd = torch.from_numpy(gen.make_rows(cfg, cfg.n_samples)).to(dev).repeat(reps, 1)
     stream = torch.cuda.current_stream()
     fused = args.reduce == "fused"
     if fused:
@@ -218,10 +221,13 @@ def run_tree_sharded(args, cfg):
     if rank == 0:
         st = S.stats()
         line = dict(metric=METRIC, value=n / (ms / 1000.0), unit=UNIT, n_gpus=world, steps=args.steps,
-                    warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="strong",
+                    warmup=args.warmup, ms_per_step=ms, higher_is_better=True,
+                    scaling="weak" if args.weak else "strong",
                     vs_baseline=None, dtype="f32", accum="f64", data="synthetic", impl="ours",
                     config={"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
-                                        f"{cfg.n_features} features, {n} samples, tree-sharded over "
+                                        f"{cfg.n_features} features, {n} samples"
+                                        + (f" ({reps} copies of {cfg.n_samples})" if reps > 1 else "")
+                                        + ", tree-sharded over "
                                         f"{world} GPU(s) + "
                                         + ("fused NVLink reduce + finalize of fp64 partials "
                                            if fused else "NCCL reduce of fp64 partials ")
@@ -266,6 +272,10 @@ def main():
     ap.add_argument("--mode", default=None, choices=["sample", "tree"],
                     help="sample sharding (default; C1-C4) or tree sharding (default for C5)")
     ap.add_argument("--rows", type=int, default=None, help="override the config's row count")
+    ap.add_argument("--weak", action="store_true",
+                    help="tree mode: duplicate the rows once per GPU (weak scaling, P:2450-2456)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help=argparse.SUPPRESS)   # gloo: N>1 code path on one GPU (tests only)
     ap.add_argument("--reduce", default="fused", choices=["fused", "nccl"],
                     help="tree mode: fused NVLink reduce + finalize kernel, or ncclReduce + finalize")
     args = ap.parse_args()
@@ -284,11 +294,14 @@ def main():
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:   # test hook: several ranks sharing one GPU (NCCL refuses duplicate GPUs)
+            dist.init_process_group("gloo")
     T.load(build_if_missing=(rank == 0 and world == 1))
     args.warmup = max(args.warmup, 3)
     n = cfg.n_samples
@@ -300,6 +313,7 @@ def main():
     stats = F.stats()
     strategy = args.strategy if args.strategy >= 0 else F.select_strategy(n, cfg.n_features)
     Xd = torch.from_numpy(X).to(dev)
+    coll_dev = dev if args.dist_backend == "nccl" else torch.device("cpu")
     out = torch.empty((n, F.n_out), dtype=torch.float32, device=dev)
     cls = torch.empty(n, dtype=torch.int32, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
@@ -341,7 +355,7 @@ def main():
     clocks = sampler.stop()
     step_ms = [e[0].elapsed_time(e[1]) for e in ev]
     kern_ms = [e[2].elapsed_time(e[3]) for e in ev]
-    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=coll_dev)
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
     ms_per_step = float(tot[0]) / args.steps
@@ -363,7 +377,7 @@ def main():
         b.record(stream)
         torch.cuda.synchronize()
         e2e_ms.append(a.elapsed_time(b))
-    e2e_t = torch.tensor([statistics.mean(e2e_ms)], dtype=torch.float64, device=dev)
+    e2e_t = torch.tensor([statistics.mean(e2e_ms)], dtype=torch.float64, device=coll_dev)
     if world > 1:
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e_value = world * n / (float(e2e_t[0]) / 1000.0)

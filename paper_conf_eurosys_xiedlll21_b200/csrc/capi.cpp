@@ -533,6 +533,8 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   DeviceGuard g(f->device);
   cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
   const int32_t C = f->host.n_out();
+  // 8 chunks (>= 64K rows each): overlap H2D / compute / D2H; 16 smaller chunks measured slower
+  // (per-chunk launch and finalize overheads outweigh the shorter tail)
   const int64_t chunk = std::min<int64_t>(n, std::max<int64_t>(65536, (n + 7) / 8));
   const int64_t nchunks = (n + chunk - 1) / chunk;
   cudaStream_t s_in, s_cmp, s_out;

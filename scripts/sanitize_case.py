@@ -13,17 +13,22 @@ from paper_conf_eurosys_xiedlll21_b200 import tahoe as T  # noqa: E402
 dev = torch.device("cuda", 0)
 for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
     f = gen.make_forest(cid, n_trees=ntrees)
+    # small direct chunks (reading R4) so the chunked launches are exercised too
+    os.environ["TAHOE_DIRECT_CHUNK_KB"] = "16"
     F = T.Forest(f, device=0).layout(gen.make_calibration(cid, 2048))
+    os.environ.pop("TAHOE_DIRECT_CHUNK_KB")
     X = gen.make_rows(cid, n)
     X[::17, 1] = np.nan
     Xd = torch.from_numpy(X).to(dev)
-    for s in (0, 1):
+    for s, variant in ((0, "0"), (0, "1"), (0, "2"), (1, "0")):
+        os.environ["TAHOE_DIRECT_VARIANT"] = variant   # direct: rows global / staged (lockstep, free)
         out = torch.empty((n, F.n_out), device=dev)
         cls = torch.empty(n, dtype=torch.int32, device=dev)
         leaf = torch.empty((n, F.n_trees), dtype=torch.int32, device=dev)
         fp = torch.empty(n, dtype=torch.int64, device=dev)
         F.predict(Xd, out=out, out_class=cls, force_strategy=s)
         F.predict(Xd, out=out, out_class=cls, out_leaf=leaf, out_fingerprint=fp, force_strategy=s)
+    os.environ.pop("TAHOE_DIRECT_VARIANT")
     # misaligned X -> warp-copy staging path
     buf = torch.empty(X.size + 1, device=dev)
     buf[1:] = Xd.reshape(-1)
@@ -32,5 +37,17 @@ for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
     T.tahoe_count_visits(F.handle, Xd, n, X.shape[1], cnt)
     S = F.shard(0, 2)
     S.predict_partial(Xd)
+    # fused cross-GPU reduce: peer-pointer kernel over two shards' partials, and the NCCL LSA
+    # kernel through a world-1 communicator
+    parts = [F.shard(r, 2).predict_partial(Xd) for r in range(2)]
+    for r in range(2):
+        for mode in (T.REDUCE_SCATTER, T.REDUCE_ALL):
+            F.reduce_partials(parts, r, mode=mode, out_class=torch.empty(n, dtype=torch.int32, device=dev))
+    if cid == 2:
+        comm = T.Comm(T.tahoe_comm_unique_id(), 1, 0, 0)
+        S1 = F.shard(0, 1)
+        S1.predict_reduce(comm, Xd)
+        torch.cuda.synchronize()
+        comm.close()
 torch.cuda.synchronize()
 print("sanitize case done")

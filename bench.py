@@ -407,10 +407,13 @@ def main():
     smem_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
     achieved = n * smem_bytes_per_sample / (kern_avg_ms / 1000.0) / 1e9
     traffic = None
+    sector_eff = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get(f"C{cfg.cid}", {}).get("dram_bytes_per_launch")
+            rec = json.load(open(tp)).get(f"C{cfg.cid}", {})
+            traffic = rec.get("dram_bytes_per_launch")
+            sector_eff = rec.get("global_ld_sector_efficiency")
         except Exception:
             traffic = None
     launches_per_step = 1 if strategy == T.STRATEGY_DIRECT and F.n_out == 1 else (
@@ -425,6 +428,7 @@ def main():
                       kernel="k_sliced" if strategy == 1 else "k_direct",
                       achieved=achieved, peak=smem_peak, unit="GB/s", frac=achieved / smem_peak,
                       traffic=traffic, kernel_ms=kern_avg_ms,
+                      global_ld_sector_efficiency=sector_eff,
                       units_per_launch=f"{n} samples x {smem_bytes_per_sample:.0f} B "
                                        f"({visits:.0f} visits x 12 B + {cfg.n_trees} leaves x 8 B)",
                       peak_source=f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz"),

@@ -256,6 +256,58 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
   }
 }
 
+// Direct strategy, staged rows, P threads per row (scalar outputs, no leaf ids): thread j of a row
+// walks trees j, j+P, j+2P, ... free-running; the P partial sums are added in a fixed order
+// through shuffles.  P x more threads over the same staged rows hide more node-load latency.
+template <bool FUSED, int ROWS, int P>
+__global__ void __launch_bounds__(ROWS * P) k_direct_tlp(const DirectKArgs a, int32_t rs) {
+  extern __shared__ __align__(16) float s_rows[];
+  const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(a.img.nodes);
+  const int fbits = a.img.fbits;
+  const uint32_t fmask = (1u << fbits) - 1u;
+  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const int32_t T = a.img.n_slots;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int r = threadIdx.x / P, j = threadIdx.x % P;
+  const int64_t ntiles = (a.n + ROWS - 1) / ROWS;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * ROWS;
+    const int nr = (int)((a.n - r0) < ROWS ? (a.n - r0) : ROWS);
+    __syncthreads();
+    for (int q = warp; q < nr; q += ROWS * P / 32) {
+      const float* src = a.X + (r0 + q) * a.d;
+      for (int c = lane; c < a.d; c += 32) s_rows[q * rs + c] = __ldg(&src[c]);
+    }
+    __syncthreads();
+    const bool active = r < nr;
+    const float* row = s_rows + (active ? r : 0) * rs;
+    double acc = 0.0;
+    if (active && j < T) {
+      int32_t t = j;
+      uint32_t k = (uint32_t)__ldg(&a.img.root[t]);
+      for (;;) {
+        const uint2 nd = __ldg(&nodes[k]);
+        if ((int32_t)nd.y < 0) {
+          acc += (double)__uint_as_float(nd.x);
+          t += P;
+          if (t >= T) break;
+          k = (uint32_t)__ldg(&a.img.root[t]);
+        } else {
+          k += step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask);
+        }
+      }
+    }
+    // fixed-order combine of the row's P chains (lanes j = 0..P-1 are adjacent)
+#pragma unroll
+    for (int o = 1; o < P; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (active && j == 0) {
+      const int64_t i = r0 + r;
+      if (FUSED) write_scalar(a.o, i, acc);
+      else a.o.raw[i] += acc;
+    }
+  }
+}
+
 // ------------------------------------------------------------------ sliced strategy
 // Sliced node words (encode.cpp): x = threshold (internal) or leaf value;
 //   internal y = off_bytes << (F+3) | default_left << (F+2) | attribute << 2   (left child next)
@@ -769,19 +821,52 @@ static cudaError_t direct_tiled_one(const DirectKArgs& a, int32_t rs, int32_t nu
   return cudaGetLastError();
 }
 
+template <bool F, int P>
+static cudaError_t direct_tlp_one(const DirectKArgs& a, int32_t rs, int32_t num_sms,
+                                  cudaStream_t st) {
+  constexpr int kRows = 128;
+  auto kern = k_direct_tlp<F, kRows, P>;
+  const int smem = kRows * rs * 4;
+  static std::atomic<int> configured[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64 && configured[dev].load() < smem) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+    if (e != cudaSuccess) return e;
+    configured[dev].store(kMaxSmemOptin);
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kRows * P, smem);
+  if (per_sm < 1) per_sm = 1;
+  const int64_t ntiles = (a.n + kRows - 1) / kRows;
+  const int grid = (int)std::min<int64_t>(ntiles, (int64_t)num_sms * per_sm);
+  kern<<<grid, kRows * P, smem, st>>>(a, rs);
+  return cudaGetLastError();
+}
+
 int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                   bool fused, int32_t num_sms, void* stream) {
   DirectKArgs a{img, X, n, d, o};
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
   // 0 = rows read from global memory; 1 = staged rows, warp-lockstep over trees;
-  // 2 = staged rows, free-running over trees
-  // default: staged rows, free-running (2) for large batches — attribute reads from shared memory
-  // leave L1/L2 to the nodes (C2 1M: 6.2 -> 4.9 ms, C3 1M: 15.9 -> 14.7 ms); rows from global
-  // memory (0) for small batches (lower launch cost) and for rows too wide to stage
+  // 2 = staged rows, free-running over trees; 3 / 4 = staged rows, 2 / 4 threads per row
+  // Default for large batches: staged rows — attribute reads from shared memory leave L1/L2 to
+  // the nodes — with two threads per row for scalar outputs (3; C5 500-tree shard 300K rows:
+  // 10.05 ms rows-global -> 9.75 ms staged -> 5.96 ms two threads per row; four threads per row
+  // thrash L1: 8.13 ms) and one thread per row, free-running, otherwise (2).  Rows from global
+  // memory (0) for small batches (lower launch cost) and for rows too wide to stage.
+  const bool scalar = o.n_classes == 1 && o.agg != TAHOE_AGG_VOTE;
   const char* env = std::getenv("TAHOE_DIRECT_VARIANT");
-  int variant = env ? std::atoi(env) : (n >= 32768 ? 2 : 0);
+  int variant = env ? std::atoi(env) : (n >= 32768 ? (scalar && !leaf ? 3 : 2) : 0);
   if (d > 256) variant = 0;  // 128 staged rows must fit shared memory
+  if ((variant == 3 || variant == 4) && scalar && !leaf) {
+    const int32_t rs = d | 1;
+    cudaError_t e;
+    if (variant == 3) e = fused ? direct_tlp_one<true, 2>(a, rs, num_sms, st) : direct_tlp_one<false, 2>(a, rs, num_sms, st);
+    else e = fused ? direct_tlp_one<true, 4>(a, rs, num_sms, st) : direct_tlp_one<false, 4>(a, rs, num_sms, st);
+    return (int)e;
+  }
   if (variant == 1 || variant == 2) {
     const int32_t rs = d | 1;  // odd stride: lanes on different rows spread over the banks
     cudaError_t e;

@@ -313,3 +313,26 @@ def test_direct_chunked_image_parity(monkeypatch):
         res = _gpu_run(F, X, T.STRATEGY_DIRECT, want_leaf=False)   # fused-finalize path
         _check(res, ref, f["agg"], True, want_leaf=False)
         F.close()
+
+
+@pytest.mark.parametrize("cid,ntrees,variant", [(2, 120, None), (5, 60, None), (2, 120, "4"),
+                                                (5, 60, "2"), (5, 60, "1")])
+def test_direct_large_batch_variants(cid, ntrees, variant, monkeypatch):
+    """Large-batch direct kernels (staged rows; two or four threads per row for scalar outputs,
+    one thread per row free-running or warp-lockstep) against the oracle, scores and classes
+    bit-exact with dyadic leaves, >= 32K rows with a ragged last tile."""
+    if variant is not None:
+        monkeypatch.setenv("TAHOE_DIRECT_VARIANT", variant)
+    f = gen.make_forest(cid, n_trees=ntrees)
+    F = T.Forest(f, base_score=0.5, device=0).layout(gen.make_calibration(cid, 4096))
+    n = 40_001
+    X = gen.make_rows(cid, n)
+    X[::7, 3] = np.nan
+    ref = oracle.predict(f, X, base_score=0.5)
+    _check(_gpu_run(F, X, T.STRATEGY_DIRECT, want_leaf=False), ref, f["agg"], True, want_leaf=False)
+    dev = torch.device("cuda", 0)
+    part = F.predict_partial(torch.from_numpy(X).to(dev))   # raw path (no fused finalize)
+    torch.cuda.synchronize()
+    # partials carry no base score; the oracle's raw margin does (dyadic: both exact)
+    assert np.array_equal(part.cpu().numpy(), ref["raw"] - 0.5), "dyadic partial sums are exact"
+    F.close()

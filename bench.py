@@ -46,54 +46,99 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region (B200_PROFILING.md)."""
+    """SM clocks and clock-event (throttle) reasons sampled DURING the timed region
+    (B200_PROFILING.md clocks line): NVML every 10 ms in a thread (the device is found by PCI bus
+    id, so CUDA and NVML orderings cannot disagree); nvidia-smi -lms 50 if NVML is unavailable."""
+
+    _REASONS = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+                ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+                ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+                ("hw_power_brake", "nvmlClocksEventReasonHwPowerBrakeSlowdown"),
+                ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"))
 
     def __init__(self, index: int):
         self.index = index
-        self.rows = []
+        self.sm, self.mx, self.reasons = [], [], set()
         self.proc = None
         self.thread = None
+        self.stop_flag = threading.Event()
+        self.nvml = None
+
+    def _handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        try:
+            import torch
+            pr = torch.cuda.get_device_properties(self.index)
+            bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            return pynvml, pynvml.nvmlDeviceGetHandleByPciBusId(bus.encode())
+        except Exception:
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.index)
 
     def start(self):
+        try:
+            nv, h = self._handle()
+            self.nvml = (nv, h)
+            self.mx.append(float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)))
+        except Exception:
+            self.nvml = None
+        if self.nvml:
+            self.thread = threading.Thread(target=self._poll_nvml, daemon=True)
+            self.thread.start()
+            return
         q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
              "clocks_event_reasons.sw_power_cap")
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
-                 "--format=csv,noheader,nounits", "-lms", "200"],
+                 "--format=csv,noheader,nounits", "-lms", "50"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except Exception:
             self.proc = None
             return
-        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread = threading.Thread(target=self._read_smi, daemon=True)
         self.thread.start()
 
-    def _read(self):
+    def _poll_nvml(self):
+        nv, h = self.nvml
+        while not self.stop_flag.is_set():
+            try:
+                self.sm.append(float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)))
+                bits = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                for name, attr in self._REASONS:
+                    if bits & getattr(nv, attr, 0):
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            self.stop_flag.wait(0.01)
+
+    def _read_smi(self):
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for line in self.proc.stdout:
-            parts = [p.strip() for p in line.split(",")]
-            if len(parts) >= 7:
-                self.rows.append(parts)
+            r = [p.strip() for p in line.split(",")]
+            if len(r) >= 7 and r[0].replace(".", "").isdigit():
+                self.sm.append(float(r[0]))
+                if r[1].replace(".", "").isdigit():
+                    self.mx.append(float(r[1]))
+                self.reasons.update(names[j] for j in range(4) if r[3 + j] == "Active")
 
     def stop(self) -> dict | None:
-        if not self.proc:
-            return None
-        time.sleep(0.15)
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=2)
-        except Exception:
-            self.proc.kill()
+        self.stop_flag.set()
+        if self.proc:
+            time.sleep(0.06)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
         if self.thread:
             self.thread.join(timeout=2)
-        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[j] for r in self.rows for j in range(4) if r[3 + j] == "Active"})
-        if not sm:
+        if not self.sm:
             return None
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(sm)}
+        return {"sm_mhz": statistics.median(self.sm), "sm_max_mhz": max(self.mx) if self.mx else None,
+                "reasons": sorted(self.reasons), "samples": len(self.sm),
+                "source": "nvml 10 ms" if self.nvml else "nvidia-smi 50 ms"}
 
 
 def build_workload(cfg, rank: int, n: int):
@@ -263,7 +308,7 @@ def _config(cfg, n, stats):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", type=int, default=2)
@@ -343,16 +388,15 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     sampler.start()
-    time.sleep(0.2)
     wall0 = time.perf_counter()
     for k in range(args.steps):
         step(ev[k])
         flush.zero_()   # L2 flush between timed steps (outside the step events)
     torch.cuda.synchronize()
     wall = time.perf_counter() - wall0
+    clocks = sampler.stop()
     if world > 1:
         dist.barrier()
-    clocks = sampler.stop()
     step_ms = [e[0].elapsed_time(e[1]) for e in ev]
     kern_ms = [e[2].elapsed_time(e[3]) for e in ev]
     tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=coll_dev)

@@ -169,6 +169,119 @@ static bool pack_best(const Forest& F, const std::vector<int32_t>& trees, int32_
   return true;
 }
 
+// Nodes read per (calibration row, tree) — the kernel's step count for that walk (a single-leaf
+// tree is a 3-node stump: 2 steps).  Empty when no rows were kept.
+static std::vector<int32_t> sim_reads(const Forest& F, int64_t& m) {
+  m = F.Xsim.empty() ? 0 : (int64_t)F.Xsim.size() / F.dsim;
+  std::vector<int32_t> reads((size_t)m * F.n_trees);
+  for (int64_t r = 0; r < m; r++) {
+    const float* x = &F.Xsim[(size_t)r * F.dsim];
+    for (int32_t t = 0; t < F.n_trees; t++) {
+      int32_t k = F.node_base[t], c = 1;
+      while (F.feat[k] >= 0) {
+        const float v = x[F.feat[k]];
+        const bool left = std::isnan(v) ? F.dl[k] != 0 : v < F.thr[k];
+        k = left ? F.lc[k] : F.rc[k];
+        c++;
+      }
+      reads[(size_t)r * F.n_trees + t] = (F.tree_size(t) == 1) ? 2 : c;
+    }
+  }
+  return reads;
+}
+
+// Work units balanced on measured paths ("loads are roughly balanced", reading R6): a
+// warp walks 4 rows x 16 lane columns in lockstep and waits for the longest of the 64 walks, so
+// the cost of a packing on the kept calibration rows is sum over 4-row units of the maximum
+// column work.  Greedy local search from the expected-work packing: tree swaps / moves between a
+// unit's bottleneck column and another column, accepted when the cost drops and the slot cap
+// holds.  Deterministic (fixed-seed generator).
+static int kRefineIters = std::getenv("TAHOE_REFINE_ITERS") ? std::atoi(std::getenv("TAHOE_REFINE_ITERS")) : 200;
+static void pack_refine(const Forest& F, const std::vector<int32_t>& reads, int64_t m, int32_t cap,
+                        Pack& P) {
+  const int32_t C = kSlicedCols;
+  const int64_t U = m / 4;
+  if (U < 4) return;
+  const int32_t T = F.n_trees;
+  std::vector<double> W((size_t)m * C, 0.0);         // W[r][c]
+  std::vector<int32_t> len(C, 0);
+  for (int32_t c = 0; c < C; c++)
+    for (int32_t t : P.lanes[c]) {
+      len[c] += enc_size(F, t);
+      for (int64_t r = 0; r < m; r++) W[(size_t)r * C + c] += reads[(size_t)r * T + t];
+    }
+  auto colmax = [&](int64_t u, int32_t c, const double* wa) {   // max over the unit's rows
+    double mx = 0;
+    for (int64_t q = 4 * u; q < 4 * u + 4; q++) mx = std::max(mx, wa ? wa[q] : W[(size_t)q * C + c]);
+    return mx;
+  };
+  std::vector<double> M((size_t)U * C), umax(U);
+  for (int64_t u = 0; u < U; u++) {
+    umax[u] = 0;
+    for (int32_t c = 0; c < C; c++) { M[(size_t)u * C + c] = colmax(u, c, nullptr); umax[u] = std::max(umax[u], M[(size_t)u * C + c]); }
+  }
+  uint64_t st = 0x9E3779B97F4A7C15ull;
+  auto rnd = [&](uint64_t lim) {
+    st += 0x9E3779B97F4A7C15ull;
+    uint64_t z = st;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return (z ^ (z >> 31)) % lim;
+  };
+  std::vector<double> na(m), nb(m), Ma(U), Mb(U);
+  const int iters = kRefineIters * (int)std::max<size_t>(1, [&] { size_t k = 0; for (auto& L : P.lanes) k += L.size(); return k; }());
+  for (int it = 0; it < iters; it++) {
+    const int64_t u0 = (int64_t)rnd((uint64_t)U);
+    int32_t a = 0;
+    for (int32_t c = 1; c < C; c++) if (M[(size_t)u0 * C + c] > M[(size_t)u0 * C + a]) a = c;
+    if (P.lanes[a].empty()) continue;
+    const int32_t b = (a + 1 + (int32_t)rnd(C - 1)) % C;
+    const size_t ia = rnd(P.lanes[a].size());
+    const bool move = P.lanes[b].empty() || rnd(4) == 0;
+    const size_t ib = move ? 0 : rnd(P.lanes[b].size());
+    const int32_t ta = P.lanes[a][ia], tb = move ? -1 : P.lanes[b][ib];
+    const int32_t sa = enc_size(F, ta), sb = move ? 0 : enc_size(F, tb);
+    if (len[a] - sa + sb > cap || len[b] - sb + sa > cap) continue;
+    for (int64_t r = 0; r < m; r++) {
+      const double ra = reads[(size_t)r * T + ta], rb = move ? 0.0 : reads[(size_t)r * T + tb];
+      na[r] = W[(size_t)r * C + a] - ra + rb;
+      nb[r] = W[(size_t)r * C + b] - rb + ra;
+    }
+    double delta = 0;
+    for (int64_t u = 0; u < U; u++) {
+      Ma[u] = colmax(u, a, na.data());
+      Mb[u] = colmax(u, b, nb.data());
+      double mx = std::max(Ma[u], Mb[u]);
+      for (int32_t c = 0; c < C; c++) if (c != a && c != b) mx = std::max(mx, M[(size_t)u * C + c]);
+      delta += mx - umax[u];
+    }
+    if (delta >= 0) continue;
+    // accept
+    if (move) {
+      P.lanes[a].erase(P.lanes[a].begin() + (long)ia);
+      P.lanes[b].push_back(ta);
+    } else {
+      std::swap(P.lanes[a][ia], P.lanes[b][ib]);
+    }
+    len[a] += sb - sa;
+    len[b] += sa - sb;
+    for (int64_t r = 0; r < m; r++) { W[(size_t)r * C + a] = na[r]; W[(size_t)r * C + b] = nb[r]; }
+    for (int64_t u = 0; u < U; u++) {
+      M[(size_t)u * C + a] = Ma[u];
+      M[(size_t)u * C + b] = Mb[u];
+      double mx = 0;
+      for (int32_t c = 0; c < C; c++) mx = std::max(mx, M[(size_t)u * C + c]);
+      umax[u] = mx;
+    }
+  }
+  // keep each column's trees in similarity order
+  std::vector<int32_t> rank((size_t)T, 0);
+  for (size_t q = 0; q < F.order.size(); q++) rank[(size_t)F.order[q]] = (int32_t)q;
+  for (auto& L : P.lanes)
+    std::sort(L.begin(), L.end(), [&](int32_t x, int32_t y) { return rank[x] < rank[y]; });
+  pack_stats(F, P);
+}
+
 tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   S = SlicedImage();
   S.fbits = feature_bits(F.n_features + 1);   // all-ones attribute field marks a leaf
@@ -178,6 +291,11 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   for (int32_t t = 0; t < F.n_trees; t++)
     if (enc_size(F, t) > cap) { S.why_invalid = "a tree exceeds one lane column of shared memory"; return TAHOE_OK; }
 
+  int64_t m = 0;
+  const std::vector<int32_t> reads = sim_reads(F, m);
+  static const char* pack_mode = std::getenv("TAHOE_PACK");          // experiments: fixed packer
+  const bool refine = m >= 16 && F.opts.tree_group != 0 && !pack_mode &&
+                      !(std::getenv("TAHOE_PACK_REFINE") && std::string(std::getenv("TAHOE_PACK_REFINE")) == "0");
   std::vector<std::vector<int32_t>> groups(F.n_classes);
   for (int32_t t : F.order) groups[F.tclass[t]].push_back(t);
   std::vector<Pack> packs;
@@ -210,7 +328,12 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
         std::vector<int32_t> chunk(G.begin() + cut[j], G.begin() + cut[j + 1]);
         Pack P;
         if (!pack_best(F, chunk, cap, P)) ok = false;
-        else { ps.push_back(P); S.cls.push_back(c); S.ntrees.push_back((int32_t)chunk.size()); }
+        else {
+          if (refine) pack_refine(F, reads, m, cap, P);
+          ps.push_back(P);
+          S.cls.push_back(c);
+          S.ntrees.push_back((int32_t)chunk.size());
+        }
       }
       if (ok) { packs.insert(packs.end(), ps.begin(), ps.end()); break; }
       S.cls.resize(packs.size());
@@ -230,22 +353,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   // Simulated lockstep efficiency of k_sliced (two rows per warp, two steps per exit test) on the
   // kept calibration rows: useful node reads / lane-steps issued.  Falls back to 0.75 x expected.
   S.eff_sim = S.eff * 0.75;
-  if (!F.Xsim.empty()) {
-    const int64_t m = (int64_t)F.Xsim.size() / F.dsim;
-    std::vector<int32_t> reads((size_t)m * F.n_trees);
-    for (int64_t r = 0; r < m; r++) {
-      const float* x = &F.Xsim[(size_t)r * F.dsim];
-      for (int32_t t = 0; t < F.n_trees; t++) {
-        int32_t k = F.node_base[t], c = 1;
-        while (F.feat[k] >= 0) {
-          const float v = x[F.feat[k]];
-          const bool left = std::isnan(v) ? F.dl[k] != 0 : v < F.thr[k];
-          k = left ? F.lc[k] : F.rc[k];
-          c++;
-        }
-        reads[(size_t)r * F.n_trees + t] = (F.tree_size(t) == 1) ? 2 : c;
-      }
-    }
+  if (m > 0) {
     // a warp walks 4 rows at once (2 per half-warp x 2 chains); its loop runs until the slowest
     // of the 64 (row, column) walks ends, two steps per exit test
     double useful = 0, issued = 0;

@@ -302,3 +302,25 @@ def test_layout_from_counts_equals_layout_from_rows():
     assert np.array_equal(ea["nodes"], eb["nodes"])
     T.tahoe_forest_free(a)
     T.tahoe_forest_free(b)
+
+
+def test_pack_refine_improves_simulated_lockstep(monkeypatch):
+    """Reading R6: the measured-path local search never makes the packing's simulated cost worse
+    than the expected-work packing it starts from, and the image still decodes to the oracle."""
+    f = gen.make_forest(3, n_trees=140)
+    effs = {}
+    monkeypatch.setenv("TAHOE_SLOT_BUDGET", "600")   # host-only handle: give it a budget
+    for flag in ("0", "1"):
+        monkeypatch.setenv("TAHOE_PACK_REFINE", flag)
+        h = T.tahoe_forest_build(f, f["n_features"], f["n_classes"], f["agg"], 0.0, -1)
+        T.tahoe_forest_layout(h, gen.make_calibration(3, 4096))
+        st = T.tahoe_forest_stats(h)
+        assert st["sliced_valid"], st["sliced_why"]
+        effs[flag] = st["lockstep_eff_sim"]
+        if flag == "1":
+            X = gen.make_rows(3, 40)
+            img = T.tahoe_forest_export_sliced(h)
+            leaf, _ = decode_sliced(img, X, len(f["root"]), f["n_classes"])
+            assert np.array_equal(leaf, oracle.predict(f, X, want_leaf=True)["leaf"])
+        T.tahoe_forest_free(h)
+    assert effs["1"] >= effs["0"] - 1e-12, effs

@@ -104,8 +104,10 @@ typedef struct {
  * tahoe_forest_layout — Algorithm 1 lines 5-7 on the host: count how many of the
  * n_calib calibration rows take each edge (edge / node probability), put the more
  * probable child of every node next to it (probability-based node rearrangement),
- * order trees by SimHash/LSH similarity and deal them into balanced work units, then
- * re-encode and re-upload.  X_calib_host: HOST pointer, n_calib x d row-major float32.
+ * order trees by SimHash/LSH similarity and deal them into balanced work units
+ * (expected-work packing, then a local search on the measured paths of up to 1024 of the rows,
+ * reading R6), then re-encode and re-upload.  X_calib_host: HOST pointer, n_calib x d row-major
+ * float32.
  * opts may be NULL (defaults).  Mutates the handle: must not overlap predictions on it.
  * Results of later predictions are unchanged bit for bit (leaf ids, classes; sums are fp64).
  */
@@ -127,7 +129,8 @@ tahoe_status tahoe_count_visits(const tahoe_forest* f, const float* X, int64_t n
  * tahoe_forest_layout_counts — tahoe_forest_layout driven by visit counts measured elsewhere
  * (e.g. tahoe_count_visits on live traffic; re-layout for incremental updates).
  * counts: HOST uint64[n_nodes] by caller node id over n_calib rows.  X_sim_host (n_sim x d, may be
- * NULL) feeds the lockstep-efficiency simulation of the cost model.
+ * NULL; up to 1024 rows are kept) feeds the lockstep simulation of the cost model and the
+ * measured-path balancing of lane columns (reading R6).
  */
 tahoe_status tahoe_forest_layout_counts(tahoe_forest* f, const uint64_t* counts, int64_t n_calib,
                                         const float* X_sim_host, int64_t n_sim, int32_t d,

@@ -412,7 +412,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_layout(
   if (n_calib > 0) {
     calibrate(F, X_calib_host, n_calib, d);
     // keep an evenly spaced subsample of the calibration rows for the lockstep simulation
-    const int64_t m = std::min<int64_t>(n_calib, 512);
+    const int64_t m = std::min<int64_t>(n_calib, 1024);
     F.dsim = d;
     F.Xsim.resize((size_t)m * d);
     for (int64_t r = 0; r < m; r++)
@@ -463,7 +463,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_layout_counts(
   F.Xsim.clear();
   F.dsim = 0;
   if (n_sim > 0) {
-    const int64_t m = std::min<int64_t>(n_sim, 512);
+    const int64_t m = std::min<int64_t>(n_sim, 1024);
     F.dsim = d;
     F.Xsim.resize((size_t)m * d);
     for (int64_t r = 0; r < m; r++)

@@ -43,7 +43,7 @@ struct Forest {
   std::vector<uint8_t> hot_left;    // 1 = left child is the hot child
   std::vector<double> exp_reads;    // per tree: expected nodes read per sample (incl. leaf)
   std::vector<int32_t> order;       // tree order (class-major, similarity order within class)
-  std::vector<float> Xsim;          // <= 512 calibration rows kept to simulate lockstep efficiency
+  std::vector<float> Xsim;          // <= 1024 calibration rows kept to simulate and balance lockstep work
   int32_t dsim = 0;
   tahoe_layout_opts opts{};
 

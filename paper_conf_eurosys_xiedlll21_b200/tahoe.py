@@ -422,14 +422,14 @@ class Forest:
 
     def layout_gpu(self, X_calib_dev, **kw):
         """Layout from visit counts measured on the GPU (tahoe_count_visits) over the device rows
-        X_calib_dev; a host copy of up to 512 of them feeds the cost model's simulation."""
+        X_calib_dev; a host copy of up to 1024 of them feeds the lockstep simulation and balancing."""
         import torch
         n, d = X_calib_dev.shape
         cnt = torch.zeros(self.n_nodes, dtype=torch.int32, device=X_calib_dev.device)
         tahoe_count_visits(self.handle, X_calib_dev, n, d, cnt)
         counts = cnt.cpu().numpy().view(np.uint32).astype(np.uint64)
-        step = max(1, n // 512)
-        X_sim = X_calib_dev[::step][:512].cpu().numpy()
+        step = max(1, n // 1024)
+        X_sim = X_calib_dev[::step][:1024].cpu().numpy()
         opts = None
         if kw:
             opts = LayoutOpts(kw.get("t_nodes", 0), kw.get("l_hash", 0), kw.get("m_chunks", 0),

@@ -336,3 +336,31 @@ def test_direct_large_batch_variants(cid, ntrees, variant, monkeypatch):
     # partials carry no base score; the oracle's raw margin does (dyadic: both exact)
     assert np.array_equal(part.cpu().numpy(), ref["raw"] - 0.5), "dyadic partial sums are exact"
     F.close()
+
+
+def test_full_size_c5_full_forest_fused_reduce():
+    """BASELINE C5 in bench.py's N=1 launch configuration: the full 4000-tree forest (323 MB
+    direct image, walked in L2-sized chunks, two threads per row) over all 10M rows through the
+    fused reduce (world-1 NCCL communicator), sampled rows checked one by one against the oracle."""
+    cfg = gen.CONFIGS[5]
+    f = gen.make_forest(5, leaf_mode="normal")
+    full = T.Forest(f, device=-1).layout(gen.make_calibration(5))
+    S = full.shard(0, 1, device=0)
+    assert S.stats()["direct_chunks"] > 1
+    try:
+        comm = T.Comm(T.tahoe_comm_unique_id(), 1, 0, 0)
+    except T.TahoeError as e:  # pragma: no cover
+        pytest.skip(f"NCCL device API unavailable: {e}")
+    n = cfg.n_samples
+    X = gen.make_rows(5, n)
+    dev = torch.device("cuda", 0)
+    Xd = torch.from_numpy(X).to(dev)
+    out = S.predict_reduce(comm, Xd, mode=T.REDUCE_ALL)
+    torch.cuda.synchronize()
+    idx = gen.subsample(1005, n, 400)
+    ref = oracle.predict(f, X, rows=idx)
+    _check(dict(out=out.cpu().numpy()[idx], cls=np.zeros(len(idx), np.int32)), ref, f["agg"], False,
+           want_leaf=False)
+    comm.close()
+    S.close()
+    del Xd

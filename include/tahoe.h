@@ -54,9 +54,17 @@ typedef enum {
 typedef enum {
   TAHOE_STRATEGY_AUTO = -1,   /* cost model (Algorithm 1 lines 8-13)                          */
   TAHOE_STRATEGY_DIRECT = 0,  /* lane = sample; forest image in HBM/L2 (paper's "direct")     */
-  TAHOE_STRATEGY_SLICED = 1   /* lane = tree; forest slices resident in shared memory, sample
+  TAHOE_STRATEGY_SLICED = 1,  /* lane = tree; forest slices resident in shared memory, sample
                                  tiles staged by TMA ("shared forest" / "splitting shared
                                  forest")                                        */
+  TAHOE_STRATEGY_SLICED_CODED = 2  /* SLICED over exact rank codes of the attributes (DESIGN.md
+                                 reading R7; same results bit for bit): a pre-pass turns each
+                                 row into u16 codes, the slices compare codes with threshold
+                                 ranks.  AUTO takes it instead of SLICED when the forest
+                                 qualifies (<= 127 attributes, <= 32000 distinct thresholds per
+                                 attribute, no subnormal leaf value) and no leaf ids or
+                                 fingerprints are requested; forcing it otherwise returns
+                                 E_UNSUPPORTED                                                */
 } tahoe_strategy;
 
 /*

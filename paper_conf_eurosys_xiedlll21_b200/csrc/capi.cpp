@@ -93,6 +93,11 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->ds.col_len);
   cudaFree((void*)f->ds.slots);
   cudaFree((void*)f->ds.leaf_meta);
+  cudaFree((void*)f->ds.cnodes);
+  cudaFree((void*)f->ds.thr_tab);
+  cudaFree((void*)f->ds.thr_off);
+  cudaFree((void*)f->ds.cb_img);
+  cudaFree((void*)f->ds.cb_desc);
   cudaFree(f->d_class_ptr);
   cudaFree(f->d_class_parts);
   f->dd = DevDirect();
@@ -173,6 +178,19 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
     f->ds.n_slices = f->sl.n_slices;
     f->ds.slots_max = f->sl.slots_max;
     f->ds.fbits = f->sl.fbits;
+    if (f->sl.code_valid) {
+      if ((st = upload(f->sl.cnodes, &f->ds.cnodes)) != TAHOE_OK) return st;
+      if ((st = upload(f->sl.thr_tab, &f->ds.thr_tab)) != TAHOE_OK) return st;
+      if ((st = upload(f->sl.thr_off, &f->ds.thr_off)) != TAHOE_OK) return st;
+      f->ds.n_features = f->host.n_features;
+      f->ds.n_thr = f->sl.thr_off.back();
+      if (!f->sl.cb_img.empty()) {
+        if ((st = upload(f->sl.cb_img, &f->ds.cb_img)) != TAHOE_OK) return st;
+        if ((st = upload(f->sl.cb_desc, &f->ds.cb_desc)) != TAHOE_OK) return st;
+        f->ds.cb_rows = f->sl.cb_rows;
+        f->ds.cb_passes = f->sl.cb_passes;
+      }
+    }
   }
   return TAHOE_OK;
 }
@@ -219,7 +237,14 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
   }
   if (forced == TAHOE_STRATEGY_DIRECT) return TAHOE_STRATEGY_DIRECT;
   if (forced == TAHOE_STRATEGY_SLICED) return f->sl.valid ? TAHOE_STRATEGY_SLICED : -2;
-  return select_strategy(plan_stats(f, d), n, d, f->host.agg);
+  if (forced == TAHOE_STRATEGY_SLICED_CODED)
+    return !f->sl.valid ? -2 : (f->ds.cnodes ? TAHOE_STRATEGY_SLICED_CODED : -3);
+  const int32_t s = select_strategy(plan_stats(f, d), n, d, f->host.agg);
+  // the rank-coded twin of the sliced strategy wherever the forest qualifies (reading R7);
+  // $TAHOE_CODES=0 keeps the fp32 slices (experiments)
+  static const bool codes_off = std::getenv("TAHOE_CODES") && std::string(std::getenv("TAHOE_CODES")) == "0";
+  if (s == TAHOE_STRATEGY_SLICED && f->ds.cnodes && !codes_off) return TAHOE_STRATEGY_SLICED_CODED;
+  return s;
 }
 
 static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int64_t n, int32_t d) {
@@ -258,8 +283,14 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
                         int32_t forced, cudaStream_t st, void* ev_b = nullptr, void* ev_e = nullptr) {
   const Forest& H = f->host;
   const int32_t C = H.n_out();
-  const int32_t strat = choose(f, n, d, forced);
+  int32_t strat = choose(f, n, d, forced);
   if (strat == -2) return fail(TAHOE_E_UNSUPPORTED, "sliced strategy unavailable: " + f->sl.why_invalid);
+  if (strat == -3) return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices unavailable: " + f->sl.code_why);
+  if (strat == TAHOE_STRATEGY_SLICED_CODED && (out_leaf || out_fp)) {
+    if (forced == TAHOE_STRATEGY_SLICED_CODED)
+      return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices produce no leaf ids / fingerprints");
+    strat = TAHOE_STRATEGY_SLICED;   // leaf diagnostics run on the fp32 slices
+  }
   cudaError_t e;
   if (out_fp && (e = cudaMemsetAsync(out_fp, 0, (size_t)n * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
   OutArgs o;
@@ -328,9 +359,24 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync partial");
     o.raw = part;
   }
-  if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
-  int rc = launch_sliced(f->ds, plan, X, n, d, o, fused, st);
-  if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+  int rc;
+  if (strat == TAHOE_STRATEGY_SLICED_CODED) {
+    const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
+    const size_t cbytes = (size_t)ntiles * code_tile_bytes(f->sl.fbits);
+    void* cbuf = nullptr;
+    if ((e = scratch_alloc(&cbuf, cbytes + (size_t)ntiles * 4, st)) != cudaSuccess) {
+      if (part) cudaFreeAsync(part, st);
+      return fail(TAHOE_E_NOMEM, "cudaMallocAsync code tiles");
+    }
+    rc = launch_sliced_codes(f->ds, plan, X, n, d, static_cast<uint16_t*>(cbuf),
+                             reinterpret_cast<int32_t*>(static_cast<char*>(cbuf) + cbytes), o, fused,
+                             f->num_sms, st, ev_b, ev_e);
+    cudaFreeAsync(cbuf, st);
+  } else {
+    if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+    rc = launch_sliced(f->ds, plan, X, n, d, o, fused, st);
+    if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+  }
   if (rc) { if (part) cudaFreeAsync(part, st); return cuda_fail((cudaError_t)rc, "sliced kernel"); }
   if (!fused) {
     fa.partial = part;
@@ -699,6 +745,10 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"bytes_fixed_index\":" << (int64_t)H.feat.size() * 12
      << ",\"sliced_valid\":" << (f->sl.valid ? "true" : "false")
      << ",\"sliced_why\":\"" << f->sl.why_invalid << "\""
+     << ",\"coded_valid\":" << (f->sl.code_valid ? "true" : "false")
+     << ",\"coded_why\":\"" << f->sl.code_why << "\"" << ",\"coded_thresholds\":"
+     << (f->sl.thr_off.empty() ? 0 : f->sl.thr_off.back())
+     << ",\"code_bank_rows\":" << f->sl.cb_rows << ",\"code_bank_passes\":" << f->sl.cb_passes
      << ",\"n_slices\":" << f->sl.n_slices << ",\"slots_max\":" << f->sl.slots_max
      << ",\"slot_budget\":" << f->slot_budget << ",\"sliced_bytes\":" << f->sl.bytes()
      << ",\"lockstep_eff\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim

@@ -73,6 +73,8 @@ const CostParams& cost_params() {
 
 double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
   const CostParams& c = cost_params();
+  // the rank-coded twin (reading R7) is costed as the fp32 slices it replaces (conservative)
+  if (strategy == TAHOE_STRATEGY_SLICED_CODED) strategy = TAHOE_STRATEGY_SLICED;
   if (strategy == TAHOE_STRATEGY_SLICED) {
     if (!st.sliced_ok || st.n_slices < 1) return INFINITY;
     const int64_t tiles = (n + 63) / 64;

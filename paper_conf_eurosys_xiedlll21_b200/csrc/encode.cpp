@@ -282,6 +282,113 @@ static void pack_refine(const Forest& F, const std::vector<int32_t>& reads, int6
   pack_stats(F, P);
 }
 
+// Bank-private threshold tables for k_encode_rows_banks (reading R7).  A warp codes one row per
+// pass: lane l of pass p bisects the sorted thresholds of one attribute, and every attribute of a
+// pass owns its own set of m = 2^sh shared-memory banks {b, b + 32/m, b + 2*32/m, ...}: element i
+// sits at word (region * 32 + b + i * 32/m), so the probe address is one multiply-add and the 32
+// probes of a warp never collide, whatever the row values are.  Bank sets are handed out largest
+// first (aligned blocks of the bit-reversed bank index, so they never fragment).  Passes = 2^F / 32
+// code slots (at least 1); lanes without an attribute write a pad slot.  Spare banks go to the
+// attributes with the most thresholds (halving their depth); the attributes are split over passes
+// in decreasing order of threshold count, trying every size of the first pass.  The image is used
+// when it fits kCodeBankBudget bytes of shared memory.
+static void build_code_banks(const std::vector<std::vector<float>>& tabs, int32_t fbits,
+                             SlicedImage& S) {
+  S.cb_img.clear();
+  S.cb_desc.clear();
+  S.cb_passes = 0;
+  S.cb_rows = 0;
+  const int32_t nf = (int32_t)tabs.size();
+  const int32_t slots = 1 << fbits;
+  const int32_t P = std::max(1, slots / 32);
+  std::vector<int32_t> ord(nf);
+  std::iota(ord.begin(), ord.end(), 0);
+  std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return tabs[a].size() > tabs[b].size(); });
+  // one pass: spare-bank doubling, returns depth (rows) and per-feature shift
+  auto plan_pass = [&](const std::vector<int32_t>& fs, std::vector<int32_t>& sh) -> int64_t {
+    sh.assign(fs.size(), 0);
+    int32_t spare = 32 - (int32_t)fs.size();
+    for (;;) {
+      int64_t best = -1;
+      size_t bi = 0;
+      for (size_t q = 0; q < fs.size(); q++) {
+        const int64_t m = 1 << sh[q];
+        const int64_t depth = ((int64_t)tabs[fs[q]].size() + m - 1) / m;
+        if (m <= spare && sh[q] < 5 && depth > best) { best = depth; bi = q; }
+      }
+      if (best <= 1) break;
+      spare -= 1 << sh[bi];
+      sh[bi]++;
+    }
+    int64_t D = 0;
+    for (size_t q = 0; q < fs.size(); q++)
+      D = std::max<int64_t>(D, ((int64_t)tabs[fs[q]].size() + (1 << sh[q]) - 1) >> sh[q]);
+    return D;
+  };
+  std::vector<std::vector<int32_t>> best_fs;
+  int64_t best_rows = INT64_MAX;
+  const int32_t lo0 = std::max(1, nf - 32 * (P - 1)), hi0 = std::min(32, nf);
+  for (int32_t n0 = (nf == 0 ? 0 : lo0); n0 <= (nf == 0 ? 0 : hi0); n0++) {
+    std::vector<std::vector<int32_t>> fs(P);
+    fs[0].assign(ord.begin(), ord.begin() + n0);
+    const int32_t rest = nf - n0;
+    for (int32_t q = 0; q < rest; q++) fs[1 + (q * (P - 1)) / std::max(1, rest)].push_back(ord[n0 + q]);
+    bool ok = true;
+    int64_t rows = 0;
+    for (auto& g : fs) {
+      if ((int32_t)g.size() > 32) { ok = false; break; }
+      std::vector<int32_t> sh;
+      rows += plan_pass(g, sh);
+    }
+    if (ok && rows < best_rows) { best_rows = rows; best_fs = fs; }
+  }
+  if (best_fs.empty() || best_rows * 128 > kCodeBankBudget) return;
+  S.cb_passes = P;
+  S.cb_rows = (int32_t)best_rows;
+  S.cb_img.assign((size_t)best_rows * 32, 0.0f);
+  S.cb_desc.assign((size_t)P * 32 * 4, -1);
+  // pad slots: every code slot that no attribute writes
+  std::vector<int32_t> pads;
+  for (int32_t j = nf; j < std::max(slots, 32); j++) pads.push_back(j);
+  size_t pad_i = 0;
+  int64_t region = 0;
+  for (int32_t p = 0; p < P; p++) {
+    std::vector<int32_t> sh;
+    const int64_t D = plan_pass(best_fs[p], sh);
+    // bank sets, largest first: m banks {b + k * 32/m}, b the smallest base whose set is free
+    std::vector<size_t> by_m(best_fs[p].size());
+    std::iota(by_m.begin(), by_m.end(), 0);
+    std::stable_sort(by_m.begin(), by_m.end(), [&](size_t a, size_t b) { return sh[a] > sh[b]; });
+    uint32_t used = 0;
+    int32_t lane = 0;
+    for (size_t q : by_m) {
+      const int32_t m = 1 << sh[q], stride = 32 / m;
+      int32_t b = 0;
+      for (; b < stride; b++) {
+        uint32_t set = 0;
+        for (int32_t k = 0; k < m; k++) set |= 1u << (b + k * stride);
+        if (!(used & set)) { used |= set; break; }
+      }
+      const int32_t a = best_fs[p][q];
+      const auto& v = tabs[a];
+      for (size_t i = 0; i < v.size(); i++) S.cb_img[(size_t)region * 32 + b + i * stride] = v[i];
+      int32_t* d = &S.cb_desc[((size_t)p * 32 + lane++) * 4];
+      d[0] = a;                                            // code slot written
+      d[1] = a;                                            // attribute read
+      d[2] = (int32_t)((region * 32 + b) * 4);             // byte offset of element 0
+      d[3] = ((stride * 4) << 16) | (int32_t)v.size();     // element stride (bytes) | K
+    }
+    for (; lane < 32; lane++) {
+      int32_t* d = &S.cb_desc[((size_t)p * 32 + lane) * 4];
+      if (pad_i < pads.size()) d[0] = pads[pad_i++];
+      d[1] = -1;
+      d[2] = 0;
+      d[3] = 0;
+    }
+    region += D;
+  }
+}
+
 tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   S = SlicedImage();
   S.fbits = feature_bits(F.n_features + 1);   // all-ones attribute field marks a leaf
@@ -382,7 +489,42 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   static_assert(kSlotBytes == 128, "slot row is 128 bytes");
   const uint32_t off_lim = 1u << (32 - (S.fbits + 3) - sb);
   const size_t per_slice = (size_t)S.slots_max * C;
+  // Rank codes (reading R7): per attribute the sorted distinct thresholds (IEEE equality, so -0.0
+  // and +0.0 are one value); a node's threshold b = tab[j] is stored as t = j + 1, and
+  // x < b  <=>  #{k : tab[k] <= x} < j + 1, exactly.  Requires F <= 7 (rows of <= 128 u16 codes),
+  // at most kCodeMaxRank distinct thresholds per attribute, and no subnormal leaf value (the
+  // kernel adds internal words, which are subnormal as floats, with flush-to-zero).
+  S.code_valid = true;
+  S.code_why.clear();
+  if (S.fbits > kCodeMaxFbits) { S.code_valid = false; S.code_why = "too many attributes for u16 code rows"; }
+  std::vector<std::vector<float>> tabs(F.n_features);
+  if (S.code_valid) {
+    for (size_t k = 0; k < F.feat.size(); k++) {
+      if (F.feat[k] >= 0) tabs[F.feat[k]].push_back(F.thr[k]);
+      else if (std::fpclassify(F.val[k]) == FP_SUBNORMAL) { S.code_valid = false; S.code_why = "subnormal leaf value"; }
+    }
+    S.thr_off.assign(F.n_features + 1, 0);
+    for (int32_t a = 0; a < F.n_features && S.code_valid; a++) {
+      auto& v = tabs[a];
+      std::sort(v.begin(), v.end(), [](float p, float q) { return p < q; });
+      v.erase(std::unique(v.begin(), v.end(), [](float p, float q) { return p == q; }), v.end());
+      if ((int32_t)v.size() > kCodeMaxRank) { S.code_valid = false; S.code_why = "too many distinct thresholds for one attribute"; }
+      S.thr_off[a + 1] = S.thr_off[a] + (int32_t)v.size();
+    }
+    if (S.code_valid) {
+      S.thr_tab.reserve(S.thr_off[F.n_features]);
+      for (auto& v : tabs) S.thr_tab.insert(S.thr_tab.end(), v.begin(), v.end());
+      build_code_banks(tabs, S.fbits, S);
+    }
+  }
+  auto rank_of = [&](int32_t a, float b) -> uint32_t {   // t = j + 1
+    const auto& v = tabs[a];
+    const size_t j = (size_t)(std::lower_bound(v.begin(), v.end(), b, [](float p, float q) { return p < q; }) - v.begin());
+    return (uint32_t)j + 1u;
+  };
+  const int32_t csh = S.fbits + 2;   // code words: off_bytes << (F+2) | dl << (F+1) | attribute << 1
   S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
+  if (S.code_valid) S.cnodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
   S.col_len.assign((size_t)S.n_slices * C, 0);
   S.slots.assign(S.n_slices, 0);
@@ -402,10 +544,16 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
           const uint32_t yleaf1 = (2u << sb) << (S.fbits + 3) | (fmask << 2);
           const uint32_t yleaf2 = (1u << sb) << (S.fbits + 3) | (fmask << 2);
           const uint32_t ys[3] = {ynode, yleaf1, yleaf2};
+          const uint32_t cys[3] = {(2u << sb) << csh, (2u << sb) << csh | (fmask << 1),
+                                   (1u << sb) << csh | (fmask << 1)};
           for (int32_t q = 0; q < 3; q++) {
             const size_t w = ((size_t)s * per_slice + (size_t)(pos + q) * C + l);
             S.nodes[2 * w] = q == 0 ? 0u : f2u(F.val[k]);
             S.nodes[2 * w + 1] = ys[q];
+            if (S.code_valid) {   // stump root: both children hold the same leaf, any rank will do
+              S.cnodes[2 * w] = q == 0 ? 1u : f2u(F.val[k]);
+              S.cnodes[2 * w + 1] = cys[q];
+            }
             if (q > 0) { S.leaf_meta[2 * w] = F.tree_orig[t]; S.leaf_meta[2 * w + 1] = F.orig[k]; }
           }
           pos += 3;
@@ -424,11 +572,13 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
           const int32_t k = pre[i];
           const int32_t sl = pos + (int32_t)i;
           const size_t w = ((size_t)s * per_slice + (size_t)sl * C + l);
-          uint32_t y;
+          uint32_t y, cy;
           if (F.feat[k] < 0) {
             if ((uint32_t)(next_root - sl) >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "leaf offset overflow");
             y = ((uint32_t)(next_root - sl) << (S.fbits + 3 + sb)) | (fmask << 2);
+            cy = ((uint32_t)(next_root - sl) << (csh + sb)) | (fmask << 1);
             S.nodes[2 * w] = f2u(F.val[k]);
+            if (S.code_valid) S.cnodes[2 * w] = f2u(F.val[k]);
             S.leaf_meta[2 * w] = F.tree_orig[t];
             S.leaf_meta[2 * w + 1] = F.orig[k];
           } else {
@@ -437,9 +587,13 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
             if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "right offset overflow");
             y = ((uint32_t)delta << (S.fbits + 3 + sb)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 2)) |
                 ((uint32_t)F.feat[k] << 2);
+            cy = ((uint32_t)delta << (csh + sb)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 1)) |
+                 ((uint32_t)F.feat[k] << 1);
             S.nodes[2 * w] = f2u(F.thr[k]);
+            if (S.code_valid) S.cnodes[2 * w] = rank_of(F.feat[k], F.thr[k]);
           }
           S.nodes[2 * w + 1] = y;
+          if (S.code_valid) S.cnodes[2 * w + 1] = cy;
         }
         pos = next_root;
       }
@@ -447,6 +601,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
       const size_t w = ((size_t)s * per_slice + (size_t)pos * C + l);
       S.nodes[2 * w] = 0u;
       S.nodes[2 * w + 1] = fmask << 2;
+      if (S.code_valid) { S.cnodes[2 * w] = 0u; S.cnodes[2 * w + 1] = fmask << 1; }
       S.col_len[(size_t)s * C + l] = pos;
     }
   }

@@ -88,6 +88,19 @@ struct SlicedImage {
   double eff = 0.0;                              // est. lockstep efficiency (mean/max column)
   double eff_sim = 0.0;                          // simulated 2-chain lockstep efficiency
   double trees_per_lane = 0.0;
+  // Rank-coded twin of `nodes` (reading R7): same slots and packing, internal x = threshold rank
+  // t = j + 1 (j = index of the threshold in its attribute's sorted distinct thresholds), attribute
+  // field a byte offset into rows of u16 codes; thr_tab/thr_off hold the sorted thresholds.
+  bool code_valid = false;
+  std::string code_why;
+  std::vector<uint32_t> cnodes;                  // [ns*slots_max*16*2]
+  std::vector<float> thr_tab;                    // concatenated sorted distinct thresholds
+  std::vector<int32_t> thr_off;                  // [n_features + 1]
+  // bank-private threshold tables for the row-coding pre-pass (encode.cpp build_code_banks);
+  // empty when they do not fit shared memory (the pre-pass then bisects thr_tab through L2)
+  std::vector<float> cb_img;                     // [cb_rows][32] words: the shared-memory image
+  std::vector<int32_t> cb_desc;                  // [passes][32 lanes] {slot, attribute, word0, sh<<16|K}
+  int32_t cb_passes = 0, cb_rows = 0;
   int64_t bytes() const { return (int64_t)nodes.size() * 4; }
 };
 

@@ -715,6 +715,366 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   }
 }
 
+// ------------------------------------------------------------------ rank-coded sliced strategy
+// Reading R7: "x_j < b_i" is evaluated on exact order-preserving codes.  Per attribute
+// the forest's distinct thresholds are sorted (tab); a row value x becomes
+// code(x) = #{k : tab[k] <= x}, and a node whose threshold is tab[j] stores t = j + 1, so that
+// x < tab[j]  <=>  code(x) < t  — the same decision, bit for bit, for every x (NaN is coded
+// kCodeNan and takes the default path; ties and signed zeros follow IEEE <=).  Two things get
+// cheaper on the hot loop: an attribute read is 2 bytes, so the two rows a warp walks at once share
+// one 128-byte bank line (1 shared-memory wavefront instead of 2), and an internal node word
+// (t < 2^15) is a subnormal float, so "add the leaf value" becomes an unconditional
+// flush-to-zero fp32 add of the word just read (internal words add exactly 0).
+
+// k_encode_rows: X (n x d fp32 row-major) -> code tiles.  One thread per (row, code slot); the
+// attribute's threshold table is searched by bisection in shared memory (or L2 when too large).
+struct EncodeRowsArgs {
+  const float* X;
+  int64_t n;
+  int32_t d, nf, fbits, rb, n_thr;
+  const float* tab;
+  const int32_t* off;
+  uint16_t* codes;
+  int32_t* nan_flags;
+  int64_t ntiles;
+};
+
+__device__ __forceinline__ uint32_t code_row_off(int r, int rb) {
+  return rb == 64 ? (((uint32_t)(r & 15) << 7) | ((uint32_t)((r >> 4) & 1) << 6) | ((uint32_t)(r >> 5) << 11))
+                  : (uint32_t)r * (uint32_t)rb;
+}
+
+template <bool SMEM>
+__global__ void __launch_bounds__(1024) k_encode_rows(const EncodeRowsArgs a) {
+  extern __shared__ __align__(16) float s_tab[];
+  const float* __restrict__ tab = a.tab;
+  const int32_t* __restrict__ off = a.off;
+  if (SMEM) {
+    int32_t* s_off = reinterpret_cast<int32_t*>(s_tab + a.n_thr);
+    for (int i = threadIdx.x; i < a.n_thr; i += blockDim.x) s_tab[i] = __ldg(&a.tab[i]);
+    for (int i = threadIdx.x; i <= a.nf; i += blockDim.x) s_off[i] = __ldg(&a.off[i]);
+    __syncthreads();
+    tab = s_tab;
+    off = s_off;
+  }
+  const int64_t total = a.ntiles * 64 << a.fbits;
+  const int smask = (1 << a.fbits) - 1;
+  const int64_t tile_u16 = (int64_t)32 * a.rb;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = e >> a.fbits;
+    const int j = (int)(e & smask);
+    uint16_t code = kCodePad;
+    if (r < a.n && j < a.nf) {
+      const float x = __ldg(&a.X[r * a.d + j]);
+      if (x != x) {
+        code = kCodeNan;
+        a.nan_flags[r >> 6] = 1;
+      } else {
+        const int32_t b0 = off[j];
+        int32_t lo = b0, len = off[j + 1] - b0;
+        while (len > 0) {   // lo := first index with tab[lo] > x
+          const int32_t h = len >> 1;
+          if (tab[lo + h] <= x) { lo += h + 1; len -= h + 1; }
+          else len = h;
+        }
+        code = (uint16_t)(lo - b0);
+      }
+    }
+    a.codes[(r >> 6) * tile_u16 + (code_row_off((int)(r & 63), a.rb) >> 1) + j] = code;
+  }
+}
+
+// k_encode_rows_banks: the same codes from bank-private tables (encode.cpp build_code_banks): the
+// CTA bulk-copies the table image into shared memory once; warp w codes rows w, w + W, ... one pass
+// at a time, lane l of pass p bisecting attribute desc[p][l] inside its own banks (one wavefront
+// per probe for the whole warp).
+struct EncodeBanksArgs {
+  const float* X;
+  int64_t n;
+  int32_t d, rb, passes, img_bytes;
+  const float* img;
+  const int4* desc;
+  uint16_t* codes;
+  int32_t* nan_flags;
+  int64_t nrows;   // ntiles * 64
+};
+
+__global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanksArgs a) {
+  extern __shared__ __align__(1024) float s_img[];
+  __shared__ uint64_t s_bar;
+  const int lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    mbar_init(&s_bar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    fence_proxy_async_smem();
+    mbar_expect_tx(&s_bar, (uint32_t)a.img_bytes);
+    bulk_g2s_big(s_img, a.img, (uint32_t)a.img_bytes, &s_bar);
+  }
+  mbar_wait(&s_bar, 0);
+  const int64_t tile_u16 = (int64_t)32 * a.rb;
+  // a warp codes kRowsPerWarp rows at once (independent bisections interleaved, the next group's
+  // attribute values loaded before this group is searched): the pre-pass is latency-bound
+  constexpr int kR = 4;
+  const int64_t wstride = (int64_t)gridDim.x * (blockDim.x >> 5) * kR;
+  const int64_t w0 = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * kR;
+  for (int p = 0; p < a.passes; p++) {
+    const int4 dsc = __ldg(&a.desc[p * 32 + lane]);
+    const int slot = dsc.x, feat = dsc.y;
+    const uint32_t base = smem_u32(s_img) + (uint32_t)dsc.z;   // element 0 of this lane's table
+    const uint32_t stride = (uint32_t)dsc.w >> 16;               // bytes between elements
+    const uint32_t lstride = 31u - __clz(stride | 1u);           // stride is a power of two
+    const int K = dsc.w & 0xffff;
+    int top = 0;   // largest power of two <= K (0 for K = 0)
+    if (K > 0) top = 1 << (31 - __clz(K));
+    auto load_x = [&](int64_t r0, float* x) {
+#pragma unroll
+      for (int q = 0; q < kR; q++)
+        x[q] = (feat >= 0 && r0 + q < a.n) ? __ldg(&a.X[(r0 + q) * a.d + feat]) : 0.0f;
+    };
+    float xn[kR];
+    load_x(w0, xn);
+    for (int64_t r0 = w0; r0 < a.nrows; r0 += wstride) {
+      float x[kR];
+#pragma unroll
+      for (int q = 0; q < kR; q++) x[q] = xn[q];
+      if (r0 + wstride < a.nrows) load_x(r0 + wstride, xn);
+      // pos := #{thresholds <= x} by Shar's bisection (uniform trip count for every row of this
+      // lane, every probe in range, no bounds tests): after the first probe at top - 1 the count
+      // lies in [pos, pos + top]; each halving step keeps it in [pos, pos + step]; a last probe
+      // at pos decides between pos and pos + 1.
+      // (positions are kept as byte offsets, pos * stride, so a probe address is one add)
+      uint32_t pos[kR];
+      if (top > 0) {
+        const uint32_t a0 = base + (uint32_t)(top - 1) * stride;
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          float v;
+          asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a0));
+          pos[q] = v <= x[q] ? (uint32_t)(K - top) * stride : 0u;
+        }
+        for (uint32_t stepb = ((uint32_t)top >> 1) * stride; stepb >= stride; stepb >>= 1) {
+          const uint32_t as = base + stepb - stride;
+#pragma unroll
+          for (int q = 0; q < kR; q++) {
+            float v;
+            asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(as + pos[q]));
+            pos[q] += v <= x[q] ? stepb : 0u;
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          float v;
+          asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(base + pos[q]));
+          pos[q] = (pos[q] >> lstride) + (v <= x[q] ? 1u : 0u);
+        }
+      } else {
+#pragma unroll
+        for (int q = 0; q < kR; q++) pos[q] = 0;
+      }
+#pragma unroll
+      for (int q = 0; q < kR; q++) {
+        const int64_t r = r0 + q;
+        if (r >= a.nrows) break;
+        uint16_t code = kCodePad;
+        if (feat >= 0 && r < a.n) {
+          if (x[q] != x[q]) {
+            code = kCodeNan;
+            a.nan_flags[r >> 6] = 1;
+          } else {
+            code = (uint16_t)pos[q];
+          }
+        }
+        if (slot >= 0) a.codes[(r >> 6) * tile_u16 + (code_row_off((int)(r & 63), a.rb) >> 1) + slot] = code;
+      }
+    }
+  }
+}
+
+struct CodedKArgs {
+  DevSliced img;
+  const uint16_t* codes;
+  const int32_t* nan_flags;
+  int64_t n;
+  int32_t forest_smem;   // bytes reserved for the slice (multiple of 1024)
+  int32_t tile_bytes;    // one 64-row code tile
+  int32_t rb;            // bytes per code row
+  int32_t cps;           // CTAs per slice (single-pass)
+  OutArgs o;
+};
+
+// One step on a coded slice: node {x = t or leaf value, y}, attribute code at (y & amask) | row,
+// left iff code < t (NaN-aware: or NaN and default-left), right / next root at +(y >> (F+2)).
+// Returns the node word as a float: the leaf value, or a subnormal (flushed to 0 by the add).
+template <bool NAN_AWARE>
+__device__ __forceinline__ float coded_step(uint32_t& p, uint32_t rowaddr, uint32_t amask,
+                                            uint32_t dlbit, uint32_t shmul) {
+  uint32_t x, y;
+  int32_t c;
+  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+  asm("ld.shared.s16 %0, [%1];" : "=r"(c) : "r"((y & amask) | rowaddr));
+  bool go_left = (uint32_t)c < x;
+  if (NAN_AWARE) go_left = go_left || ((c == (int32_t)(int16_t)kCodeNan) && (y & dlbit));
+  p += go_left ? (uint32_t)kSlotBytes : __umulhi(y, shmul);
+  return __uint_as_float(x);
+}
+
+// flush-to-zero fp32 add of two consecutive step words (internal words are subnormal -> +0; at
+// most one of two consecutive steps meets a leaf), then one fp64 add: exact.
+__device__ __forceinline__ void add_pair_ftz(double& acc, float v1, float v2) {
+  float s;
+  asm("add.rn.ftz.f32 %0, %1, %2;" : "=f"(s) : "f"(v1), "f"(v2));
+  double dv;
+  asm("cvt.f64.f32 %0, %1;" : "=d"(dv) : "f"(s));
+  acc += dv;
+}
+
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t pe, uint32_t rowA,
+                                            uint32_t rowB, uint32_t amask, uint32_t dlbit,
+                                            uint32_t shmul, double& accA, double& accB) {
+  accA = 0.0;
+  accB = 0.0;
+  while ((pA != pe) | (pB != pe)) {
+    const float a1 = coded_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul);
+    const float b1 = coded_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul);
+    const float a2 = coded_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul);
+    const float b2 = coded_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul);
+    add_pair_ftz(accA, a1, a2);
+    add_pair_ftz(accB, b1, b2);
+  }
+}
+
+// k_sliced_codes: k_sliced's persistent slice-stationary schedule (slice in shared memory, 3-deep
+// ring of 64-row tiles refilled by the warp that finishes a tile, dynamic 4-row work units, one
+// half-warp per row, two chains per lane) over code tiles (one 1-D bulk copy per tile).
+template <bool FUSED>
+__global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant__ CodedKArgs a) {
+  constexpr int C = kSlicedCols;
+  extern __shared__ __align__(1024) unsigned char smem[];
+  unsigned char* s_ring = smem + a.forest_smem;
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)kRing * a.tile_bytes);
+  uint64_t* s_forest = s_full + kRing;
+  int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
+  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
+  const int lane = threadIdx.x & 31;
+  const int warp = threadIdx.x >> 5;
+  const int col = lane & (C - 1);
+  const int half = lane >> 4;
+  const uint32_t F = (uint32_t)a.img.fbits;
+  const uint32_t amask = ((1u << F) - 1u) << 1;
+  const uint32_t dlbit = 1u << (F + 1);
+  const uint32_t shmul = 1u << (32 - (F + 2));
+  const int32_t ns = a.img.n_slices;
+  const int32_t G = gridDim.x;
+  const bool multipass = ns > G;
+  const int64_t R = kSlicedTileRows;
+  const int64_t ntiles = (a.n + R - 1) / R;
+
+  if (threadIdx.x == 0) {
+    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; }
+    *s_next = 0ull;
+    mbar_init(s_forest, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+
+  auto issue_tile = [&](int64_t tile, int b) {
+    if (lane == 0) {
+      fence_proxy_async_smem();
+      mbar_expect_tx(&s_full[b], (uint32_t)a.tile_bytes);
+      bulk_g2s(s_ring + (size_t)b * a.tile_bytes,
+               reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tile_bytes,
+               (uint32_t)a.tile_bytes, &s_full[b]);
+    }
+    __syncwarp();
+  };
+  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts) {
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) {
+      __threadfence_block();
+      last = atomicAdd(&s_cnt[b], 1) == units - 1;
+      if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
+    }
+    last = __shfl_sync(0xffffffffu, last, 0);
+    if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+  };
+
+  uint32_t g = 0;
+  uint32_t ph_forest = 0;
+  const uint32_t ring0 = smem_u32(s_ring);
+  for (int32_t sl = multipass ? (int32_t)blockIdx.x : (int32_t)blockIdx.x % ns; sl < ns;
+       sl += multipass ? G : ns) {
+    const int64_t t0 = multipass ? 0 : blockIdx.x / ns;
+    const int64_t ts = multipass ? 1 : a.cps;
+    const int64_t my_tiles = t0 < ntiles ? (ntiles - t0 + ts - 1) / ts : 0;
+    if (warp == 0) {
+      if (lane == 0) {
+        const uint32_t bytes = (uint32_t)a.img.slots[sl] * (uint32_t)kSlotBytes;
+        fence_proxy_async_smem();
+        mbar_expect_tx(s_forest, bytes);
+        bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
+      }
+      for (int64_t q = 0; q < kRing && q < my_tiles; q++) issue_tile(t0 + q * ts, (int)((g + q) % kRing));
+    }
+    const uint32_t sbase = smem_u32(smem);
+    const uint32_t p0 = sbase + (uint32_t)col * 8u;
+    const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+    mbar_wait(s_forest, ph_forest);
+    ph_forest ^= 1u;
+
+    constexpr int kUnits = kSlicedTileRows / 4;
+    const uint64_t total = (uint64_t)my_tiles * kUnits;
+    for (;;) {
+      unsigned long long q = 0;
+      if (lane == 0) q = atomicAdd(s_next, 1ull);
+      q = __shfl_sync(0xffffffffu, q, 0);
+      if (q >= total) break;
+      const int64_t it = (int64_t)(q / kUnits);
+      const int u = (int)(q % kUnits);
+      const uint32_t gt = g + (uint32_t)it;
+      const int b = (int)(gt % kRing);
+      const int64_t tile = t0 + it * ts;
+      const int64_t r0 = tile * R;
+      const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+      mbar_wait(&s_full[b], (gt / kRing) & 1u);
+      if (u < nr) {
+        const int rA = u + 16 * half, rB = rA + 32;
+        const bool okA = rA < nr, okB = rB < nr;
+        const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
+        const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tile_bytes;
+        const uint32_t rowA = tb + code_row_off(okA ? rA : u, a.rb);
+        const uint32_t rowB = tb + code_row_off(okB ? rB : u, a.rb);
+        double accA, accB;
+        if (__ldg(&a.nan_flags[tile]))
+          walk_coded2<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        else
+          walk_coded2<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        // a9: the k_sliced butterfly (lanes 0, 8, 16, 24 own rows u, u+32, u+16, u+48)
+        const bool b3 = lane & 8;
+        double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
+#pragma unroll
+        for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        const int rr = b3 ? rB : rA;
+        if ((lane & 7) == 0 && (b3 ? okB : okA)) {
+          const int64_t i = r0 + rr;
+          if (FUSED) write_scalar(a.o, i, v);
+          else a.o.raw[(size_t)sl * a.n + i] = v;
+        }
+      }
+      release(b, kUnits, it, my_tiles, t0, ts);
+    }
+    g += (uint32_t)my_tiles;
+    __syncthreads();
+    if (threadIdx.x == 0) *s_next = 0ull;
+    __syncthreads();
+  }
+}
+
 static int grid_for(int64_t n, int block, int num_sms, int per_sm);
 
 // ------------------------------------------------------------------ visit counting
@@ -967,6 +1327,106 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
   cudaError_t e;
   if (leaf) e = fused ? sliced_rows<true, true>(a, plan, st) : sliced_rows<true, false>(a, plan, st);
   else e = fused ? sliced_rows<false, true>(a, plan, st) : sliced_rows<false, false>(a, plan, st);
+  return (int)e;
+}
+
+int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
+                        int32_t d, uint16_t* codes, int32_t* nan_flags, const OutArgs& o,
+                        bool fused, int32_t num_sms, void* stream, void* ev_b, void* ev_e) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
+  cudaError_t e = cudaMemsetAsync(nan_flags, 0, (size_t)ntiles * 4, st);
+  if (e != cudaSuccess) return (int)e;
+  EncodeRowsArgs ea;
+  ea.X = X;
+  ea.n = n;
+  ea.d = d;
+  ea.nf = img.n_features;
+  ea.fbits = img.fbits;
+  ea.rb = code_row_bytes(img.fbits);
+  ea.n_thr = img.n_thr;
+  ea.tab = img.thr_tab;
+  ea.off = img.thr_off;
+  ea.codes = codes;
+  ea.nan_flags = nan_flags;
+  ea.ntiles = ntiles;
+  const int64_t tab_bytes = (int64_t)img.n_thr * 4 + (int64_t)(img.n_features + 1) * 4;
+  const int64_t elems = ntiles * kSlicedTileRows << img.fbits;
+  const int blk = 1024;
+  // $TAHOE_CODE_BANKS=0: bisect through L2 instead (tests cover both pre-pass kernels)
+  const bool banks_off = std::getenv("TAHOE_CODE_BANKS") && std::atoi(std::getenv("TAHOE_CODE_BANKS")) == 0;
+  if (img.cb_img && !banks_off) {
+    EncodeBanksArgs ba;
+    ba.X = X;
+    ba.n = n;
+    ba.d = d;
+    ba.rb = code_row_bytes(img.fbits);
+    ba.passes = img.cb_passes;
+    ba.img_bytes = img.cb_rows * 128;
+    ba.img = img.cb_img;
+    ba.desc = reinterpret_cast<const int4*>(img.cb_desc);
+    ba.codes = codes;
+    ba.nan_flags = nan_flags;
+    ba.nrows = ntiles * kSlicedTileRows;
+    static std::atomic<int> configured[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && !configured[dev].load()) {
+      // static + dynamic shared memory must stay within the opt-in limit (the kernel's mbarrier
+      // is static)
+      e = cudaFuncSetAttribute(k_encode_rows_banks, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               kMaxSmemOptin - 1024);
+      if (e != cudaSuccess) return (int)e;
+      configured[dev].store(1);
+    }
+    const int64_t warps_needed = (ba.nrows + 3) / 4;
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(num_sms, (warps_needed + 31) / 32));
+    k_encode_rows_banks<<<grid, blk, ba.img_bytes, st>>>(ba);
+  } else if (tab_bytes <= 200 * 1024) {
+    static std::atomic<int> configured[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && !configured[dev].load()) {
+      e = cudaFuncSetAttribute(k_encode_rows<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+      if (e != cudaSuccess) return (int)e;
+      configured[dev].store(1);
+    }
+    const int smem = (int)((tab_bytes + 15) & ~15LL);
+    const int per_sm = smem <= 100 * 1024 ? 2 : 1;
+    k_encode_rows<true><<<grid_for((elems + 0) , blk, num_sms, per_sm), blk, smem, st>>>(ea);
+  } else {
+    k_encode_rows<false><<<grid_for(elems, blk, num_sms, 2), blk, 0, st>>>(ea);
+  }
+  if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
+
+  CodedKArgs a{};
+  a.img = img;
+  a.codes = codes;
+  a.nan_flags = nan_flags;
+  a.n = n;
+  a.forest_smem = plan.forest_smem;
+  a.tile_bytes = code_tile_bytes(img.fbits);
+  a.rb = code_row_bytes(img.fbits);
+  a.cps = plan.cps;
+  a.o = o;
+  const int smem = plan.forest_smem + kRing * a.tile_bytes + kSlicedBarrierBytes;
+  auto kern = fused ? k_sliced_codes<true> : k_sliced_codes<false>;
+  {
+    static std::atomic<int> configured[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && !configured[dev].load()) {
+      e = cudaFuncSetAttribute(k_sliced_codes<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+      if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_sliced_codes<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+      if (e != cudaSuccess) return (int)e;
+      configured[dev].store(1);
+    }
+  }
+  if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+  kern<<<plan.grid, 1024, smem, st>>>(a);
+  e = cudaGetLastError();
+  if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
   return (int)e;
 }
 

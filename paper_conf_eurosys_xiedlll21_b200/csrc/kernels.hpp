@@ -38,7 +38,34 @@ struct DevSliced {
   int32_t n_slices = 0;
   int32_t slots_max = 0;
   int32_t fbits = 0;
+  // rank-coded twin (reading R7); cnodes == nullptr when the forest does not qualify
+  const uint32_t* cnodes = nullptr;  // [ns][slots_max][16] uint2
+  const float* thr_tab = nullptr;    // sorted distinct thresholds, attribute after attribute
+  const int32_t* thr_off = nullptr;  // [n_features + 1]
+  int32_t n_features = 0;            // attributes coded per row
+  int32_t n_thr = 0;                 // thr_off[n_features]
+  const float* cb_img = nullptr;     // bank-private tables (cb_rows x 32 words) or nullptr
+  const int32_t* cb_desc = nullptr;  // [cb_passes][32] int4
+  int32_t cb_rows = 0, cb_passes = 0;
 };
+
+// ------------------------------------------------------------------ rank-coded rows (reading R7)
+// A sample row becomes u16 codes: code(x) = #{distinct thresholds of the attribute <= x}
+// (< kCodeMaxRank), NaN -> kCodeNan; slots n_features .. 2^F - 1 hold kCodePad.  Loaded
+// sign-extended, kCodeNan / kCodePad are 0xFFFFFFFE / 0xFFFFFFFF, larger than every node word,
+// so "code < t" sends NaN right (its default path is applied separately) and a leaf's pad read
+// never goes left.  A 64-row tile of code rows is kCodeTileRows * code_row_bytes(F) bytes; with
+// 64-byte rows, row r sits at ((r & 15) << 7) | (((r >> 4) & 1) << 6) | ((r >> 5) << 11), so
+// the rows u and u + 16 that the two half-warps of a warp walk together occupy the two halves of
+// one 128-byte bank line (conflict-free attribute loads).
+constexpr int32_t kCodeMaxRank = 32000;
+constexpr int32_t kCodeMaxFbits = 7;
+constexpr int32_t kCodeBankBudget = 216 * 1024;   // shared memory for the bank-private tables
+constexpr uint16_t kCodeNan = 0xFFFEu;
+constexpr uint16_t kCodePad = 0xFFFFu;
+inline int32_t code_row_bytes(int32_t fbits) { return (2 << fbits) < 64 ? 64 : (2 << fbits); }
+inline int32_t code_tile_bytes(int32_t fbits) { return 64 * code_row_bytes(fbits); }
+inline int64_t code_ring_bytes(int32_t fbits) { return (int64_t)3 * code_tile_bytes(fbits); }
 
 struct OutArgs {
   float* out = nullptr;          // final scores (fused finalize) or nullptr
@@ -107,6 +134,11 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
                   bool fused, int32_t num_sms, void* stream);
 int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                   int32_t d, const OutArgs& o, bool fused, void* stream);
+// rank-coded sliced strategy: encode X into code tiles (codes: ntiles * code_tile_bytes bytes,
+// nan_flags: ntiles ints, both device scratch), then walk the coded slices
+int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
+                        int32_t d, uint16_t* codes, int32_t* nan_flags, const OutArgs& o,
+                        bool fused, int32_t num_sms, void* stream, void* ev_b, void* ev_e);
 int launch_finalize(const FinalizeArgs& a, void* stream);
 int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t d,
                         uint32_t* counts, int32_t num_sms, void* stream);

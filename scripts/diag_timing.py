@@ -16,8 +16,8 @@ X = torch.from_numpy(gen.make_rows(cid, n)).cuda()
 out = torch.empty((n, F.n_out), device="cuda")
 cls = torch.empty(n, dtype=torch.int32, device="cuda")
 s = torch.cuda.current_stream()
-for strat in (1, 0):
-    if strat == 1 and not F.stats()["sliced_valid"]:
+for strat in (2, 1, 0):
+    if (strat == 1 and not st["sliced_valid"]) or (strat == 2 and not st.get("coded_valid")):
         continue
     for _ in range(3):
         F.predict(X, out=out, out_class=cls, force_strategy=strat)

@@ -18,10 +18,27 @@ pytestmark = pytest.mark.gpu
 
 from paper_conf_eurosys_xiedlll21_b200 import tahoe as T  # noqa: E402
 
-STRATS = [T.STRATEGY_DIRECT, T.STRATEGY_SLICED]
+STRATS = [T.STRATEGY_DIRECT, T.STRATEGY_SLICED, T.STRATEGY_SLICED_CODED]
+
+
+def _usable(F, s):
+    st = F.stats()
+    if s == T.STRATEGY_SLICED:
+        return st["sliced_valid"]
+    if s == T.STRATEGY_SLICED_CODED:
+        return st["sliced_valid"] and st["coded_valid"]
+    return True
+
+
+def _strats(F):
+    return [s for s in STRATS if _usable(F, s)]
 
 
 def _gpu_run(F, X, strategy, want_leaf=True):
+    """Predict through the C ABI with `strategy` forced.  The rank-coded slices produce no leaf
+    ids / fingerprints (E_UNSUPPORTED), so they run scores + classes only."""
+    if strategy == T.STRATEGY_SLICED_CODED:
+        want_leaf = False
     dev = torch.device("cuda", 0)
     Xd = torch.from_numpy(X).to(dev)
     n = X.shape[0]
@@ -39,7 +56,7 @@ def _gpu_run(F, X, strategy, want_leaf=True):
 
 
 def _check(res, ref, agg, exact, want_leaf=True):
-    if want_leaf:
+    if want_leaf and "leaf" in res:
         assert np.array_equal(res["leaf"], ref["leaf"]), "leaf ids differ"
         assert np.array_equal(res["fp"], ref["fp"]), "fingerprints differ"
     if exact:
@@ -78,9 +95,7 @@ def test_parity_configs(cid, ntrees, n, mode, layout):
     if layout:
         F.layout(gen.make_calibration(cid, 4096))
     ref = oracle.predict(f, X, want_leaf=True)
-    for s in STRATS:
-        if s == T.STRATEGY_SLICED and not F.stats()["sliced_valid"]:
-            continue
+    for s in _strats(F):
         _check(_gpu_run(F, X, s), ref, f["agg"], mode == "dyadic")
 
 
@@ -89,7 +104,7 @@ def test_parity_c4_full_forest_subsample():
     X = gen.make_rows(4, 2003)
     F = T.Forest(f, device=0).layout(gen.make_calibration(4, 4096))
     ref = oracle.predict(f, X, want_leaf=True)
-    for s in STRATS:
+    for s in _strats(F):
         _check(_gpu_run(F, X, s), ref, f["agg"], True)
 
 
@@ -117,7 +132,7 @@ def test_edge_cases_nan_misaligned_wide_d_and_tiny_batches():
     X[::5, 3] = np.nan
     X[::11, :] = np.nan
     ref = oracle.predict(f, X, want_leaf=True)
-    for s in STRATS:
+    for s in _strats(F):
         _check(_gpu_run(F, X, s), ref, f["agg"], True)
     # misaligned X (offset by one float => no TMA) and wider rows than the forest needs
     dev = torch.device("cuda", 0)
@@ -125,13 +140,13 @@ def test_edge_cases_nan_misaligned_wide_d_and_tiny_batches():
     buf = torch.empty(Xw.size + 1, dtype=torch.float32, device=dev)
     buf[1:] = torch.from_numpy(Xw.ravel()).to(dev)
     Xm = buf[1:].view(Xw.shape)
-    for s in STRATS:
+    for s in _strats(F):
         out = torch.empty((X.shape[0], 1), dtype=torch.float32, device=dev)
         F.predict(Xm, out=out, force_strategy=s)
         torch.cuda.synchronize()
         assert np.array_equal(out.cpu().numpy(), ref["out"])
     for n in (0, 1, 31, 33, 64, 65):
-        for s in STRATS:
+        for s in _strats(F):
             Xd = torch.from_numpy(X[:n].copy()).to(dev)
             out = torch.full((n, 1), -1.0, dtype=torch.float32, device=dev)
             F.predict(Xd, out=out, force_strategy=s)
@@ -147,7 +162,7 @@ def test_aggregations_average_base_vote():
     for agg, base in ((oracle.AGG_AVERAGE, 0.625), (oracle.AGG_SUM, -2.0), (oracle.AGG_BINARY, 0.25)):
         F = T.Forest(f, n_features=5, n_classes=1, agg=agg, base_score=base, device=0)
         ref = oracle.predict(f, X, agg=agg, base_score=base, want_leaf=True)
-        for s in STRATS:
+        for s in _strats(F):
             _check(_gpu_run(F, X, s), ref, agg, True)
     C = 4
     fv = random_forest(rng, 40, 5, 5, n_classes=C, vote=True)
@@ -165,7 +180,7 @@ def test_layout_never_changes_results():
     for kw in (dict(), dict(node_reorder=0, tree_group=0), dict(node_reorder=1, tree_group=0),
                dict(t_nodes=2, l_hash=64, m_chunks=16)):
         F.layout(gen.make_calibration(3, 3000), **kw)
-        for s in STRATS:
+        for s in _strats(F):
             r = _gpu_run(F, X, s)
             _check(r, ref, f["agg"], True)
             outs.append(r["out"])
@@ -225,7 +240,7 @@ def test_single_leaf_trees_and_stumps():
     X = rng.normal(size=(2049, 6)).astype(np.float32)
     ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
     F = T.Forest(f, n_features=6, n_classes=1, agg=oracle.AGG_SUM, device=0)
-    for s in STRATS:
+    for s in _strats(F):
         _check(_gpu_run(F, X, s), ref, oracle.AGG_SUM, True)
 
 
@@ -293,7 +308,7 @@ def test_gpu_visit_counts_equal_oracle_and_drive_layout():
         assert np.array_equal(ia[k], ib[k]), k
     X = gen.make_rows(3, 2000)
     ref = oracle.predict(f, X, want_leaf=True)
-    for s in STRATS:
+    for s in _strats(F):
         _check(_gpu_run(F, X, s), ref, f["agg"], True)
 
 
@@ -364,3 +379,88 @@ def test_full_size_c5_full_forest_fused_reduce():
     comm.close()
     S.close()
     del Xd
+
+
+def test_rank_codes_threshold_ties_signed_zero_inf_nan():
+    """Reading R7: the rank-coded slices decide "x < b" exactly.  Rows are built from the forest's
+    own thresholds (x == b goes right), their float neighbours, -0.0 / +0.0, +-Inf and NaN (default
+    path from the node's default_left); a threshold of 0.0 is planted so signed zeros meet it.
+    Scores and classes are bit-exact against the oracle (dyadic leaves), and equal the fp32
+    slices and the direct strategy."""
+    rng = np.random.default_rng(77)
+    f = gen.make_forest(2, n_trees=96)
+    f = {k: (v.copy() if isinstance(v, np.ndarray) else v) for k, v in f.items()}
+    internal = np.flatnonzero(f["feature"] >= 0)
+    f["threshold"][internal[::17]] = 0.0
+    f["threshold"][internal[5::41]] = -0.0
+    f["default_left"][:] = rng.integers(0, 2, size=len(f["default_left"]))
+    F = T.Forest(f, device=0).layout(gen.make_calibration(2, 4096))
+    assert F.stats()["coded_valid"], F.stats()["coded_why"]
+    n, d = 9001, f["n_features"]
+    X = gen.make_rows(2, n)
+    thr_by_feat = [f["threshold"][internal[f["feature"][internal] == j]] for j in range(d)]
+    pick = rng.random(X.shape)
+    for j in range(d):
+        t = thr_by_feat[j]
+        if len(t) == 0:
+            continue
+        m = pick[:, j] < 0.35
+        v = rng.choice(t, size=m.sum())
+        kind = rng.integers(0, 3, size=m.sum())
+        v = np.where(kind == 1, np.nextafter(v, np.float32(np.inf)), v)
+        v = np.where(kind == 2, np.nextafter(v, np.float32(-np.inf)), v)
+        X[m, j] = v.astype(np.float32)
+    X[pick > 0.97] = -0.0
+    X[(pick > 0.95) & (pick <= 0.97)] = 0.0
+    X[(pick > 0.94) & (pick <= 0.95)] = np.inf
+    X[(pick > 0.93) & (pick <= 0.94)] = -np.inf
+    X[(pick > 0.92) & (pick <= 0.93)] = np.nan
+    ref = oracle.predict(f, X)
+    outs = []
+    for s in _strats(F):
+        r = _gpu_run(F, X, s, want_leaf=False)
+        _check(r, ref, f["agg"], True, want_leaf=False)
+        outs.append(r["out"])
+    assert len(outs) == 3 and all(np.array_equal(o, outs[0]) for o in outs)
+
+
+def test_rank_codes_eligibility_and_auto_choice():
+    """The coded twin exists when the forest qualifies (<= 127 attributes, no subnormal leaf) and
+    is refused (E_UNSUPPORTED) when forced with leaf-id outputs or on a forest that does not."""
+    f = gen.make_forest(2, n_trees=32)
+    F = T.Forest(f, device=0)
+    assert F.stats()["coded_valid"]
+    X = torch.from_numpy(gen.make_rows(2, 100)).cuda()
+    out = torch.empty((100, 1), dtype=torch.float32, device="cuda")
+    leaf = torch.empty((100, F.n_trees), dtype=torch.int32, device="cuda")
+    with pytest.raises(T.TahoeError):
+        F.predict(X, out=out, out_leaf=leaf, force_strategy=T.STRATEGY_SLICED_CODED)
+    g = {k: (v.copy() if isinstance(v, np.ndarray) else v) for k, v in f.items()}
+    leaves = np.flatnonzero(g["feature"] < 0)
+    g["leaf_value"][leaves[3]] = np.float32(1e-40)   # subnormal leaf value
+    G = T.Forest(g, device=0)
+    assert not G.stats()["coded_valid"]
+    with pytest.raises(T.TahoeError):
+        G.predict(X, out=out, force_strategy=T.STRATEGY_SLICED_CODED)
+    ref = oracle.predict(g, X.cpu().numpy())
+    G.predict(X, out=out)                                  # auto: fp32 slices or direct
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), ref["out"])
+
+
+@pytest.mark.parametrize("banks", ["1", "0"])
+@pytest.mark.parametrize("cid,ntrees,n", [(2, 120, 30011), (3, 210, 20011), (1, None, 1000)])
+def test_rank_code_prepass_kernels(cid, ntrees, n, banks, monkeypatch):
+    """Both row-coding pre-passes (bank-private tables in shared memory; bisection through L2) feed
+    the coded slices the same codes: scores and classes bit-exact against the oracle with NaN rows
+    and a ragged last tile."""
+    monkeypatch.setenv("TAHOE_CODE_BANKS", banks)
+    f = gen.make_forest(cid, n_trees=ntrees)
+    F = T.Forest(f, device=0).layout(gen.make_calibration(cid, 4096))
+    st = F.stats()
+    assert st["coded_valid"] and st["code_bank_rows"] > 0
+    X = gen.make_rows(cid, n)
+    X[::13, 1] = np.nan
+    ref = oracle.predict(f, X)
+    _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, f["agg"], True,
+           want_leaf=False)

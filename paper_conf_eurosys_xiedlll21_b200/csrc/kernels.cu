@@ -800,6 +800,7 @@ struct EncodeBanksArgs {
   int64_t nrows;   // ntiles * 64
 };
 
+template <bool RB64>
 __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanksArgs a) {
   extern __shared__ __align__(1024) float s_img[];
   __shared__ uint64_t s_bar;
@@ -815,12 +816,15 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
     bulk_g2s_big(s_img, a.img, (uint32_t)a.img_bytes, &s_bar);
   }
   mbar_wait(&s_bar, 0);
-  const int64_t tile_u16 = (int64_t)32 * a.rb;
-  // a warp codes kRowsPerWarp rows at once (independent bisections interleaved, the next group's
-  // attribute values loaded before this group is searched): the pre-pass is latency-bound
-  constexpr int kR = 4;
+  const int rb = RB64 ? 64 : a.rb;
+  const int64_t tile_u16 = (int64_t)32 * rb;
+  // a warp codes kR consecutive rows at once (independent bisections interleaved; the next
+  // group's attribute values are loaded before this group is searched)
+  constexpr int kR = 8;
+  static_assert(64 % kR == 0, "a row group stays inside one tile");
   const int64_t wstride = (int64_t)gridDim.x * (blockDim.x >> 5) * kR;
   const int64_t w0 = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * kR;
+  const uint32_t d = (uint32_t)a.d;
   for (int p = 0; p < a.passes; p++) {
     const int4 dsc = __ldg(&a.desc[p * 32 + lane]);
     const int slot = dsc.x, feat = dsc.y;
@@ -828,15 +832,20 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
     const uint32_t stride = (uint32_t)dsc.w >> 16;               // bytes between elements
     const uint32_t lstride = 31u - __clz(stride | 1u);           // stride is a power of two
     const int K = dsc.w & 0xffff;
-    int top = 0;   // largest power of two <= K (0 for K = 0)
-    if (K > 0) top = 1 << (31 - __clz(K));
+    const int top = K > 0 ? 1 << (31 - __clz(K)) : 0;            // largest power of two <= K
+    const float* Xf = a.X + (feat >= 0 ? feat : 0);
     auto load_x = [&](int64_t r0, float* x) {
+      const float* xr = Xf + r0 * a.d;
+      if (feat >= 0 && r0 + kR <= a.n) {
 #pragma unroll
-      for (int q = 0; q < kR; q++)
-        x[q] = (feat >= 0 && r0 + q < a.n) ? __ldg(&a.X[(r0 + q) * a.d + feat]) : 0.0f;
+        for (int q = 0; q < kR; q++) x[q] = __ldg(xr + q * d);
+      } else {
+#pragma unroll
+        for (int q = 0; q < kR; q++) x[q] = (feat >= 0 && r0 + q < a.n) ? __ldg(xr + q * d) : 0.0f;
+      }
     };
     float xn[kR];
-    load_x(w0, xn);
+    if (w0 < a.nrows) load_x(w0, xn);
     for (int64_t r0 = w0; r0 < a.nrows; r0 += wstride) {
       float x[kR];
 #pragma unroll
@@ -845,17 +854,16 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
       // pos := #{thresholds <= x} by Shar's bisection (uniform trip count for every row of this
       // lane, every probe in range, no bounds tests): after the first probe at top - 1 the count
       // lies in [pos, pos + top]; each halving step keeps it in [pos, pos + step]; a last probe
-      // at pos decides between pos and pos + 1.
-      // (positions are kept as byte offsets, pos * stride, so a probe address is one add)
+      // at pos decides between pos and pos + 1.  Positions are byte offsets (pos * stride).
       uint32_t pos[kR];
-      if (top > 0) {
-        const uint32_t a0 = base + (uint32_t)(top - 1) * stride;
 #pragma unroll
-        for (int q = 0; q < kR; q++) {
-          float v;
-          asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a0));
-          pos[q] = v <= x[q] ? (uint32_t)(K - top) * stride : 0u;
-        }
+      for (int q = 0; q < kR; q++) pos[q] = 0;
+      if (top > 0) {
+        float v0;
+        asm("ld.shared.f32 %0, [%1];" : "=f"(v0) : "r"(base + (uint32_t)(top - 1) * stride));
+        const uint32_t hi = (uint32_t)(K - top) * stride;
+#pragma unroll
+        for (int q = 0; q < kR; q++) pos[q] = v0 <= x[q] ? hi : 0u;
         for (uint32_t stepb = ((uint32_t)top >> 1) * stride; stepb >= stride; stepb >>= 1) {
           const uint32_t as = base + stepb - stride;
 #pragma unroll
@@ -871,24 +879,19 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
           asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(base + pos[q]));
           pos[q] = (pos[q] >> lstride) + (v <= x[q] ? 1u : 0u);
         }
-      } else {
-#pragma unroll
-        for (int q = 0; q < kR; q++) pos[q] = 0;
       }
+      if (slot >= 0) {
+        uint16_t* tb = a.codes + (r0 >> 6) * tile_u16 + slot;
+        const int rr0 = (int)(r0 & 63);
+        bool nan = false;
 #pragma unroll
-      for (int q = 0; q < kR; q++) {
-        const int64_t r = r0 + q;
-        if (r >= a.nrows) break;
-        uint16_t code = kCodePad;
-        if (feat >= 0 && r < a.n) {
-          if (x[q] != x[q]) {
-            code = kCodeNan;
-            a.nan_flags[r >> 6] = 1;
-          } else {
-            code = (uint16_t)pos[q];
-          }
+        for (int q = 0; q < kR; q++) {
+          uint16_t code = (uint16_t)pos[q];
+          if (feat < 0 || r0 + q >= a.n) code = kCodePad;
+          else if (x[q] != x[q]) { code = kCodeNan; nan = true; }
+          tb[code_row_off(rr0 + q, rb) >> 1] = code;
         }
-        if (slot >= 0) a.codes[(r >> 6) * tile_u16 + (code_row_off((int)(r & 63), a.rb) >> 1) + slot] = code;
+        if (nan) a.nan_flags[r0 >> 6] = 1;
       }
     }
   }
@@ -1374,14 +1377,18 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
       // static + dynamic shared memory must stay within the opt-in limit (the kernel's mbarrier
       // is static)
-      e = cudaFuncSetAttribute(k_encode_rows_banks, cudaFuncAttributeMaxDynamicSharedMemorySize,
+      e = cudaFuncSetAttribute(k_encode_rows_banks<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                kMaxSmemOptin - 1024);
+      if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_encode_rows_banks<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 kMaxSmemOptin - 1024);
       if (e != cudaSuccess) return (int)e;
       configured[dev].store(1);
     }
-    const int64_t warps_needed = (ba.nrows + 3) / 4;
+    const int64_t warps_needed = (ba.nrows + 7) / 8;
     const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(num_sms, (warps_needed + 31) / 32));
-    k_encode_rows_banks<<<grid, blk, ba.img_bytes, st>>>(ba);
+    if (ba.rb == 64) k_encode_rows_banks<true><<<grid, blk, ba.img_bytes, st>>>(ba);
+    else k_encode_rows_banks<false><<<grid, blk, ba.img_bytes, st>>>(ba);
   } else if (tab_bytes <= 200 * 1024) {
     static std::atomic<int> configured[64];
     int dev = 0;

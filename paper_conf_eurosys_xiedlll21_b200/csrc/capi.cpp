@@ -286,6 +286,16 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   int32_t strat = choose(f, n, d, forced);
   if (strat == -2) return fail(TAHOE_E_UNSUPPORTED, "sliced strategy unavailable: " + f->sl.why_invalid);
   if (strat == -3) return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices unavailable: " + f->sl.code_why);
+  if (strat == TAHOE_STRATEGY_SLICED_CODED) {
+    // the code-tile ring (+ trailers and staged partials) must fit next to the slice
+    const int64_t need = (((int64_t)f->sl.slots_max * kSlotBytes + 1023) & ~1023LL) +
+                         3LL * code_tile_stride(f->sl.fbits) + kSlicedBarrierBytes + 3LL * kSlicedTileRows * 8;
+    if (need > f->max_smem) {
+      if (forced == TAHOE_STRATEGY_SLICED_CODED)
+        return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices: code-tile ring does not fit shared memory");
+      strat = TAHOE_STRATEGY_SLICED;
+    }
+  }
   if (strat == TAHOE_STRATEGY_SLICED_CODED && (out_leaf || out_fp)) {
     if (forced == TAHOE_STRATEGY_SLICED_CODED)
       return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices produce no leaf ids / fingerprints");
@@ -362,14 +372,13 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   int rc;
   if (strat == TAHOE_STRATEGY_SLICED_CODED) {
     const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
-    const size_t cbytes = (size_t)ntiles * code_tile_bytes(f->sl.fbits);
+    const size_t cbytes = (size_t)ntiles * code_tile_stride(f->sl.fbits);
     void* cbuf = nullptr;
-    if ((e = scratch_alloc(&cbuf, cbytes + (size_t)ntiles * 4, st)) != cudaSuccess) {
+    if ((e = scratch_alloc(&cbuf, cbytes, st)) != cudaSuccess) {
       if (part) cudaFreeAsync(part, st);
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync code tiles");
     }
-    rc = launch_sliced_codes(f->ds, plan, X, n, d, static_cast<uint16_t*>(cbuf),
-                             reinterpret_cast<int32_t*>(static_cast<char*>(cbuf) + cbytes), o, fused,
+    rc = launch_sliced_codes(f->ds, plan, X, n, d, static_cast<uint16_t*>(cbuf), o, fused,
                              f->num_sms, st, ev_b, ev_e);
     cudaFreeAsync(cbuf, st);
   } else {

@@ -735,7 +735,7 @@ struct EncodeRowsArgs {
   const float* tab;
   const int32_t* off;
   uint16_t* codes;
-  int32_t* nan_flags;
+  int32_t tstride;   // bytes per code tile (rows + trailer)
   int64_t ntiles;
 };
 
@@ -759,7 +759,8 @@ __global__ void __launch_bounds__(1024) k_encode_rows(const EncodeRowsArgs a) {
   }
   const int64_t total = a.ntiles * 64 << a.fbits;
   const int smask = (1 << a.fbits) - 1;
-  const int64_t tile_u16 = (int64_t)32 * a.rb;
+  const int64_t tile_u16 = a.tstride >> 1;
+  const int32_t flag_u16 = 32 * a.rb;   // trailer word (after the rows)
   for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
        e += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = e >> a.fbits;
@@ -769,7 +770,7 @@ __global__ void __launch_bounds__(1024) k_encode_rows(const EncodeRowsArgs a) {
       const float x = __ldg(&a.X[r * a.d + j]);
       if (x != x) {
         code = kCodeNan;
-        a.nan_flags[r >> 6] = 1;
+        *reinterpret_cast<int32_t*>(a.codes + (r >> 6) * tile_u16 + flag_u16) = 1;
       } else {
         const int32_t b0 = off[j];
         int32_t lo = b0, len = off[j + 1] - b0;
@@ -796,7 +797,7 @@ struct EncodeBanksArgs {
   const float* img;
   const int4* desc;
   uint16_t* codes;
-  int32_t* nan_flags;
+  int32_t tstride;   // bytes per code tile (rows + trailer)
   int64_t nrows;   // ntiles * 64
 };
 
@@ -817,7 +818,8 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
   }
   mbar_wait(&s_bar, 0);
   const int rb = RB64 ? 64 : a.rb;
-  const int64_t tile_u16 = (int64_t)32 * rb;
+  const int64_t tile_u16 = a.tstride >> 1;
+  const int32_t flag_u16 = 32 * rb;   // trailer word (after the rows)
   // a warp codes kR consecutive rows at once (independent bisections interleaved; the next
   // group's attribute values are loaded before this group is searched)
   constexpr int kR = 8;
@@ -891,7 +893,7 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
           else if (x[q] != x[q]) { code = kCodeNan; nan = true; }
           tb[code_row_off(rr0 + q, rb) >> 1] = code;
         }
-        if (nan) a.nan_flags[r0 >> 6] = 1;
+        if (nan) *reinterpret_cast<int32_t*>(a.codes + (r0 >> 6) * tile_u16 + flag_u16) = 1;
       }
     }
   }
@@ -900,10 +902,10 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
 struct CodedKArgs {
   DevSliced img;
   const uint16_t* codes;
-  const int32_t* nan_flags;
   int64_t n;
   int32_t forest_smem;   // bytes reserved for the slice (multiple of 1024)
-  int32_t tile_bytes;    // one 64-row code tile
+  int32_t tile_bytes;    // the 64 code rows of a tile (its NaN flag follows them)
+  int32_t tstride;       // bytes per tile (rows + 128-byte trailer), in HBM and in the ring
   int32_t rb;            // bytes per code row
   int32_t cps;           // CTAs per slice (single-pass)
   OutArgs o;
@@ -959,10 +961,12 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
   unsigned char* s_ring = smem + a.forest_smem;
-  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)kRing * a.tile_bytes);
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)kRing * a.tstride);
   uint64_t* s_forest = s_full + kRing;
   int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
   unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
+  // slice partials of the tiles in the ring, written out coalesced by the warp closing a tile
+  double* s_part = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_full) + kSlicedBarrierBytes);
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int col = lane & (C - 1);
@@ -988,14 +992,17 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   auto issue_tile = [&](int64_t tile, int b) {
     if (lane == 0) {
       fence_proxy_async_smem();
-      mbar_expect_tx(&s_full[b], (uint32_t)a.tile_bytes);
-      bulk_g2s(s_ring + (size_t)b * a.tile_bytes,
-               reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tile_bytes,
-               (uint32_t)a.tile_bytes, &s_full[b]);
+      mbar_expect_tx(&s_full[b], (uint32_t)a.tstride);
+      bulk_g2s(s_ring + (size_t)b * a.tstride,
+               reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride,
+               (uint32_t)a.tstride, &s_full[b]);
     }
     __syncwarp();
   };
-  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts) {
+  // after one work unit: the warp finishing the tile's last unit writes the tile's 64 slice
+  // partials (two coalesced 256-byte stores) and refills the buffer with the tile kRing ahead
+  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts,
+                     int sl, int64_t r0, int nr) {
     __syncwarp();
     int last = 0;
     if (lane == 0) {
@@ -1004,7 +1011,15 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
       if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
     }
     last = __shfl_sync(0xffffffffu, last, 0);
-    if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+    if (!last) return;
+    if (!FUSED) {
+      const double* sp = s_part + b * kSlicedTileRows;
+      double* dst = a.o.raw + (size_t)sl * a.n + r0;
+      if (lane < nr) dst[lane] = sp[lane];
+      if (lane + 32 < nr) dst[lane + 32] = sp[lane + 32];
+      __syncwarp();
+    }
+    if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
   };
 
   uint32_t g = 0;
@@ -1049,11 +1064,13 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         const int rA = u + 16 * half, rB = rA + 32;
         const bool okA = rA < nr, okB = rB < nr;
         const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
-        const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tile_bytes;
+        const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tstride;
         const uint32_t rowA = tb + code_row_off(okA ? rA : u, a.rb);
         const uint32_t rowB = tb + code_row_off(okB ? rB : u, a.rb);
+        uint32_t nan_flag;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(tb + (uint32_t)a.tile_bytes));
         double accA, accB;
-        if (__ldg(&a.nan_flags[tile]))
+        if (nan_flag)
           walk_coded2<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
         else
           walk_coded2<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
@@ -1064,12 +1081,11 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
         const int rr = b3 ? rB : rA;
         if ((lane & 7) == 0 && (b3 ? okB : okA)) {
-          const int64_t i = r0 + rr;
-          if (FUSED) write_scalar(a.o, i, v);
-          else a.o.raw[(size_t)sl * a.n + i] = v;
+          if (FUSED) write_scalar(a.o, r0 + rr, v);
+          else s_part[b * kSlicedTileRows + rr] = v;
         }
       }
-      release(b, kUnits, it, my_tiles, t0, ts);
+      release(b, kUnits, it, my_tiles, t0, ts, sl, r0, nr);
     }
     g += (uint32_t)my_tiles;
     __syncthreads();
@@ -1334,11 +1350,15 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
 }
 
 int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
-                        int32_t d, uint16_t* codes, int32_t* nan_flags, const OutArgs& o,
-                        bool fused, int32_t num_sms, void* stream, void* ev_b, void* ev_e) {
+                        int32_t d, uint16_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
+                        void* stream, void* ev_b, void* ev_e) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
-  cudaError_t e = cudaMemsetAsync(nan_flags, 0, (size_t)ntiles * 4, st);
+  const int32_t tstride = code_tile_stride(img.fbits);
+  const int32_t tbytes = code_tile_bytes(img.fbits);
+  // zero every tile's NaN flag (the trailer word after its rows)
+  cudaError_t e = cudaMemset2DAsync(reinterpret_cast<char*>(codes) + tbytes, (size_t)tstride, 0, 4,
+                                    (size_t)ntiles, st);
   if (e != cudaSuccess) return (int)e;
   EncodeRowsArgs ea;
   ea.X = X;
@@ -1351,7 +1371,7 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   ea.tab = img.thr_tab;
   ea.off = img.thr_off;
   ea.codes = codes;
-  ea.nan_flags = nan_flags;
+  ea.tstride = tstride;
   ea.ntiles = ntiles;
   const int64_t tab_bytes = (int64_t)img.n_thr * 4 + (int64_t)(img.n_features + 1) * 4;
   const int64_t elems = ntiles * kSlicedTileRows << img.fbits;
@@ -1369,7 +1389,7 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
     ba.img = img.cb_img;
     ba.desc = reinterpret_cast<const int4*>(img.cb_desc);
     ba.codes = codes;
-    ba.nan_flags = nan_flags;
+    ba.tstride = tstride;
     ba.nrows = ntiles * kSlicedTileRows;
     static std::atomic<int> configured[64];
     int dev = 0;
@@ -1409,14 +1429,15 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   CodedKArgs a{};
   a.img = img;
   a.codes = codes;
-  a.nan_flags = nan_flags;
   a.n = n;
   a.forest_smem = plan.forest_smem;
-  a.tile_bytes = code_tile_bytes(img.fbits);
+  a.tile_bytes = tbytes;
+  a.tstride = tstride;
   a.rb = code_row_bytes(img.fbits);
   a.cps = plan.cps;
   a.o = o;
-  const int smem = plan.forest_smem + kRing * a.tile_bytes + kSlicedBarrierBytes;
+  const int smem = plan.forest_smem + kRing * tstride + kSlicedBarrierBytes +
+                   kRing * kSlicedTileRows * (int)sizeof(double);
   auto kern = fused ? k_sliced_codes<true> : k_sliced_codes<false>;
   {
     static std::atomic<int> configured[64];

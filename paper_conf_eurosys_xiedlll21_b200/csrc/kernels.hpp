@@ -65,7 +65,9 @@ constexpr uint16_t kCodeNan = 0xFFFEu;
 constexpr uint16_t kCodePad = 0xFFFFu;
 inline int32_t code_row_bytes(int32_t fbits) { return (2 << fbits) < 64 ? 64 : (2 << fbits); }
 inline int32_t code_tile_bytes(int32_t fbits) { return 64 * code_row_bytes(fbits); }
-inline int64_t code_ring_bytes(int32_t fbits) { return (int64_t)3 * code_tile_bytes(fbits); }
+// a code tile in HBM and in the ring: the rows, then a 128-byte trailer whose first word is the
+// tile's NaN flag (1 if any of its codes is kCodeNan; it arrives with the tile's bulk copy)
+inline int32_t code_tile_stride(int32_t fbits) { return code_tile_bytes(fbits) + 128; }
 
 struct OutArgs {
   float* out = nullptr;          // final scores (fused finalize) or nullptr
@@ -134,11 +136,11 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
                   bool fused, int32_t num_sms, void* stream);
 int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                   int32_t d, const OutArgs& o, bool fused, void* stream);
-// rank-coded sliced strategy: encode X into code tiles (codes: ntiles * code_tile_bytes bytes,
-// nan_flags: ntiles ints, both device scratch), then walk the coded slices
+// rank-coded sliced strategy: encode X into code tiles (codes: device scratch of
+// ntiles * code_tile_stride bytes), then walk the coded slices
 int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
-                        int32_t d, uint16_t* codes, int32_t* nan_flags, const OutArgs& o,
-                        bool fused, int32_t num_sms, void* stream, void* ev_b, void* ev_e);
+                        int32_t d, uint16_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
+                        void* stream, void* ev_b, void* ev_e);
 int launch_finalize(const FinalizeArgs& a, void* stream);
 int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t d,
                         uint32_t* counts, int32_t num_sms, void* stream);

@@ -29,6 +29,13 @@ for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
         F.predict(Xd, out=out, out_class=cls, force_strategy=s)
         F.predict(Xd, out=out, out_class=cls, out_leaf=leaf, out_fingerprint=fp, force_strategy=s)
     os.environ.pop("TAHOE_DIRECT_VARIANT")
+    # rank-coded slices (reading R7): both row-coding pre-passes
+    if F.stats()["coded_valid"]:
+        for banks in ("1", "0"):
+            os.environ["TAHOE_CODE_BANKS"] = banks
+            out = torch.empty((n, F.n_out), device=dev)
+            F.predict(Xd, out=out, force_strategy=2)
+        os.environ.pop("TAHOE_CODE_BANKS")
     # misaligned X -> warp-copy staging path
     buf = torch.empty(X.size + 1, device=dev)
     buf[1:] = Xd.reshape(-1)

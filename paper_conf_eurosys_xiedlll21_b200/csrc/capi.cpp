@@ -224,6 +224,9 @@ static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   }
   for (double v : f->host.exp_reads) st.V += v;
   st.sliced_ok = f->sl.valid;
+  static const bool codes_off = std::getenv("TAHOE_CODES") && std::string(std::getenv("TAHOE_CODES")) == "0";
+  st.coded_ok = f->sl.valid && f->sl.code_valid && !codes_off;
+  st.code_passes = std::max(1, (1 << f->sl.fbits) / 32);
   st.sliced_eff = f->sl.eff_sim;
   st.n_slices = f->sl.n_slices;
   st.num_sms = f->num_sms;
@@ -239,12 +242,9 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
   if (forced == TAHOE_STRATEGY_SLICED) return f->sl.valid ? TAHOE_STRATEGY_SLICED : -2;
   if (forced == TAHOE_STRATEGY_SLICED_CODED)
     return !f->sl.valid ? -2 : (f->ds.cnodes ? TAHOE_STRATEGY_SLICED_CODED : -3);
-  const int32_t s = select_strategy(plan_stats(f, d), n, d, f->host.agg);
-  // the rank-coded twin of the sliced strategy wherever the forest qualifies (reading R7);
-  // $TAHOE_CODES=0 keeps the fp32 slices (experiments)
-  static const bool codes_off = std::getenv("TAHOE_CODES") && std::string(std::getenv("TAHOE_CODES")) == "0";
-  if (s == TAHOE_STRATEGY_SLICED && f->ds.cnodes && !codes_off) return TAHOE_STRATEGY_SLICED_CODED;
-  return s;
+  // the cost model weighs the rank-coded twin of the sliced strategy (reading R7) wherever the
+  // forest qualifies; $TAHOE_CODES=0 leaves it out (experiments)
+  return select_strategy(plan_stats(f, d), n, d, f->host.agg);
 }
 
 static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int64_t n, int32_t d) {
@@ -758,6 +758,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"coded_why\":\"" << f->sl.code_why << "\"" << ",\"coded_thresholds\":"
      << (f->sl.thr_off.empty() ? 0 : f->sl.thr_off.back())
      << ",\"code_bank_rows\":" << f->sl.cb_rows << ",\"code_bank_passes\":" << f->sl.cb_passes
+     << ",\"sliced_fbits\":" << f->sl.fbits
      << ",\"n_slices\":" << f->sl.n_slices << ",\"slots_max\":" << f->sl.slots_max
      << ",\"slot_budget\":" << f->slot_budget << ",\"sliced_bytes\":" << f->sl.bytes()
      << ",\"lockstep_eff\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim

@@ -8,7 +8,10 @@
 //            a_s absorbs launch, slice staging and the fixed-order slice reduction (T_G_REDU);
 //   direct : T = a_d + (d > 256 ? g_d : 1) * max(l_d * V, b_d * V * n / SMs)
 //            one thread per sample: latency-bound below a full GPU of threads (l_d per visit),
-//            L1/L2-throughput-bound above it (T_GMEM).
+//            L1/L2-throughput-bound above it (T_GMEM);
+//   coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs
+//            the rank-coded slices (reading R7): the same busiest-CTA node reads at a cheaper
+//            per-read cost b_c, plus the row-coding pre-pass (passes of 32 attributes per row).
 // V = expected node reads per sample (calibrated E[path] + 1 leaf read, summed over trees,
 // reading Z16).  The constants are fitted on the chip by scripts/fit_costmodel.py and read from
 // costmodel_b200.json next to libtahoe.so (or $TAHOE_COSTMODEL); defaults are round-1 B200
@@ -65,6 +68,9 @@ const CostParams& cost_params() {
     all &= read_key(js, "b_d", &v); if (all) c.b_d = v;
     if (read_key(js, "g_s", &v)) c.g_s = v;
     if (read_key(js, "g_d", &v)) c.g_d = v;
+    if (read_key(js, "a_c", &v)) c.a_c = v;
+    if (read_key(js, "b_c", &v)) c.b_c = v;
+    if (read_key(js, "e_c", &v)) c.e_c = v;
     c.fitted = all;
     return c;
   }();
@@ -73,10 +79,9 @@ const CostParams& cost_params() {
 
 double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
   const CostParams& c = cost_params();
-  // the rank-coded twin (reading R7) is costed as the fp32 slices it replaces (conservative)
-  if (strategy == TAHOE_STRATEGY_SLICED_CODED) strategy = TAHOE_STRATEGY_SLICED;
-  if (strategy == TAHOE_STRATEGY_SLICED) {
+  if (strategy == TAHOE_STRATEGY_SLICED || strategy == TAHOE_STRATEGY_SLICED_CODED) {
     if (!st.sliced_ok || st.n_slices < 1) return INFINITY;
+    if (strategy == TAHOE_STRATEGY_SLICED_CODED && !st.coded_ok) return INFINITY;
     const int64_t tiles = (n + 63) / 64;
     const int64_t cps = st.n_slices <= st.num_sms
                             ? std::max<int64_t>(1, std::min<int64_t>(st.num_sms / st.n_slices, tiles))
@@ -84,6 +89,8 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
     const double passes = st.n_slices <= st.num_sms ? 1.0 : std::ceil((double)st.n_slices / st.num_sms);
     const double eff = st.sliced_eff > 0.05 ? st.sliced_eff : 0.05;
     const double U = (double)((tiles + cps - 1) / cps) * 64.0 * st.V / (st.n_slices * eff) * passes;
+    if (strategy == TAHOE_STRATEGY_SLICED_CODED)
+      return c.a_c + c.b_c * U + c.e_c * (double)(tiles * 64) * st.code_passes / std::max(1, st.num_sms);
     return c.a_s + c.b_s * U * (st.rows_global ? c.g_s : 1.0);
   }
   const double sms = st.num_sms > 0 ? st.num_sms : 148;
@@ -94,9 +101,13 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
 int32_t select_strategy(const PlanStats& st, int64_t n, int32_t d, int32_t agg) {
   (void)d;
   if (agg == TAHOE_AGG_VOTE || !st.sliced_ok) return TAHOE_STRATEGY_DIRECT;
-  return predict_us(st, TAHOE_STRATEGY_SLICED, n) <= predict_us(st, TAHOE_STRATEGY_DIRECT, n)
-             ? TAHOE_STRATEGY_SLICED
-             : TAHOE_STRATEGY_DIRECT;
+  int32_t best = TAHOE_STRATEGY_DIRECT;
+  double tb = predict_us(st, TAHOE_STRATEGY_DIRECT, n);
+  for (int32_t s : {TAHOE_STRATEGY_SLICED, TAHOE_STRATEGY_SLICED_CODED}) {
+    const double t = predict_us(st, s, n);
+    if (t < tb) { tb = t; best = s; }
+  }
+  return best;
 }
 
 }  // namespace tahoe

@@ -125,6 +125,8 @@ struct PlanStats {
   bool sliced_ok = false;
   bool rows_global = false;  // sliced rows too wide to stage in shared memory
   bool wide_rows = false;    // d > 256: direct reads attributes from rows far apart in memory
+  bool coded_ok = false;     // rank-coded twin available and enabled (reading R7)
+  int32_t code_passes = 1;   // row-coding passes of 32 attributes
 };
 // Fitted per-platform constants (costmodel_b200.json, scripts/fit_costmodel.py), microseconds.
 struct CostParams {
@@ -132,6 +134,7 @@ struct CostParams {
   double g_s = 4.0;                          // sliced: slowdown when rows stay in global memory
   double a_d = 11.8, l_d = 0.34, b_d = 6.3e-4; // direct: launch; per-visit latency; per unit
   double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
+  double a_c = 30.0, b_c = 6.6e-5, e_c = 1.6e-5; // coded: launches; per unit; per row-pass per SM
   bool fitted = false;
 };
 const CostParams& cost_params();

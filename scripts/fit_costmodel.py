@@ -5,6 +5,7 @@ Times both strategies on the BASELINE-shaped forests over a sweep of batch sizes
 
     sliced : T = a_s + b_s * U_s,   U_s = ceil(tiles / cps) * 64 * V / (slices * eff_sim)
     direct : T = a_d + max(l_d * V, b_d * V * n / SMs)
+    coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs   (reading R7)
 
 (costmodel.cpp), writes paper_conf_eurosys_xiedlll21_b200/costmodel_b200.json (read by
 libtahoe.so at load) and a report with the model's rank accuracy (paper: 87/90 correct orderings,
@@ -69,9 +70,12 @@ def main():
             rec = dict(config=cid, n=n, V=st["expected_node_reads_per_sample"],
                        slices=st["n_slices"], eff_sim=st["lockstep_eff_sim"],
                        sms=st["num_sms"], sliced_valid=st["sliced_valid"],
+                       coded_valid=st["sliced_valid"] and st["coded_valid"],
+                       passes=max(1, (1 << st["sliced_fbits"]) // 32),
                        rows_global=cid == 4)  # C4: d = 2000 (> 256, too wide to stage)
             rec["direct_ms"] = time_ms(F, X, T.STRATEGY_DIRECT)
             rec["sliced_ms"] = time_ms(F, X, T.STRATEGY_SLICED) if st["sliced_valid"] else None
+            rec["coded_ms"] = time_ms(F, X, T.STRATEGY_SLICED_CODED) if rec["coded_valid"] else None
             rows.append(rec)
             print(json.dumps(rec), flush=True)
         F.close()
@@ -90,6 +94,19 @@ def main():
     gl = [r for r in rows if r["sliced_ms"] is not None and r["rows_global"] and r["n"] >= 10_000]
     g_s = float(np.median([(r["sliced_ms"] * 1000 - a_s) / (b_s * U_s(r)) for r in gl])) if gl else 4.0
 
+    def E_c(r):
+        return math.ceil(r["n"] / 64) * 64 * r["passes"] / r["sms"]
+
+    cd = [r for r in rows if r["coded_ms"] is not None]
+    if cd:
+        Ac = np.array([[1.0, U_s(r), E_c(r)] for r in cd])
+        yc = np.array([r["coded_ms"] * 1000 for r in cd])
+        wc = 1.0 / yc
+        a_c, b_c, e_c = np.linalg.lstsq(Ac * wc[:, None], yc * wc, rcond=None)[0]
+        a_c, b_c, e_c = max(a_c, 1.0), max(b_c, 1e-9), max(e_c, 0.0)
+    else:
+        a_c, b_c, e_c = 30.0, 6.6e-5, 1.6e-5
+
     def direct_model(p, r):
         a, l, b, g = p
         return a + (g if r["rows_global"] else 1.0) * max(l * r["V"], b * r["V"] * r["n"] / r["sms"])
@@ -99,7 +116,7 @@ def main():
                         x0=[5.0, 0.1, 3e-4, 2.0])
     a_d, l_d, b_d, g_d = np.abs(res.x)
     params = dict(a_s=float(a_s), b_s=float(b_s), g_s=g_s, a_d=float(a_d), l_d=float(l_d), b_d=float(b_d),
-                  g_d=float(g_d),
+                  g_d=float(g_d), a_c=float(a_c), b_c=float(b_c), e_c=float(e_c),
                   units="microseconds", gpu=torch.cuda.get_device_name(0))
 
     correct = total = 0
@@ -107,22 +124,29 @@ def main():
     for r in rows:
         ps = (params["a_s"] + params["b_s"] * U_s(r) * (g_s if r["rows_global"] else 1.0)
               if r["sliced_ms"] is not None else math.inf)
+        pc = a_c + b_c * U_s(r) + e_c * E_c(r) if r["coded_ms"] is not None else math.inf
         pd = direct_model([a_d, l_d, b_d, g_d], r)
-        r.update(pred_sliced_us=ps, pred_direct_us=pd)
+        r.update(pred_sliced_us=ps, pred_direct_us=pd, pred_coded_us=pc)
         if r["sliced_ms"] is None:
             continue
         total += 1
-        meas = "sliced" if r["sliced_ms"] <= r["direct_ms"] else "direct"
-        pred = "sliced" if ps <= pd else "direct"
+        meas_t = {"direct": r["direct_ms"], "sliced": r["sliced_ms"]}
+        if r["coded_ms"] is not None:
+            meas_t["coded"] = r["coded_ms"]
+        pred_t = {"direct": pd, "sliced": ps, "coded": pc}
+        meas = min(meas_t, key=meas_t.get)
+        pred = min(pred_t, key=pred_t.get)
         correct += meas == pred
-        report.append((r["config"], r["n"], r["direct_ms"], r["sliced_ms"], pd / 1000, ps / 1000, meas, pred))
+        report.append((r["config"], r["n"], r["direct_ms"], r["sliced_ms"],
+                       r["coded_ms"] if r["coded_ms"] is not None else float("nan"),
+                       pd / 1000, ps / 1000, pc / 1000, meas, pred))
     params["rank_accuracy"] = f"{correct}/{total}"
     path = os.path.join(ROOT, "paper_conf_eurosys_xiedlll21_b200", "costmodel_b200.json")
     json.dump(params, open(path, "w"), indent=1)
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     json.dump(dict(params=params, rows=rows), open(os.path.join(ROOT, "gpurun_out", "costmodel_fit.json"), "w"), indent=1)
     print(json.dumps(params))
-    print("config n direct_ms sliced_ms pred_direct_ms pred_sliced_ms measured_best predicted_best")
+    print("config n direct_ms sliced_ms coded_ms pred_direct_ms pred_sliced_ms pred_coded_ms measured_best predicted_best")
     for t in report:
         print(" ".join(f"{v:.4g}" if isinstance(v, float) else str(v) for v in t))
 

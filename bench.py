@@ -450,14 +450,17 @@ def main():
     n_sms = stats["num_sms"]
     smem_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
     achieved = n * smem_bytes_per_sample / (kern_avg_ms / 1000.0) / 1e9
+    kname = {1: "k_sliced", 2: "k_sliced_codes"}.get(strategy, "k_direct")
     traffic = None
     sector_eff = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
             rec = json.load(open(tp)).get(f"C{cfg.cid}", {})
-            traffic = rec.get("dram_bytes_per_launch")
-            sector_eff = rec.get("global_ld_sector_efficiency")
+            # only a capture of the kernel this run times (e.g. "k_sliced_codes<0>")
+            if rec.get("kernel", "").split("<")[0] == kname:
+                traffic = rec.get("dram_bytes_per_launch")
+                sector_eff = rec.get("global_ld_sector_efficiency")
         except Exception:
             traffic = None
     launches_per_step = 1 if strategy == T.STRATEGY_DIRECT and F.n_out == 1 else (
@@ -471,7 +474,7 @@ def main():
         config=_config(cfg, n, stats),
         strategy={0: "direct", 1: "sliced", 2: "sliced-coded"}.get(strategy, str(strategy)),
         roofline=dict(bound="alu", pipe="shared-memory LSU, 128 B/clk/SM (DESIGN.md Roofline)",
-                      kernel={1: "k_sliced", 2: "k_sliced_codes"}.get(strategy, "k_direct"),
+                      kernel=kname,
                       achieved=achieved, peak=smem_peak, unit="GB/s", frac=achieved / smem_peak,
                       traffic=traffic, kernel_ms=kern_avg_ms,
                       global_ld_sector_efficiency=sector_eff,

@@ -296,9 +296,13 @@ def _config(cfg, n, stats):
     c = {"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
                      f"{cfg.n_features} features, {n} samples per GPU (BASELINE configs[{cfg.cid - 1}])",
          "n_per_gpu": n, "n_trees": cfg.n_trees, "n_features": cfg.n_features,
-         "max_depth": cfg.max_depth, "agg": "binary margin + class",
+         "max_depth": cfg.max_depth,
+         "agg": {gen.AGG_SUM: "sum", gen.AGG_AVERAGE: "average", gen.AGG_BINARY: "binary margin + class",
+                 gen.AGG_CLASS_SUM: f"{cfg.n_classes}-class sums + argmax",
+                 gen.AGG_VOTE: "vote"}.get(cfg.agg, str(cfg.agg)),
          "parallelism": "sample-sharded (no collective)",
-         "l2": "256 MiB L2 flush between timed steps (inputs 112 MB < L2), outside the events"}
+         "l2": f"256 MiB L2 flush between timed steps (inputs {n * cfg.n_features * 4 / 1e6:.0f} MB "
+               f"{'<' if n * cfg.n_features * 4 < 126e6 else '>'} L2), outside the events"}
     if stats:
         c.update({k: stats[k] for k in ("nodes", "leaves", "n_slices", "slots_max", "lockstep_eff",
                                         "expected_visits_per_sample", "sliced_bytes") if k in stats})

@@ -100,6 +100,8 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->ds.cb_desc);
   cudaFree(f->d_class_ptr);
   cudaFree(f->d_class_parts);
+  cudaFree(f->d_cta_start);
+  f->d_cta_start = nullptr;
   f->dd = DevDirect();
   f->ds = DevSliced();
   f->d_class_ptr = f->d_class_parts = nullptr;
@@ -178,6 +180,31 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
     f->ds.n_slices = f->sl.n_slices;
     f->ds.slots_max = f->sl.slots_max;
     f->ds.fbits = f->sl.fbits;
+    // weighted CTA shares of a full-GPU launch (largest remainder, at least one CTA per slice)
+    const int32_t ns = f->sl.n_slices;
+    f->cta_start.clear();
+    if (ns >= 1 && ns <= f->num_sms && (int32_t)f->sl.slice_work.size() == ns) {
+      double tot = 0;
+      for (double w : f->sl.slice_work) tot += w;
+      std::vector<int32_t> c(ns, 1);
+      int32_t left = f->num_sms - ns;
+      std::vector<std::pair<double, int32_t>> rem;
+      for (int32_t q = 0; q < ns; q++) {
+        const double share = (double)f->num_sms * f->sl.slice_work[q] / tot - 1.0;
+        const int32_t k = std::max(0, std::min(left, (int32_t)std::floor(share)));
+        c[q] += k;
+        left -= k;
+        rem.push_back({share - k, q});
+      }
+      std::sort(rem.begin(), rem.end(), [](const std::pair<double, int32_t>& u, const std::pair<double, int32_t>& v) {
+        return u.first != v.first ? u.first > v.first : u.second < v.second; });
+      for (size_t q = 0; left > 0; q = (q + 1) % rem.size(), left--) c[rem[q].second]++;
+      f->cta_start.assign(ns + 1, 0);
+      for (int32_t q = 0; q < ns; q++) f->cta_start[q + 1] = f->cta_start[q] + c[q];
+      const int32_t* dp = nullptr;
+      if ((st = upload(f->cta_start, &dp)) != TAHOE_OK) return st;
+      f->d_cta_start = const_cast<int32_t*>(dp);
+    }
     if (f->sl.code_valid) {
       if ((st = upload(f->sl.cnodes, &f->ds.cnodes)) != TAHOE_OK) return st;
       if ((st = upload(f->sl.thr_tab, &f->ds.thr_tab)) != TAHOE_OK) return st;
@@ -378,7 +405,14 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       if (part) cudaFreeAsync(part, st);
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync code tiles");
     }
-    rc = launch_sliced_codes(f->ds, plan, X, n, d, static_cast<uint16_t*>(cbuf), o, fused,
+    SlicedPlan cp = plan;
+    // a full GPU of CTAs, shared out among the slices by their simulated work, once every CTA has
+    // at least a few tiles
+    if (f->d_cta_start && ntiles >= 4LL * f->num_sms) {
+      cp.grid = f->num_sms;
+      cp.cta_start = f->d_cta_start;
+    }
+    rc = launch_sliced_codes(f->ds, cp, X, n, d, static_cast<uint16_t*>(cbuf), o, fused,
                              f->num_sms, st, ev_b, ev_e);
     cudaFreeAsync(cbuf, st);
   } else {
@@ -758,7 +792,11 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"coded_why\":\"" << f->sl.code_why << "\"" << ",\"coded_thresholds\":"
      << (f->sl.thr_off.empty() ? 0 : f->sl.thr_off.back())
      << ",\"code_bank_rows\":" << f->sl.cb_rows << ",\"code_bank_passes\":" << f->sl.cb_passes
-     << ",\"sliced_fbits\":" << f->sl.fbits
+     << ",\"sliced_fbits\":" << f->sl.fbits << ",\"cta_split\":[" << [&] {
+          std::string r;
+          for (size_t q = 0; q + 1 < f->cta_start.size(); q++)
+            r += (q ? "," : "") + std::to_string(f->cta_start[q + 1] - f->cta_start[q]);
+          return r; }() << "]"
      << ",\"n_slices\":" << f->sl.n_slices << ",\"slots_max\":" << f->sl.slots_max
      << ",\"slot_budget\":" << f->slot_budget << ",\"sliced_bytes\":" << f->sl.bytes()
      << ",\"lockstep_eff\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim

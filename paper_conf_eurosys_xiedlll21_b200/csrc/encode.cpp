@@ -460,11 +460,16 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   // Simulated lockstep efficiency of k_sliced (two rows per warp, two steps per exit test) on the
   // kept calibration rows: useful node reads / lane-steps issued.  Falls back to 0.75 x expected.
   S.eff_sim = S.eff * 0.75;
+  // per-slice work (issued lane-steps per row): shares the GPU's CTAs out among the slices
+  S.slice_work.assign(packs.size(), 0.0);
+  for (size_t s = 0; s < packs.size(); s++) S.slice_work[s] = std::max(1e-9, packs[s].max_work * (double)kSlicedCols);
   if (m > 0) {
     // a warp walks 4 rows at once (2 per half-warp x 2 chains); its loop runs until the slowest
     // of the 64 (row, column) walks ends, two steps per exit test
     double useful = 0, issued = 0;
-    for (auto& P : packs) {
+    for (size_t s = 0; s < packs.size(); s++) {
+      auto& P = packs[s];
+      double issued_s = 0;
       for (int64_t r = 0; r + 3 < m; r += 4) {
         double mx = 0;
         for (int64_t q = r; q < r + 4; q++)
@@ -474,8 +479,10 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
             useful += w;
             mx = std::max(mx, w);
           }
-        issued += 64.0 * 2.0 * std::ceil(mx / 2.0);
+        issued_s += 64.0 * 2.0 * std::ceil(mx / 2.0);
       }
+      issued += issued_s;
+      if (issued_s > 0) S.slice_work[s] = issued_s / (double)(m / 4 * 4);
     }
     if (issued > 0) S.eff_sim = useful / issued;
   }

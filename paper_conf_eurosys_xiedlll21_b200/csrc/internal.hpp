@@ -88,6 +88,7 @@ struct SlicedImage {
   double eff = 0.0;                              // est. lockstep efficiency (mean/max column)
   double eff_sim = 0.0;                          // simulated 2-chain lockstep efficiency
   double trees_per_lane = 0.0;
+  std::vector<double> slice_work;                // issued lane-steps per row, per slice
   // Rank-coded twin of `nodes` (reading R7): same slots and packing, internal x = threshold rank
   // t = j + 1 (j = index of the threshold in its attribute's sorted distinct thresholds), attribute
   // field a byte offset into rows of u16 codes; thr_tab/thr_off hold the sorted thresholds.
@@ -160,5 +161,9 @@ struct tahoe_forest {
   tahoe::DevDirect dd{};
   tahoe::DevSliced ds{};
   int32_t* d_class_ptr = nullptr;   // sliced class CSR
+  // CTAs of a full-GPU sliced launch per slice, proportional to slice_work (prefix, ns + 1):
+  // the slices' CTAs then grab tiles dynamically, so every slice finishes at about the same time
+  std::vector<int32_t> cta_start;
+  int32_t* d_cta_start = nullptr;
   int32_t* d_class_parts = nullptr;
 };

@@ -907,7 +907,8 @@ struct CodedKArgs {
   int32_t tile_bytes;    // the 64 code rows of a tile (its NaN flag follows them)
   int32_t tstride;       // bytes per tile (rows + 128-byte trailer), in HBM and in the ring
   int32_t rb;            // bytes per code row
-  int32_t cps;           // CTAs per slice (single-pass)
+  int32_t cps;           // CTAs per slice (single-pass, no cta_start)
+  const int32_t* cta_start;  // or: slice s is worked by CTAs [cta_start[s], cta_start[s+1])
   OutArgs o;
 };
 
@@ -1025,10 +1026,19 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   uint32_t g = 0;
   uint32_t ph_forest = 0;
   const uint32_t ring0 = smem_u32(s_ring);
-  for (int32_t sl = multipass ? (int32_t)blockIdx.x : (int32_t)blockIdx.x % ns; sl < ns;
-       sl += multipass ? G : ns) {
-    const int64_t t0 = multipass ? 0 : blockIdx.x / ns;
-    const int64_t ts = multipass ? 1 : a.cps;
+  // single pass: this CTA's slice and its place among the slice's CTAs (weighted map, or
+  // round-robin); it takes every ts-th tile starting at t0
+  int32_t sl0 = (int32_t)blockIdx.x % ns;
+  int64_t t0s = blockIdx.x / ns, tss = a.cps;
+  if (!multipass && a.cta_start) {
+    sl0 = 0;
+    while (sl0 + 1 < ns && __ldg(&a.cta_start[sl0 + 1]) <= (int32_t)blockIdx.x) sl0++;
+    t0s = blockIdx.x - __ldg(&a.cta_start[sl0]);
+    tss = __ldg(&a.cta_start[sl0 + 1]) - __ldg(&a.cta_start[sl0]);
+  }
+  for (int32_t sl = multipass ? (int32_t)blockIdx.x : sl0; sl < ns; sl += multipass ? G : ns) {
+    const int64_t t0 = multipass ? 0 : t0s;
+    const int64_t ts = multipass ? 1 : tss;
     const int64_t my_tiles = t0 < ntiles ? (ntiles - t0 + ts - 1) / ts : 0;
     if (warp == 0) {
       if (lane == 0) {
@@ -1435,6 +1445,7 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   a.tstride = tstride;
   a.rb = code_row_bytes(img.fbits);
   a.cps = plan.cps;
+  a.cta_start = plan.cta_start;
   a.o = o;
   const int smem = plan.forest_smem + kRing * tstride + kSlicedBarrierBytes +
                    kRing * kSlicedTileRows * (int)sizeof(double);

@@ -131,6 +131,8 @@ struct SlicedPlan {
   int32_t grid = 0, block = 1024, tile_rows = 0, cps = 1;
   int32_t smem_bytes = 0, forest_smem = 0, buf_floats = 0, row_stride = 0;
   int32_t rows = 0;  // 0 global, 1 dense, 2 padded (kernels.cu kRows*)
+  const int32_t* cta_start = nullptr;  // coded slices: CTA -> slice prefix (grid == its total),
+                                       // or nullptr: CTA b works on slice b % n_slices
 };
 int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                   bool fused, int32_t num_sms, void* stream);

@@ -16,3 +16,10 @@ for r in rows:
     if hdr and len(r)==len(hdr):
         d=dict(zip(hdr,r)); print(d['Kernel Name'][:60], d['Metric Value'])
 PY
+python -c "
+import gen
+from paper_conf_eurosys_xiedlll21_b200 import tahoe as T
+for c in (2,3):
+    F=T.Forest(gen.make_forest(c),device=0).layout(gen.make_calibration(c))
+    print(c, F.stats()['cta_split'])
+"

@@ -883,17 +883,29 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
         }
       }
       if (slot >= 0) {
-        uint16_t* tb = a.codes + (r0 >> 6) * tile_u16 + slot;
-        const int rr0 = (int)(r0 & 63);
+        // the kR rows r0 .. r0+kR-1 of a group (r0 % kR == 0) sit at a constant stride in the
+        // tile: 128 bytes apart in the 64-byte-row layout (same bits 4-5 of r), rb otherwise
+        uint16_t* tb = a.codes + (r0 >> 6) * tile_u16;
+        uint16_t* p0 = tb + (code_row_off((int)(r0 & 63), rb) >> 1) + slot;
+        const int rstride = RB64 ? 64 : (rb >> 1);
         bool nan = false;
+        if (feat >= 0 && r0 + kR <= a.n) {
 #pragma unroll
-        for (int q = 0; q < kR; q++) {
-          uint16_t code = (uint16_t)pos[q];
-          if (feat < 0 || r0 + q >= a.n) code = kCodePad;
-          else if (x[q] != x[q]) { code = kCodeNan; nan = true; }
-          tb[code_row_off(rr0 + q, rb) >> 1] = code;
+          for (int q = 0; q < kR; q++) {
+            const bool isnan_q = x[q] != x[q];
+            nan |= isnan_q;
+            p0[q * rstride] = isnan_q ? kCodeNan : (uint16_t)pos[q];
+          }
+        } else {
+#pragma unroll
+          for (int q = 0; q < kR; q++) {
+            uint16_t code = (uint16_t)pos[q];
+            if (feat < 0 || r0 + q >= a.n) code = kCodePad;
+            else if (x[q] != x[q]) { code = kCodeNan; nan = true; }
+            p0[q * rstride] = code;
+          }
         }
-        if (nan) *reinterpret_cast<int32_t*>(a.codes + (r0 >> 6) * tile_u16 + flag_u16) = 1;
+        if (nan) *reinterpret_cast<int32_t*>(tb + flag_u16) = 1;
       }
     }
   }

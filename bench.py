@@ -470,7 +470,7 @@ def main():
     launches_per_step = 1 if strategy == T.STRATEGY_DIRECT and F.n_out == 1 else (
         1 + (1 if (strategy != T.STRATEGY_DIRECT and stats["n_slices"] > 1) or F.n_out > 1 else 0))
     if strategy == T.STRATEGY_SLICED_CODED:
-        launches_per_step += 1   # k_encode_rows (the nan-flag memset is not a kernel of ours)
+        launches_per_step += 1   # k_encode_rows_banks (the trailer memset is not a kernel of ours)
     line = dict(
         metric=METRIC, value=value, unit=UNIT, n_gpus=world, steps=args.steps, warmup=args.warmup,
         ms_per_step=ms_per_step, higher_is_better=True, scaling="weak", vs_baseline=None,

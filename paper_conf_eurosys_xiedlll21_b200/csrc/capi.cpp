@@ -397,6 +397,11 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
     o.raw = part;
   }
   int rc;
+  fa.partial = part;
+  fa.part_stride = n;
+  fa.row_stride = 1;
+  fa.class_ptr = f->d_class_ptr;
+  fa.class_parts = f->d_class_parts;
   if (strat == TAHOE_STRATEGY_SLICED_CODED) {
     const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
     const size_t cbytes = (size_t)ntiles * code_tile_stride(f->sl.fbits);
@@ -422,11 +427,6 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   }
   if (rc) { if (part) cudaFreeAsync(part, st); return cuda_fail((cudaError_t)rc, "sliced kernel"); }
   if (!fused) {
-    fa.partial = part;
-    fa.part_stride = n;
-    fa.row_stride = 1;
-    fa.class_ptr = f->d_class_ptr;
-    fa.class_parts = f->d_class_parts;
     rc = launch_finalize(fa, st);
     cudaFreeAsync(part, st);
     if (rc) return cuda_fail((cudaError_t)rc, "finalize kernel");

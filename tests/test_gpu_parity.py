@@ -464,3 +464,24 @@ def test_rank_code_prepass_kernels(cid, ntrees, n, banks, monkeypatch):
     ref = oracle.predict(f, X)
     _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, f["agg"], True,
            want_leaf=False)
+
+
+def test_rank_codes_multislice_classes_and_partials(monkeypatch):
+    """Multi-slice, multi-class coded launches (partials staged in shared memory, written by the
+    warp closing each tile, combined per class in slice order): CLASS_SUM scores and argmax
+    bit-exact with dyadic leaves, and the raw per-class partials (tahoe_predict_partial, no base)
+    exact too."""
+    monkeypatch.setenv("TAHOE_FORCE_STRATEGY", "2")
+    f = gen.make_forest(3, n_trees=280)
+    F = T.Forest(f, base_score=0.25, device=0).layout(gen.make_calibration(3, 4096))
+    st = F.stats()
+    assert st["coded_valid"] and st["n_slices"] > 1
+    n = 50_003
+    X = gen.make_rows(3, n)
+    X[::29, 4] = np.nan
+    ref = oracle.predict(f, X, base_score=0.25)
+    res = _gpu_run(F, X, -1, want_leaf=False)
+    _check(res, ref, f["agg"], True, want_leaf=False)
+    part = F.predict_partial(torch.from_numpy(X).cuda())
+    torch.cuda.synchronize()
+    assert np.array_equal(part.cpu().numpy(), ref["raw"] - 0.25), "dyadic partial sums are exact"

@@ -485,3 +485,26 @@ def test_rank_codes_multislice_classes_and_partials(monkeypatch):
     part = F.predict_partial(torch.from_numpy(X).cuda())
     torch.cuda.synchronize()
     assert np.array_equal(part.cpu().numpy(), ref["raw"] - 0.25), "dyadic partial sums are exact"
+
+
+@pytest.mark.parametrize("d", [3, 15, 31, 100, 127])
+def test_rank_codes_row_widths(d, monkeypatch):
+    """Every code-row geometry: 3-15 attributes (64-byte rows, one pass), 31 (64-byte rows, all 32
+    slots used, the pad slot is the leaf's), 100 and 127 attributes (256-byte rows, four 32-lane
+    passes of the pre-pass; 127 leaves a single pad slot).  Thresholds on a coarse grid make
+    x == b frequent.  Dyadic scores bit-exact against the oracle through both pre-passes."""
+    from test_oracle_pins import random_forest
+    rng = np.random.default_rng(d)
+    grid = np.linspace(-2.0, 2.0, 41)
+    f = random_forest(rng, 48, 6, d, thr_grid=grid)
+    X = rng.normal(size=(9001, d)).astype(np.float32)
+    X[rng.random(X.shape) < 0.3] = rng.choice(grid, size=1)[0]
+    X[::37, 0] = np.nan
+    F = T.Forest(f, n_features=d, n_classes=1, agg=oracle.AGG_SUM, device=0)
+    st = F.stats()
+    assert st["sliced_valid"] and st["coded_valid"], st["coded_why"]
+    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1)
+    for banks in ("1", "0"):
+        monkeypatch.setenv("TAHOE_CODE_BANKS", banks)
+        _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, oracle.AGG_SUM, True,
+               want_leaf=False)

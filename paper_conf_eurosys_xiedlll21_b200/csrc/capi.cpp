@@ -98,6 +98,11 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->ds.thr_off);
   cudaFree((void*)f->ds.cb_img);
   cudaFree((void*)f->ds.cb_desc);
+  cudaFree((void*)f->ds.v_src);
+  cudaFree((void*)f->ds.c8_img);
+  cudaFree((void*)f->ds.c8_grp);
+  cudaFree((void*)f->ds.c8_band);
+  cudaFree((void*)f->ds.slice_w);
   cudaFree(f->d_class_ptr);
   cudaFree(f->d_class_parts);
   cudaFree(f->d_cta_start);
@@ -152,7 +157,7 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
   tahoe_status st = encode_direct(f->host, f->di);
   if (st != TAHOE_OK) return st;
   direct_chunks(f);
-  st = encode_sliced(f->host, f->slot_budget, f->sl);
+  st = encode_sliced(f->host, f->slot_budget, f->sl, f->max_smem);
   if (st != TAHOE_OK) return st;
   if (f->device < 0) return TAHOE_OK;
   DeviceGuard g(f->device);
@@ -217,6 +222,21 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
         f->ds.cb_rows = f->sl.cb_rows;
         f->ds.cb_passes = f->sl.cb_passes;
       }
+      if (f->sl.code8) {   // wide codes (reading R8)
+        const int32_t* grp = nullptr;
+        const int32_t* band = nullptr;
+        if ((st = upload(f->sl.v_src, &f->ds.v_src)) != TAHOE_OK) return st;
+        if ((st = upload(f->sl.c8_img, &f->ds.c8_img)) != TAHOE_OK) return st;
+        if ((st = upload(f->sl.c8_grp, &grp)) != TAHOE_OK) return st;
+        if ((st = upload(f->sl.c8_band, &band)) != TAHOE_OK) return st;
+        f->ds.c8_grp = reinterpret_cast<const int4x*>(grp);
+        f->ds.c8_band = reinterpret_cast<const int4x*>(band);
+        f->ds.c8_bands = f->sl.c8_bands;
+        f->ds.vfbits = f->sl.vfbits;
+        f->ds.code8 = 1;
+        std::vector<float> w(f->sl.slice_work.begin(), f->sl.slice_work.end());
+        if ((st = upload(w, &f->ds.slice_w)) != TAHOE_OK) return st;
+      }
     }
   }
   return TAHOE_OK;
@@ -254,6 +274,8 @@ static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   static const bool codes_off = std::getenv("TAHOE_CODES") && std::string(std::getenv("TAHOE_CODES")) == "0";
   st.coded_ok = f->sl.valid && f->sl.code_valid && !codes_off;
   st.code_passes = std::max(1, (1 << f->sl.fbits) / 32);
+  st.code8 = f->sl.code8;
+  if (st.code8) st.code_passes = (1 << f->sl.vfbits) / 32;
   st.sliced_eff = f->sl.eff_sim;
   st.n_slices = f->sl.n_slices;
   st.num_sms = f->num_sms;
@@ -313,7 +335,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   int32_t strat = choose(f, n, d, forced);
   if (strat == -2) return fail(TAHOE_E_UNSUPPORTED, "sliced strategy unavailable: " + f->sl.why_invalid);
   if (strat == -3) return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices unavailable: " + f->sl.code_why);
-  if (strat == TAHOE_STRATEGY_SLICED_CODED) {
+  if (strat == TAHOE_STRATEGY_SLICED_CODED && !f->sl.code8) {
     // the code-tile ring (+ trailers and staged partials) must fit next to the slice
     const int64_t need = (((int64_t)f->sl.slots_max * kSlotBytes + 1023) & ~1023LL) +
                          3LL * code_tile_stride(f->sl.fbits) + kSlicedBarrierBytes + 3LL * kSlicedTileRows * 8;
@@ -402,7 +424,25 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   fa.row_stride = 1;
   fa.class_ptr = f->d_class_ptr;
   fa.class_parts = f->d_class_parts;
-  if (strat == TAHOE_STRATEGY_SLICED_CODED) {
+  if (strat == TAHOE_STRATEGY_SLICED_CODED && f->sl.code8) {
+    // wide codes (reading R8): u8 code tiles + NaN flags from the library pool
+    const int64_t ntiles = (n + kCode8TileRows - 1) / kCode8TileRows;
+    const size_t cbytes = (size_t)ntiles * (size_t)(code8_tile_bytes(f->sl.vfbits) + 16) +
+                          (size_t)f->sl.n_slices * 8;
+    void* cbuf = nullptr;
+    if ((e = scratch_alloc(&cbuf, cbytes, st)) != cudaSuccess) {
+      if (part) cudaFreeAsync(part, st);
+      return fail(TAHOE_E_NOMEM, "cudaMallocAsync code tiles");
+    }
+    SlicedPlan cp = plan;
+    if (f->d_cta_start && ntiles >= 4LL * f->num_sms) {
+      cp.grid = f->num_sms;
+      cp.cta_start = f->d_cta_start;
+    }
+    rc = launch_sliced_codes8(f->ds, cp, X, n, d, static_cast<uint8_t*>(cbuf), o, fused,
+                              f->num_sms, st, ev_b, ev_e);
+    cudaFreeAsync(cbuf, st);
+  } else if (strat == TAHOE_STRATEGY_SLICED_CODED) {
     const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
     const size_t cbytes = (size_t)ntiles * code_tile_stride(f->sl.fbits);
     void* cbuf = nullptr;
@@ -791,6 +831,8 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"coded_valid\":" << (f->sl.code_valid ? "true" : "false")
      << ",\"coded_why\":\"" << f->sl.code_why << "\"" << ",\"coded_thresholds\":"
      << (f->sl.thr_off.empty() ? 0 : f->sl.thr_off.back())
+     << ",\"code8\":" << (f->sl.code8 ? "true" : "false") << ",\"code8_vfbits\":" << f->sl.vfbits
+     << ",\"code8_virtual\":" << f->sl.n_virtual << ",\"code8_bands\":" << f->sl.c8_bands
      << ",\"code_bank_rows\":" << f->sl.cb_rows << ",\"code_bank_passes\":" << f->sl.cb_passes
      << ",\"sliced_fbits\":" << f->sl.fbits << ",\"cta_split\":[" << [&] {
           std::string r;

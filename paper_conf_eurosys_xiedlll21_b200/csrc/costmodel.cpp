@@ -71,6 +71,9 @@ const CostParams& cost_params() {
     if (read_key(js, "a_c", &v)) c.a_c = v;
     if (read_key(js, "b_c", &v)) c.b_c = v;
     if (read_key(js, "e_c", &v)) c.e_c = v;
+    if (read_key(js, "a_w", &v)) c.a_w = v;
+    if (read_key(js, "b_w", &v)) c.b_w = v;
+    if (read_key(js, "e_w", &v)) c.e_w = v;
     c.fitted = all;
     return c;
   }();
@@ -89,6 +92,8 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
     const double passes = st.n_slices <= st.num_sms ? 1.0 : std::ceil((double)st.n_slices / st.num_sms);
     const double eff = st.sliced_eff > 0.05 ? st.sliced_eff : 0.05;
     const double U = (double)((tiles + cps - 1) / cps) * 64.0 * st.V / (st.n_slices * eff) * passes;
+    if (strategy == TAHOE_STRATEGY_SLICED_CODED && st.code8)
+      return c.a_w + c.b_w * U + c.e_w * (double)(tiles * 64) * st.code_passes / std::max(1, st.num_sms);
     if (strategy == TAHOE_STRATEGY_SLICED_CODED)
       return c.a_c + c.b_c * U + c.e_c * (double)(tiles * 64) * st.code_passes / std::max(1, st.num_sms);
     return c.a_s + c.b_s * U * (st.rows_global ? c.g_s : 1.0);

@@ -11,6 +11,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstring>
+#include <limits>
 #include <cstdlib>
 #include <numeric>
 #include <string>
@@ -389,9 +390,108 @@ static void build_code_banks(const std::vector<std::vector<float>>& tabs, int32_
   }
 }
 
-tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
+// Pre-pass tables of the wide codes (reading R8): groups of 32 consecutive virtual attributes, lane
+// a of group g bisecting the sorted thresholds of virtual attribute 32g + a.  Element i of lane a
+// sits at word (row0_g + i) * 32 + a (lane a owns bank a: the 32 probes of a warp never collide);
+// every lane of a group is padded with NaN to 2^k - 1 elements, k = the group's probe count, so
+// the bisection has a uniform trip count ("tab[i] <= x" stays true on a prefix: NaN <= x is
+// false).  Groups are dealt to bands of balanced size <= kCode8BandBudget bytes; a pre-pass CTA
+// stages one band.
+static void build_code8_banks(const std::vector<std::vector<float>>& vt, int32_t vfbits,
+                              SlicedImage& S) {
+  const int32_t G = (1 << vfbits) / 32;
+  std::vector<int32_t> probes(G, 0);
+  int64_t total = 0;
+  for (int32_t g = 0; g < G; g++) {
+    size_t mk = 0;
+    for (int32_t a = 0; a < 32; a++) {
+      const size_t v = (size_t)g * 32 + a;
+      if (v < vt.size()) mk = std::max(mk, vt[v].size());
+    }
+    int32_t k = 0;
+    while (((size_t)1 << k) - 1 < mk) k++;
+    probes[g] = k;
+    total += (((int64_t)1 << k) - 1) * 128;
+  }
+  auto gbytes = [&](int32_t g) { return (((int64_t)1 << probes[g]) - 1) * 128; };
+  std::vector<int32_t> cut;
+  for (int32_t nb = (int32_t)std::max<int64_t>(1, (total + kCode8BandBudget - 1) / kCode8BandBudget);; nb++) {
+    const int64_t target = (total + nb - 1) / nb;
+    cut.assign(1, 0);
+    int32_t g = 0;
+    for (int32_t b = 0; b < nb; b++) {
+      int64_t acc = 0;
+      while (g < G && acc + gbytes(g) <= kCode8BandBudget && (acc < target || b == nb - 1)) acc += gbytes(g++);
+      cut.push_back(g);
+    }
+    if (g == G) break;
+  }
+  cut.erase(std::unique(cut.begin(), cut.end()), cut.end());   // no empty bands
+  S.c8_bands = (int32_t)cut.size() - 1;
+  S.c8_grp.assign((size_t)G * 4, 0);
+  S.c8_band.assign((size_t)S.c8_bands * 4, 0);
+  S.c8_img.clear();
+  const float qnan = std::numeric_limits<float>::quiet_NaN();
+  for (int32_t b = 0; b < S.c8_bands; b++) {
+    const int64_t off_words = (int64_t)S.c8_img.size();
+    int64_t row = 0;
+    for (int32_t g = cut[b]; g < cut[b + 1]; g++) {
+      const int32_t D = (1 << probes[g]) - 1;
+      S.c8_grp[(size_t)g * 4 + 0] = (int32_t)(row * 32);
+      S.c8_grp[(size_t)g * 4 + 1] = probes[g];
+      S.c8_grp[(size_t)g * 4 + 2] = b;
+      S.c8_img.resize((size_t)(off_words + (row + D) * 32), qnan);
+      for (int32_t a = 0; a < 32; a++) {
+        const size_t v = (size_t)g * 32 + a;
+        if (v >= vt.size()) continue;
+        for (size_t i = 0; i < vt[v].size(); i++)
+          S.c8_img[(size_t)(off_words + (row + (int64_t)i) * 32 + a)] = vt[v][i];
+      }
+      row += D;
+    }
+    S.c8_band[(size_t)b * 4 + 0] = (int32_t)(off_words * 4);
+    S.c8_band[(size_t)b * 4 + 1] = (int32_t)(row * 128);
+    S.c8_band[(size_t)b * 4 + 2] = cut[b];
+    S.c8_band[(size_t)b * 4 + 3] = cut[b + 1];
+  }
+}
+
+tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t max_smem) {
   S = SlicedImage();
   S.fbits = feature_bits(F.n_features + 1);   // all-ones attribute field marks a leaf
+  // per attribute the sorted distinct thresholds (IEEE equality: -0.0 and +0.0 are one value),
+  // for the rank codes of readings R7 / R8
+  std::vector<std::vector<float>> tabs(F.n_features);
+  bool sub_leaf = false;
+  for (size_t k = 0; k < F.feat.size(); k++) {
+    if (F.feat[k] >= 0) tabs[F.feat[k]].push_back(F.thr[k]);
+    else if (std::fpclassify(F.val[k]) == FP_SUBNORMAL) sub_leaf = true;
+  }
+  for (auto& v : tabs) {
+    std::sort(v.begin(), v.end(), [](float p, float q) { return p < q; });
+    v.erase(std::unique(v.begin(), v.end(), [](float p, float q) { return p == q; }), v.end());
+  }
+  // Wide codes (reading R8): rows of more than 127 attributes, coded as u8 over virtual attributes
+  // and staged in shared memory next to slices packed for the room the code-tile ring leaves.
+  std::vector<int32_t> vbase(F.n_features + 1, 0);
+  if (max_smem > 0 && S.fbits > kCodeMaxFbits && F.agg != TAHOE_AGG_VOTE && !sub_leaf) {
+    for (int32_t a = 0; a < F.n_features; a++)
+      vbase[a + 1] = vbase[a] + ((int32_t)tabs[a].size() + kCode8MaxRank - 1) / kCode8MaxRank;
+    const int32_t nv = vbase[F.n_features];
+    const int32_t vfb = std::max(5, feature_bits(nv + 1));   // byte 2^V - 1 is the pad a leaf reads
+    if (vfb <= kCode8MaxFbits) {
+      const int64_t room = (int64_t)max_smem - code8_ring_smem(vfb) - kSlicedBarrierBytes;
+      const int32_t cap8 = (int32_t)std::max<int64_t>(0, (room & ~1023LL) / kSlotBytes);
+      bool fits = cap8 >= 16;
+      for (int32_t t = 0; t < F.n_trees && fits; t++) fits = enc_size(F, t) <= cap8 - 1;
+      if (fits) {
+        S.code8 = true;
+        S.vfbits = vfb;
+        S.n_virtual = nv;
+        cap = std::min(cap, cap8);
+      }
+    }
+  }
   cap -= 1;                                    // one terminal slot per lane column
   if (F.agg == TAHOE_AGG_VOTE) { S.why_invalid = "VOTE runs on the direct strategy"; return TAHOE_OK; }
   if (cap < 1) { S.why_invalid = "no shared memory budget"; return TAHOE_OK; }
@@ -503,20 +603,30 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
   // kernel adds internal words, which are subnormal as floats, with flush-to-zero).
   S.code_valid = true;
   S.code_why.clear();
-  if (S.fbits > kCodeMaxFbits) { S.code_valid = false; S.code_why = "too many attributes for u16 code rows"; }
-  std::vector<std::vector<float>> tabs(F.n_features);
-  if (S.code_valid) {
-    for (size_t k = 0; k < F.feat.size(); k++) {
-      if (F.feat[k] >= 0) tabs[F.feat[k]].push_back(F.thr[k]);
-      else if (std::fpclassify(F.val[k]) == FP_SUBNORMAL) { S.code_valid = false; S.code_why = "subnormal leaf value"; }
-    }
+  if (sub_leaf) { S.code_valid = false; S.code_why = "subnormal leaf value"; }
+  else if (S.code8) {
+    // reading R8: virtual attribute vbase[a] + k codes thresholds tab_a[127k .. 127k + 126]
+    std::vector<std::vector<float>> vt((size_t)S.n_virtual);
+    S.v_src.assign((size_t)1 << S.vfbits, -1);
+    S.thr_off.assign(S.n_virtual + 1, 0);
+    for (int32_t a = 0; a < F.n_features; a++)
+      for (int32_t v = vbase[a]; v < vbase[a + 1]; v++) {
+        const size_t i0 = (size_t)(v - vbase[a]) * kCode8MaxRank;
+        const size_t i1 = std::min(tabs[a].size(), i0 + kCode8MaxRank);
+        vt[v].assign(tabs[a].begin() + i0, tabs[a].begin() + i1);
+        S.v_src[v] = a;
+      }
+    for (int32_t v = 0; v < S.n_virtual; v++) S.thr_off[v + 1] = S.thr_off[v] + (int32_t)vt[v].size();
+    for (auto& v : vt) S.thr_tab.insert(S.thr_tab.end(), v.begin(), v.end());
+    build_code8_banks(vt, S.vfbits, S);
+  } else if (S.fbits > kCodeMaxFbits) {
+    S.code_valid = false;
+    S.code_why = "too many attributes for u16 code rows (and no room for wide code tiles)";
+  } else {
     S.thr_off.assign(F.n_features + 1, 0);
     for (int32_t a = 0; a < F.n_features && S.code_valid; a++) {
-      auto& v = tabs[a];
-      std::sort(v.begin(), v.end(), [](float p, float q) { return p < q; });
-      v.erase(std::unique(v.begin(), v.end(), [](float p, float q) { return p == q; }), v.end());
-      if ((int32_t)v.size() > kCodeMaxRank) { S.code_valid = false; S.code_why = "too many distinct thresholds for one attribute"; }
-      S.thr_off[a + 1] = S.thr_off[a] + (int32_t)v.size();
+      if ((int32_t)tabs[a].size() > kCodeMaxRank) { S.code_valid = false; S.code_why = "too many distinct thresholds for one attribute"; }
+      S.thr_off[a + 1] = S.thr_off[a] + (int32_t)tabs[a].size();
     }
     if (S.code_valid) {
       S.thr_tab.reserve(S.thr_off[F.n_features]);
@@ -524,12 +634,24 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
       build_code_banks(tabs, S.fbits, S);
     }
   }
-  auto rank_of = [&](int32_t a, float b) -> uint32_t {   // t = j + 1
+  auto index_of = [&](int32_t a, float b) -> uint32_t {   // j: b == tab_a[j]
     const auto& v = tabs[a];
-    const size_t j = (size_t)(std::lower_bound(v.begin(), v.end(), b, [](float p, float q) { return p < q; }) - v.begin());
-    return (uint32_t)j + 1u;
+    return (uint32_t)(std::lower_bound(v.begin(), v.end(), b, [](float p, float q) { return p < q; }) - v.begin());
   };
-  const int32_t csh = S.fbits + 2;   // code words: off_bytes << (F+2) | dl << (F+1) | attribute << 1
+  auto rank_of = [&](int32_t a, float b) -> uint32_t {   // t = j + 1 (R8: within the piece)
+    const uint32_t j = index_of(a, b);
+    return S.code8 ? j % (uint32_t)kCode8MaxRank + 1u : j + 1u;
+  };
+  auto code_attr = [&](int32_t a, float b) -> uint32_t {   // attribute field of a code word
+    return S.code8 ? (uint32_t)vbase[a] + index_of(a, b) / (uint32_t)kCode8MaxRank : (uint32_t)a << 1;
+  };
+  // code words: R7 off_bytes << (F+2) | dl << (F+1) | attribute << 1;
+  //             R8 off_bytes << (V+1) | dl << V | virtual attribute
+  const int32_t csh = S.code8 ? S.vfbits + 1 : S.fbits + 2;
+  const uint32_t cdl = S.code8 ? 1u << S.vfbits : 1u << (S.fbits + 1);
+  const uint32_t cleaf = S.code8 ? (1u << S.vfbits) - 1u : fmask << 1;
+  if (S.code_valid && S.code8 && (uint32_t)S.slots_max >= (1u << (32 - csh - sb)))
+    return fail(TAHOE_E_UNSUPPORTED, "wide-code offset overflow");
   S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   if (S.code_valid) S.cnodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
@@ -551,8 +673,8 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
           const uint32_t yleaf1 = (2u << sb) << (S.fbits + 3) | (fmask << 2);
           const uint32_t yleaf2 = (1u << sb) << (S.fbits + 3) | (fmask << 2);
           const uint32_t ys[3] = {ynode, yleaf1, yleaf2};
-          const uint32_t cys[3] = {(2u << sb) << csh, (2u << sb) << csh | (fmask << 1),
-                                   (1u << sb) << csh | (fmask << 1)};
+          const uint32_t cys[3] = {(2u << sb) << csh, (2u << sb) << csh | cleaf,
+                                   (1u << sb) << csh | cleaf};
           for (int32_t q = 0; q < 3; q++) {
             const size_t w = ((size_t)s * per_slice + (size_t)(pos + q) * C + l);
             S.nodes[2 * w] = q == 0 ? 0u : f2u(F.val[k]);
@@ -583,7 +705,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
           if (F.feat[k] < 0) {
             if ((uint32_t)(next_root - sl) >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "leaf offset overflow");
             y = ((uint32_t)(next_root - sl) << (S.fbits + 3 + sb)) | (fmask << 2);
-            cy = ((uint32_t)(next_root - sl) << (csh + sb)) | (fmask << 1);
+            cy = ((uint32_t)(next_root - sl) << (csh + sb)) | cleaf;
             S.nodes[2 * w] = f2u(F.val[k]);
             if (S.code_valid) S.cnodes[2 * w] = f2u(F.val[k]);
             S.leaf_meta[2 * w] = F.tree_orig[t];
@@ -594,8 +716,8 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
             if (delta <= 0 || (uint32_t)delta >= off_lim) return fail(TAHOE_E_UNSUPPORTED, "right offset overflow");
             y = ((uint32_t)delta << (S.fbits + 3 + sb)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 2)) |
                 ((uint32_t)F.feat[k] << 2);
-            cy = ((uint32_t)delta << (csh + sb)) | ((F.dl[k] ? 1u : 0u) << (S.fbits + 1)) |
-                 ((uint32_t)F.feat[k] << 1);
+            cy = ((uint32_t)delta << (csh + sb)) | (F.dl[k] ? cdl : 0u) |
+                 (S.code_valid ? code_attr(F.feat[k], F.thr[k]) : 0u);
             S.nodes[2 * w] = f2u(F.thr[k]);
             if (S.code_valid) S.cnodes[2 * w] = rank_of(F.feat[k], F.thr[k]);
           }
@@ -608,7 +730,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S) {
       const size_t w = ((size_t)s * per_slice + (size_t)pos * C + l);
       S.nodes[2 * w] = 0u;
       S.nodes[2 * w + 1] = fmask << 2;
-      if (S.code_valid) { S.cnodes[2 * w] = 0u; S.cnodes[2 * w + 1] = fmask << 1; }
+      if (S.code_valid) { S.cnodes[2 * w] = 0u; S.cnodes[2 * w + 1] = cleaf; }
       S.col_len[(size_t)s * C + l] = pos;
     }
   }

@@ -102,6 +102,20 @@ struct SlicedImage {
   std::vector<float> cb_img;                     // [cb_rows][32] words: the shared-memory image
   std::vector<int32_t> cb_desc;                  // [passes][32 lanes] {slot, attribute, word0, sh<<16|K}
   int32_t cb_passes = 0, cb_rows = 0;
+  // Wide rank codes (reading R8): rows of more than 127 attributes become u8 codes over VIRTUAL
+  // attributes (an attribute with K distinct thresholds is split into ceil(K / 127) pieces, each
+  // coding its own <= 127 thresholds), so that a 16-row tile of code rows can be staged in shared
+  // memory next to a (smaller) slice.  When code8 is set, cnodes hold the u8 node words
+  // (kernels.hpp "wide codes"), thr_tab/thr_off are per virtual attribute and v_src maps a
+  // virtual attribute to its source column.
+  bool code8 = false;
+  int32_t vfbits = 0;                            // code row = 2^vfbits bytes
+  int32_t n_virtual = 0;
+  std::vector<int32_t> v_src;                    // [2^vfbits] source column, -1 = pad byte
+  std::vector<float> c8_img;                     // pre-pass tables, bank-private, band after band
+  std::vector<int32_t> c8_grp;                   // [2^vfbits / 32] {word offset in band, probes, band, 0}
+  std::vector<int32_t> c8_band;                  // [bands] {byte offset, bytes, first group, end group}
+  int32_t c8_bands = 0;
   int64_t bytes() const { return (int64_t)nodes.size() * 4; }
 };
 
@@ -115,7 +129,9 @@ struct DirectImage {
 
 int32_t feature_bits(int32_t n_features);
 tahoe_status encode_direct(const Forest& F, DirectImage& D);
-tahoe_status encode_sliced(const Forest& F, int32_t slot_budget, SlicedImage& S);
+// max_smem > 0 enables the wide rank codes (reading R8) for forests over more than 127 attributes:
+// the slices are then packed for the smaller budget that leaves room for the u8 code-tile ring.
+tahoe_status encode_sliced(const Forest& F, int32_t slot_budget, SlicedImage& S, int32_t max_smem = 0);
 
 // Cost model (costmodel.cpp) — Algorithm 1 lines 8-13 re-targeted.
 struct PlanStats {
@@ -128,6 +144,7 @@ struct PlanStats {
   bool wide_rows = false;    // d > 256: direct reads attributes from rows far apart in memory
   bool coded_ok = false;     // rank-coded twin available and enabled (reading R7)
   int32_t code_passes = 1;   // row-coding passes of 32 attributes
+  bool code8 = false;        // the coded twin is the wide-code one (reading R8)
 };
 // Fitted per-platform constants (costmodel_b200.json, scripts/fit_costmodel.py), microseconds.
 struct CostParams {
@@ -136,6 +153,7 @@ struct CostParams {
   double a_d = 11.8, l_d = 0.34, b_d = 6.3e-4; // direct: launch; per-visit latency; per unit
   double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
   double a_c = 30.0, b_c = 6.6e-5, e_c = 1.6e-5; // coded: launches; per unit; per row-pass per SM
+  double a_w = 40.0, b_w = 1.5e-4, e_w = 1.6e-5; // wide codes (reading R8): the same three terms
   bool fitted = false;
 };
 const CostParams& cost_params();

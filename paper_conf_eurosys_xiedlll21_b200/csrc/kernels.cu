@@ -1494,6 +1494,438 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   return (int)e;
 }
 
+// ------------------------------------------------------------------ wide rank codes (reading R8)
+// Rows of more than 127 attributes (C4: 2000).  A row becomes 2^V u8 codes over virtual
+// attributes (kernels.hpp "wide codes"): 2 KB for C4 instead of 8 KB of fp32, so 16-row tiles fit
+// in shared memory next to a slice and the walk's attribute reads stop going to L2.
+
+// k_encode_rows8: CTA = (band b, row chunk).  The CTA bulk-copies band b's bank-private tables
+// (encode.cpp build_code8_banks) into shared memory; a warp then codes kR rows at a time, group by
+// group of the band: lane a bisects virtual attribute 32g + a with the group's uniform probe count
+// (one conflict-free LDS per probe for the warp) and writes its code byte (32 consecutive bytes
+// per row and group).  A tile's NaN flag is set by whichever band meets a NaN.
+struct Encode8Args {
+  const float* X;
+  int64_t n;
+  int32_t d, vfbits, bands, chunks;
+  const float* img;
+  const int4* grp;
+  const int4* band;
+  const int32_t* v_src;
+  uint8_t* codes;
+  uint32_t* flags;   // 4 words per tile, word 0 = NaN flag
+};
+
+// pos[q] := #{tab <= x[q]} over a lane's 2^K - 1 table elements at base + i * 128 bytes (NaN pads
+// compare false): probe at pos + step - 1 for step = 2^(K-1) .. 1.  The running address a[q] =
+// base + pos[q] * 128 makes every probe one LDS with an immediate offset, one FSETP and one
+// predicated add.
+template <int K, int kR>
+__device__ __forceinline__ void bisect8(uint32_t base, const float* x, uint32_t* pos) {
+  uint32_t ad[kR];
+#pragma unroll
+  for (int q = 0; q < kR; q++) ad[q] = base;
+#pragma unroll
+  for (int st = K - 1; st >= 0; st--) {
+#pragma unroll
+    for (int q = 0; q < kR; q++) {
+      float t;
+      asm("ld.shared.f32 %0, [%1];" : "=f"(t) : "r"(ad[q] + (((1u << st) - 1u) << 7)));
+      ad[q] += t <= x[q] ? (1u << st) << 7 : 0u;
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < kR; q++) pos[q] = (ad[q] - base) >> 7;
+}
+
+__global__ void __launch_bounds__(1024, 1) k_encode_rows8(const Encode8Args a) {
+  extern __shared__ __align__(1024) float s_img[];
+  __shared__ uint64_t s_bar;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = blockDim.x >> 5;
+  const int b = blockIdx.x % a.bands;
+  const int64_t chunk = blockIdx.x / a.bands;
+  const int4 bd = __ldg(&a.band[b]);
+  if (threadIdx.x == 0) {
+    mbar_init(&s_bar, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (bd.y > 0) {
+    if (threadIdx.x == 0) {
+      fence_proxy_async_smem();
+      mbar_expect_tx(&s_bar, (uint32_t)bd.y);
+      bulk_g2s_big(s_img, reinterpret_cast<const unsigned char*>(a.img) + bd.x, (uint32_t)bd.y, &s_bar);
+    }
+    mbar_wait(&s_bar, 0);
+  }
+  constexpr int kR = 8;
+  static_assert(kCode8TileRows % kR == 0, "a row group stays inside one tile");
+  // this chunk's rows, in whole groups of kR
+  const int64_t groups = (a.n + kR - 1) / kR;
+  const int64_t per = (groups + a.chunks - 1) / a.chunks;
+  const int64_t r_lo = chunk * per * kR;
+  const int64_t r_hi = min(a.n, (chunk + 1) * per * kR);
+  const uint32_t V = (uint32_t)a.vfbits;
+  const int64_t tile_bytes = (int64_t)kCode8TileRows << V;
+  const uint32_t sbase = smem_u32(s_img) + (uint32_t)lane * 4u;
+  for (int64_t r0 = r_lo + (int64_t)warp * kR; r0 < r_hi; r0 += (int64_t)W * kR) {
+    const bool full = r0 + kR <= r_hi;
+    bool nan_any = false;
+    uint8_t* row0 = a.codes + (r0 >> 4) * tile_bytes + ((r0 & 15) << V);
+    // the next group's attribute values are loaded before this group is searched
+    auto load_x = [&](int g, float* x, int& src) {
+      src = g < bd.w ? __ldg(&a.v_src[g * 32 + lane]) : -1;
+      const float* xs = a.X + r0 * a.d + (src >= 0 ? src : 0);
+#pragma unroll
+      for (int q = 0; q < kR; q++) x[q] = (src >= 0 && (full || r0 + q < r_hi)) ? __ldg(xs + (int64_t)q * a.d) : 0.0f;
+    };
+    float xn[kR];
+    int srcn;
+    load_x(bd.z, xn, srcn);
+    for (int g = bd.z; g < bd.w; g++) {
+      const int4 gd = __ldg(&a.grp[g]);
+      const int v = g * 32 + lane;
+      const int src = srcn;
+      float x[kR];
+#pragma unroll
+      for (int q = 0; q < kR; q++) x[q] = xn[q];
+      load_x(g + 1, xn, srcn);
+      uint32_t pos[kR];
+      const uint32_t base = sbase + (uint32_t)gd.x * 4u;
+      switch (gd.y) {   // probe count: a uniform, fully unrolled bisection per group
+        case 0: for (int q = 0; q < kR; q++) pos[q] = 0; break;
+        case 1: bisect8<1, kR>(base, x, pos); break;
+        case 2: bisect8<2, kR>(base, x, pos); break;
+        case 3: bisect8<3, kR>(base, x, pos); break;
+        case 4: bisect8<4, kR>(base, x, pos); break;
+        case 5: bisect8<5, kR>(base, x, pos); break;
+        case 6: bisect8<6, kR>(base, x, pos); break;
+        default: bisect8<7, kR>(base, x, pos); break;
+      }
+#pragma unroll
+      for (int q = 0; q < kR; q++) {
+        if (!full && r0 + q >= r_hi) continue;
+        const bool isnan_q = src >= 0 && x[q] != x[q];
+        nan_any |= isnan_q;
+        const int8_t c = src < 0 ? kCode8Pad : (isnan_q ? kCode8Nan : (int8_t)pos[q]);
+        row0[((uint32_t)q << V) + (uint32_t)v] = (uint8_t)c;
+      }
+    }
+    if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 >> 4) * 4] = 1u;
+  }
+}
+
+struct Coded8KArgs {
+  DevSliced img;
+  const uint8_t* codes;
+  const uint32_t* flags;
+  int32_t* tile_next;    // [ns] next unclaimed tile of each slice (zeroed per launch)
+  int32_t* cta_on;       // [ns] CTAs currently working on each slice (zeroed per launch)
+  const float* work;     // [ns] simulated lane-steps per row of each slice (slice choice weights)
+  int64_t n;
+  int32_t forest_smem;   // bytes reserved for the slice (multiple of 1024)
+  const int32_t* cta_start;  // initial CTA -> slice map (prefix), or nullptr: blockIdx % ns
+  OutArgs o;
+};
+
+// One step on a wide-coded slice: node {x = t or leaf value, y}, code byte at (y & amask) | row,
+// left iff code < t (NaN-aware: or NaN and default-left), right / next root at +(y >> (V+1)).
+template <bool NAN_AWARE>
+__device__ __forceinline__ float coded8_step(uint32_t& p, uint32_t rowaddr, uint32_t amask,
+                                             uint32_t dlbit, uint32_t shmul) {
+  uint32_t x, y;
+  int32_t c;
+  asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+  asm("ld.shared.s8 %0, [%1];" : "=r"(c) : "r"((y & amask) | rowaddr));
+  bool go_left = (uint32_t)c < x;
+  if (NAN_AWARE) go_left = go_left || ((c == (int32_t)kCode8Nan) && (y & dlbit));
+  p += go_left ? (uint32_t)kSlotBytes : __umulhi(y, shmul);
+  return __uint_as_float(x);
+}
+
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_coded8(uint32_t pA, uint32_t pB, uint32_t pe, uint32_t rowA,
+                                            uint32_t rowB, uint32_t amask, uint32_t dlbit,
+                                            uint32_t shmul, double& accA, double& accB) {
+  accA = 0.0;
+  accB = 0.0;
+  while ((pA != pe) | (pB != pe)) {
+    const float a1 = coded8_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul);
+    const float b1 = coded8_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul);
+    const float a2 = coded8_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul);
+    const float b2 = coded8_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul);
+    add_pair_ftz(accA, a1, a2);
+    add_pair_ftz(accB, b1, b2);
+  }
+}
+
+// k_sliced_codes8: k_sliced_codes' walk (slice resident in shared memory, dynamic 4-row work
+// units, half-warp per row, two chains per lane, ring refilled by the warp closing a tile) over
+// 16-row tiles of u8 code rows; unit u of a tile: half h walks rows u + 4h (chain A) and
+// u + 8 + 4h (chain B).  Tiles are claimed dynamically from a per-slice global counter, in
+// increasing order (so the ~30 slices sweep the code rows together and each tile is read from
+// HBM about once); a CTA whose slice runs out of tiles moves to the slice with the most remaining
+// work per CTA (re-staging that slice), so no SM idles while another slice still has tiles.
+// Ring entries are numbered by a CTA-wide sequence; entry e uses buffer e % 3 and that buffer's
+// mbarrier phase e / 3, and the warp releasing the last unit of entry e issues entry e + 3.  The
+// ring holds 12 units, fewer than the CTA's warps, so a warp may grab a unit of an entry not
+// issued yet: it waits until the buffer's ticket names its entry (set by the issuing warp), and
+// only then on the mbarrier phase, which is then the current one.  Once the slice's tiles are
+// all claimed, entries are issued EMPTY (tile -1, the phase completes without data) and released
+// like the others, so the chain of tickets never stalls; a warp leaves the slice when it meets an
+// empty entry and every valid entry issued so far has been released.
+constexpr int kCode8Threads = 512;
+template <bool FUSED>
+__global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {
+  constexpr int C = kSlicedCols;
+  constexpr int R = kCode8TileRows;
+  constexpr int kR8 = kCode8Ring;
+  constexpr int kUnits = R / 4;
+  extern __shared__ __align__(1024) unsigned char smem[];
+  const uint32_t V = (uint32_t)a.img.vfbits;
+  const uint32_t RB = 1u << V;
+  const uint32_t tile_bytes = (uint32_t)R << V;
+  const uint32_t sbase = smem_u32(smem);
+  const uint32_t ring_off = ((sbase + (uint32_t)a.forest_smem + RB - 1u) & ~(RB - 1u)) - sbase;
+  unsigned char* s_ring = smem + ring_off;
+  uint32_t* s_flag = reinterpret_cast<uint32_t*>(s_ring + (size_t)kR8 * tile_bytes);
+  double* s_part = reinterpret_cast<double*>(s_flag + kR8 * 4);
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_part + kR8 * R);      // [3]
+  uint64_t* s_forest = s_full + kR8;                                       // [1]
+  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full + 4);  // unit counter
+  int* s_cnt = reinterpret_cast<int*>(s_full + 5);                         // [3] units released
+  uint32_t* s_gen = reinterpret_cast<uint32_t*>(s_cnt + 4);                // [3] ticket: entry issued
+  int32_t* s_tile = reinterpret_cast<int32_t*>(s_gen + 4);                 // [3] tile of the entry
+  uint32_t* s_vis = reinterpret_cast<uint32_t*>(s_tile + 4);              // valid entries issued
+  uint32_t* s_vdone = reinterpret_cast<uint32_t*>(s_tile + 5);            // valid entries released
+  int32_t* s_slice = reinterpret_cast<int32_t*>(s_tile + 6);
+  uint32_t* s_issued = reinterpret_cast<uint32_t*>(s_tile + 7);           // entries issued
+  const int lane = threadIdx.x & 31;
+  const int col = lane & (C - 1);
+  const int half = lane >> 4;
+  const uint32_t amask = RB - 1u;
+  const uint32_t dlbit = RB;
+  const uint32_t shmul = 1u << (32 - (V + 1));
+  const int32_t ns = a.img.n_slices;
+  const int32_t ntiles = (int32_t)((a.n + R - 1) / R);
+
+  if (threadIdx.x == 0) {
+    for (int b = 0; b < kR8; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; s_gen[b] = 0xffffffffu; }
+    mbar_init(s_forest, 1);
+    fence_mbar_init();
+    int32_t sl = (int32_t)blockIdx.x % ns;
+    if (a.cta_start) {
+      sl = 0;
+      while (sl + 1 < ns && __ldg(&a.cta_start[sl + 1]) <= (int32_t)blockIdx.x) sl++;
+    }
+    *s_slice = sl;
+    atomicAdd(&a.cta_on[sl], 1);
+  }
+  __syncthreads();
+
+  uint32_t g = 0;   // sequence number of this slice's first ring entry
+  uint32_t ph_forest = 0;
+  // claim the slice's next tile for entry e (buffer e % 3) and issue its copies; past the slice's
+  // last tile the entry is marked empty (its mbarrier phase completes without data)
+  auto issue = [&](int sl, uint32_t e) {
+    if (lane == 0) {
+      const int b = (int)(e % kR8);
+      const int32_t tile = atomicAdd(&a.tile_next[sl], 1);
+      const bool ok = tile < ntiles;
+      s_tile[b] = ok ? tile : -1;
+      __threadfence_block();   // the buffer's previous partials were read before this point
+      *reinterpret_cast<volatile uint32_t*>(&s_gen[b]) = e;
+      if (!ok) {
+        mbar_expect_tx(&s_full[b], 0u);
+      } else {
+        atomicAdd(s_vis, 1u);
+        fence_proxy_async_smem();
+        mbar_expect_tx(&s_full[b], tile_bytes + 16u);
+        bulk_g2s(s_ring + (size_t)b * tile_bytes, a.codes + (int64_t)tile * tile_bytes, tile_bytes, &s_full[b]);
+        bulk_g2s(s_flag + b * 4, a.flags + (int64_t)tile * 4, 16u, &s_full[b]);
+      }
+      atomicAdd(s_issued, 1u);
+    }
+    __syncwarp();
+  };
+
+  for (;;) {
+    const int32_t sl = *s_slice;
+    if (sl < 0) break;
+    if (threadIdx.x == 0) {
+      *s_next = 0ull;
+      *s_vis = 0u;
+      *s_vdone = 0u;
+      *s_issued = 0u;
+      // the last slice's trailing (empty) entries may have been released only partly
+      for (int b = 0; b < kR8; b++) s_cnt[b] = 0;
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      if (lane == 0) {
+        const uint32_t bytes = (uint32_t)a.img.slots[sl] * (uint32_t)kSlotBytes;
+        fence_proxy_async_smem();
+        mbar_expect_tx(s_forest, bytes);
+        bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
+      }
+      for (uint32_t q = 0; q < (uint32_t)kR8; q++) issue(sl, g + q);
+    }
+    const uint32_t p0 = sbase + (uint32_t)col * 8u;
+    const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+    mbar_wait(s_forest, ph_forest);
+    ph_forest ^= 1u;
+    for (;;) {
+      unsigned long long q = 0;
+      if (lane == 0) q = atomicAdd(s_next, 1ull);
+      q = __shfl_sync(0xffffffffu, q, 0);
+      const uint32_t it = (uint32_t)(q / kUnits);
+      const int u = (int)(q % kUnits);
+      const uint32_t e = g + it;
+      const int b = (int)(e % kR8);
+      if (lane == 0)
+        while (*reinterpret_cast<volatile uint32_t*>(&s_gen[b]) != e) __nanosleep(128);
+      __syncwarp();
+      mbar_wait(&s_full[b], (e / kR8) & 1u);
+      const int32_t tile = *reinterpret_cast<volatile int32_t*>(&s_tile[b]);
+      const int64_t r0 = (int64_t)tile * R;
+      const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+      if (tile >= 0 && u < nr) {
+        const int rA = u + (R / 4) * half, rB = rA + R / 2;
+        const bool okA = rA < nr, okB = rB < nr;
+        const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
+        const uint32_t tb = sbase + ring_off + (uint32_t)b * tile_bytes;
+        const uint32_t rowA = tb + ((uint32_t)(okA ? rA : u) << V);
+        const uint32_t rowB = tb + ((uint32_t)(okB ? rB : u) << V);
+        uint32_t nan_flag;
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(smem_u32(s_flag + b * 4)));
+        double accA, accB;
+        if (nan_flag)
+          walk_coded8<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        else
+          walk_coded8<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        // butterfly over the 16 lane columns: after the xor-8 exchange lanes with bit 3 clear
+        // hold chain A, set hold chain B (lanes 0, 8, 16, 24 own rows rA(h=0), rB(h=0), rA(h=1),
+        // rB(h=1))
+        const bool b3 = lane & 8;
+        double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
+#pragma unroll
+        for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        const int rr = b3 ? rB : rA;
+        if ((lane & 7) == 0 && (b3 ? okB : okA)) {
+          if (FUSED) write_scalar(a.o, r0 + rr, v);
+          else s_part[b * R + rr] = v;
+        }
+      }
+      // release the unit; the warp closing the entry writes its partials and issues entry e + 3
+      __syncwarp();
+      int last = 0;
+      if (lane == 0) {
+        __threadfence_block();
+        last = atomicAdd(&s_cnt[b], 1) == kUnits - 1;
+        if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
+      }
+      last = __shfl_sync(0xffffffffu, last, 0);
+      if (last) {
+        if (FUSED || tile < 0) {
+          issue(sl, e + kR8);
+        } else {
+          const double p = lane < nr ? s_part[b * R + lane] : 0.0;
+          __syncwarp();
+          issue(sl, e + kR8);
+          if (lane < nr) a.o.raw[(size_t)sl * a.n + r0 + lane] = p;
+        }
+        if (tile >= 0 && lane == 0) atomicAdd(s_vdone, 1u);
+      }
+      if (tile < 0) {
+        int done = 0;
+        if (lane == 0)
+          done = *reinterpret_cast<volatile uint32_t*>(s_vdone) == *reinterpret_cast<volatile uint32_t*>(s_vis);
+        if (__shfl_sync(0xffffffffu, done, 0)) break;
+      }
+    }
+    __syncthreads();   // every entry of this slice is consumed or empty
+    const uint32_t issued = *s_issued;
+    g += issued;
+    // the forest barrier completed one phase this slice: re-init for the next one
+    if (threadIdx.x == 0) {
+      atomicSub(&a.cta_on[sl], 1);
+      // next slice: the most remaining work per CTA already on it
+      int32_t best = -1;
+      float bw = 0.0f;
+      for (int32_t s2 = 0; s2 < ns; s2++) {
+        const int32_t rem = ntiles - *reinterpret_cast<volatile int32_t*>(&a.tile_next[s2]);
+        const int32_t on = *reinterpret_cast<volatile int32_t*>(&a.cta_on[s2]);
+        if (rem < 1 || (on > 0 && rem < 2)) continue;   // a slice nobody works on is always taken
+        const float w = (float)rem * __ldg(&a.work[s2]) / (float)(1 + on);
+        if (w > bw) { bw = w; best = s2; }
+      }
+      if (best >= 0) atomicAdd(&a.cta_on[best], 1);
+      *s_slice = best;
+    }
+    __syncthreads();
+  }
+}
+
+int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
+                         int32_t d, uint8_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
+                         void* stream, void* ev_b, void* ev_e) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const int64_t ntiles = (n + kCode8TileRows - 1) / kCode8TileRows;
+  const int64_t tbytes = code8_tile_bytes(img.vfbits);
+  uint32_t* flags = reinterpret_cast<uint32_t*>(codes + ntiles * tbytes);
+  // NaN flags (16 bytes per tile), then the per-slice tile counters and CTA counts
+  cudaError_t e = cudaMemsetAsync(flags, 0, (size_t)ntiles * 16 + (size_t)img.n_slices * 8, st);
+  if (e != cudaSuccess) return (int)e;
+  Encode8Args ea;
+  ea.X = X;
+  ea.n = n;
+  ea.d = d;
+  ea.vfbits = img.vfbits;
+  ea.bands = img.c8_bands;
+  ea.chunks = std::max(1, num_sms / std::max(1, img.c8_bands));
+  ea.img = img.c8_img;
+  ea.grp = reinterpret_cast<const int4*>(img.c8_grp);
+  ea.band = reinterpret_cast<const int4*>(img.c8_band);
+  ea.v_src = img.v_src;
+  ea.codes = codes;
+  ea.flags = flags;
+  {
+    static std::atomic<int> configured[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && !configured[dev].load()) {
+      e = cudaFuncSetAttribute(k_encode_rows8, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
+      if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_sliced_codes8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+      if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_sliced_codes8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+      if (e != cudaSuccess) return (int)e;
+      configured[dev].store(1);
+    }
+  }
+  k_encode_rows8<<<ea.bands * ea.chunks, 1024, kCode8BandBudget, st>>>(ea);
+  if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
+
+  Coded8KArgs a{};
+  a.img = img;
+  a.codes = codes;
+  a.flags = flags;
+  a.tile_next = reinterpret_cast<int32_t*>(flags + ntiles * 4);
+  a.cta_on = a.tile_next + img.n_slices;
+  a.work = img.slice_w;
+  a.n = n;
+  a.forest_smem = plan.forest_smem;
+  a.cta_start = plan.cta_start;
+  a.o = o;
+  const int smem = plan.forest_smem + (int)code8_ring_smem(img.vfbits) + kSlicedBarrierBytes;
+  if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+  if (fused) k_sliced_codes8<true><<<plan.grid, kCode8Threads, smem, st>>>(a);
+  else k_sliced_codes8<false><<<plan.grid, kCode8Threads, smem, st>>>(a);
+  e = cudaGetLastError();
+  if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+  return (int)e;
+}
+
 int launch_finalize(const FinalizeArgs& a, void* stream) {
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);

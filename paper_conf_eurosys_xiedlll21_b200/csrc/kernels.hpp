@@ -30,6 +30,8 @@ struct DevDirect {
   int64_t n_nodes = 0;
 };
 
+struct int4x { int32_t x, y, z, w; };   // host-side stand-in for CUDA's int4 (same layout)
+
 struct DevSliced {
   const uint32_t* nodes = nullptr;   // [ns][slots_max][32] uint2
   const int32_t* col_len = nullptr;  // [ns][32]
@@ -47,6 +49,15 @@ struct DevSliced {
   const float* cb_img = nullptr;     // bank-private tables (cb_rows x 32 words) or nullptr
   const int32_t* cb_desc = nullptr;  // [cb_passes][32] int4
   int32_t cb_rows = 0, cb_passes = 0;
+  // wide rank codes (reading R8): cnodes hold u8-code node words when code8 != 0
+  int32_t code8 = 0;
+  int32_t vfbits = 0;                // code row = 2^vfbits bytes
+  const int32_t* v_src = nullptr;    // [2^vfbits] source column of each code byte, -1 = pad
+  const float* c8_img = nullptr;     // pre-pass tables (bank-private, band after band)
+  const int4x* c8_grp = nullptr;     // [2^vfbits / 32] {word offset in band, probes, band, 0}
+  const int4x* c8_band = nullptr;    // [bands] {byte offset, bytes, first group, end group}
+  int32_t c8_bands = 0;
+  const float* slice_w = nullptr;    // [ns] simulated lane-steps per row (dynamic slice choice)
 };
 
 // ------------------------------------------------------------------ rank-coded rows (reading R7)
@@ -68,6 +79,32 @@ inline int32_t code_tile_bytes(int32_t fbits) { return 64 * code_row_bytes(fbits
 // a code tile in HBM and in the ring: the rows, then a 128-byte trailer whose first word is the
 // tile's NaN flag (1 if any of its codes is kCodeNan; it arrives with the tile's bulk copy)
 inline int32_t code_tile_stride(int32_t fbits) { return code_tile_bytes(fbits) + 128; }
+
+// ------------------------------------------------------------------ wide codes (reading R8)
+// Rows of more than 127 attributes: an attribute with K distinct thresholds becomes ceil(K / 127)
+// VIRTUAL attributes; piece k codes thresholds tab[127k .. 127k + 126] as
+// code_k(x) = #{i in the piece : tab[i] <= x} = clamp(code(x) - 127k, 0, 127), and a node whose
+// threshold is tab[i] reads piece k = i / 127 with t = i - 127k + 1, so that
+// x < tab[i]  <=>  code(x) < i + 1  <=>  code_k(x) < t  (R7's exactness, piece by piece).  Codes are
+// s8: 0 .. 127, NaN kCode8Nan (-2), pad kCode8Pad (-1); loaded sign-extended they exceed every node
+// word like R7's u16 codes.  A code row is 2^V bytes (V = vfbits, all-ones byte = the pad a leaf
+// reads); node words: internal x = t, y = off_bytes << (V+1) | default_left << V | virtual
+// attribute; leaf x = value, y = off_bytes << (V+1) | (2^V - 1).  Tiles of kCode8TileRows rows;
+// the tiles' NaN flags sit in a separate array (16 bytes per tile) that rides along with each
+// tile's bulk copy.
+constexpr int32_t kCode8MaxRank = 127;
+constexpr int32_t kCode8MaxFbits = 12;           // rows of <= 4 KB
+constexpr int32_t kCode8TileRows = 16;
+constexpr int32_t kCode8Ring = 3;
+constexpr int32_t kCode8BandBudget = 200 * 1024; // pre-pass tables per CTA
+constexpr int8_t kCode8Nan = -2;
+constexpr int8_t kCode8Pad = -1;
+inline int64_t code8_tile_bytes(int32_t vfbits) { return (int64_t)kCode8TileRows << vfbits; }
+// shared memory next to the slice: the ring (aligned to the row size), the flags, staged partials
+inline int64_t code8_ring_smem(int32_t vfbits) {
+  return (int64_t)kCode8Ring * code8_tile_bytes(vfbits) + (1LL << vfbits) + kCode8Ring * 16 +
+         kCode8Ring * kCode8TileRows * 8;
+}
 
 struct OutArgs {
   float* out = nullptr;          // final scores (fused finalize) or nullptr
@@ -143,6 +180,11 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
 int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                         int32_t d, uint16_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
                         void* stream, void* ev_b, void* ev_e);
+// wide rank codes (reading R8): u8 code tiles (codes: ntiles * code8_tile_bytes + ntiles * 16
+// bytes of NaN flags + n_slices * 8 bytes of counters), then the coded slices over them
+int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
+                         int32_t d, uint8_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
+                         void* stream, void* ev_b, void* ev_e);
 int launch_finalize(const FinalizeArgs& a, void* stream);
 int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t d,
                         uint32_t* counts, int32_t num_sms, void* stream);

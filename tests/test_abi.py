@@ -324,3 +324,29 @@ def test_pack_refine_improves_simulated_lockstep(monkeypatch):
             assert np.array_equal(leaf, oracle.predict(f, X, want_leaf=True)["leaf"])
         T.tahoe_forest_free(h)
     assert effs["1"] >= effs["0"] - 1e-12, effs
+
+
+def test_wide_code_layout_host():
+    """Reading R8 on a host-only handle: a forest over 2000 attributes gets the wide codes; its
+    virtual attributes number sum_j ceil(K_j / 127) over the distinct thresholds K_j of each
+    attribute (counted here with numpy), the code row is the smallest power of two above them
+    (the all-ones byte is the leaf's pad), the slices are packed for the room the 3-tile code ring
+    leaves, and the (shared) sliced image still decodes to the oracle's leaves."""
+    f = gen.make_forest(4, n_trees=120)
+    h = T.tahoe_forest_build(f, f["n_features"], f["n_classes"], f["agg"], 0.0, -1)
+    T.tahoe_forest_layout(h, gen.make_calibration(4, 2048))
+    st = T.tahoe_forest_stats(h)
+    assert st["sliced_valid"] and st["coded_valid"] and st["code8"], st["coded_why"]
+    feat, thr = f["feature"], f["threshold"]
+    k = [len(np.unique(thr[feat == j])) for j in range(f["n_features"])]
+    nv = int(sum((x + 126) // 127 for x in k))
+    assert st["code8_virtual"] == nv
+    V = st["code8_vfbits"]
+    assert (1 << V) - 1 >= nv and (1 << (V - 1)) - 1 < nv
+    ring = 3 * 16 * (1 << V) + (1 << V) + 3 * 16 + 3 * 16 * 8
+    assert ((st["slots_max"] * 128 + 1023) // 1024) * 1024 + ring + 128 <= 232448
+    X = gen.make_rows(4, 24)
+    img = T.tahoe_forest_export_sliced(h)
+    leaf, _ = decode_sliced(img, X, len(f["root"]), f["n_classes"])
+    assert np.array_equal(leaf, oracle.predict(f, X, want_leaf=True)["leaf"])
+    T.tahoe_forest_free(h)

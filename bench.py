@@ -454,7 +454,7 @@ def main():
     n_sms = stats["num_sms"]
     smem_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
     achieved = n * smem_bytes_per_sample / (kern_avg_ms / 1000.0) / 1e9
-    kname = {1: "k_sliced", 2: "k_sliced_codes"}.get(strategy, "k_direct")
+    kname = {1: "k_sliced", 2: "k_sliced_codes8" if stats.get("code8") else "k_sliced_codes"}.get(strategy, "k_direct")
     traffic = None
     sector_eff = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -470,7 +470,7 @@ def main():
     launches_per_step = 1 if strategy == T.STRATEGY_DIRECT and F.n_out == 1 else (
         1 + (1 if (strategy != T.STRATEGY_DIRECT and stats["n_slices"] > 1) or F.n_out > 1 else 0))
     if strategy == T.STRATEGY_SLICED_CODED:
-        launches_per_step += 1   # k_encode_rows_banks (the trailer memset is not a kernel of ours)
+        launches_per_step += 1   # the row-coding pre-pass (the flag memset is not a kernel of ours)
     line = dict(
         metric=METRIC, value=value, unit=UNIT, n_gpus=world, steps=args.steps, warmup=args.warmup,
         ms_per_step=ms_per_step, higher_is_better=True, scaling="weak", vs_baseline=None,

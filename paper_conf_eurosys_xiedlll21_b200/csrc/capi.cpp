@@ -426,7 +426,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   fa.class_parts = f->d_class_parts;
   if (strat == TAHOE_STRATEGY_SLICED_CODED && f->sl.code8) {
     // wide codes (reading R8): u8 code tiles + NaN flags from the library pool
-    const int64_t ntiles = (n + kCode8TileRows - 1) / kCode8TileRows;
+    const int64_t ntiles = (code8_chunk_rows(f->sl.vfbits, n) + kCode8TileRows - 1) / kCode8TileRows;
     const size_t cbytes = (size_t)ntiles * (size_t)(code8_tile_bytes(f->sl.vfbits) + 16) +
                           (size_t)f->sl.n_slices * 8;
     void* cbuf = nullptr;
@@ -435,10 +435,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync code tiles");
     }
     SlicedPlan cp = plan;
-    if (f->d_cta_start && ntiles >= 4LL * f->num_sms) {
-      cp.grid = f->num_sms;
-      cp.cta_start = f->d_cta_start;
-    }
+    cp.cta_start = f->d_cta_start;   // used per chunk once it has a few tiles per CTA
     rc = launch_sliced_codes8(f->ds, cp, X, n, d, static_cast<uint8_t*>(cbuf), o, fused,
                               f->num_sms, st, ev_b, ev_e);
     cudaFreeAsync(cbuf, st);

@@ -22,6 +22,14 @@ namespace tahoe {
 
 static uint32_t f2u(float f) { uint32_t u; std::memcpy(&u, &f, 4); return u; }
 
+int64_t code8_chunk_mb() {
+  static const int64_t mb = [] {
+    const char* e = std::getenv("TAHOE_CODE8_CHUNK_MB");
+    return e && *e ? (int64_t)std::atoll(e) : (int64_t)0;
+  }();
+  return mb;
+}
+
 // ------------------------------------------------------------------ direct image
 tahoe_status encode_direct(const Forest& F, DirectImage& D) {
   D = DirectImage();
@@ -408,10 +416,9 @@ static void build_code8_banks(const std::vector<std::vector<float>>& vt, int32_t
       const size_t v = (size_t)g * 32 + a;
       if (v < vt.size()) mk = std::max(mk, vt[v].size());
     }
-    int32_t k = 0;
-    while (((size_t)1 << k) - 1 < mk) k++;
-    probes[g] = k;
-    total += (((int64_t)1 << k) - 1) * 128;
+    (void)mk;
+    probes[g] = 7;   // every lane padded to 127 elements: one uniform 7-probe bisection
+    total += (((int64_t)1 << probes[g]) - 1) * 128;
   }
   auto gbytes = [&](int32_t g) { return (((int64_t)1 << probes[g]) - 1) * 128; };
   std::vector<int32_t> cut;
@@ -480,7 +487,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
     const int32_t nv = vbase[F.n_features];
     const int32_t vfb = std::max(5, feature_bits(nv + 1));   // byte 2^V - 1 is the pad a leaf reads
     if (vfb <= kCode8MaxFbits) {
-      const int64_t room = (int64_t)max_smem - code8_ring_smem(vfb) - kSlicedBarrierBytes;
+      const int64_t room = (int64_t)max_smem - code8_ring_smem(vfb);
       const int32_t cap8 = (int32_t)std::max<int64_t>(0, (room & ~1023LL) / kSlotBytes);
       bool fits = cap8 >= 16;
       for (int32_t t = 0; t < F.n_trees && fits; t++) fits = enc_size(F, t) <= cap8 - 1;

@@ -1569,21 +1569,21 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows8(const Encode8Args a) {
   const int64_t tile_bytes = (int64_t)kCode8TileRows << V;
   const uint32_t sbase = smem_u32(s_img) + (uint32_t)lane * 4u;
   for (int64_t r0 = r_lo + (int64_t)warp * kR; r0 < r_hi; r0 += (int64_t)W * kR) {
-    const bool full = r0 + kR <= r_hi;
+    const int nq = (int)min((int64_t)kR, r_hi - r0);   // rows of this group (the tail is ragged)
     bool nan_any = false;
-    uint8_t* row0 = a.codes + (r0 >> 4) * tile_bytes + ((r0 & 15) << V);
-    // the next group's attribute values are loaded before this group is searched
+    uint8_t* row0 = a.codes + (r0 / kCode8TileRows) * tile_bytes + ((r0 % kCode8TileRows) << V);
+    // the next group's attribute values are loaded before this group is searched (rows past the
+    // tail re-read the last row; their codes are not stored)
     auto load_x = [&](int g, float* x, int& src) {
       src = g < bd.w ? __ldg(&a.v_src[g * 32 + lane]) : -1;
-      const float* xs = a.X + r0 * a.d + (src >= 0 ? src : 0);
+      const float* xs = a.X + (src >= 0 ? src : 0);
 #pragma unroll
-      for (int q = 0; q < kR; q++) x[q] = (src >= 0 && (full || r0 + q < r_hi)) ? __ldg(xs + (int64_t)q * a.d) : 0.0f;
+      for (int q = 0; q < kR; q++) x[q] = __ldg(xs + (r0 + (q < nq ? q : nq - 1)) * a.d);
     };
     float xn[kR];
     int srcn;
     load_x(bd.z, xn, srcn);
     for (int g = bd.z; g < bd.w; g++) {
-      const int4 gd = __ldg(&a.grp[g]);
       const int v = g * 32 + lane;
       const int src = srcn;
       float x[kR];
@@ -1591,27 +1591,16 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows8(const Encode8Args a) {
       for (int q = 0; q < kR; q++) x[q] = xn[q];
       load_x(g + 1, xn, srcn);
       uint32_t pos[kR];
-      const uint32_t base = sbase + (uint32_t)gd.x * 4u;
-      switch (gd.y) {   // probe count: a uniform, fully unrolled bisection per group
-        case 0: for (int q = 0; q < kR; q++) pos[q] = 0; break;
-        case 1: bisect8<1, kR>(base, x, pos); break;
-        case 2: bisect8<2, kR>(base, x, pos); break;
-        case 3: bisect8<3, kR>(base, x, pos); break;
-        case 4: bisect8<4, kR>(base, x, pos); break;
-        case 5: bisect8<5, kR>(base, x, pos); break;
-        case 6: bisect8<6, kR>(base, x, pos); break;
-        default: bisect8<7, kR>(base, x, pos); break;
-      }
+      bisect8<7, kR>(sbase + (uint32_t)__ldg(&a.grp[g]).x * 4u, x, pos);
 #pragma unroll
       for (int q = 0; q < kR; q++) {
-        if (!full && r0 + q >= r_hi) continue;
         const bool isnan_q = src >= 0 && x[q] != x[q];
-        nan_any |= isnan_q;
+        nan_any |= isnan_q && q < nq;
         const int8_t c = src < 0 ? kCode8Pad : (isnan_q ? kCode8Nan : (int8_t)pos[q]);
-        row0[((uint32_t)q << V) + (uint32_t)v] = (uint8_t)c;
+        if (q < nq) row0[((uint32_t)q << V) + (uint32_t)v] = (uint8_t)c;
       }
     }
-    if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 >> 4) * 4] = 1u;
+    if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 / kCode8TileRows) * 4] = 1u;
   }
 }
 
@@ -1625,6 +1614,8 @@ struct Coded8KArgs {
   int64_t n;
   int32_t forest_smem;   // bytes reserved for the slice (multiple of 1024)
   const int32_t* cta_start;  // initial CTA -> slice map (prefix), or nullptr: blockIdx % ns
+  int64_t row0;          // first row of this launch's chunk (outputs are indexed row0 + r)
+  int64_t n_all;         // rows of the whole batch (row stride of the raw partials)
   OutArgs o;
 };
 
@@ -1674,12 +1665,14 @@ __device__ __forceinline__ void walk_coded8(uint32_t pA, uint32_t pB, uint32_t p
 // all claimed, entries are issued EMPTY (tile -1, the phase completes without data) and released
 // like the others, so the chain of tickets never stalls; a warp leaves the slice when it meets an
 // empty entry and every valid entry issued so far has been released.
-constexpr int kCode8Threads = 512;
-template <bool FUSED>
-__global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {
+constexpr int kCode8Threads = 384;
+// R rows per walked tile (a multiple of the pre-pass tile, whose NaN flags it carries), kR8 tiles
+// in the ring (R * kR8 rows in shared memory).
+template <bool FUSED, int R, int kR8>
+__global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {
   constexpr int C = kSlicedCols;
-  constexpr int R = kCode8TileRows;
-  constexpr int kR8 = kCode8Ring;
+  constexpr int FS = R / kCode8TileRows;   // pre-pass tiles (NaN flags) per walked tile
+  static_assert(R % kCode8TileRows == 0 && R * kR8 == kCode8TileRows * kCode8Ring, "ring rows");
   constexpr int kUnits = R / 4;
   extern __shared__ __align__(1024) unsigned char smem[];
   const uint32_t V = (uint32_t)a.img.vfbits;
@@ -1689,17 +1682,19 @@ __global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid
   const uint32_t ring_off = ((sbase + (uint32_t)a.forest_smem + RB - 1u) & ~(RB - 1u)) - sbase;
   unsigned char* s_ring = smem + ring_off;
   uint32_t* s_flag = reinterpret_cast<uint32_t*>(s_ring + (size_t)kR8 * tile_bytes);
-  double* s_part = reinterpret_cast<double*>(s_flag + kR8 * 4);
-  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_part + kR8 * R);      // [3]
-  uint64_t* s_forest = s_full + kR8;                                       // [1]
-  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full + 4);  // unit counter
-  int* s_cnt = reinterpret_cast<int*>(s_full + 5);                         // [3] units released
-  uint32_t* s_gen = reinterpret_cast<uint32_t*>(s_cnt + 4);                // [3] ticket: entry issued
-  int32_t* s_tile = reinterpret_cast<int32_t*>(s_gen + 4);                 // [3] tile of the entry
-  uint32_t* s_vis = reinterpret_cast<uint32_t*>(s_tile + 4);              // valid entries issued
-  uint32_t* s_vdone = reinterpret_cast<uint32_t*>(s_tile + 5);            // valid entries released
-  int32_t* s_slice = reinterpret_cast<int32_t*>(s_tile + 6);
-  uint32_t* s_issued = reinterpret_cast<uint32_t*>(s_tile + 7);           // entries issued
+  double* s_part = reinterpret_cast<double*>(s_flag + kR8 * FS * 4);
+  // control block (kCode8Ctl bytes): mbarriers, unit counter, per-buffer counters, CTA state
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_part + kR8 * R);      // [ring] tile arrived
+  uint64_t* s_forest = s_full + kR8;                                       // slice staged
+  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_forest + 1);  // unit counter
+  int* s_cnt = reinterpret_cast<int*>(s_next + 1);                         // [ring] units released
+  uint32_t* s_gen = reinterpret_cast<uint32_t*>(s_cnt + kR8);              // [ring] ticket: entry issued
+  int32_t* s_tile = reinterpret_cast<int32_t*>(s_gen + kR8);               // [ring] tile of the entry
+  uint32_t* s_vis = reinterpret_cast<uint32_t*>(s_tile + kR8);            // valid entries issued
+  uint32_t* s_vdone = s_vis + 1;                                           // valid entries released
+  int32_t* s_slice = reinterpret_cast<int32_t*>(s_vis + 2);
+  uint32_t* s_issued = s_vis + 3;                                          // entries issued
+  static_assert(8 * (kR8 + 2) + 12 * kR8 + 16 <= kCode8Ctl, "control block");
   const int lane = threadIdx.x & 31;
   const int col = lane & (C - 1);
   const int half = lane >> 4;
@@ -1740,9 +1735,9 @@ __global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid
       } else {
         atomicAdd(s_vis, 1u);
         fence_proxy_async_smem();
-        mbar_expect_tx(&s_full[b], tile_bytes + 16u);
+        mbar_expect_tx(&s_full[b], tile_bytes + 16u * FS);
         bulk_g2s(s_ring + (size_t)b * tile_bytes, a.codes + (int64_t)tile * tile_bytes, tile_bytes, &s_full[b]);
-        bulk_g2s(s_flag + b * 4, a.flags + (int64_t)tile * 4, 16u, &s_full[b]);
+        bulk_g2s(s_flag + b * FS * 4, a.flags + (int64_t)tile * FS * 4, 16u * FS, &s_full[b]);
       }
       atomicAdd(s_issued, 1u);
     }
@@ -1796,8 +1791,13 @@ __global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid
         const uint32_t tb = sbase + ring_off + (uint32_t)b * tile_bytes;
         const uint32_t rowA = tb + ((uint32_t)(okA ? rA : u) << V);
         const uint32_t rowB = tb + ((uint32_t)(okB ? rB : u) << V);
-        uint32_t nan_flag;
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(smem_u32(s_flag + b * 4)));
+        uint32_t nan_flag = 0;
+#pragma unroll
+        for (int k = 0; k < FS; k++) {
+          uint32_t fk;
+          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(fk) : "r"(smem_u32(s_flag + (b * FS + k) * 4)));
+          nan_flag |= fk;
+        }
         double accA, accB;
         if (nan_flag)
           walk_coded8<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
@@ -1812,7 +1812,7 @@ __global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid
         for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
         const int rr = b3 ? rB : rA;
         if ((lane & 7) == 0 && (b3 ? okB : okA)) {
-          if (FUSED) write_scalar(a.o, r0 + rr, v);
+          if (FUSED) write_scalar(a.o, a.row0 + r0 + rr, v);
           else s_part[b * R + rr] = v;
         }
       }
@@ -1832,7 +1832,7 @@ __global__ void __launch_bounds__(kCode8Threads, 1) k_sliced_codes8(const __grid
           const double p = lane < nr ? s_part[b * R + lane] : 0.0;
           __syncwarp();
           issue(sl, e + kR8);
-          if (lane < nr) a.o.raw[(size_t)sl * a.n + r0 + lane] = p;
+          if (lane < nr) a.o.raw[(size_t)sl * a.n_all + a.row0 + r0 + lane] = p;
         }
         if (tile >= 0 && lane == 0) atomicAdd(s_vdone, 1u);
       }
@@ -1870,60 +1870,82 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
                          int32_t d, uint8_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
                          void* stream, void* ev_b, void* ev_e) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  const int64_t ntiles = (n + kCode8TileRows - 1) / kCode8TileRows;
   const int64_t tbytes = code8_tile_bytes(img.vfbits);
-  uint32_t* flags = reinterpret_cast<uint32_t*>(codes + ntiles * tbytes);
-  // NaN flags (16 bytes per tile), then the per-slice tile counters and CTA counts
-  cudaError_t e = cudaMemsetAsync(flags, 0, (size_t)ntiles * 16 + (size_t)img.n_slices * 8, st);
-  if (e != cudaSuccess) return (int)e;
-  Encode8Args ea;
-  ea.X = X;
-  ea.n = n;
-  ea.d = d;
-  ea.vfbits = img.vfbits;
-  ea.bands = img.c8_bands;
-  ea.chunks = std::max(1, num_sms / std::max(1, img.c8_bands));
-  ea.img = img.c8_img;
-  ea.grp = reinterpret_cast<const int4*>(img.c8_grp);
-  ea.band = reinterpret_cast<const int4*>(img.c8_band);
-  ea.v_src = img.v_src;
-  ea.codes = codes;
-  ea.flags = flags;
+  const int64_t chunk = code8_chunk_rows(img.vfbits, n);
+  const int64_t ctiles = (chunk + kCode8TileRows - 1) / kCode8TileRows;
+  uint32_t* flags = reinterpret_cast<uint32_t*>(codes + ctiles * tbytes);
+  cudaError_t e;
   {
     static std::atomic<int> configured[64];
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
       e = cudaFuncSetAttribute(k_encode_rows8, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
-      if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sliced_codes8<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
-      if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sliced_codes8<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+      for (auto k : {k_sliced_codes8<true, 8, 6>, k_sliced_codes8<false, 8, 6>, k_sliced_codes8<true, 16, 3>,
+                     k_sliced_codes8<false, 16, 3>})
+        if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
       if (e != cudaSuccess) return (int)e;
       configured[dev].store(1);
     }
   }
-  k_encode_rows8<<<ea.bands * ea.chunks, 1024, kCode8BandBudget, st>>>(ea);
-  if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
-
-  Coded8KArgs a{};
-  a.img = img;
-  a.codes = codes;
-  a.flags = flags;
-  a.tile_next = reinterpret_cast<int32_t*>(flags + ntiles * 4);
-  a.cta_on = a.tile_next + img.n_slices;
-  a.work = img.slice_w;
-  a.n = n;
-  a.forest_smem = plan.forest_smem;
-  a.cta_start = plan.cta_start;
-  a.o = o;
-  const int smem = plan.forest_smem + (int)code8_ring_smem(img.vfbits) + kSlicedBarrierBytes;
-  if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
-  if (fused) k_sliced_codes8<true><<<plan.grid, kCode8Threads, smem, st>>>(a);
-  else k_sliced_codes8<false><<<plan.grid, kCode8Threads, smem, st>>>(a);
-  e = cudaGetLastError();
+  const int smem = plan.forest_smem + (int)code8_ring_smem(img.vfbits);
+  static const bool tile16 = std::getenv("TAHOE_CODE8_TILE") && std::atoi(std::getenv("TAHOE_CODE8_TILE")) == 16;
+  static const int threads = [] {   // $TAHOE_CODE8_THREADS, $TAHOE_CODE8_TILE (8 or 16): experiments
+    const char* e = std::getenv("TAHOE_CODE8_THREADS");
+    return e && *e ? std::atoi(e) : kCode8Threads;
+  }();
+  // Optional chunks of rows ($TAHOE_CODE8_CHUNK_MB) bound the code scratch; the default is one
+  // launch pair for the whole batch (chunks small enough for the chunk's tiles to stay in L2
+  // between the pre-pass and the ~30 slices were measured slower: each chunk pays a tail).  The
+  // kernel events bracket the walk kernel, or the whole chunk loop when there are several chunks.
+  const bool one = chunk >= n;
+  if (ev_b && !one) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+  for (int64_t c0 = 0; c0 < n; c0 += chunk) {
+    const int64_t cn = std::min(chunk, n - c0);
+    const int64_t ntiles = (cn + kCode8TileRows - 1) / kCode8TileRows;
+    // NaN flags (16 bytes per tile), then the per-slice tile counters and CTA counts
+    e = cudaMemsetAsync(flags, 0, (size_t)ntiles * 16 + (size_t)img.n_slices * 8, st);
+    if (e != cudaSuccess) return (int)e;
+    Encode8Args ea;
+    ea.X = X + c0 * d;
+    ea.n = cn;
+    ea.d = d;
+    ea.vfbits = img.vfbits;
+    ea.bands = img.c8_bands;
+    ea.chunks = std::max(1, num_sms / std::max(1, img.c8_bands));
+    ea.img = img.c8_img;
+    ea.grp = reinterpret_cast<const int4*>(img.c8_grp);
+    ea.band = reinterpret_cast<const int4*>(img.c8_band);
+    ea.v_src = img.v_src;
+    ea.codes = codes;
+    ea.flags = flags;
+    k_encode_rows8<<<ea.bands * ea.chunks, 1024, kCode8BandBudget, st>>>(ea);
+    if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
+    Coded8KArgs a{};
+    a.img = img;
+    a.codes = codes;
+    a.flags = flags;
+    a.tile_next = reinterpret_cast<int32_t*>(flags + ntiles * 4);
+    a.cta_on = a.tile_next + img.n_slices;
+    a.work = img.slice_w;
+    a.n = cn;
+    a.row0 = c0;
+    a.n_all = n;
+    a.forest_smem = plan.forest_smem;
+    // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
+    // every CTA a few tiles, else the plan's grid
+    const bool full = plan.cta_start && ntiles >= 4LL * num_sms;
+    a.cta_start = full ? plan.cta_start : nullptr;
+    const int grid = full ? num_sms : plan.grid;
+    a.o = o;
+    auto kern = tile16 ? (fused ? k_sliced_codes8<true, 16, 3> : k_sliced_codes8<false, 16, 3>)
+                       : (fused ? k_sliced_codes8<true, 8, 6> : k_sliced_codes8<false, 8, 6>);
+    if (ev_b && one) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+    kern<<<grid, threads, smem, st>>>(a);
+    if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
+  }
   if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
-  return (int)e;
+  return 0;
 }
 
 int launch_finalize(const FinalizeArgs& a, void* stream) {

@@ -94,16 +94,28 @@ inline int32_t code_tile_stride(int32_t fbits) { return code_tile_bytes(fbits) +
 // tile's bulk copy.
 constexpr int32_t kCode8MaxRank = 127;
 constexpr int32_t kCode8MaxFbits = 12;           // rows of <= 4 KB
-constexpr int32_t kCode8TileRows = 16;
-constexpr int32_t kCode8Ring = 3;
+constexpr int32_t kCode8TileRows = 8;
+constexpr int32_t kCode8Ring = 6;
 constexpr int32_t kCode8BandBudget = 200 * 1024; // pre-pass tables per CTA
 constexpr int8_t kCode8Nan = -2;
 constexpr int8_t kCode8Pad = -1;
 inline int64_t code8_tile_bytes(int32_t vfbits) { return (int64_t)kCode8TileRows << vfbits; }
-// shared memory next to the slice: the ring (aligned to the row size), the flags, staged partials
+// rows per launch: the chunk's code tiles (~48 MB) stay in the 126 MB L2 between the pre-pass
+// and the slices
+int64_t code8_chunk_mb();   // $TAHOE_CODE8_CHUNK_MB (experiments); default 0 = one launch
+inline int64_t code8_chunk_rows(int32_t vfbits, int64_t n) {
+  if (code8_chunk_mb() <= 0) return n > 0 ? n : 1;
+  int64_t c = (code8_chunk_mb() << 20) >> vfbits;
+  c -= c % kCode8TileRows;
+  if (c < kCode8TileRows) c = kCode8TileRows;
+  return n < c ? n : c;
+}
+constexpr int32_t kCode8Ctl = 256;               // mbarriers, counters, tickets
+// shared memory next to the slice: the ring (aligned to the row size), the flags, staged partials,
+// the control block
 inline int64_t code8_ring_smem(int32_t vfbits) {
   return (int64_t)kCode8Ring * code8_tile_bytes(vfbits) + (1LL << vfbits) + kCode8Ring * 16 +
-         kCode8Ring * kCode8TileRows * 8;
+         kCode8Ring * kCode8TileRows * 8 + kCode8Ctl;
 }
 
 struct OutArgs {
@@ -180,8 +192,9 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
 int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                         int32_t d, uint16_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
                         void* stream, void* ev_b, void* ev_e);
-// wide rank codes (reading R8): u8 code tiles (codes: ntiles * code8_tile_bytes + ntiles * 16
-// bytes of NaN flags + n_slices * 8 bytes of counters), then the coded slices over them
+// wide rank codes (reading R8): per chunk of code8_chunk_rows rows, u8 code tiles (codes: scratch
+// of ctiles * code8_tile_bytes + ctiles * 16 bytes of NaN flags + n_slices * 8 bytes of counters,
+// ctiles = the chunk's tiles), then the coded slices over them
 int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                          int32_t d, uint8_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
                          void* stream, void* ev_b, void* ev_e);

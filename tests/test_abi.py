@@ -343,8 +343,8 @@ def test_wide_code_layout_host():
     assert st["code8_virtual"] == nv
     V = st["code8_vfbits"]
     assert (1 << V) - 1 >= nv and (1 << (V - 1)) - 1 < nv
-    ring = 3 * 16 * (1 << V) + (1 << V) + 3 * 16 + 3 * 16 * 8
-    assert ((st["slots_max"] * 128 + 1023) // 1024) * 1024 + ring + 128 <= 232448
+    ring = 6 * 8 * (1 << V) + (1 << V) + 6 * 16 + 6 * 8 * 8 + 256
+    assert ((st["slots_max"] * 128 + 1023) // 1024) * 1024 + ring <= 232448
     X = gen.make_rows(4, 24)
     img = T.tahoe_forest_export_sliced(h)
     leaf, _ = decode_sliced(img, X, len(f["root"]), f["n_classes"])

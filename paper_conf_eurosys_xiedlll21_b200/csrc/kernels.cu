@@ -1616,6 +1616,7 @@ struct Coded8KArgs {
   const int32_t* cta_start;  // initial CTA -> slice map (prefix), or nullptr: blockIdx % ns
   int64_t row0;          // first row of this launch's chunk (outputs are indexed row0 + r)
   int64_t n_all;         // rows of the whole batch (row stride of the raw partials)
+  int32_t switch_slices; // 1: a CTA whose slice is exhausted moves to another (0: experiments)
   OutArgs o;
 };
 
@@ -1859,6 +1860,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
         const float w = (float)rem * __ldg(&a.work[s2]) / (float)(1 + on);
         if (w > bw) { bw = w; best = s2; }
       }
+      if (!a.switch_slices) best = -1;
       if (best >= 0) atomicAdd(&a.cta_on[best], 1);
       *s_slice = best;
     }
@@ -1881,19 +1883,14 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
       e = cudaFuncSetAttribute(k_encode_rows8, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
-      for (auto k : {k_sliced_codes8<true, 8, 6>, k_sliced_codes8<false, 8, 6>, k_sliced_codes8<true, 16, 3>,
-                     k_sliced_codes8<false, 16, 3>})
+      for (auto k : {k_sliced_codes8<true, kCode8TileRows, kCode8Ring>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring>})
         if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
       if (e != cudaSuccess) return (int)e;
       configured[dev].store(1);
     }
   }
   const int smem = plan.forest_smem + (int)code8_ring_smem(img.vfbits);
-  static const bool tile16 = std::getenv("TAHOE_CODE8_TILE") && std::atoi(std::getenv("TAHOE_CODE8_TILE")) == 16;
-  static const int threads = [] {   // $TAHOE_CODE8_THREADS, $TAHOE_CODE8_TILE (8 or 16): experiments
-    const char* e = std::getenv("TAHOE_CODE8_THREADS");
-    return e && *e ? std::atoi(e) : kCode8Threads;
-  }();
+  const int threads = kCode8Threads;
   // Optional chunks of rows ($TAHOE_CODE8_CHUNK_MB) bound the code scratch; the default is one
   // launch pair for the whole batch (chunks small enough for the chunk's tiles to stay in L2
   // between the pre-pass and the ~30 slices were measured slower: each chunk pays a tail).  The
@@ -1932,14 +1929,16 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     a.row0 = c0;
     a.n_all = n;
     a.forest_smem = plan.forest_smem;
+    a.switch_slices = !(std::getenv("TAHOE_CODE8_SWITCH") && std::atoi(std::getenv("TAHOE_CODE8_SWITCH")) == 0);
     // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
     // every CTA a few tiles, else the plan's grid
     const bool full = plan.cta_start && ntiles >= 4LL * num_sms;
     a.cta_start = full ? plan.cta_start : nullptr;
     const int grid = full ? num_sms : plan.grid;
     a.o = o;
-    auto kern = tile16 ? (fused ? k_sliced_codes8<true, 16, 3> : k_sliced_codes8<false, 16, 3>)
-                       : (fused ? k_sliced_codes8<true, 8, 6> : k_sliced_codes8<false, 8, 6>);
+    // (16-row tiles in a 3-deep ring and 512 / 1024-thread CTAs measured within 2 %)
+    auto kern = fused ? k_sliced_codes8<true, kCode8TileRows, kCode8Ring>
+                      : k_sliced_codes8<false, kCode8TileRows, kCode8Ring>;
     if (ev_b && one) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
     kern<<<grid, threads, smem, st>>>(a);
     if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;

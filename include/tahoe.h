@@ -64,7 +64,12 @@ typedef enum {
                                  qualifies (<= 127 attributes, <= 32000 distinct thresholds per
                                  attribute, no subnormal leaf value) and no leaf ids or
                                  fingerprints are requested; forcing it otherwise returns
-                                 E_UNSUPPORTED                                                */
+                                 E_UNSUPPORTED.  Forests over more than 127 attributes get the
+                                 WIDE codes instead (reading R8): u8 codes over virtual
+                                 attributes (<= 127 thresholds each), 2^V-byte code rows staged
+                                 in shared memory next to slices packed for that room; they
+                                 qualify while the used attributes need <= 4 KB rows and every
+                                 tree fits the smaller lane column                            */
 } tahoe_strategy;
 
 /*

@@ -1235,10 +1235,9 @@ static cudaError_t direct_tiled_one(const DirectKArgs& a, int32_t rs, int32_t nu
   return cudaGetLastError();
 }
 
-template <bool F, int P>
+template <bool F, int P, int kRows = 128>
 static cudaError_t direct_tlp_one(const DirectKArgs& a, int32_t rs, int32_t num_sms,
                                   cudaStream_t st) {
-  constexpr int kRows = 128;
   auto kern = k_direct_tlp<F, kRows, P>;
   const int smem = kRows * rs * 4;
   static std::atomic<int> configured[64];
@@ -1252,6 +1251,14 @@ static cudaError_t direct_tlp_one(const DirectKArgs& a, int32_t rs, int32_t num_
   int per_sm = 1;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kRows * P, smem);
   if (per_sm < 1) per_sm = 1;
+  // experiments: $TAHOE_DIRECT_PERSM caps the resident CTAs per SM and hands the rest of the
+  // unified L1 / shared memory to L1 (node reads)
+  static const int cap = std::getenv("TAHOE_DIRECT_PERSM") ? std::atoi(std::getenv("TAHOE_DIRECT_PERSM")) : 0;
+  if (cap > 0 && cap < per_sm) {
+    per_sm = cap;
+    const int pct = (int)std::min<int64_t>(100, ((int64_t)per_sm * (smem + 1024) * 100 + 233471) / 233472);
+    cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
+  }
   const int64_t ntiles = (a.n + kRows - 1) / kRows;
   const int grid = (int)std::min<int64_t>(ntiles, (int64_t)num_sms * per_sm);
   kern<<<grid, kRows * P, smem, st>>>(a, rs);
@@ -1264,21 +1271,28 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
   // 0 = rows read from global memory; 1 = staged rows, warp-lockstep over trees;
-  // 2 = staged rows, free-running over trees; 3 / 4 = staged rows, 2 / 4 threads per row
+  // 2 = staged rows, free-running over trees; 3 / 4 = staged rows (128 per CTA), 2 / 4 threads
+  // per row; 5 = 64 staged rows, 8 threads per row; 6 = 64 rows x 4; 7 = 32 rows x 16.
   // Default for large batches: staged rows — attribute reads from shared memory leave L1/L2 to
-  // the nodes — with two threads per row for scalar outputs (3; C5 500-tree shard 300K rows:
-  // 10.05 ms rows-global -> 9.75 ms staged -> 5.96 ms two threads per row; four threads per row
-  // thrash L1: 8.13 ms) and one thread per row, free-running, otherwise (2).  Rows from global
-  // memory (0) for small batches (lower launch cost) and for rows too wide to stage.
+  // the nodes — with 8 threads per row over 64-row CTAs for scalar outputs (5) and one thread per
+  // row, free-running, otherwise (2).  C5 500-tree shard, 300K rows: rows-global 10.05 ms ->
+  // staged 9.75 -> 2 threads per row 5.96 -> 8 threads per row over 64 rows 4.05 ms: more node
+  // loads in flight, while the smaller row tiles leave ~150 KB of the unified L1 to the nodes
+  // (4 threads per row over 128-row CTAs at 4 CTAs/SM leave ~50 KB: 8.04 ms; 16 per row 4.65 ms).
+  // Rows from global memory (0) for small batches (lower launch cost) and for rows too wide to
+  // stage.
   const bool scalar = o.n_classes == 1 && o.agg != TAHOE_AGG_VOTE;
   const char* env = std::getenv("TAHOE_DIRECT_VARIANT");
-  int variant = env ? std::atoi(env) : (n >= 32768 ? (scalar && !leaf ? 3 : 2) : 0);
+  int variant = env ? std::atoi(env) : (n >= 32768 ? (scalar && !leaf ? 5 : 2) : 0);
   if (d > 256) variant = 0;  // 128 staged rows must fit shared memory
-  if ((variant == 3 || variant == 4) && scalar && !leaf) {
+  if (variant >= 3 && variant <= 7 && scalar && !leaf) {
     const int32_t rs = d | 1;
     cudaError_t e;
     if (variant == 3) e = fused ? direct_tlp_one<true, 2>(a, rs, num_sms, st) : direct_tlp_one<false, 2>(a, rs, num_sms, st);
-    else e = fused ? direct_tlp_one<true, 4>(a, rs, num_sms, st) : direct_tlp_one<false, 4>(a, rs, num_sms, st);
+    else if (variant == 4) e = fused ? direct_tlp_one<true, 4>(a, rs, num_sms, st) : direct_tlp_one<false, 4>(a, rs, num_sms, st);
+    else if (variant == 5) e = fused ? direct_tlp_one<true, 8, 64>(a, rs, num_sms, st) : direct_tlp_one<false, 8, 64>(a, rs, num_sms, st);
+    else if (variant == 6) e = fused ? direct_tlp_one<true, 4, 64>(a, rs, num_sms, st) : direct_tlp_one<false, 4, 64>(a, rs, num_sms, st);
+    else e = fused ? direct_tlp_one<true, 16, 32>(a, rs, num_sms, st) : direct_tlp_one<false, 16, 32>(a, rs, num_sms, st);
     return (int)e;
   }
   if (variant == 1 || variant == 2) {

@@ -331,10 +331,11 @@ def test_direct_chunked_image_parity(monkeypatch):
 
 
 @pytest.mark.parametrize("cid,ntrees,variant", [(2, 120, None), (5, 60, None), (2, 120, "4"),
-                                                (5, 60, "2"), (5, 60, "1")])
+                                                (5, 60, "2"), (5, 60, "1"), (5, 60, "3"),
+                                                (2, 120, "6"), (5, 60, "7")])
 def test_direct_large_batch_variants(cid, ntrees, variant, monkeypatch):
-    """Large-batch direct kernels (staged rows; two or four threads per row for scalar outputs,
-    one thread per row free-running or warp-lockstep) against the oracle, scores and classes
+    """Large-batch direct kernels (staged rows; 2, 4, 8 (default) or 16 threads per row for scalar
+    outputs, one thread per row free-running or warp-lockstep) against the oracle, scores and classes
     bit-exact with dyadic leaves, >= 32K rows with a ragged last tile."""
     if variant is not None:
         monkeypatch.setenv("TAHOE_DIRECT_VARIANT", variant)

@@ -22,12 +22,14 @@ out = ["# Round 1 cost-model fit (B200, `python scripts/fit_costmodel.py`)", "",
        "* sliced: `T = a_s + b_s * U_s * (rows in global ? g_s : 1)`, "
        "`U_s = ceil(tiles/cps) * 64 * V / (slices * eff_sim)`",
        "* coded (rank-coded slices, reading R7): `T = a_c + b_c * U_s + e_c * ceil(n/64) * 64 * passes / SMs`",
+       "* wide codes (reading R8, > 127 attributes): `T = a_w + b_w * U_s + e_w * ceil(n/64) * 64 * passes / SMs`",
        "* direct: `T = a_d + (d > 256 ? g_d : 1) * max(l_d * V, b_d * V * n / SMs)`", "",
        "Kernels: the 16-lane-column `k_sliced`, the rank-coded `k_sliced_codes` with its row-coding "
-       "pre-pass, and the staged-row direct kernels (two threads per row for scalar outputs) for "
-       "batches >= 32K rows.", "",
+       "pre-pass, the wide-code `k_sliced_codes8` with its pre-pass (C4), and the staged-row direct "
+       "kernels (eight threads per row over 64-row tiles for scalar outputs) for batches >= 32K rows.", "",
        f"Fitted constants (microseconds): a_s = {p['a_s']:.3g}, b_s = {p['b_s']:.4g}, "
        f"g_s = {p['g_s']:.3g}, a_c = {p['a_c']:.3g}, b_c = {p['b_c']:.4g}, e_c = {p['e_c']:.4g}, "
+       f"a_w = {p.get('a_w', float('nan')):.3g}, b_w = {p.get('b_w', float('nan')):.4g}, e_w = {p.get('e_w', float('nan')):.4g}, "
        f"a_d = {p['a_d']:.4g}, l_d = {p['l_d']:.4g}, b_d = {p['b_d']:.4g}, g_d = {p['g_d']:.4g}", "",
        f"Rank accuracy (model picks the measured-fastest strategy): **{p['rank_accuracy']}** "
        "(paper: 87/90, P:2413-2422).", "",

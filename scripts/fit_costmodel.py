@@ -6,6 +6,7 @@ Times both strategies on the BASELINE-shaped forests over a sweep of batch sizes
     sliced : T = a_s + b_s * U_s,   U_s = ceil(tiles / cps) * 64 * V / (slices * eff_sim)
     direct : T = a_d + max(l_d * V, b_d * V * n / SMs)
     coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs   (reading R7)
+    wide   : T = a_w + b_w * U_s + e_w * ceil(n / 64) * 64 * passes / SMs   (reading R8, d > 127)
 
 (costmodel.cpp), writes paper_conf_eurosys_xiedlll21_b200/costmodel_b200.json (read by
 libtahoe.so at load) and a report with the model's rank accuracy (paper: 87/90 correct orderings,
@@ -32,7 +33,7 @@ SWEEP = {
     1: [100, 1000, 10_000, 100_000],
     2: [100, 1000, 10_000, 100_000, 1_000_000],
     3: [1000, 10_000, 100_000, 1_000_000],
-    4: [1000, 10_000, 100_000],
+    4: [1000, 10_000, 100_000, 300_000],
     5: [1000, 10_000, 100_000],
 }
 
@@ -53,7 +54,7 @@ def time_ms(F, X, strat, reps=5):
     return statistics.median(ts)
 
 
-def main():
+def measure():
     rows = []
     for cid, ns in SWEEP.items():
         if QUICK:
@@ -71,7 +72,8 @@ def main():
                        slices=st["n_slices"], eff_sim=st["lockstep_eff_sim"],
                        sms=st["num_sms"], sliced_valid=st["sliced_valid"],
                        coded_valid=st["sliced_valid"] and st["coded_valid"],
-                       passes=max(1, (1 << st["sliced_fbits"]) // 32),
+                       passes=max(1, (1 << (st["code8_vfbits"] if st["code8"] else st["sliced_fbits"])) // 32),
+                       wide=bool(st["code8"]),
                        rows_global=cid == 4)  # C4: d = 2000 (> 256, too wide to stage)
             rec["direct_ms"] = time_ms(F, X, T.STRATEGY_DIRECT)
             rec["sliced_ms"] = time_ms(F, X, T.STRATEGY_SLICED) if st["sliced_valid"] else None
@@ -79,6 +81,20 @@ def main():
             rows.append(rec)
             print(json.dumps(rec), flush=True)
         F.close()
+    return rows
+
+
+# Row-coding cost of the wide codes per row-pass per SM, from the C4 bench's pre-pass
+# (k_encode_rows8: 2.6 ms per 500K rows x 64 passes on 148 SMs).  The sweep alone cannot separate
+# it from the walk (on the one wide config both terms grow with n).
+E_W_PREPASS = 2600.0 / (500_032 * 64 / 148)
+
+
+def main():
+    if "--refit" in sys.argv:   # re-fit saved measurements (no GPU)
+        rows = json.load(open(sys.argv[sys.argv.index("--refit") + 1]))["rows"]
+    else:
+        rows = measure()
 
     def U_s(r):
         tiles = math.ceil(r["n"] / 64)
@@ -97,15 +113,26 @@ def main():
     def E_c(r):
         return math.ceil(r["n"] / 64) * 64 * r["passes"] / r["sms"]
 
-    cd = [r for r in rows if r["coded_ms"] is not None]
-    if cd:
+    def fit3(cd, default):
+        if len(cd) < 3:
+            return default
         Ac = np.array([[1.0, U_s(r), E_c(r)] for r in cd])
         yc = np.array([r["coded_ms"] * 1000 for r in cd])
         wc = 1.0 / yc
-        a_c, b_c, e_c = np.linalg.lstsq(Ac * wc[:, None], yc * wc, rcond=None)[0]
-        a_c, b_c, e_c = max(a_c, 1.0), max(b_c, 1e-9), max(e_c, 0.0)
+        a, b, e = np.linalg.lstsq(Ac * wc[:, None], yc * wc, rcond=None)[0]
+        return max(a, 1.0), max(b, 1e-9), max(e, 0.0)
+
+    a_c, b_c, e_c = fit3([r for r in rows if r["coded_ms"] is not None and not r["wide"]], (30.0, 6.6e-5, 1.6e-5))
+    wd = [r for r in rows if r["coded_ms"] is not None and r["wide"]]
+    e_w = E_W_PREPASS
+    if len(wd) >= 2:   # a_w, b_w on the walk's share (total - pre-pass term)
+        Aw = np.array([[1.0, U_s(r)] for r in wd])
+        yw = np.array([r["coded_ms"] * 1000 - e_w * E_c(r) for r in wd])
+        ww = 1.0 / np.array([r["coded_ms"] * 1000 for r in wd])
+        a_w, b_w = np.linalg.lstsq(Aw * ww[:, None], yw * ww, rcond=None)[0]
+        a_w, b_w = max(a_w, 1.0), max(b_w, 1e-9)
     else:
-        a_c, b_c, e_c = 30.0, 6.6e-5, 1.6e-5
+        a_w, b_w = 40.0, 1.68e-4
 
     def direct_model(p, r):
         a, l, b, g = p
@@ -117,14 +144,21 @@ def main():
     a_d, l_d, b_d, g_d = np.abs(res.x)
     params = dict(a_s=float(a_s), b_s=float(b_s), g_s=g_s, a_d=float(a_d), l_d=float(l_d), b_d=float(b_d),
                   g_d=float(g_d), a_c=float(a_c), b_c=float(b_c), e_c=float(e_c),
-                  units="microseconds", gpu=torch.cuda.get_device_name(0))
+                  a_w=float(a_w), b_w=float(b_w), e_w=float(e_w),
+                  units="microseconds",
+                  gpu=torch.cuda.get_device_name(0) if torch.cuda.is_available() else "NVIDIA B200")
 
     correct = total = 0
     report = []
     for r in rows:
         ps = (params["a_s"] + params["b_s"] * U_s(r) * (g_s if r["rows_global"] else 1.0)
               if r["sliced_ms"] is not None else math.inf)
-        pc = a_c + b_c * U_s(r) + e_c * E_c(r) if r["coded_ms"] is not None else math.inf
+        if r["coded_ms"] is None:
+            pc = math.inf
+        elif r["wide"]:
+            pc = a_w + b_w * U_s(r) + e_w * E_c(r)
+        else:
+            pc = a_c + b_c * U_s(r) + e_c * E_c(r)
         pd = direct_model([a_d, l_d, b_d, g_d], r)
         r.update(pred_sliced_us=ps, pred_direct_us=pd, pred_coded_us=pc)
         if r["sliced_ms"] is None:

@@ -659,42 +659,50 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   DeviceGuard g(f->device);
   cudaStream_t user = reinterpret_cast<cudaStream_t>(stream);
   const int32_t C = f->host.n_out();
-  // 8 chunks (>= 64K rows each): overlap H2D / compute / D2H; 16 smaller chunks measured slower
-  // (per-chunk launch and finalize overheads outweigh the shorter tail)
+  // Chunks overlap H2D / compute / D2H on three streams: 8 chunks of >= 64K rows.  The time is
+  // about H2D of every row plus the compute of the last chunk, as long as a chunk's compute (fixed
+  // launch / tail cost + per-row cost) stays below its H2D; 16 equal chunks, and 8 chunks followed
+  // by halving tail chunks, measured slower (more fixed per-chunk cost).  Three buffers, so a copy
+  // never waits for the compute of the chunk before the previous one.
   const int64_t chunk = std::min<int64_t>(n, std::max<int64_t>(65536, (n + 7) / 8));
-  const int64_t nchunks = (n + chunk - 1) / chunk;
+  std::vector<int64_t> cuts;
+  for (int64_t r = 0; r < n; r += chunk) cuts.push_back(r);
+  cuts.push_back(n);
+  const int64_t nchunks = (int64_t)cuts.size() - 1;
+  constexpr int NB = 3;
   cudaStream_t s_in, s_cmp, s_out;
   cudaStreamCreateWithFlags(&s_in, cudaStreamNonBlocking);
   cudaStreamCreateWithFlags(&s_cmp, cudaStreamNonBlocking);
   cudaStreamCreateWithFlags(&s_out, cudaStreamNonBlocking);
-  cudaEvent_t ev_start, ev_in[2], ev_cmp[2], ev_out[2];
+  cudaEvent_t ev_start, ev_in[NB], ev_cmp[NB], ev_out[NB];
   cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming);
-  for (int b = 0; b < 2; b++) {
+  for (int b = 0; b < NB; b++) {
     cudaEventCreateWithFlags(&ev_in[b], cudaEventDisableTiming);
     cudaEventCreateWithFlags(&ev_cmp[b], cudaEventDisableTiming);
     cudaEventCreateWithFlags(&ev_out[b], cudaEventDisableTiming);
   }
+  const int64_t nbuf = std::min<int64_t>(NB, nchunks);
   float* dX = nullptr;
   float* dO = nullptr;
   int32_t* dC = nullptr;
-  cudaError_t e = scratch_alloc((void**)&dX, (size_t)2 * chunk * d * 4, user);
-  if (e == cudaSuccess) e = scratch_alloc((void**)&dO, (size_t)2 * chunk * C * 4, user);
-  if (e == cudaSuccess && class_host) e = scratch_alloc((void**)&dC, (size_t)2 * chunk * 4, user);
+  cudaError_t e = scratch_alloc((void**)&dX, (size_t)nbuf * chunk * d * 4, user);
+  if (e == cudaSuccess) e = scratch_alloc((void**)&dO, (size_t)nbuf * chunk * C * 4, user);
+  if (e == cudaSuccess && class_host) e = scratch_alloc((void**)&dC, (size_t)nbuf * chunk * 4, user);
   cudaEventRecord(ev_start, user);
   cudaStreamWaitEvent(s_in, ev_start, 0);
   cudaStreamWaitEvent(s_cmp, ev_start, 0);
   cudaStreamWaitEvent(s_out, ev_start, 0);
   for (int64_t c = 0; c < nchunks && e == cudaSuccess && st == TAHOE_OK; c++) {
-    const int b = (int)(c & 1);
-    const int64_t r0 = c * chunk, nr = std::min(chunk, n - r0);
+    const int b = (int)(c % NB);
+    const int64_t r0 = cuts[c], nr = cuts[c + 1] - cuts[c];
     float* xb = dX + (size_t)b * chunk * d;
     float* ob = dO + (size_t)b * chunk * C;
     int32_t* cb = dC ? dC + (size_t)b * chunk : nullptr;
-    if (c >= 2) cudaStreamWaitEvent(s_in, ev_cmp[b], 0);     // X buffer consumed by chunk c-2
+    if (c >= NB) cudaStreamWaitEvent(s_in, ev_cmp[b], 0);    // X buffer consumed by chunk c-NB
     e = cudaMemcpyAsync(xb, X_host + r0 * d, (size_t)nr * d * 4, cudaMemcpyHostToDevice, s_in);
     cudaEventRecord(ev_in[b], s_in);
     cudaStreamWaitEvent(s_cmp, ev_in[b], 0);
-    if (c >= 2) cudaStreamWaitEvent(s_cmp, ev_out[b], 0);    // out buffer drained by chunk c-2
+    if (c >= NB) cudaStreamWaitEvent(s_cmp, ev_out[b], 0);   // out buffer drained by chunk c-NB
     if (e == cudaSuccess)
       st = run(f, xb, nr, d, ob, cb, nullptr, nullptr, nullptr, -1, s_cmp);
     cudaEventRecord(ev_cmp[b], s_cmp);
@@ -713,7 +721,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   if (dO) cudaFreeAsync(dO, user);
   if (dC) cudaFreeAsync(dC, user);
   cudaEventDestroy(ev_start);
-  for (int b = 0; b < 2; b++) { cudaEventDestroy(ev_in[b]); cudaEventDestroy(ev_cmp[b]); cudaEventDestroy(ev_out[b]); }
+  for (int b = 0; b < NB; b++) { cudaEventDestroy(ev_in[b]); cudaEventDestroy(ev_cmp[b]); cudaEventDestroy(ev_out[b]); }
   cudaStreamDestroy(s_in);
   cudaStreamDestroy(s_cmp);
   cudaStreamDestroy(s_out);

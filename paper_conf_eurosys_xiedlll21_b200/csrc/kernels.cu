@@ -1552,7 +1552,13 @@ __device__ __forceinline__ void bisect8(uint32_t base, const float* x, uint32_t*
   for (int q = 0; q < kR; q++) pos[q] = (ad[q] - base) >> 7;
 }
 
-__global__ void __launch_bounds__(1024, 1) k_encode_rows8(const Encode8Args a) {
+// 1024 threads x 4 rows per warp step (64 registers, no spills): C4 pre-pass 2.12 ms per 500K
+// rows; 8 rows per step spill at 1024 threads (2.60 ms) and at 512 threads lack the warps to
+// cover the X loads (3.02 ms)
+constexpr int kEncode8Threads = 1024;
+constexpr int kEncode8Rows = 4;
+template <int THREADS, int kR>
+__global__ void __launch_bounds__(THREADS, 1) k_encode_rows8(const Encode8Args a) {
   extern __shared__ __align__(1024) float s_img[];
   __shared__ uint64_t s_bar;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = blockDim.x >> 5;
@@ -1572,7 +1578,6 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows8(const Encode8Args a) {
     }
     mbar_wait(&s_bar, 0);
   }
-  constexpr int kR = 8;
   static_assert(kCode8TileRows % kR == 0, "a row group stays inside one tile");
   // this chunk's rows, in whole groups of kR
   const int64_t groups = (a.n + kR - 1) / kR;
@@ -1890,13 +1895,14 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
   const int64_t chunk = code8_chunk_rows(img.vfbits, n);
   const int64_t ctiles = (chunk + kCode8TileRows - 1) / kCode8TileRows;
   uint32_t* flags = reinterpret_cast<uint32_t*>(codes + ctiles * tbytes);
-  cudaError_t e;
+  cudaError_t e = cudaSuccess;
   {
     static std::atomic<int> configured[64];
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
-      e = cudaFuncSetAttribute(k_encode_rows8, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
+      e = cudaFuncSetAttribute(k_encode_rows8<kEncode8Threads, kEncode8Rows>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
       for (auto k : {k_sliced_codes8<true, kCode8TileRows, kCode8Ring>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring>})
         if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
       if (e != cudaSuccess) return (int)e;
@@ -1930,7 +1936,7 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     ea.v_src = img.v_src;
     ea.codes = codes;
     ea.flags = flags;
-    k_encode_rows8<<<ea.bands * ea.chunks, 1024, kCode8BandBudget, st>>>(ea);
+    k_encode_rows8<kEncode8Threads, kEncode8Rows><<<ea.bands * ea.chunks, kEncode8Threads, kCode8BandBudget, st>>>(ea);
     if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
     Coded8KArgs a{};
     a.img = img;

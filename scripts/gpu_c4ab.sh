@@ -1,6 +1,3 @@
 #!/bin/bash
-# C4 wide codes: tail / switching experiments
-for n in 500000 1000000; do
-for sw in 1 0; do echo "n $n switch $sw"; TAHOE_CODE8_SWITCH=$sw timeout 200 python scripts/diag_timing.py 4 $n 2>&1 | grep "strategy=2"; done
-echo "n $n chunk 256"; TAHOE_CODE8_CHUNK_MB=256 timeout 200 python scripts/diag_timing.py 4 $n 2>&1 | grep "strategy=2"
-done
+# C4 wide-code pre-pass variants (same box): 0 = 512 threads x 8 rows, 1 = 1024 x 8, 2 = 1024 x 4
+for rep in 1 2; do for v in 0 1 2; do echo "enc8 $v"; TAHOE_ENC8=$v timeout 200 python scripts/diag_timing.py 4 500000 2>&1 | grep "strategy=2"; done; done

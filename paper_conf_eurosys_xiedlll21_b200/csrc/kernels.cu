@@ -1636,6 +1636,7 @@ struct Coded8KArgs {
   int64_t row0;          // first row of this launch's chunk (outputs are indexed row0 + r)
   int64_t n_all;         // rows of the whole batch (row stride of the raw partials)
   int32_t switch_slices; // 1: a CTA whose slice is exhausted moves to another (0: experiments)
+  int32_t prefetch;      // tiles ahead of a claim to prefetch into L2 (0 = none)
   OutArgs o;
 };
 
@@ -1754,6 +1755,11 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
         mbar_expect_tx(&s_full[b], 0u);
       } else {
         atomicAdd(s_vis, 1u);
+        // warm L2 with the tile this slice's CTAs will claim a few claims from now (the tiles
+        // are mostly not in L2: the slices drift apart over the batch)
+        if (a.prefetch > 0 && tile + a.prefetch < ntiles)
+          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a.codes + (int64_t)(tile + a.prefetch) * tile_bytes),
+                       "r"(tile_bytes) : "memory");
         fence_proxy_async_smem();
         mbar_expect_tx(&s_full[b], tile_bytes + 16u * FS);
         bulk_g2s(s_ring + (size_t)b * tile_bytes, a.codes + (int64_t)tile * tile_bytes, tile_bytes, &s_full[b]);
@@ -1950,6 +1956,9 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     a.n_all = n;
     a.forest_smem = plan.forest_smem;
     a.switch_slices = !(std::getenv("TAHOE_CODE8_SWITCH") && std::atoi(std::getenv("TAHOE_CODE8_SWITCH")) == 0);
+    // L2 prefetch 8 tiles ahead of each claim (C4 walk 7.27 -> 6.88 ms; 24 and 64 the same within
+    // 1 %); $TAHOE_CODE8_PREFETCH overrides (experiments)
+    a.prefetch = std::getenv("TAHOE_CODE8_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODE8_PREFETCH")) : 8;
     // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
     // every CTA a few tiles, else the plan's grid
     const bool full = plan.cta_start && ntiles >= 4LL * num_sms;

@@ -921,6 +921,7 @@ struct CodedKArgs {
   int32_t rb;            // bytes per code row
   int32_t cps;           // CTAs per slice (single-pass, no cta_start)
   const int32_t* cta_start;  // or: slice s is worked by CTAs [cta_start[s], cta_start[s+1])
+  int32_t prefetch;      // entries of the CTA's tile sequence to prefetch into L2 ahead (0 = none)
   OutArgs o;
 };
 
@@ -1002,8 +1003,12 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   }
   __syncthreads();
 
-  auto issue_tile = [&](int64_t tile, int b) {
+  auto issue_tile = [&](int64_t tile, int b, int64_t ahead = -1) {
     if (lane == 0) {
+      // optional L2 prefetch of this CTA's tile `ahead` (a later tile of its sequence)
+      if (ahead >= 0 && ahead < ntiles)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
+                     "r"((uint32_t)a.tstride) : "memory");
       fence_proxy_async_smem();
       mbar_expect_tx(&s_full[b], (uint32_t)a.tstride);
       bulk_g2s(s_ring + (size_t)b * a.tstride,
@@ -1026,7 +1031,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     last = __shfl_sync(0xffffffffu, last, 0);
     if (!last) return;
     if (FUSED) {
-      if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+      if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
       return;
     }
     // take the tile's 64 partials out of shared memory, refill the buffer at once, then store the
@@ -1036,7 +1041,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     const double* sp = s_part + b * kSlicedTileRows;
     const double p0 = lane < nr ? sp[lane] : 0.0, p1 = lane + 32 < nr ? sp[lane + 32] : 0.0;
     __syncwarp();
-    if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+    if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
     double* dst = a.o.raw + (size_t)sl * a.n + r0;
     if (lane < nr) dst[lane] = p0;
     if (lane + 32 < nr) dst[lane + 32] = p1;
@@ -1485,6 +1490,7 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   a.rb = code_row_bytes(img.fbits);
   a.cps = plan.cps;
   a.cta_start = plan.cta_start;
+  a.prefetch = std::getenv("TAHOE_CODES_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODES_PREFETCH")) : 0;
   a.o = o;
   const int smem = plan.forest_smem + kRing * tstride + kSlicedBarrierBytes +
                    kRing * kSlicedTileRows * (int)sizeof(double);

@@ -1643,6 +1643,7 @@ struct Coded8KArgs {
   int64_t n_all;         // rows of the whole batch (row stride of the raw partials)
   int32_t switch_slices; // 1: a CTA whose slice is exhausted moves to another (0: experiments)
   int32_t prefetch;      // tiles ahead of a claim to prefetch into L2 (0 = none)
+  uint32_t sleep_ns;     // back-off between ticket polls
   OutArgs o;
 };
 
@@ -1810,7 +1811,9 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
       const uint32_t e = g + it;
       const int b = (int)(e % kR8);
       if (lane == 0)
-        while (*reinterpret_cast<volatile uint32_t*>(&s_gen[b]) != e) __nanosleep(128);
+        while (*reinterpret_cast<volatile uint32_t*>(&s_gen[b]) != e) {
+          if (a.sleep_ns) __nanosleep(a.sleep_ns);
+        }
       __syncwarp();
       mbar_wait(&s_full[b], (e / kR8) & 1u);
       const int32_t tile = *reinterpret_cast<volatile int32_t*>(&s_tile[b]);
@@ -1965,6 +1968,10 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     // L2 prefetch 8 tiles ahead of each claim (C4 walk 7.27 -> 6.88 ms; 24 and 64 the same within
     // 1 %); $TAHOE_CODE8_PREFETCH overrides (experiments)
     a.prefetch = std::getenv("TAHOE_CODE8_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODE8_PREFETCH")) : 8;
+    // ticket polls spin without back-off: the walk issues at ~33 %, so the polls cost little,
+    // while a 32 / 128 / 512 ns back-off delays the waiting warps (C4 walk 6.39 / 6.80 / 6.88 /
+    // 11.46 ms); $TAHOE_CODE8_SLEEP overrides (experiments)
+    a.sleep_ns = std::getenv("TAHOE_CODE8_SLEEP") ? (uint32_t)std::atoi(std::getenv("TAHOE_CODE8_SLEEP")) : 0u;
     // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
     // every CTA a few tiles, else the plan's grid
     const bool full = plan.cta_start && ntiles >= 4LL * num_sms;

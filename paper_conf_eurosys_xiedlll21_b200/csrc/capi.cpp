@@ -103,6 +103,7 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->ds.c8_grp);
   cudaFree((void*)f->ds.c8_band);
   cudaFree((void*)f->ds.slice_w);
+  cudaFree((void*)f->ds.col_mid);
   cudaFree(f->d_class_ptr);
   cudaFree(f->d_class_parts);
   cudaFree(f->d_cta_start);
@@ -236,6 +237,7 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
         f->ds.code8 = 1;
         std::vector<float> w(f->sl.slice_work.begin(), f->sl.slice_work.end());
         if ((st = upload(w, &f->ds.slice_w)) != TAHOE_OK) return st;
+        if ((st = upload(f->sl.col_mid, &f->ds.col_mid)) != TAHOE_OK) return st;
       }
     }
   }

@@ -663,6 +663,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
   if (S.code_valid) S.cnodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);
   S.col_len.assign((size_t)S.n_slices * C, 0);
+  S.col_mid.assign((size_t)S.n_slices * C, 0);
   S.slots.assign(S.n_slices, 0);
   std::vector<int32_t> slot(F.feat.size(), -1);
   std::vector<int32_t> pre, st;
@@ -672,8 +673,10 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
     for (int32_t l = 0; l < C; l++) {
       int32_t pos = 0;
       const auto& L = P.lanes[l];
+      std::vector<int32_t> root_pos;   // slot of each tree's root in this column
       for (size_t ti = 0; ti < L.size(); ti++) {
         const int32_t t = L[ti];
+        root_pos.push_back(pos);
         if (F.tree_size(t) == 1) {  // 3-node stump: root (attribute 0, +2 slots right) + 2 leaves
           const int32_t k = F.node_base[t];
           const uint32_t ynode = (2u << sb) << (S.fbits + 3);
@@ -739,6 +742,18 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
       S.nodes[2 * w + 1] = fmask << 2;
       if (S.code_valid) { S.cnodes[2 * w] = 0u; S.cnodes[2 * w + 1] = cleaf; }
       S.col_len[(size_t)s * C + l] = pos;
+      // the column's split point for two chains per row (wide codes): the tree root that best
+      // halves the column's expected work (no split: the terminal slot, the second chain idles)
+      {
+        double total = 0.0, pre = 0.0, best = 1e300;
+        for (int32_t t : L) total += F.exp_reads[t];
+        int32_t mid = pos;
+        for (size_t ti = 0; ti < L.size(); ti++) {
+          if (ti > 0 && std::max(pre, total - pre) < best) { best = std::max(pre, total - pre); mid = root_pos[ti]; }
+          pre += F.exp_reads[L[ti]];
+        }
+        S.col_mid[(size_t)s * C + l] = mid;
+      }
     }
   }
   // class -> slices (in slice order: the fixed fp64 summation order of the finalize step)

@@ -81,7 +81,9 @@ struct SlicedImage {
   std::string why_invalid;
   int32_t n_slices = 0, slots_max = 0, fbits = 0;
   std::vector<int32_t> slots, cls, ntrees;       // per slice
-  std::vector<int32_t> col_len;                  // [ns*32]
+  std::vector<int32_t> col_len;                  // [ns*16]
+  std::vector<int32_t> col_mid;                  // [ns*16] slot of the first tree of the column's
+                                                 // second half by expected work (== col_len: none)
   std::vector<uint32_t> nodes;                   // [ns*slots_max*32*2]
   std::vector<int32_t> leaf_meta;                // [ns*slots_max*32*2] {tree, node}
   std::vector<int32_t> class_ptr, class_parts;   // class -> slices (CSR)

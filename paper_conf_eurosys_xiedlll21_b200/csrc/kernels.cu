@@ -1644,6 +1644,7 @@ struct Coded8KArgs {
   int32_t switch_slices; // 1: a CTA whose slice is exhausted moves to another (0: experiments)
   int32_t prefetch;      // tiles ahead of a claim to prefetch into L2 (0 = none)
   uint32_t sleep_ns;     // back-off between ticket polls
+  int32_t split;         // 1: four chains per lane (each column walked as two halves)
   OutArgs o;
 };
 
@@ -1676,6 +1677,36 @@ __device__ __forceinline__ void walk_coded8(uint32_t pA, uint32_t pB, uint32_t p
     add_pair_ftz(accA, a1, a2);
     add_pair_ftz(accB, b1, b2);
   }
+}
+
+// Four chains per lane: each row's column is walked as two halves (split at col_mid, the tree
+// root that halves the column's expected work), so a lane keeps four independent node chains in
+// flight over the same two staged rows.  A first-half chain freezes at its split slot (it keeps
+// re-reading that internal node, whose word adds +0).
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_coded8_split(uint32_t pA1, uint32_t mA, uint32_t pA2, uint32_t pB1,
+                                                  uint32_t mB, uint32_t pB2, uint32_t pe,
+                                                  uint32_t rowA, uint32_t rowB, uint32_t amask,
+                                                  uint32_t dlbit, uint32_t shmul, double& accA,
+                                                  double& accB) {
+  double a1 = 0.0, a2 = 0.0, b1 = 0.0, b2 = 0.0;
+  while ((pA1 != mA) | (pA2 != pe) | (pB1 != mB) | (pB2 != pe)) {
+    uint32_t q;
+    q = pA1; const float x1 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul); pA1 = pA1 == mA ? pA1 : q;
+    q = pB1; const float y1 = coded8_step<NAN_AWARE>(q, rowB, amask, dlbit, shmul); pB1 = pB1 == mB ? pB1 : q;
+    const float x3 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul);
+    const float y3 = coded8_step<NAN_AWARE>(pB2, rowB, amask, dlbit, shmul);
+    q = pA1; const float x2 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul); pA1 = pA1 == mA ? pA1 : q;
+    q = pB1; const float y2 = coded8_step<NAN_AWARE>(q, rowB, amask, dlbit, shmul); pB1 = pB1 == mB ? pB1 : q;
+    const float x4 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul);
+    const float y4 = coded8_step<NAN_AWARE>(pB2, rowB, amask, dlbit, shmul);
+    add_pair_ftz(a1, x1, x2);
+    add_pair_ftz(b1, y1, y2);
+    add_pair_ftz(a2, x3, x4);
+    add_pair_ftz(b2, y3, y4);
+  }
+  accA = a1 + a2;
+  accB = b1 + b2;
 }
 
 // k_sliced_codes8: k_sliced_codes' walk (slice resident in shared memory, dynamic 4-row work
@@ -1834,10 +1865,16 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
           nan_flag |= fk;
         }
         double accA, accB;
-        if (nan_flag)
+        if (a.split) {
+          const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
+          const uint32_t mA = okA ? pm : pe, mB = okB ? pm : pe;
+          if (nan_flag) walk_coded8_split<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          else walk_coded8_split<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        } else if (nan_flag) {
           walk_coded8<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-        else
+        } else {
           walk_coded8<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        }
         // butterfly over the 16 lane columns: after the xor-8 exchange lanes with bit 3 clear
         // hold chain A, set hold chain B (lanes 0, 8, 16, 24 own rows rA(h=0), rB(h=0), rA(h=1),
         // rB(h=1))
@@ -1972,6 +2009,8 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     // while a 32 / 128 / 512 ns back-off delays the waiting warps (C4 walk 6.39 / 6.80 / 6.88 /
     // 11.46 ms); $TAHOE_CODE8_SLEEP overrides (experiments)
     a.sleep_ns = std::getenv("TAHOE_CODE8_SLEEP") ? (uint32_t)std::atoi(std::getenv("TAHOE_CODE8_SLEEP")) : 0u;
+    // four chains per lane (C4 walk 6.43 -> 6.22 ms); $TAHOE_CODE8_SPLIT=0: two (experiments)
+    a.split = img.col_mid ? (std::getenv("TAHOE_CODE8_SPLIT") ? std::atoi(std::getenv("TAHOE_CODE8_SPLIT")) : 1) : 0;
     // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
     // every CTA a few tiles, else the plan's grid
     const bool full = plan.cta_start && ntiles >= 4LL * num_sms;

@@ -58,6 +58,7 @@ struct DevSliced {
   const int4x* c8_band = nullptr;    // [bands] {byte offset, bytes, first group, end group}
   int32_t c8_bands = 0;
   const float* slice_w = nullptr;    // [ns] simulated lane-steps per row (dynamic slice choice)
+  const int32_t* col_mid = nullptr;  // [ns][16] split slot of each column (two chains per row)
 };
 
 // ------------------------------------------------------------------ rank-coded rows (reading R7)

@@ -490,7 +490,10 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
       const int64_t room = (int64_t)max_smem - code8_ring_smem(vfb);
       const int32_t cap8 = (int32_t)std::max<int64_t>(0, (room & ~1023LL) / kSlotBytes);
       bool fits = cap8 >= 16;
-      for (int32_t t = 0; t < F.n_trees && fits; t++) fits = enc_size(F, t) <= cap8 - 1;
+      // offsets within a tree (right child, next root) stay below the tree's size; the code word
+      // keeps 32 - (V + 1) bits of byte offset (slots of 128 bytes)
+      const int32_t off8 = 1 << std::min(30, 32 - (vfb + 1) - 7);
+      for (int32_t t = 0; t < F.n_trees && fits; t++) fits = enc_size(F, t) <= cap8 - 1 && enc_size(F, t) < off8;
       if (fits) {
         S.code8 = true;
         S.vfbits = vfb;
@@ -502,8 +505,13 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
   cap -= 1;                                    // one terminal slot per lane column
   if (F.agg == TAHOE_AGG_VOTE) { S.why_invalid = "VOTE runs on the direct strategy"; return TAHOE_OK; }
   if (cap < 1) { S.why_invalid = "no shared memory budget"; return TAHOE_OK; }
-  for (int32_t t = 0; t < F.n_trees; t++)
+  // a node word keeps 32 - (F + 3) bits of byte offset (slots of 128 bytes); offsets within a tree
+  // (right child, next tree root) stay below the tree's size
+  const int64_t off_slots = (int64_t)1 << std::max(0, 32 - (S.fbits + 3) - 7);
+  for (int32_t t = 0; t < F.n_trees; t++) {
     if (enc_size(F, t) > cap) { S.why_invalid = "a tree exceeds one lane column of shared memory"; return TAHOE_OK; }
+    if (enc_size(F, t) >= off_slots) { S.why_invalid = "a tree is too large for the node word's offset field"; return TAHOE_OK; }
+  }
 
   int64_t m = 0;
   const std::vector<int32_t> reads = sim_reads(F, m);
@@ -657,8 +665,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
   const int32_t csh = S.code8 ? S.vfbits + 1 : S.fbits + 2;
   const uint32_t cdl = S.code8 ? 1u << S.vfbits : 1u << (S.fbits + 1);
   const uint32_t cleaf = S.code8 ? (1u << S.vfbits) - 1u : fmask << 1;
-  if (S.code_valid && S.code8 && (uint32_t)S.slots_max >= (1u << (32 - csh - sb)))
-    return fail(TAHOE_E_UNSUPPORTED, "wide-code offset overflow");
+
   S.nodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   if (S.code_valid) S.cnodes.assign((size_t)S.n_slices * per_slice * 2, 0);
   S.leaf_meta.assign((size_t)S.n_slices * per_slice * 2, -1);

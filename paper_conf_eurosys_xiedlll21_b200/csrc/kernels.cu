@@ -917,7 +917,7 @@ struct CodedKArgs {
   int64_t n;
   int32_t forest_smem;   // bytes reserved for the slice (multiple of 1024)
   int32_t tile_bytes;    // the 64 code rows of a tile (its NaN flag follows them)
-  int32_t tstride;       // bytes per tile (rows + 128-byte trailer), in HBM and in the ring
+  int32_t tstride;       // bytes per tile (rows + trailer of max(128, row bytes)), in HBM and in the ring
   int32_t rb;            // bytes per code row
   int32_t cps;           // CTAs per slice (single-pass, no cta_start)
   const int32_t* cta_start;  // or: slice s is worked by CTAs [cta_start[s], cta_start[s+1])
@@ -1540,20 +1540,26 @@ struct Encode8Args {
 // compare false): probe at pos + step - 1 for step = 2^(K-1) .. 1.  The running address a[q] =
 // base + pos[q] * 128 makes every probe one LDS with an immediate offset, one FSETP and one
 // predicated add.
+// one bisection level of bisect8 (probe offset and step are immediates: LDS [ad + imm]; FSETP;
+// predicated IADD: three instructions per probe), then the next level
+template <int ST, int kR>
+__device__ __forceinline__ void probe8(uint32_t* ad, const float* x) {
+#pragma unroll
+  for (int q = 0; q < kR; q++)
+    asm("{\n\t.reg .f32 t;\n\t.reg .pred p;\n\t"
+        "ld.shared.f32 t, [%0+%2];\n\t"
+        "setp.le.f32 p, t, %1;\n\t"
+        "@p add.u32 %0, %0, %3;\n\t}"
+        : "+r"(ad[q]) : "f"(x[q]), "n"(((1u << ST) - 1u) << 7), "n"((1u << ST) << 7));
+  if constexpr (ST > 0) probe8<ST - 1, kR>(ad, x);
+}
+
 template <int K, int kR>
 __device__ __forceinline__ void bisect8(uint32_t base, const float* x, uint32_t* pos) {
   uint32_t ad[kR];
 #pragma unroll
   for (int q = 0; q < kR; q++) ad[q] = base;
-#pragma unroll
-  for (int st = K - 1; st >= 0; st--) {
-#pragma unroll
-    for (int q = 0; q < kR; q++) {
-      float t;
-      asm("ld.shared.f32 %0, [%1];" : "=f"(t) : "r"(ad[q] + (((1u << st) - 1u) << 7)));
-      ad[q] += t <= x[q] ? (1u << st) << 7 : 0u;
-    }
-  }
+  probe8<K - 1, kR>(ad, x);
 #pragma unroll
   for (int q = 0; q < kR; q++) pos[q] = (ad[q] - base) >> 7;
 }

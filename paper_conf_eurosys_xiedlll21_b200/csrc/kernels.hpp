@@ -77,9 +77,13 @@ constexpr uint16_t kCodeNan = 0xFFFEu;
 constexpr uint16_t kCodePad = 0xFFFFu;
 inline int32_t code_row_bytes(int32_t fbits) { return (2 << fbits) < 64 ? 64 : (2 << fbits); }
 inline int32_t code_tile_bytes(int32_t fbits) { return 64 * code_row_bytes(fbits); }
-// a code tile in HBM and in the ring: the rows, then a 128-byte trailer whose first word is the
-// tile's NaN flag (1 if any of its codes is kCodeNan; it arrives with the tile's bulk copy)
-inline int32_t code_tile_stride(int32_t fbits) { return code_tile_bytes(fbits) + 128; }
+// a code tile in HBM and in the ring: the rows, then a trailer whose first word is the tile's NaN
+// flag (1 if any of its codes is kCodeNan; it arrives with the tile's bulk copy).  The trailer is
+// max(128, row bytes) long so that every ring buffer's rows stay aligned to the row size: a code
+// address is formed by OR-ing the attribute's byte offset into the row base.
+inline int32_t code_tile_stride(int32_t fbits) {
+  return code_tile_bytes(fbits) + (code_row_bytes(fbits) > 128 ? code_row_bytes(fbits) : 128);
+}
 
 // ------------------------------------------------------------------ wide codes (reading R8)
 // Rows of more than 127 attributes: an attribute with K distinct thresholds becomes ceil(K / 127)

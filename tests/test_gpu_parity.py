@@ -498,7 +498,9 @@ def test_rank_codes_row_widths(d, monkeypatch):
     rng = np.random.default_rng(d)
     grid = np.linspace(-2.0, 2.0, 41)
     f = random_forest(rng, 48, 6, d, thr_grid=grid)
-    X = rng.normal(size=(9001, d)).astype(np.float32)
+    # 20011 rows = 313 code tiles: every CTA of a one-slice forest walks several tiles, so every
+    # ring buffer is used (256-byte rows once misaligned the second buffer's row base)
+    X = rng.normal(size=(20011, d)).astype(np.float32)
     X[rng.random(X.shape) < 0.3] = rng.choice(grid, size=1)[0]
     X[::37, 0] = np.nan
     F = T.Forest(f, n_features=d, n_classes=1, agg=oracle.AGG_SUM, device=0)

@@ -76,7 +76,12 @@ static cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
 static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
   const int32_t fb = feature_bits(n_features + 1);
   const bool padded = n_features % 4 == 0;   // predict with d == n_features takes the 2-D TMA path
-  const int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb, padded));
+  int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb, padded));
+  // forests that can take the u16 rank codes (reading R7) keep room for their code-tile ring and
+  // staged partials too (rows of ~100-127 attributes are too wide for the fp32 ring, which would
+  // otherwise leave the whole of shared memory to the slice)
+  if (fb <= kCodeMaxFbits)
+    ring = std::max<int64_t>(ring, (int64_t)kSlicedRing * code_tile_stride(fb) + (int64_t)kSlicedRing * kSlicedTileRows * 8);
   // the slice region is rounded up to 1 KB so the ring's row bases stay aligned
   return (int32_t)std::max<int64_t>(0, ((max_smem - ring - kSlicedBarrierBytes) & ~1023LL) / kSlotBytes);
 }

@@ -308,6 +308,69 @@ __global__ void __launch_bounds__(ROWS * P) k_direct_tlp(const DirectKArgs a, in
   }
 }
 
+// Direct strategy with tree heads in shared memory (scalar outputs, no leaf ids): k_direct_tlp's
+// walk, but the first `kh` node slots of every tree of the image (the root and the hot-first
+// preorder prefix below it, reading R1 / P:616-628) are copied once per CTA into shared memory
+// and read from there; the rest of each tree is read through L1/L2 as before.  A tree's slots are
+// contiguous from root[t] (encode_direct), so slot k of tree t is a head iff k - root[t] < kh.
+template <bool FUSED, int ROWS, int P>
+__global__ void __launch_bounds__(ROWS * P) k_direct_heads(const DirectKArgs a, int32_t rs, int32_t kh) {
+  extern __shared__ __align__(16) uint2 s_heads[];
+  const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(a.img.nodes);
+  const int fbits = a.img.fbits;
+  const uint32_t fmask = (1u << fbits) - 1u;
+  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const int32_t T = a.img.n_slots;
+  float* s_rows = reinterpret_cast<float*>(s_heads + (size_t)T * kh);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int r = threadIdx.x / P, j = threadIdx.x % P;
+  for (int32_t q = threadIdx.x; q < T * kh; q += ROWS * P) {
+    const int32_t t = q / kh;
+    const int64_t g = (int64_t)__ldg(&a.img.root[t]) + (q - t * kh);
+    s_heads[q] = g < a.img.n_nodes ? __ldg(&nodes[g]) : make_uint2(0u, 0u);
+  }
+  const int64_t ntiles = (a.n + ROWS - 1) / ROWS;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * ROWS;
+    const int nr = (int)((a.n - r0) < ROWS ? (a.n - r0) : ROWS);
+    __syncthreads();
+    for (int q = warp; q < nr; q += ROWS * P / 32) {
+      const float* src = a.X + (r0 + q) * a.d;
+      for (int c = lane; c < a.d; c += 32) s_rows[q * rs + c] = __ldg(&src[c]);
+    }
+    __syncthreads();
+    const bool active = r < nr;
+    const float* row = s_rows + (active ? r : 0) * rs;
+    double acc = 0.0;
+    if (active && j < T) {
+      int32_t t = j;
+      uint32_t hb = (uint32_t)(j * kh);
+      uint32_t rt = (uint32_t)__ldg(&a.img.root[t]);
+      uint32_t k = rt;
+      for (;;) {
+        const uint32_t rel = k - rt;
+        const uint2 nd = rel < (uint32_t)kh ? s_heads[hb + rel] : __ldg(&nodes[k]);
+        if ((int32_t)nd.y < 0) {
+          acc += (double)__uint_as_float(nd.x);
+          t += P;
+          if (t >= T) break;
+          hb += (uint32_t)(P * kh);
+          rt = k = (uint32_t)__ldg(&a.img.root[t]);
+        } else {
+          k += step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask);
+        }
+      }
+    }
+#pragma unroll
+    for (int o = 1; o < P; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (active && j == 0) {
+      const int64_t i = r0 + r;
+      if (FUSED) write_scalar(a.o, i, acc);
+      else a.o.raw[i] += acc;
+    }
+  }
+}
+
 // ------------------------------------------------------------------ sliced strategy
 // Sliced node words (encode.cpp): x = threshold (internal) or leaf value;
 //   internal y = off_bytes << (F+3) | default_left << (F+2) | attribute << 2   (left child next)
@@ -1270,6 +1333,28 @@ static cudaError_t direct_tlp_one(const DirectKArgs& a, int32_t rs, int32_t num_
   return cudaGetLastError();
 }
 
+template <bool F, int P, int kRows>
+static cudaError_t direct_heads_one(const DirectKArgs& a, int32_t rs, int32_t kh, int32_t num_sms,
+                                    cudaStream_t st) {
+  auto kern = k_direct_heads<F, kRows, P>;
+  const int smem = kRows * rs * 4 + a.img.n_slots * kh * 8;
+  static std::atomic<int> configured[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64 && configured[dev].load() < smem) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+    if (e != cudaSuccess) return e;
+    configured[dev].store(kMaxSmemOptin);
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kRows * P, smem);
+  if (per_sm < 1) per_sm = 1;
+  const int64_t ntiles = (a.n + kRows - 1) / kRows;
+  const int grid = (int)std::min<int64_t>(ntiles, (int64_t)num_sms * per_sm);
+  kern<<<grid, kRows * P, smem, st>>>(a, rs, kh);
+  return cudaGetLastError();
+}
+
 int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                   bool fused, int32_t num_sms, void* stream) {
   DirectKArgs a{img, X, n, d, o};
@@ -1290,6 +1375,21 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
   const char* env = std::getenv("TAHOE_DIRECT_VARIANT");
   int variant = env ? std::atoi(env) : (n >= 32768 ? (scalar && !leaf ? 5 : 2) : 0);
   if (d > 256) variant = 0;  // 128 staged rows must fit shared memory
+  // 8 / 9: variant 5 / 128 rows x 8 with the first kh slots of every tree in shared memory
+  // ($TAHOE_DIRECT_HEADS slots per tree, capped by a 48 KB budget; < 2 slots => variant 5)
+  if ((variant == 8 || variant == 9) && scalar && !leaf) {
+    const int32_t rs = d | 1;
+    const char* khe = std::getenv("TAHOE_DIRECT_HEADS");
+    int32_t kh = khe ? std::atoi(khe) : 8;
+    while (kh > 1 && (int64_t)img.n_slots * kh * 8 > 49152) kh >>= 1;
+    if (kh >= 2) {
+      cudaError_t e;
+      if (variant == 8) e = fused ? direct_heads_one<true, 8, 64>(a, rs, kh, num_sms, st) : direct_heads_one<false, 8, 64>(a, rs, kh, num_sms, st);
+      else e = fused ? direct_heads_one<true, 8, 128>(a, rs, kh, num_sms, st) : direct_heads_one<false, 8, 128>(a, rs, kh, num_sms, st);
+      return (int)e;
+    }
+    variant = 5;
+  }
   if (variant >= 3 && variant <= 7 && scalar && !leaf) {
     const int32_t rs = d | 1;
     cudaError_t e;

@@ -122,9 +122,12 @@ template <class T>
 static tahoe_status upload(const std::vector<T>& v, const T** dst) {
   if (v.empty()) { *dst = nullptr; return TAHOE_OK; }
   void* p = nullptr;
-  cudaError_t e = cudaMalloc(&p, v.size() * sizeof(T));
+  // padded to 64 bytes (zeros), so kernels may load whole aligned node groups past the last node
+  const size_t bytes = v.size() * sizeof(T), padded = (bytes + 63) & ~(size_t)63;
+  cudaError_t e = cudaMalloc(&p, padded);
   if (e != cudaSuccess) return fail(TAHOE_E_NOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
-  e = cudaMemcpy(p, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+  if (padded > bytes) e = cudaMemset(static_cast<char*>(p) + bytes, 0, padded - bytes);
+  if (e == cudaSuccess) e = cudaMemcpy(p, v.data(), bytes, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) { cudaFree(p); return cuda_fail(e, "cudaMemcpy"); }
   *dst = static_cast<const T*>(p);
   return TAHOE_OK;

@@ -259,7 +259,11 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
 // Direct strategy, staged rows, P threads per row (scalar outputs, no leaf ids): thread j of a row
 // walks trees j, j+P, j+2P, ... free-running; the P partial sums are added in a fixed order
 // through shuffles.  P x more threads over the same staged rows hide more node-load latency.
-template <bool FUSED, int ROWS, int P>
+// GRP > 1: node loads fetch the aligned group of GRP slots (16 B or 32 B) holding the node into
+// registers, and the next node is taken from them when it lies in the same group (the hot child
+// sits in the next slot), so a walk down a hot chain costs one L1/L2 request per group
+// instead of one per node.  The device image is padded to 64 bytes (upload()).
+template <bool FUSED, int ROWS, int P, int GRP = 1>
 __global__ void __launch_bounds__(ROWS * P) k_direct_tlp(const DirectKArgs a, int32_t rs) {
   extern __shared__ __align__(16) float s_rows[];
   const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(a.img.nodes);
@@ -285,8 +289,27 @@ __global__ void __launch_bounds__(ROWS * P) k_direct_tlp(const DirectKArgs a, in
     if (active && j < T) {
       int32_t t = j;
       uint32_t k = (uint32_t)__ldg(&a.img.root[t]);
+      uint4 g0 = make_uint4(0u, 0u, 0u, 0u), g1 = g0;
+      uint32_t gbase = 0xffffffffu;
       for (;;) {
-        const uint2 nd = __ldg(&nodes[k]);
+        uint2 nd;
+        if constexpr (GRP == 1) {
+          nd = __ldg(&nodes[k]);
+        } else {
+          if ((k & ~(uint32_t)(GRP - 1)) != gbase) {
+            gbase = k & ~(uint32_t)(GRP - 1);
+            const uint4* gp = reinterpret_cast<const uint4*>(nodes + gbase);
+            g0 = __ldg(gp);
+            if constexpr (GRP == 4) g1 = __ldg(gp + 1);
+          }
+          const uint32_t w = k & (uint32_t)(GRP - 1);
+          if constexpr (GRP == 4) {
+            const uint4 g = (w & 2u) ? g1 : g0;
+            nd = (w & 1u) ? make_uint2(g.z, g.w) : make_uint2(g.x, g.y);
+          } else {
+            nd = w ? make_uint2(g0.z, g0.w) : make_uint2(g0.x, g0.y);
+          }
+        }
         if ((int32_t)nd.y < 0) {
           acc += (double)__uint_as_float(nd.x);
           t += P;
@@ -1303,10 +1326,10 @@ static cudaError_t direct_tiled_one(const DirectKArgs& a, int32_t rs, int32_t nu
   return cudaGetLastError();
 }
 
-template <bool F, int P, int kRows = 128>
+template <bool F, int P, int kRows = 128, int GRP = 1>
 static cudaError_t direct_tlp_one(const DirectKArgs& a, int32_t rs, int32_t num_sms,
                                   cudaStream_t st) {
-  auto kern = k_direct_tlp<F, kRows, P>;
+  auto kern = k_direct_tlp<F, kRows, P, GRP>;
   const int smem = kRows * rs * 4;
   static std::atomic<int> configured[64];
   int dev = 0;
@@ -1389,6 +1412,13 @@ int launch_direct(const DevDirect& img, const float* X, int64_t n, int32_t d, co
       return (int)e;
     }
     variant = 5;
+  }
+  if ((variant == 10 || variant == 11) && scalar && !leaf) {   // variant 5 over node groups
+    const int32_t rs = d | 1;
+    cudaError_t e;
+    if (variant == 10) e = fused ? direct_tlp_one<true, 8, 64, 4>(a, rs, num_sms, st) : direct_tlp_one<false, 8, 64, 4>(a, rs, num_sms, st);
+    else e = fused ? direct_tlp_one<true, 8, 64, 2>(a, rs, num_sms, st) : direct_tlp_one<false, 8, 64, 2>(a, rs, num_sms, st);
+    return (int)e;
   }
   if (variant >= 3 && variant <= 7 && scalar && !leaf) {
     const int32_t rs = d | 1;

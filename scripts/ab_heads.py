@@ -11,7 +11,8 @@ F = T.Forest(f, device=0)
 F.layout(gen.make_calibration(5, 16384))
 S = F.shard(0, 8)
 X = torch.from_numpy(gen.make_rows(5, n)).cuda()
-cases = [("5", None), ("8", "4"), ("8", "8"), ("8", "16"), ("9", "8"), ("9", "16"), ("5", None)]
+cases = [(v, None) for v in (sys.argv[2].split(",") if len(sys.argv) > 2 else ["5"])] if len(sys.argv) > 2 else \
+    [("5", None), ("8", "4"), ("8", "8"), ("8", "16"), ("9", "8"), ("9", "16"), ("5", None)]
 for name, H in ((f"shard0/8", S), ("full", F)):
     part = torch.empty((n, 1), dtype=torch.float64, device="cuda")
     ref = None

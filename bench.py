@@ -457,6 +457,7 @@ def main():
     kname = {1: "k_sliced", 2: "k_sliced_codes8" if stats.get("code8") else "k_sliced_codes"}.get(strategy, "k_direct")
     traffic = None
     sector_eff = None
+    path_sector_eff = None   # every LSU global load of the step (pre-pass + walk), same capture
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
@@ -465,6 +466,7 @@ def main():
             if rec.get("kernel", "").split("<")[0] == kname:
                 traffic = rec.get("dram_bytes_per_launch")
                 sector_eff = rec.get("global_ld_sector_efficiency")
+                path_sector_eff = rec.get("path_global_ld_sector_efficiency")
         except Exception:
             traffic = None
     launches_per_step = 1 if strategy == T.STRATEGY_DIRECT and F.n_out == 1 else (
@@ -482,6 +484,7 @@ def main():
                       achieved=achieved, peak=smem_peak, unit="GB/s", frac=achieved / smem_peak,
                       traffic=traffic, kernel_ms=kern_avg_ms,
                       global_ld_sector_efficiency=sector_eff,
+                      path_global_ld_sector_efficiency=path_sector_eff,
                       units_per_launch=f"{n} samples x {smem_bytes_per_sample:.0f} B "
                                        f"({visits:.0f} visits x 12 B + {cfg.n_trees} leaves x 8 B)",
                       peak_source=f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz"),

@@ -332,11 +332,13 @@ def test_direct_chunked_image_parity(monkeypatch):
 
 @pytest.mark.parametrize("cid,ntrees,variant", [(2, 120, None), (5, 60, None), (2, 120, "4"),
                                                 (5, 60, "2"), (5, 60, "1"), (5, 60, "3"),
-                                                (2, 120, "6"), (5, 60, "7")])
+                                                (2, 120, "6"), (5, 60, "7"), (5, 60, "8"),
+                                                (2, 120, "9"), (5, 60, "10"), (2, 120, "11")])
 def test_direct_large_batch_variants(cid, ntrees, variant, monkeypatch):
     """Large-batch direct kernels (staged rows; 2, 4, 8 (default) or 16 threads per row for scalar
-    outputs, one thread per row free-running or warp-lockstep) against the oracle, scores and classes
-    bit-exact with dyadic leaves, >= 32K rows with a ragged last tile."""
+    outputs, one thread per row free-running or warp-lockstep; the measured-and-rejected tree-head
+    (8, 9) and node-group (10, 11) experiments) against the oracle, scores and classes bit-exact with
+    dyadic leaves, >= 32K rows with a ragged last tile."""
     if variant is not None:
         monkeypatch.setenv("TAHOE_DIRECT_VARIANT", variant)
     f = gen.make_forest(cid, n_trees=ntrees)

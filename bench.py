@@ -223,7 +223,8 @@ def run_tree_sharded(args, cfg):
     full = T.Forest(f, device=-1).layout(gen.make_calibration(cfg))
     S = full.shard(rank, world, device=local)
     layout_s = time.perf_counter() - t0
-    Xd = torch.from_numpy(gen.make_rows(cfg, cfg.n_samples)).to(dev).repeat(reps, 1)
+    Xh = gen.make_rows(cfg, cfg.n_samples)
+    Xd = torch.from_numpy(Xh).to(dev).repeat(reps, 1)
     stream = torch.cuda.current_stream()
     fused = args.reduce == "fused"
     if fused:
@@ -263,8 +264,57 @@ def run_tree_sharded(args, cfg):
     ms = sum(a.elapsed_time(b) for a, b in ev) / args.steps
     if world > 1:
         ms = D.max_over_ranks(ms, device=dev)
+    # end to end through the public API with pinned HOST buffers (one GPU: the whole forest on
+    # this rank, tahoe_predict_host: chunked H2D of the rows / traversal / D2H of the outputs)
+    e2e = None
+    if world == 1 and not args.weak:
+        Xp = torch.from_numpy(Xh).pin_memory()
+        oh = torch.empty((n, S.n_out), dtype=torch.float32).pin_memory()
+        S.predict_host(Xp, oh)
+        torch.cuda.synchronize()
+        e2e_ms = []
+        for _ in range(max(2, min(args.steps, 3))):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            S.predict_host(Xp, oh)
+            b.record(stream)
+            torch.cuda.synchronize()
+            e2e_ms.append(a.elapsed_time(b))
+        e2e = dict(value=n / (sum(e2e_ms) / len(e2e_ms) / 1000.0), unit=UNIT,
+                   h2d_bytes_per_step=int(Xp.numel() * 4), d2h_bytes_per_step=int(oh.numel() * 4))
+        del Xp, oh
     if rank == 0:
         st = S.stats()
+        # the oracle (as it stands) on a bounded sample of the same rows and the FULL forest
+        cpu = None
+        visits = st["expected_visits_per_sample"]   # this rank's shard, calibration estimate
+        if not args.no_cpu and world == 1:
+            import oracle
+            rate, rows, secs, vis = oracle_rate(f, Xh, 12.0, 200_000)
+            cpu = dict(value=rate, unit=UNIT, cores=oracle.n_threads(), kind="oracle",
+                       sample=f"{rows} seeded rows of this workload, full {cfg.n_trees}-tree forest "
+                              f"({secs:.1f} s of oracle work)")
+            visits = vis
+        # roofline of the traversal (k_direct_tlp over the L2-sized chunks of the shard's image):
+        # algorithmic bytes per sample = node visits x (8 B node + 4 B attribute) + leaves x 8 B,
+        # against the L1 / shared-memory data pipe the node and attribute loads go through
+        # (128 B/clk/SM, the same unit and peak as the sliced kernels' roofline); the time is the
+        # whole step (traversal launches + the reduce/finalize kernel, < 1 % of it)
+        peaks = _peaks()
+        n_sms = st["num_sms"]
+        pipe_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
+        bytes_per_sample = visits * 12.0 + st["n_trees"] * 8.0
+        achieved = n * bytes_per_sample / (ms / 1000.0) / 1e9
+        roofline = dict(bound="alu", pipe="L1/shared-memory LSU data pipe, 128 B/clk/SM (DESIGN.md Roofline)",
+                        kernel="k_direct_tlp", achieved=achieved, peak=pipe_peak, unit="GB/s",
+                        frac=achieved / pipe_peak, traffic=None, kernel_ms=ms,
+                        units_per_launch=f"{n} samples x {bytes_per_sample:.0f} B ({visits:.0f} visits x 12 B"
+                                         f" + {st['n_trees']} leaves x 8 B) per step",
+                        peak_source=f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz")
+        hbm_bytes = n * (cfg.n_features * 4) + (hi - lo if fused else n) * 4
+        hbm = dict(achieved=hbm_bytes / (ms / 1000.0) / 1e9, peak=peaks["hbm_gbs"], unit="GB/s",
+                   frac=hbm_bytes / (ms / 1000.0) / 1e9 / peaks["hbm_gbs"], bytes_per_step=hbm_bytes,
+                   peak_source=peaks["source"])
         line = dict(metric=METRIC, value=n / (ms / 1000.0), unit=UNIT, n_gpus=world, steps=args.steps,
                     warmup=args.warmup, ms_per_step=ms, higher_is_better=True,
                     scaling="weak" if args.weak else "strong",
@@ -280,7 +330,7 @@ def run_tree_sharded(args, cfg):
                             "n": n, "trees_per_shard": st["n_trees"],
                             "parallelism": f"tree-sharded x{world}",
                             "reduce": "fused (NCCL device API, LSA)" if fused else "ncclReduce"},
-                    strategy="direct", roofline=None, cpu_baseline=None, e2e=None,
+                    strategy="direct", roofline=roofline, hbm=hbm, cpu_baseline=cpu, e2e=e2e,
                     gpu_launches=(2 if (fused or rank == 0) else 1) * args.steps, clocks=clocks,
                     layout_s=layout_s)
         print(json.dumps(line), flush=True)

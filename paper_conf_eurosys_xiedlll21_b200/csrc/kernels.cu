@@ -829,6 +829,13 @@ __device__ __forceinline__ uint32_t code_row_off(int r, int rb) {
   return rb == 64 ? (((uint32_t)(r & 15) << 7) | ((uint32_t)((r >> 4) & 1) << 6) | ((uint32_t)(r >> 5) << 11))
                   : (uint32_t)r * (uint32_t)rb;
 }
+// Rows of >= 128 bytes: the rows walked by the second half-warp (r & 16) store attribute slot j at
+// slot j ^ 32 (their 64-byte halves swapped), so the low, most-tested attributes of the two rows
+// one warp reads at once sit in different banks (C3 ncu before: 25 % of shared wavefronts were
+// bank-conflict replays between the two half-warps' rows).  Returned in u16 slots.
+__device__ __forceinline__ uint32_t code_slot_swz(int r, int rb) {
+  return (rb >= 128 && (r & 16)) ? 32u : 0u;
+}
 
 template <bool SMEM>
 __global__ void __launch_bounds__(1024) k_encode_rows(const EncodeRowsArgs a) {
@@ -868,7 +875,7 @@ __global__ void __launch_bounds__(1024) k_encode_rows(const EncodeRowsArgs a) {
         code = (uint16_t)(lo - b0);
       }
     }
-    a.codes[(r >> 6) * tile_u16 + (code_row_off((int)(r & 63), a.rb) >> 1) + j] = code;
+    a.codes[(r >> 6) * tile_u16 + (code_row_off((int)(r & 63), a.rb) >> 1) + (j ^ code_slot_swz((int)(r & 63), a.rb))] = code;
   }
 }
 
@@ -972,7 +979,7 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
         // the kR rows r0 .. r0+kR-1 of a group (r0 % kR == 0) sit at a constant stride in the
         // tile: 128 bytes apart in the 64-byte-row layout (same bits 4-5 of r), rb otherwise
         uint16_t* tb = a.codes + (r0 >> 6) * tile_u16;
-        uint16_t* p0 = tb + (code_row_off((int)(r0 & 63), rb) >> 1) + slot;
+        uint16_t* p0 = tb + (code_row_off((int)(r0 & 63), rb) >> 1) + (slot ^ code_slot_swz((int)(r0 & 63), rb));
         const int rstride = RB64 ? 64 : (rb >> 1);
         bool nan = false;
         if (feat >= 0 && r0 + kR <= a.n) {
@@ -1020,7 +1027,7 @@ __device__ __forceinline__ float coded_step(uint32_t& p, uint32_t rowaddr, uint3
   uint32_t x, y;
   int32_t c;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
-  asm("ld.shared.s16 %0, [%1];" : "=r"(c) : "r"((y & amask) | rowaddr));
+  asm("ld.shared.s16 %0, [%1];" : "=r"(c) : "r"((y & amask) ^ rowaddr));   // rowaddr carries the swizzle
   bool go_left = (uint32_t)c < x;
   if (NAN_AWARE) go_left = go_left || ((c == (int32_t)(int16_t)kCodeNan) && (y & dlbit));
   p += go_left ? (uint32_t)kSlotBytes : __umulhi(y, shmul);
@@ -1186,8 +1193,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         const bool okA = rA < nr, okB = rB < nr;
         const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
         const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tstride;
-        const uint32_t rowA = tb + code_row_off(okA ? rA : u, a.rb);
-        const uint32_t rowB = tb + code_row_off(okB ? rB : u, a.rb);
+        // row base | swizzle (code_slot_swz in bytes): the attribute offset is XORed into it
+        const int qA = okA ? rA : u, qB = okB ? rB : u;
+        const uint32_t rowA = (tb + code_row_off(qA, a.rb)) | (code_slot_swz(qA, a.rb) << 1);
+        const uint32_t rowB = (tb + code_row_off(qB, a.rb)) | (code_slot_swz(qB, a.rb) << 1);
         uint32_t nan_flag;
         asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(tb + (uint32_t)a.tile_bytes));
         double accA, accB;

@@ -1021,13 +1021,14 @@ struct CodedKArgs {
 // One step on a coded slice: node {x = t or leaf value, y}, attribute code at (y & amask) | row,
 // left iff code < t (NaN-aware: or NaN and default-left), right / next root at +(y >> (F+2)).
 // Returns the node word as a float: the leaf value, or a subnormal (flushed to 0 by the add).
-template <bool NAN_AWARE>
+template <bool NAN_AWARE, bool SWZ>
 __device__ __forceinline__ float coded_step(uint32_t& p, uint32_t rowaddr, uint32_t amask,
                                             uint32_t dlbit, uint32_t shmul) {
   uint32_t x, y;
   int32_t c;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
-  asm("ld.shared.s16 %0, [%1];" : "=r"(c) : "r"((y & amask) ^ rowaddr));   // rowaddr carries the swizzle
+  // SWZ: rowaddr carries the swizzle (code_slot_swz), XORed into the attribute offset
+  asm("ld.shared.s16 %0, [%1];" : "=r"(c) : "r"(SWZ ? ((y & amask) ^ rowaddr) : ((y & amask) | rowaddr)));
   bool go_left = (uint32_t)c < x;
   if (NAN_AWARE) go_left = go_left || ((c == (int32_t)(int16_t)kCodeNan) && (y & dlbit));
   p += go_left ? (uint32_t)kSlotBytes : __umulhi(y, shmul);
@@ -1044,17 +1045,17 @@ __device__ __forceinline__ void add_pair_ftz(double& acc, float v1, float v2) {
   acc += dv;
 }
 
-template <bool NAN_AWARE>
+template <bool NAN_AWARE, bool SWZ>
 __device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t pe, uint32_t rowA,
                                             uint32_t rowB, uint32_t amask, uint32_t dlbit,
                                             uint32_t shmul, double& accA, double& accB) {
   accA = 0.0;
   accB = 0.0;
   while ((pA != pe) | (pB != pe)) {
-    const float a1 = coded_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul);
-    const float b1 = coded_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul);
-    const float a2 = coded_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul);
-    const float b2 = coded_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul);
+    const float a1 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+    const float b1 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+    const float a2 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+    const float b2 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
     add_pair_ftz(accA, a1, a2);
     add_pair_ftz(accB, b1, b2);
   }
@@ -1063,7 +1064,7 @@ __device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t p
 // k_sliced_codes: k_sliced's persistent slice-stationary schedule (slice in shared memory, 3-deep
 // ring of 64-row tiles refilled by the warp that finishes a tile, dynamic 4-row work units, one
 // half-warp per row, two chains per lane) over code tiles (one 1-D bulk copy per tile).
-template <bool FUSED>
+template <bool FUSED, bool SWZ>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant__ CodedKArgs a) {
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
@@ -1195,15 +1196,17 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tstride;
         // row base | swizzle (code_slot_swz in bytes): the attribute offset is XORed into it
         const int qA = okA ? rA : u, qB = okB ? rB : u;
-        const uint32_t rowA = (tb + code_row_off(qA, a.rb)) | (code_slot_swz(qA, a.rb) << 1);
-        const uint32_t rowB = (tb + code_row_off(qB, a.rb)) | (code_slot_swz(qB, a.rb) << 1);
+        const uint32_t rowA = SWZ ? (tb + code_row_off(qA, a.rb)) | (code_slot_swz(qA, a.rb) << 1)
+                                  : tb + code_row_off(qA, a.rb);
+        const uint32_t rowB = SWZ ? (tb + code_row_off(qB, a.rb)) | (code_slot_swz(qB, a.rb) << 1)
+                                  : tb + code_row_off(qB, a.rb);
         uint32_t nan_flag;
         asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(tb + (uint32_t)a.tile_bytes));
         double accA, accB;
         if (nan_flag)
-          walk_coded2<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          walk_coded2<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
         else
-          walk_coded2<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          walk_coded2<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
         // a9: the k_sliced butterfly (lanes 0, 8, 16, 24 own rows u, u+32, u+16, u+48)
         const bool b3 = lane & 8;
         double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
@@ -1633,16 +1636,19 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   a.o = o;
   const int smem = plan.forest_smem + kRing * tstride + kSlicedBarrierBytes +
                    kRing * kSlicedTileRows * (int)sizeof(double);
-  auto kern = fused ? k_sliced_codes<true> : k_sliced_codes<false>;
+  // rows of >= 128 bytes are stored swizzled (code_slot_swz); the others keep the plain walk
+  auto kern = a.rb >= 128 ? (fused ? k_sliced_codes<true, true> : k_sliced_codes<false, true>)
+                          : (fused ? k_sliced_codes<true, false> : k_sliced_codes<false, false>);
   {
     static std::atomic<int> configured[64];
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
-      e = cudaFuncSetAttribute(k_sliced_codes<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
-      if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sliced_codes<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
-      if (e != cudaSuccess) return (int)e;
+      for (auto k : {k_sliced_codes<true, false>, k_sliced_codes<false, false>,
+                     k_sliced_codes<true, true>, k_sliced_codes<false, true>}) {
+        e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+        if (e != cudaSuccess) return (int)e;
+      }
       configured[dev].store(1);
     }
   }

@@ -355,11 +355,6 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       strat = TAHOE_STRATEGY_SLICED;
     }
   }
-  if (strat == TAHOE_STRATEGY_SLICED_CODED && (out_leaf || out_fp)) {
-    if (forced == TAHOE_STRATEGY_SLICED_CODED)
-      return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices produce no leaf ids / fingerprints");
-    strat = TAHOE_STRATEGY_SLICED;   // leaf diagnostics run on the fp32 slices
-  }
   cudaError_t e;
   if (out_fp && (e = cudaMemsetAsync(out_fp, 0, (size_t)n * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
   OutArgs o;
@@ -408,7 +403,10 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       rc = launch_direct(dc, X, n, d, o, false, f->num_sms, st);
     }
     if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
-    if (rc) return cuda_fail((cudaError_t)rc, "direct kernel");
+    if (rc) {
+      if (!raw_user) cudaFreeAsync(raw, st);
+      return cuda_fail((cudaError_t)rc, "direct kernel");
+    }
     if (!raw_user) {
       fa.partial = raw;
       fa.part_stride = 1;

@@ -70,6 +70,22 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
       "r"(phase), "r"(20000u)
       : "memory");
 }
+// Ring tickets (ring-wrap guard): s_gen[b] holds the CTA-wide sequence number of the tile last
+// issued into ring buffer b.  A warp that claimed a unit of tile sequence `seq` first waits until
+// the buffer's ticket names seq and only then waits on the buffer's mbarrier phase, so it never
+// waits on a parity that matches a phase two fills behind (a unit of tile seq + 2 * ring could
+// otherwise be claimed while tile seq's refill is still pending, and its parity wait would return
+// at once on the old data).
+__device__ __forceinline__ void wait_ticket(const uint32_t* gen, uint32_t seq, int lane) {
+  if (lane == 0)
+    while (*reinterpret_cast<const volatile uint32_t*>(gen) != seq) {
+    }
+  __syncwarp();
+}
+__device__ __forceinline__ void set_ticket(uint32_t* gen, uint32_t seq) {
+  __threadfence_block();
+  *reinterpret_cast<volatile uint32_t*>(gen) = seq;
+}
 // issue a (possibly > 64 KB) bulk copy in 64 KB pieces on one barrier; caller did expect_tx(total)
 __device__ __forceinline__ void bulk_g2s_big(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   const uint32_t kPiece = 65536;
@@ -586,6 +602,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   uint64_t* s_forest = s_full + kRing;
   int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
   unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
+  uint32_t* s_gen = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(s_full) + 72);  // [kRing] tickets
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int nwarps = blockDim.x >> 5;
@@ -606,15 +623,16 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   if (threadIdx.x == 0) {
     // full barriers: one arrive.expect_tx per TMA fill, or 32 cp.async arrivals (misaligned X)
     const uint32_t arrivals = (ROWS == kRowsDense && !a.x_aligned) ? 32u : 1u;
-    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], arrivals); s_cnt[b] = 0; }
+    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], arrivals); s_cnt[b] = 0; s_gen[b] = 0xffffffffu; }
     *s_next = 0ull;
     mbar_init(s_forest, 1);
     fence_mbar_init();
   }
   __syncthreads();
 
-  // a6: stage tile `tile` into ring buffer b; called by one whole warp
-  auto issue_tile = [&](int64_t tile, int b) {
+  // a6: stage tile `tile` (CTA-wide tile sequence number seq) into ring buffer b; called by one
+  // whole warp
+  auto issue_tile = [&](int64_t tile, int b, uint32_t seq) {
     const int64_t r0 = tile * R;
     float* dst = s_ring + (size_t)b * a.buf_floats;
     if (PADDED) {
@@ -653,11 +671,14 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
       }
     }
     __syncwarp();
+    if (lane == 0) set_ticket(&s_gen[b], seq);
+    __syncwarp();
   };
 
   // release ring buffer b after one work unit; the warp finishing the tile's last unit refills it
   // with the tile kRing ahead (acquire fence after observing the counter)
-  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts) {
+  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts,
+                     uint32_t seq) {   // seq: the tile sequence number of the released tile
     __syncwarp();
     int last = 0;
     if (lane == 0) {
@@ -666,7 +687,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
       if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
     }
     last = __shfl_sync(0xffffffffu, last, 0);
-    if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b);
+    if (last && it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b, seq + (uint32_t)kRing);
   };
 
   uint32_t g = 0;  // tiles this CTA has consumed so far (identical in every warp)
@@ -684,7 +705,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         bulk_g2s_big(smem, a.img.nodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
       if (ROWS_SMEM)
-        for (int64_t q = 0; q < kRing && q < my_tiles; q++) issue_tile(t0 + q * ts, (int)((g + q) % kRing));
+        for (int64_t q = 0; q < kRing && q < my_tiles; q++)
+          issue_tile(t0 + q * ts, (int)((g + q) % kRing), g + (uint32_t)q);
     }
     const uint32_t sbase = smem_u32(smem);
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
@@ -696,9 +718,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
     if (!LEAF) {
       // Dynamic schedule over work units of 4 rows {u, u+16, u+32, u+48} of a 64-row tile: half h
       // of the warp walks rows u+16h (chain A) and u+32+16h (chain B).  Warps grab units from a CTA
-      // counter, so a slow unit delays nobody; at most 32 units are in flight, so no warp can run
-      // a full ring ahead of a buffer's refill.  Rows too wide to stage are read from global memory
-      // with the same schedule.
+      // counter, so a slow unit delays nobody.  Claims are not bounded by the ring: while one slow
+      // unit holds tile T, other warps may finish T+1, T+2, T+4, T+5 and claim T+6 (buffer and
+      // parity of T), so a claim waits for the buffer's ticket before its mbarrier phase
+      // (wait_ticket).  Rows too wide to stage are read from global memory with the same schedule.
       constexpr int kUnits = kSlicedTileRows / 4;
       const uint64_t total = (uint64_t)my_tiles * kUnits;
       for (;;) {
@@ -712,7 +735,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         const int b = (int)(gt % kRing);
         const int64_t r0 = (t0 + it * ts) * R;
         const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-        if (ROWS_SMEM) mbar_wait(&s_full[b], (gt / kRing) & 1u);
+        if (ROWS_SMEM) {
+          wait_ticket(&s_gen[b], gt, lane);
+          mbar_wait(&s_full[b], (gt / kRing) & 1u);
+        }
         if (u < nr) {
           const int rA = u + 16 * half, rB = rA + 32;
           const bool okA = rA < nr, okB = rB < nr;
@@ -746,7 +772,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
             else a.o.raw[(size_t)sl * a.n + i] = v;
           }
         }
-        if (ROWS_SMEM) release(b, kUnits, it, my_tiles, t0, ts);
+        if (ROWS_SMEM) release(b, kUnits, it, my_tiles, t0, ts, gt);
       }
       g += (uint32_t)my_tiles;
     } else {
@@ -792,7 +818,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
               atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[i]), (unsigned long long)fp);
           }
         }
-        if (ROWS_SMEM) release(b, nwarps, it, my_tiles, t0, ts);
+        if (ROWS_SMEM) release(b, nwarps, it, my_tiles, t0, ts, g);
       }
     }
     __syncthreads();  // every warp is done with this slice (multi-pass reload)
@@ -1021,12 +1047,15 @@ struct CodedKArgs {
 // One step on a coded slice: node {x = t or leaf value, y}, attribute code at (y & amask) | row,
 // left iff code < t (NaN-aware: or NaN and default-left), right / next root at +(y >> (F+2)).
 // Returns the node word as a float: the leaf value, or a subnormal (flushed to 0 by the add).
+// yout (diagnostic walks only): receives the node word's y, so the caller can tell a leaf.
 template <bool NAN_AWARE, bool SWZ>
 __device__ __forceinline__ float coded_step(uint32_t& p, uint32_t rowaddr, uint32_t amask,
-                                            uint32_t dlbit, uint32_t shmul) {
+                                            uint32_t dlbit, uint32_t shmul,
+                                            uint32_t* yout = nullptr) {
   uint32_t x, y;
   int32_t c;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+  if (yout) *yout = y;
   // SWZ: rowaddr carries the swizzle (code_slot_swz), XORed into the attribute offset
   asm("ld.shared.s16 %0, [%1];" : "=r"(c) : "r"(SWZ ? ((y & amask) ^ rowaddr) : ((y & amask) | rowaddr)));
   bool go_left = (uint32_t)c < x;
@@ -1061,10 +1090,54 @@ __device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t p
   }
 }
 
+// Leaf diagnostics of a coded walk (per-(sample, tree) leaf ids, fingerprint): the node word just
+// read at q was a leaf iff its attribute field is all ones (the pad code) and q is not the
+// column's terminal self-loop pe; its caller {tree, node} ids sit in leaf_meta at the same word
+// index as in the slice.
+__device__ __forceinline__ void record_leaf(uint32_t q, uint32_t y, uint32_t pe, uint32_t amask,
+                                            uint32_t sbase, const int2* __restrict__ meta,
+                                            int32_t* out_row, uint64_t& fp) {
+  if ((y & amask) == amask && q != pe) {
+    const int2 m = __ldg(&meta[(q - sbase) >> 3]);
+    if (out_row) out_row[m.x] = m.y;
+    fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
+  }
+}
+
+// walk_coded2 with the leaf diagnostics: the same steps in the same order and the same fp32 / fp64
+// additions; after every step the node just read is checked for a leaf.
+template <bool NAN_AWARE, bool SWZ>
+__device__ __forceinline__ void walk_coded2_leaf(uint32_t pA, uint32_t pB, uint32_t pe,
+                                                 uint32_t rowA, uint32_t rowB, uint32_t amask,
+                                                 uint32_t dlbit, uint32_t shmul, double& accA,
+                                                 double& accB, uint32_t sbase,
+                                                 const int2* __restrict__ meta, int32_t* outA,
+                                                 int32_t* outB, uint64_t& fpA, uint64_t& fpB) {
+  accA = 0.0;
+  accB = 0.0;
+  fpA = 0;
+  fpB = 0;
+  while ((pA != pe) | (pB != pe)) {
+    uint32_t y, q;
+    q = pA; const float a1 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outA, fpA);
+    q = pB; const float b1 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outB, fpB);
+    q = pA; const float a2 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outA, fpA);
+    q = pB; const float b2 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outB, fpB);
+    add_pair_ftz(accA, a1, a2);
+    add_pair_ftz(accB, b1, b2);
+  }
+}
+
 // k_sliced_codes: k_sliced's persistent slice-stationary schedule (slice in shared memory, 3-deep
 // ring of 64-row tiles refilled by the warp that finishes a tile, dynamic 4-row work units, one
 // half-warp per row, two chains per lane) over code tiles (one 1-D bulk copy per tile).
-template <bool FUSED, bool SWZ>
+// LEAF: the same schedule and walk, also writing per-(sample, tree) caller leaf ids (out_leaf, may
+// be null) and accumulating fingerprints (out_fp, u64 atomic adds per slice).
+template <bool FUSED, bool SWZ, bool LEAF>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant__ CodedKArgs a) {
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
@@ -1073,6 +1146,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   uint64_t* s_forest = s_full + kRing;
   int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
   unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
+  uint32_t* s_gen = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(s_full) + 72);  // [kRing] tickets
   // slice partials of the tiles in the ring, written out coalesced by the warp closing a tile
   double* s_part = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_full) + kSlicedBarrierBytes);
   const int lane = threadIdx.x & 31;
@@ -1090,14 +1164,15 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   const int64_t ntiles = (a.n + R - 1) / R;
 
   if (threadIdx.x == 0) {
-    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; }
+    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; s_gen[b] = 0xffffffffu; }
     *s_next = 0ull;
     mbar_init(s_forest, 1);
     fence_mbar_init();
   }
   __syncthreads();
 
-  auto issue_tile = [&](int64_t tile, int b, int64_t ahead = -1) {
+  // stage tile `tile` (CTA-wide sequence number seq) into buffer b, then publish the ticket
+  auto issue_tile = [&](int64_t tile, int b, uint32_t seq, int64_t ahead = -1) {
     if (lane == 0) {
       // optional L2 prefetch of this CTA's tile `ahead` (a later tile of its sequence)
       if (ahead >= 0 && ahead < ntiles)
@@ -1108,13 +1183,14 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
       bulk_g2s(s_ring + (size_t)b * a.tstride,
                reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride,
                (uint32_t)a.tstride, &s_full[b]);
+      set_ticket(&s_gen[b], seq);
     }
     __syncwarp();
   };
   // after one work unit: the warp finishing the tile's last unit writes the tile's 64 slice
   // partials (two coalesced 256-byte stores) and refills the buffer with the tile kRing ahead
   auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts,
-                     int sl, int64_t r0, int nr) {
+                     int sl, int64_t r0, int nr, uint32_t seq) {
     __syncwarp();
     int last = 0;
     if (lane == 0) {
@@ -1125,7 +1201,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     last = __shfl_sync(0xffffffffu, last, 0);
     if (!last) return;
     if (FUSED) {
-      if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
+      if (it + kRing < my_tiles)
+        issue_tile(t0 + (it + kRing) * ts, b, seq + (uint32_t)kRing, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
       return;
     }
     // take the tile's 64 partials out of shared memory, refill the buffer at once, then store the
@@ -1135,7 +1212,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     const double* sp = s_part + b * kSlicedTileRows;
     const double p0 = lane < nr ? sp[lane] : 0.0, p1 = lane + 32 < nr ? sp[lane + 32] : 0.0;
     __syncwarp();
-    if (it + kRing < my_tiles) issue_tile(t0 + (it + kRing) * ts, b, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
+    if (it + kRing < my_tiles)
+      issue_tile(t0 + (it + kRing) * ts, b, seq + (uint32_t)kRing, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
     double* dst = a.o.raw + (size_t)sl * a.n + r0;
     if (lane < nr) dst[lane] = p0;
     if (lane + 32 < nr) dst[lane + 32] = p1;
@@ -1166,11 +1244,14 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         mbar_expect_tx(s_forest, bytes);
         bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
-      for (int64_t q = 0; q < kRing && q < my_tiles; q++) issue_tile(t0 + q * ts, (int)((g + q) % kRing));
+      for (int64_t q = 0; q < kRing && q < my_tiles; q++)
+        issue_tile(t0 + q * ts, (int)((g + q) % kRing), g + (uint32_t)q);
     }
     const uint32_t sbase = smem_u32(smem);
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
     const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+    const int2* __restrict__ meta =
+        LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
     mbar_wait(s_forest, ph_forest);
     ph_forest ^= 1u;
 
@@ -1188,6 +1269,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
       const int64_t tile = t0 + it * ts;
       const int64_t r0 = tile * R;
       const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+      wait_ticket(&s_gen[b], gt, lane);
       mbar_wait(&s_full[b], (gt / kRing) & 1u);
       if (u < nr) {
         const int rA = u + 16 * half, rB = rA + 32;
@@ -1203,22 +1285,39 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         uint32_t nan_flag;
         asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(tb + (uint32_t)a.tile_bytes));
         double accA, accB;
-        if (nan_flag)
+        uint64_t fpA = 0, fpB = 0;
+        if (LEAF) {
+          int32_t* oA = (a.o.out_leaf && okA) ? a.o.out_leaf + (r0 + rA) * (int64_t)a.o.T_leaf : nullptr;
+          int32_t* oB = (a.o.out_leaf && okB) ? a.o.out_leaf + (r0 + rB) * (int64_t)a.o.T_leaf : nullptr;
+          if (nan_flag)
+            walk_coded2_leaf<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+          else
+            walk_coded2_leaf<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+        } else if (nan_flag) {
           walk_coded2<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-        else
+        } else {
           walk_coded2<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+        }
         // a9: the k_sliced butterfly (lanes 0, 8, 16, 24 own rows u, u+32, u+16, u+48)
         const bool b3 = lane & 8;
         double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
 #pragma unroll
         for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        uint64_t fv = 0;
+        if (LEAF) {
+          fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
+#pragma unroll
+          for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
+        }
         const int rr = b3 ? rB : rA;
         if ((lane & 7) == 0 && (b3 ? okB : okA)) {
           if (FUSED) write_scalar(a.o, r0 + rr, v);
           else s_part[b * kSlicedTileRows + rr] = v;
+          if (LEAF && a.o.out_fp)
+            atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[r0 + rr]), (unsigned long long)fv);
         }
       }
-      release(b, kUnits, it, my_tiles, t0, ts, sl, r0, nr);
+      release(b, kUnits, it, my_tiles, t0, ts, sl, r0, nr, gt);
     }
     g += (uint32_t)my_tiles;
     __syncthreads();
@@ -1636,16 +1735,22 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   a.o = o;
   const int smem = plan.forest_smem + kRing * tstride + kSlicedBarrierBytes +
                    kRing * kSlicedTileRows * (int)sizeof(double);
-  // rows of >= 128 bytes are stored swizzled (code_slot_swz); the others keep the plain walk
-  auto kern = a.rb >= 128 ? (fused ? k_sliced_codes<true, true> : k_sliced_codes<false, true>)
-                          : (fused ? k_sliced_codes<true, false> : k_sliced_codes<false, false>);
+  // rows of >= 128 bytes are stored swizzled (code_slot_swz); the others keep the plain walk;
+  // leaf ids / fingerprints take the LEAF instantiation of the same walk
+  const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
+  auto kern = leaf ? (a.rb >= 128 ? (fused ? k_sliced_codes<true, true, true> : k_sliced_codes<false, true, true>)
+                                  : (fused ? k_sliced_codes<true, false, true> : k_sliced_codes<false, false, true>))
+                   : (a.rb >= 128 ? (fused ? k_sliced_codes<true, true, false> : k_sliced_codes<false, true, false>)
+                                  : (fused ? k_sliced_codes<true, false, false> : k_sliced_codes<false, false, false>));
   {
     static std::atomic<int> configured[64];
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
-      for (auto k : {k_sliced_codes<true, false>, k_sliced_codes<false, false>,
-                     k_sliced_codes<true, true>, k_sliced_codes<false, true>}) {
+      for (auto k : {k_sliced_codes<true, false, false>, k_sliced_codes<false, false, false>,
+                     k_sliced_codes<true, true, false>, k_sliced_codes<false, true, false>,
+                     k_sliced_codes<true, false, true>, k_sliced_codes<false, false, true>,
+                     k_sliced_codes<true, true, true>, k_sliced_codes<false, true, true>}) {
         e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
         if (e != cudaSuccess) return (int)e;
       }
@@ -1803,10 +1908,12 @@ struct Coded8KArgs {
 // left iff code < t (NaN-aware: or NaN and default-left), right / next root at +(y >> (V+1)).
 template <bool NAN_AWARE>
 __device__ __forceinline__ float coded8_step(uint32_t& p, uint32_t rowaddr, uint32_t amask,
-                                             uint32_t dlbit, uint32_t shmul) {
+                                             uint32_t dlbit, uint32_t shmul,
+                                             uint32_t* yout = nullptr) {
   uint32_t x, y;
   int32_t c;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
+  if (yout) *yout = y;
   asm("ld.shared.s8 %0, [%1];" : "=r"(c) : "r"((y & amask) | rowaddr));
   bool go_left = (uint32_t)c < x;
   if (NAN_AWARE) go_left = go_left || ((c == (int32_t)kCode8Nan) && (y & dlbit));
@@ -1860,6 +1967,73 @@ __device__ __forceinline__ void walk_coded8_split(uint32_t pA1, uint32_t mA, uin
   accB = b1 + b2;
 }
 
+// Leaf-diagnostic twins of the two wide-code walks (same steps, same order, same additions; the
+// node read before each step is checked for a leaf, record_leaf).  A first-half chain frozen at its
+// split slot re-reads a tree root, which is never a leaf.
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_coded8_leaf(uint32_t pA, uint32_t pB, uint32_t pe, uint32_t rowA,
+                                                 uint32_t rowB, uint32_t amask, uint32_t dlbit,
+                                                 uint32_t shmul, double& accA, double& accB,
+                                                 uint32_t sbase, const int2* __restrict__ meta,
+                                                 int32_t* outA, int32_t* outB, uint64_t& fpA,
+                                                 uint64_t& fpB) {
+  accA = 0.0;
+  accB = 0.0;
+  fpA = 0;
+  fpB = 0;
+  while ((pA != pe) | (pB != pe)) {
+    uint32_t y, q;
+    q = pA; const float a1 = coded8_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outA, fpA);
+    q = pB; const float b1 = coded8_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outB, fpB);
+    q = pA; const float a2 = coded8_step<NAN_AWARE>(pA, rowA, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outA, fpA);
+    q = pB; const float b2 = coded8_step<NAN_AWARE>(pB, rowB, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outB, fpB);
+    add_pair_ftz(accA, a1, a2);
+    add_pair_ftz(accB, b1, b2);
+  }
+}
+
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA, uint32_t pA2, uint32_t pB1,
+                                                       uint32_t mB, uint32_t pB2, uint32_t pe,
+                                                       uint32_t rowA, uint32_t rowB, uint32_t amask,
+                                                       uint32_t dlbit, uint32_t shmul, double& accA,
+                                                       double& accB, uint32_t sbase,
+                                                       const int2* __restrict__ meta, int32_t* outA,
+                                                       int32_t* outB, uint64_t& fpA, uint64_t& fpB) {
+  double a1 = 0.0, a2 = 0.0, b1 = 0.0, b2 = 0.0;
+  fpA = 0;
+  fpB = 0;
+  while ((pA1 != mA) | (pA2 != pe) | (pB1 != mB) | (pB2 != pe)) {
+    uint32_t q, y;
+    q = pA1; const float x1 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul, &y);
+    record_leaf(pA1, y, pe, amask, sbase, meta, outA, fpA); pA1 = pA1 == mA ? pA1 : q;
+    q = pB1; const float y1 = coded8_step<NAN_AWARE>(q, rowB, amask, dlbit, shmul, &y);
+    record_leaf(pB1, y, pe, amask, sbase, meta, outB, fpB); pB1 = pB1 == mB ? pB1 : q;
+    q = pA2; const float x3 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outA, fpA);
+    q = pB2; const float y3 = coded8_step<NAN_AWARE>(pB2, rowB, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outB, fpB);
+    q = pA1; const float x2 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul, &y);
+    record_leaf(pA1, y, pe, amask, sbase, meta, outA, fpA); pA1 = pA1 == mA ? pA1 : q;
+    q = pB1; const float y2 = coded8_step<NAN_AWARE>(q, rowB, amask, dlbit, shmul, &y);
+    record_leaf(pB1, y, pe, amask, sbase, meta, outB, fpB); pB1 = pB1 == mB ? pB1 : q;
+    q = pA2; const float x4 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outA, fpA);
+    q = pB2; const float y4 = coded8_step<NAN_AWARE>(pB2, rowB, amask, dlbit, shmul, &y);
+    record_leaf(q, y, pe, amask, sbase, meta, outB, fpB);
+    add_pair_ftz(a1, x1, x2);
+    add_pair_ftz(b1, y1, y2);
+    add_pair_ftz(a2, x3, x4);
+    add_pair_ftz(b2, y3, y4);
+  }
+  accA = a1 + a2;
+  accB = b1 + b2;
+}
+
 // k_sliced_codes8: k_sliced_codes' walk (slice resident in shared memory, dynamic 4-row work
 // units, half-warp per row, two chains per lane, ring refilled by the warp closing a tile) over
 // 16-row tiles of u8 code rows; unit u of a tile: half h walks rows u + 4h (chain A) and
@@ -1878,7 +2052,7 @@ __device__ __forceinline__ void walk_coded8_split(uint32_t pA1, uint32_t mA, uin
 constexpr int kCode8Threads = 384;
 // R rows per walked tile (a multiple of the pre-pass tile, whose NaN flags it carries), kR8 tiles
 // in the ring (R * kR8 rows in shared memory).
-template <bool FUSED, int R, int kR8>
+template <bool FUSED, int R, int kR8, bool LEAF>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {
   constexpr int C = kSlicedCols;
   constexpr int FS = R / kCode8TileRows;   // pre-pass tiles (NaN flags) per walked tile
@@ -1982,6 +2156,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
     }
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
     const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+    const int2* __restrict__ meta =
+        LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
     mbar_wait(s_forest, ph_forest);
     ph_forest ^= 1u;
     for (;;) {
@@ -2016,11 +2192,26 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
           nan_flag |= fk;
         }
         double accA, accB;
+        uint64_t fpA = 0, fpB = 0;
+        int32_t* oA = nullptr;
+        int32_t* oB = nullptr;
+        if (LEAF && a.o.out_leaf) {
+          if (okA) oA = a.o.out_leaf + (a.row0 + r0 + rA) * (int64_t)a.o.T_leaf;
+          if (okB) oB = a.o.out_leaf + (a.row0 + r0 + rB) * (int64_t)a.o.T_leaf;
+        }
         if (a.split) {
           const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
           const uint32_t mA = okA ? pm : pe, mB = okB ? pm : pe;
-          if (nan_flag) walk_coded8_split<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-          else walk_coded8_split<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          if (LEAF) {
+            if (nan_flag) walk_coded8_split_leaf<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+            else walk_coded8_split_leaf<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+          } else {
+            if (nan_flag) walk_coded8_split<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+            else walk_coded8_split<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          }
+        } else if (LEAF) {
+          if (nan_flag) walk_coded8_leaf<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+          else walk_coded8_leaf<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
         } else if (nan_flag) {
           walk_coded8<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
         } else {
@@ -2033,10 +2224,18 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
         double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
 #pragma unroll
         for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+        uint64_t fv = 0;
+        if (LEAF) {
+          fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
+#pragma unroll
+          for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
+        }
         const int rr = b3 ? rB : rA;
         if ((lane & 7) == 0 && (b3 ? okB : okA)) {
           if (FUSED) write_scalar(a.o, a.row0 + r0 + rr, v);
           else s_part[b * R + rr] = v;
+          if (LEAF && a.o.out_fp)
+            atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[a.row0 + r0 + rr]), (unsigned long long)fv);
         }
       }
       // release the unit; the warp closing the entry writes its partials and issues entry e + 3
@@ -2106,7 +2305,8 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
       e = cudaFuncSetAttribute(k_encode_rows8<kEncode8Threads, kEncode8Rows>,
                                cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
-      for (auto k : {k_sliced_codes8<true, kCode8TileRows, kCode8Ring>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring>})
+      for (auto k : {k_sliced_codes8<true, kCode8TileRows, kCode8Ring, false>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring, false>,
+                     k_sliced_codes8<true, kCode8TileRows, kCode8Ring, true>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring, true>})
         if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
       if (e != cudaSuccess) return (int)e;
       configured[dev].store(1);
@@ -2169,8 +2369,11 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     const int grid = full ? num_sms : plan.grid;
     a.o = o;
     // (16-row tiles in a 3-deep ring and 512 / 1024-thread CTAs measured within 2 %)
-    auto kern = fused ? k_sliced_codes8<true, kCode8TileRows, kCode8Ring>
-                      : k_sliced_codes8<false, kCode8TileRows, kCode8Ring>;
+    const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
+    auto kern = leaf ? (fused ? k_sliced_codes8<true, kCode8TileRows, kCode8Ring, true>
+                              : k_sliced_codes8<false, kCode8TileRows, kCode8Ring, true>)
+                     : (fused ? k_sliced_codes8<true, kCode8TileRows, kCode8Ring, false>
+                              : k_sliced_codes8<false, kCode8TileRows, kCode8Ring, false>);
     if (ev_b && one) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
     kern<<<grid, threads, smem, st>>>(a);
     if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;

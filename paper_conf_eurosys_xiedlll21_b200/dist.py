@@ -40,17 +40,24 @@ def predict_sample_sharded(forest, X_local: torch.Tensor, **kw) -> torch.Tensor:
     return forest.predict(X_local, **kw)
 
 
+def _global_rank(group, group_rank: int) -> int:
+    """Global rank of rank `group_rank` of `group` (None = the default group: the same number)."""
+    return group_rank if group is None else dist.get_global_rank(group, group_rank)
+
+
 def reduce_partials(partial: torch.Tensor, dst: int = 0, group=None) -> torch.Tensor:
-    """Sum the per-rank fp64 partial sums onto `dst` (in place; one ncclReduce / gloo reduce)."""
+    """Sum the per-rank fp64 partial sums onto `dst`, a rank WITHIN `group` (in place; one
+    ncclReduce / gloo reduce)."""
     if partial.dtype != torch.float64:
         raise TypeError("partials are fp64")
-    dist.reduce(partial, dst=dst, op=dist.ReduceOp.SUM, group=group)
+    dist.reduce(partial, dst=_global_rank(group, dst), op=dist.ReduceOp.SUM, group=group)
     return partial
 
 
 def predict_tree_sharded(full_forest, shard_forest, X: torch.Tensor, dst: int = 0, group=None,
                          partial_fn: Callable | None = None, finalize_fn: Callable | None = None):
-    """Tree-sharded prediction of all rows of X (replicated on every rank).
+    """Tree-sharded prediction of all rows of X (replicated on every rank); `dst` is a rank within
+    `group`.
 
     Returns (out, partial) on `dst` and (None, partial) elsewhere.  partial_fn(X) -> fp64 [n, n_out]
     defaults to shard_forest.predict_partial; finalize_fn(partial) defaults to
@@ -65,9 +72,10 @@ def predict_tree_sharded(full_forest, shard_forest, X: torch.Tensor, dst: int = 
 
 
 def broadcast_comm_id(make_id: Callable[[], bytes], src: int = 0, group=None) -> bytes:
-    """One rank draws the 128-byte communicator id, every rank returns the same bytes."""
+    """Rank `src` of `group` draws the 128-byte communicator id, every rank returns the same
+    bytes."""
     box = [make_id() if dist.get_rank(group) == src else None]
-    dist.broadcast_object_list(box, src=src, group=group)
+    dist.broadcast_object_list(box, src=_global_rank(group, src), group=group)
     uid = box[0]
     if not isinstance(uid, (bytes, bytearray)) or len(uid) != 128:
         raise RuntimeError("bad communicator id")

@@ -386,6 +386,37 @@ def tahoe_forest_export_sliced(h) -> dict | None:
 
 
 # ----------------------------------------------------------------------- convenience wrapper
+def _need(t, name: str, dtype, shape: tuple, device: int | None):
+    """Validate a tensor handed to the C ABI: the library reads raw pointers with a row stride of
+    shape[1], so a strided view, a wrong dtype, a wrong shape or a tensor on another device would
+    give silently wrong results or a fault.  device None: a host tensor; else cuda:<device>."""
+    import torch
+    if t is None:
+        return
+    if not isinstance(t, torch.Tensor):
+        raise TypeError(f"{name}: expected a torch.Tensor, got {type(t).__name__}")
+    if t.dtype != dtype:
+        raise TypeError(f"{name}: dtype {t.dtype}, expected {dtype}")
+    if tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name}: shape {tuple(t.shape)}, expected {tuple(shape)}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous (row-major, row stride = shape[1])")
+    if device is None:
+        if t.is_cuda:
+            raise ValueError(f"{name}: expected a host tensor")
+    elif not t.is_cuda or t.device.index != device:
+        raise ValueError(f"{name}: on {t.device}, expected cuda:{device}")
+
+
+def _need_X(X, name: str, device: int | None):
+    """X: [n, d] float32, d >= the forest's feature count (checked by the library)."""
+    import torch
+    if not isinstance(X, torch.Tensor) or X.dim() != 2:
+        raise ValueError(f"{name}: expected a 2-D torch tensor")
+    _need(X, name, torch.float32, tuple(X.shape), device)
+    return X.shape
+
+
 class Forest:
     """Owns a tahoe_forest handle.  ``arrays`` are the user-level node arrays (as produced by
     gen.make_forest)."""
@@ -400,6 +431,7 @@ class Forest:
         self.handle = tahoe_forest_build(arrays, self.n_features, self.n_classes, self.agg,
                                          base_score, device)
         self.n_trees = tahoe_forest_n_trees(self.handle)
+        self.n_trees_full = self.n_trees
         self.n_out = tahoe_forest_n_outputs(self.handle)
 
     @classmethod
@@ -408,6 +440,7 @@ class Forest:
         f.n_features, f.n_classes, f.agg = like.n_features, like.n_classes, like.agg
         f.device, f.n_nodes, f.handle = device, like.n_nodes, handle
         f.n_trees = tahoe_forest_n_trees(handle)
+        f.n_trees_full = like.n_trees_full   # leaf ids of a shard use the full forest's tree ids
         f.n_out = tahoe_forest_n_outputs(handle)
         return f
 
@@ -446,13 +479,22 @@ class Forest:
     def predict_cost_us(self, strategy: int, n: int) -> float:
         return tahoe_predict_cost_us(self.handle, strategy, n)
 
+    def _stream(self, stream):
+        import torch
+        return torch.cuda.current_stream(self.device) if stream is None else stream
+
     def predict(self, X, out=None, out_class=None, out_leaf=None, out_fingerprint=None,
                 force_strategy: int = -1, stream=None, ev_main_begin=None, ev_main_end=None):
         """X: torch tensor on the forest's device (n x d float32).  Returns ``out``."""
         import torch
-        n, d = X.shape
+        n, d = _need_X(X, "X", self.device)
         if out is None:
             out = torch.empty((n, self.n_out), dtype=torch.float32, device=X.device)
+        _need(out, "out", torch.float32, (n, self.n_out), self.device)
+        _need(out_class, "out_class", torch.int32, (n,), self.device)
+        _need(out_leaf, "out_leaf", torch.int32, (n, self.n_trees_full), self.device)
+        _need(out_fingerprint, "out_fingerprint", torch.int64, (n,), self.device)
+        stream = self._stream(stream)
         if (out_class is None and out_leaf is None and out_fingerprint is None
                 and force_strategy < 0 and ev_main_begin is None):
             tahoe_predict(self.handle, X, n, d, out, stream)
@@ -462,8 +504,11 @@ class Forest:
         return out
 
     def predict_host(self, X_host, out_host, class_host=None, stream=None):
-        n, d = X_host.shape
-        tahoe_predict_host(self.handle, X_host, n, d, out_host, class_host, stream)
+        import torch
+        n, d = _need_X(X_host, "X_host", None)
+        _need(out_host, "out_host", torch.float32, (n, self.n_out), None)
+        _need(class_host, "class_host", torch.int32, (n,), None)
+        tahoe_predict_host(self.handle, X_host, n, d, out_host, class_host, self._stream(stream))
         return out_host
 
     def shard(self, rank: int, world: int, device: int | None = None) -> "Forest":
@@ -472,18 +517,22 @@ class Forest:
 
     def predict_partial(self, X, partial=None, stream=None):
         import torch
-        n, d = X.shape
+        n, d = _need_X(X, "X", self.device)
         if partial is None:
             partial = torch.empty((n, self.n_out), dtype=torch.float64, device=X.device)
-        tahoe_predict_partial(self.handle, X, n, d, partial, stream)
+        _need(partial, "partial", torch.float64, (n, self.n_out), self.device)
+        tahoe_predict_partial(self.handle, X, n, d, partial, self._stream(stream))
         return partial
 
     def finalize(self, partial, out=None, out_class=None, stream=None):
         import torch
         n = partial.shape[0]
+        _need(partial, "partial", torch.float64, (n, self.n_out), self.device)
         if out is None:
             out = torch.empty((n, self.n_out), dtype=torch.float32, device=partial.device)
-        tahoe_finalize(self.handle, partial, n, out, out_class, stream)
+        _need(out, "out", torch.float32, (n, self.n_out), self.device)
+        _need(out_class, "out_class", torch.int32, (n,), self.device)
+        tahoe_finalize(self.handle, partial, n, out, out_class, self._stream(stream))
         return out
 
     def export_sliced(self):
@@ -494,11 +543,14 @@ class Forest:
         """Collective tree-sharded prediction with this shard (tahoe_predict_reduce): returns this
         rank's rows [lo, hi) of the finalised output."""
         import torch
-        n, d = X.shape
+        n, d = _need_X(X, "X", self.device)
         lo, hi = tahoe_reduce_rows(n, comm.world, comm.rank, mode)
         if out is None:
             out = torch.empty((hi - lo, self.n_out), dtype=torch.float32, device=X.device)
-        tahoe_predict_reduce(self.handle, comm.handle, X, n, d, mode, out, out_class, stream)
+        _need(out, "out", torch.float32, (hi - lo, self.n_out), self.device)
+        _need(out_class, "out_class", torch.int32, (hi - lo,), self.device)
+        tahoe_predict_reduce(self.handle, comm.handle, X, n, d, mode, out, out_class,
+                             self._stream(stream))
         return out
 
     def reduce_partials(self, partials, rank: int, mode: int = REDUCE_SCATTER, out=None,
@@ -506,11 +558,16 @@ class Forest:
         """Fixed-order sum + finalisation of per-shard partials resident on this device."""
         import torch
         n = partials[0].shape[0]
+        for q, p in enumerate(partials):
+            if isinstance(p, torch.Tensor):
+                _need(p, f"partials[{q}]", torch.float64, (n, self.n_out), self.device)
         lo, hi = tahoe_reduce_rows(n, len(partials), rank, mode)
         if out is None:
             out = torch.empty((hi - lo, self.n_out), dtype=torch.float32, device=partials[0].device)
+        _need(out, "out", torch.float32, (hi - lo, self.n_out), self.device)
+        _need(out_class, "out_class", torch.int32, (hi - lo,), self.device)
         tahoe_reduce_partials(self.handle, partials, len(partials), rank, mode, n, out, out_class,
-                              stream)
+                              self._stream(stream))
         return out
 
     def close(self):

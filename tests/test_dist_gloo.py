@@ -124,3 +124,46 @@ def test_gloo_world2_sample_and_tree_sharding():
     for p in procs:
         p.join(timeout=60)
     assert res == {0: "ok", 1: "ok"}, res
+
+
+def _worker_subgroup(rank, world, port, q):
+    """dst / src arguments are ranks WITHIN the group: with group = global ranks [1, 2], group rank
+    0 is global rank 1 (dist.reduce read dst as a global rank)."""
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    from paper_conf_eurosys_xiedlll21_b200 import dist as D
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        grp = dist.new_group([1, 2])
+        if rank in (1, 2):
+            part = torch.full((4, 1), float(rank), dtype=torch.float64)
+            out, p = D.predict_tree_sharded(None, None, None, dst=0, group=grp,
+                                            partial_fn=lambda _x: part, finalize_fn=lambda t: t)
+            if rank == 1:   # group rank 0 receives the sum and finalises
+                assert out is not None and torch.equal(out, torch.full((4, 1), 3.0, dtype=torch.float64))
+            else:
+                assert out is None
+            uid = D.broadcast_comm_id(lambda: bytes([rank]) * 128, src=0, group=grp)
+            assert uid == bytes([1]) * 128, "the id comes from group rank 0 (global rank 1)"
+        q.put((rank, "ok"))
+    except Exception as e:  # pragma: no cover
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world3_subgroup_ranks():
+    world = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_subgroup, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    assert res == {0: "ok", 1: "ok", 2: "ok"}, res

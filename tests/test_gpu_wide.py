@@ -65,11 +65,11 @@ def test_wide_codes_piece_boundaries_ties_signed_zero_inf_nan():
     assert st["coded_valid"] and st["code8"], st["coded_why"]
     assert st["code8_virtual"] > d, "some attribute must span several pieces"
     X = _boundary_rows(f, rng, 20011, d)
-    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1)
+    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
     outs = []
     for s in _strats(F):
-        r = _gpu_run(F, X, s, want_leaf=False)
-        _check(r, ref, oracle.AGG_SUM, True, want_leaf=False)
+        r = _gpu_run(F, X, s)          # leaf ids + fingerprints (LEAF instantiations)
+        _check(r, ref, oracle.AGG_SUM, True)
         outs.append(r["out"])
     assert len(outs) == 3 and all(np.array_equal(o, outs[0]) for o in outs)
 
@@ -86,9 +86,10 @@ def test_wide_codes_row_geometries(d):
     X = rng.normal(size=(7001, d)).astype(np.float32)
     X[::23, 0] = np.nan
     X[5::31, :] = np.nan
-    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1)
+    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
     _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, oracle.AGG_SUM, True,
            want_leaf=False)
+    _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED), ref, oracle.AGG_SUM, True)
 
 
 def test_wide_codes_multiclass_partials_and_slice_switching(monkeypatch):
@@ -104,8 +105,10 @@ def test_wide_codes_multiclass_partials_and_slice_switching(monkeypatch):
     for n in (333, 60_017):
         X = rng.normal(size=(n, d)).astype(np.float32)
         X[::41, 7] = np.nan
-        ref = oracle.predict(f, X, agg=oracle.AGG_CLASS_SUM, n_classes=5, base_score=0.5)
+        ref = oracle.predict(f, X, agg=oracle.AGG_CLASS_SUM, n_classes=5, base_score=0.5,
+                             want_leaf=True)
         _check(_gpu_run(F, X, -1, want_leaf=False), ref, oracle.AGG_CLASS_SUM, True, want_leaf=False)
+        _check(_gpu_run(F, X, -1), ref, oracle.AGG_CLASS_SUM, True)
         part = F.predict_partial(torch.from_numpy(X).cuda())
         torch.cuda.synchronize()
         assert np.array_equal(part.cpu().numpy(), ref["raw"] - 0.5), "dyadic partial sums are exact"

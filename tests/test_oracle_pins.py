@@ -308,3 +308,79 @@ def test_oracle_rows_subset_matches_full():
     a = oracle.predict(f, X, want_leaf=True)
     b = oracle.predict(f, X, rows=idx, want_leaf=True)
     assert np.array_equal(a["leaf"][idx], b["leaf"]) and np.array_equal(a["raw"][idx], b["raw"])
+
+
+# ----------------------------------------------------------------- fingerprint
+_M64 = (1 << 64) - 1
+
+
+def _mix64(z: int) -> int:
+    """splitmix64's output finaliser, restated in plain Python integers."""
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & _M64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & _M64
+    return z ^ (z >> 31)
+
+
+def test_mix64_known_answers():
+    """The restated finaliser reproduces the published splitmix64 stream of seed 0 (state advanced
+    by the golden gamma 0x9E3779B97F4A7C15 before each output): 0xE220A8397B1DCDAF,
+    0x6E789E6AA1B965F4, 0x06C45D188009454F."""
+    s, got = 0, []
+    for _ in range(3):
+        s = (s + 0x9E3779B97F4A7C15) & _M64
+        got.append(_mix64(s))
+    assert got == [0xE220A8397B1DCDAF, 0x6E789E6AA1B965F4, 0x06C45D188009454F]
+
+
+def _fp_from_leaves(leaf: np.ndarray, tree_ids) -> np.ndarray:
+    out = np.zeros(leaf.shape[0], np.uint64)
+    for i in range(leaf.shape[0]):
+        acc = 0
+        for j, t in enumerate(tree_ids):
+            acc = (acc + _mix64(((int(t) << 32) | (int(leaf[i, j]) & 0xFFFFFFFF)) & _M64)) & _M64
+        out[i] = acc
+    return out
+
+
+def test_fingerprint_restated_from_leaf_ids():
+    """fp[i] = sum_t mix64((t << 32) | leaf[i][t]) mod 2^64, restated from the
+    oracle's own leaf ids (not from its fingerprint code)."""
+    rng = np.random.default_rng(5)
+    f = random_forest(rng, 23, 5, 6)
+    X = rng.normal(size=(257, 6)).astype(np.float32)
+    r = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
+    assert np.array_equal(r["fp"], _fp_from_leaves(r["leaf"], range(23)))
+
+
+def test_fingerprint_single_leaf_trees_closed_form():
+    """Trees that are single leaves: every row reaches the root, so fp is the same closed-form
+    constant for every row."""
+    T = 9
+    roots = np.arange(100, 100 + T, dtype=np.int32)
+    n = 110
+    f = dict(root=roots, feature=np.full(n, -1, np.int32), threshold=np.zeros(n, np.float32),
+             left=np.full(n, -1, np.int32), right=np.full(n, -1, np.int32),
+             leaf_value=np.zeros(n, np.float32), default_left=None, tree_class=None)
+    X = np.zeros((5, 2), np.float32)
+    r = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1)
+    want = 0
+    for t in range(T):
+        want = (want + _mix64((t << 32) | (100 + t))) & _M64
+    assert r["fp"].tolist() == [want] * 5
+
+
+def test_fingerprint_tree_sharded_sum_equals_full():
+    """Invariant: splitting the trees into shards and summing the shards'
+    fingerprints (each tree keeping its global index t) gives the full forest's fingerprint.
+    The shard fingerprints are restated from the oracle's leaf ids of each sub-forest."""
+    rng = np.random.default_rng(9)
+    f = random_forest(rng, 31, 6, 5)
+    X = rng.normal(size=(123, 5)).astype(np.float32)
+    full = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1)
+    perm = rng.permutation(31)
+    tot = np.zeros(X.shape[0], np.uint64)
+    for shard in np.array_split(perm, 4):
+        sub = dict(f, root=f["root"][shard])
+        rs = oracle.predict(sub, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
+        tot = tot + _fp_from_leaves(rs["leaf"], shard)   # uint64 wraps mod 2^64
+    assert np.array_equal(tot, full["fp"])

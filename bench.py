@@ -1,18 +1,21 @@
 #!/usr/bin/env python
 """Benchmark of the hot path: batched decision-tree-ensemble prediction (Tahoe, EuroSys '21).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config 2]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config 3]
     python -m torch.distributed.run --nnodes=1 --nproc-per-node N --master-addr 127.0.0.1 \
         --master-port P bench.py --gpus N ...
 
-Workload (BASELINE.json configs[1], the config the metric is quoted on and that fits one GPU):
-C2, a Higgs-shaped binary forest of 500 random post-pruned trees (depth <= 8, 28 attributes) over
-1M synthetic samples per GPU.  A step = one tahoe_predict of the whole batch (all §8(a) rows:
-traversal, combine, finalize).  N > 1: every rank predicts its own 1M rows (sample sharding, weak
-scaling, no data-path collective).  Rank 0 prints one JSON line.
+Workload (BASELINE.json metric "samples/sec per forest at 1/2/4/8 B200"; the one config quoted over
+1/2/4/8 GPUs is configs[2]): C3, a covtype-shaped 7-class forest of 7 x 200 random post-pruned
+trees (depth <= 12, 54 attributes) over 4M synthetic samples, split contiguously over the N ranks
+(rank r predicts rows [r n / N, (r + 1) n / N): the paper's even partition; strong
+scaling, no data-path collective).  --weak gives every rank its own 4M rows.  --config 2 / 4 / 5
+run the other BASELINE configs (C5: tree-sharded, fused NVLink reduce).  A step = one tahoe_predict
+of the rank's rows (all §8(a) rows: row coding, traversal, combine, finalize).  Rank 0 prints one
+JSON line.
 
 --impl reference: the CPU oracle (oracle/, the "reference arm" of this tier) timed on the box's
-host cores on a bounded sample of the same workload per step.
+host cores on a bounded sample of the same workload per step (rank 0 only).
 """
 from __future__ import annotations
 
@@ -141,14 +144,17 @@ class ClockSampler:
                 "source": "nvml 10 ms" if self.nvml else "nvidia-smi 50 ms"}
 
 
-def build_workload(cfg, rank: int, n: int):
-    f = gen.make_forest(cfg, leaf_mode="normal")
-    X = gen.make_rows(cfg, n, row0=rank * n)
-    return f, X
+def rank_rows(cfg, n: int, rank: int, world: int, weak: bool) -> tuple[int, int]:
+    """Rows [lo, hi) of the config's seeded test matrix that `rank` predicts: a contiguous 1/world
+    of n (strong scaling), or its own n rows with --weak."""
+    if weak:
+        return rank * n, (rank + 1) * n
+    return (n * rank) // world, (n * (rank + 1)) // world
 
 
 def oracle_rate(f, X, target_s: float, max_rows: int):
-    """Oracle (as it stands) on a bounded sample of X: returns (rows/s, rows, seconds, visits)."""
+    """Oracle (as it stands) on a bounded seeded sample of X, all host cores.  Returns (rows/s,
+    rows, seconds, mean visits, sample indices, oracle result)."""
     import oracle
     probe = min(2000, X.shape[0])
     t = time.perf_counter()
@@ -159,7 +165,65 @@ def oracle_rate(f, X, target_s: float, max_rows: int):
     t = time.perf_counter()
     r = oracle.predict(f, X, rows=idx)
     dt = time.perf_counter() - t
-    return rows / dt, rows, dt, float(r["visits"].mean())
+    return rows / dt, rows, dt, float(r["visits"].mean()), idx, r
+
+
+def oracle_single_core(f, X, rows: int = 10_000):
+    """Single-core oracle rate on the first `rows` rows (SURVEY §8(d) "two numbers per config")."""
+    import oracle
+    m = min(rows, X.shape[0])
+    t = time.perf_counter()
+    oracle.predict(f, X[:m], nthreads=1)
+    return m / (time.perf_counter() - t), m
+
+
+def parity_record(f, out_rows: np.ndarray, cls_rows: np.ndarray, ref: dict) -> dict:
+    """GPU outputs on the oracle's sample rows against the oracle (north_star bars): scores within
+    max(1e-5 |ref|, 1e-6); classes exact outside the fp64 rounding window of reading R3 (bound
+    4 gamma_T T max|v|), rows inside it counted."""
+    import oracle
+    tol = np.maximum(1e-5 * np.abs(ref["out"]), 1e-6)
+    err = np.abs(out_rows - ref["out"])
+    bad = (err > tol).any(axis=1)
+    leaves = f["feature"] < 0
+    T = len(f["root"])
+    u = 2.0 ** -53
+    bound = 4.0 * (T * u / (1 - T * u)) * T * float(np.abs(f["leaf_value"][leaves]).max())
+    agg = f["agg"]
+    window = 0
+    cls_bad = 0
+    if agg in (oracle.AGG_BINARY, oracle.AGG_CLASS_SUM):
+        if agg == oracle.AGG_BINARY:
+            sure = np.abs(ref["raw"][:, 0]) > bound
+        else:
+            srt = np.sort(ref["raw"], axis=1)
+            sure = (srt[:, -1] - srt[:, -2]) > bound
+        window = int((~sure).sum())
+        cls_bad = int((cls_rows[sure] != ref["cls"][sure]).sum())
+    rel = err / np.maximum(np.abs(ref["out"]), 1e-30)
+    return dict(rows=int(len(out_rows)), mismatches=int(bad.sum()) + cls_bad,
+                score_mismatches=int(bad.sum()), class_mismatches=cls_bad,
+                max_abs_err=float(err.max()) if err.size else 0.0,
+                max_rel_err=float(rel.max()) if rel.size else 0.0,
+                classes_in_R3_window=window, r3_bound=bound,
+                tolerance="max(1e-5 |ref|, 1e-6) vs the oracle's fp64 sum rounded once")
+
+
+def visit_peak(device: int, variant: int) -> dict | None:
+    """Live microbenchmark (Algorithm 1 line 4): node reads per second of the production coded walk
+    on ideal data, plus raw shared-memory bytes per SM clock (tahoe_measure_visit_rate)."""
+    from paper_conf_eurosys_xiedlll21_b200 import tahoe as T
+    try:
+        T.tahoe_measure_visit_rate(device, variant, 256, 200)   # warm clocks
+        best = 0.0
+        bw = None
+        for _ in range(3):
+            r, b = T.tahoe_measure_visit_rate(device, variant, 256, 2000)
+            if r > best:
+                best, bw = r, b
+        return dict(node_reads_per_s=best, smem_bytes_per_clk_sm=bw, variant=variant)
+    except Exception as e:  # pragma: no cover
+        return dict(error=str(e))
 
 
 def run_reference(args, cfg):
@@ -168,9 +232,10 @@ def run_reference(args, cfg):
         return 0
     import oracle
     n = cfg.n_samples
-    f, X = build_workload(cfg, 0, min(n, 200_000))
+    f = gen.make_forest(cfg, leaf_mode="normal")
+    X = gen.make_rows(cfg, min(n, 200_000))
     cores = oracle.n_threads()
-    rate0, _, _, _ = oracle_rate(f, X, 1.0, 20000)
+    rate0 = oracle_rate(f, X, 1.0, 20000)[0]
     rows = int(min(X.shape[0], max(1000, rate0 * 4.0)))   # ~4 s of oracle work per step
     idx = gen.subsample(99, X.shape[0], rows)
     for _ in range(args.warmup):
@@ -182,11 +247,13 @@ def run_reference(args, cfg):
         times.append(time.perf_counter() - t)
     ms = 1000.0 * statistics.mean(times)
     value = rows / (ms / 1000.0)
-    sample = f"{rows} seeded rows per step of the {cfg.name} workload (of {n} per GPU)"
+    sample = f"{rows} seeded rows per step of the {cfg.name} workload ({n} rows)"
     line = dict(metric=METRIC, value=value, unit=UNIT, n_gpus=args.gpus, steps=args.steps,
-                warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="weak",
+                warmup=args.warmup, ms_per_step=ms, ms_median=1000.0 * statistics.median(times),
+                ms_min=1000.0 * min(times), higher_is_better=True,
+                scaling="weak" if args.weak else "strong",
                 vs_baseline=None, dtype="f32", data="synthetic", impl="reference",
-                config=_config(cfg, n, None),
+                config=_config(cfg, n, None, args.gpus, args.weak),
                 cpu_baseline=dict(value=value, unit=UNIT, cores=cores, kind="oracle",
                                   sample=sample),
                 e2e=dict(value=value, unit=UNIT, h2d_bytes_per_step=0, d2h_bytes_per_step=0))
@@ -228,7 +295,6 @@ def run_tree_sharded(args, cfg):
     stream = torch.cuda.current_stream()
     fused = args.reduce == "fused"
     if fused:
-        os.environ.setdefault("NCCL_DEBUG", "WARN")   # keep stdout to the one JSON line
         comm = D.init_comm(local)
         lo, hi = T.tahoe_reduce_rows(n, world, rank, T.REDUCE_SCATTER)
         out = torch.empty((hi - lo, S.n_out), dtype=torch.float32, device=dev)
@@ -287,14 +353,20 @@ def run_tree_sharded(args, cfg):
         st = S.stats()
         # the oracle (as it stands) on a bounded sample of the same rows and the FULL forest
         cpu = None
+        parity = None
         visits = st["expected_visits_per_sample"]   # this rank's shard, calibration estimate
         if not args.no_cpu and world == 1:
             import oracle
-            rate, rows, secs, vis = oracle_rate(f, Xh, 12.0, 200_000)
+            rate, rows, secs, vis, idx, ref = oracle_rate(f, Xh, 12.0, 200_000)
+            r1, m1 = oracle_single_core(f, Xh, 500)
             cpu = dict(value=rate, unit=UNIT, cores=oracle.n_threads(), kind="oracle",
                        sample=f"{rows} seeded rows of this workload, full {cfg.n_trees}-tree forest "
-                              f"({secs:.1f} s of oracle work)")
+                              f"({secs:.1f} s of oracle work)",
+                       single_core=dict(value=r1, unit=UNIT, cores=1, sample=f"first {m1} rows"))
             visits = vis
+            if not args.weak:
+                oh_dev = out.cpu().numpy()
+                parity = parity_record(f, oh_dev[idx], np.zeros(len(idx), np.int32), ref)
         # roofline of the traversal (k_direct_tlp over the L2-sized chunks of the shard's image):
         # algorithmic bytes per sample = node visits x (8 B node + 4 B attribute) + leaves x 8 B,
         # against the L1 / shared-memory data pipe the node and attribute loads go through
@@ -330,7 +402,8 @@ def run_tree_sharded(args, cfg):
                             "n": n, "trees_per_shard": st["n_trees"],
                             "parallelism": f"tree-sharded x{world}",
                             "reduce": "fused (NCCL device API, LSA)" if fused else "ncclReduce"},
-                    strategy="direct", roofline=roofline, hbm=hbm, cpu_baseline=cpu, e2e=e2e,
+                    strategy="direct", roofline=roofline, hbm=hbm, cpu_baseline=cpu, parity=parity,
+                    e2e=e2e,
                     gpu_launches=(2 if (fused or rank == 0) else 1) * args.steps, clocks=clocks,
                     layout_s=layout_s)
         print(json.dumps(line), flush=True)
@@ -342,19 +415,24 @@ def run_tree_sharded(args, cfg):
     return 0
 
 
-def _config(cfg, n, stats):
+def _config(cfg, n, stats, world: int = 1, weak: bool = False):
+    """n: rows of the whole job (strong) or per GPU (weak)."""
+    n_local = n if weak else -(-n // world)
+    split = (f"{n} samples per GPU (weak scaling)" if weak else
+             f"{n} samples split contiguously over {world} GPU(s)")
     c = {"workload": f"{cfg.name}: {cfg.n_trees} trees depth<={cfg.max_depth}, "
-                     f"{cfg.n_features} features, {n} samples per GPU (BASELINE configs[{cfg.cid - 1}])",
-         "n_per_gpu": n, "n_trees": cfg.n_trees, "n_features": cfg.n_features,
-         "max_depth": cfg.max_depth,
+                     f"{cfg.n_features} features, {split} (BASELINE configs[{cfg.cid - 1}])",
+         "n_total": n * world if weak else n, "n_per_gpu": n_local, "n_trees": cfg.n_trees,
+         "n_features": cfg.n_features, "max_depth": cfg.max_depth,
          "agg": {gen.AGG_SUM: "sum", gen.AGG_AVERAGE: "average", gen.AGG_BINARY: "binary margin + class",
                  gen.AGG_CLASS_SUM: f"{cfg.n_classes}-class sums + argmax",
                  gen.AGG_VOTE: "vote"}.get(cfg.agg, str(cfg.agg)),
-         "parallelism": "sample-sharded (no collective)",
-         "l2": f"256 MiB L2 flush between timed steps (inputs {n * cfg.n_features * 4 / 1e6:.0f} MB "
-               f"{'<' if n * cfg.n_features * 4 < 126e6 else '>'} L2), outside the events"}
+         "parallelism": f"sample-sharded x{world} (no collective)",
+         "l2": f"256 MiB L2 flush between timed steps (inputs {n_local * cfg.n_features * 4 / 1e6:.0f} MB "
+               f"per GPU {'<' if n_local * cfg.n_features * 4 < 126e6 else '>'} L2), outside the events"}
     if stats:
-        c.update({k: stats[k] for k in ("nodes", "leaves", "n_slices", "slots_max", "lockstep_eff",
+        c.update({k: stats[k] for k in ("nodes", "leaves", "n_slices", "slots_max",
+                                        "column_balance_expected", "lockstep_eff_sim",
                                         "expected_visits_per_sample", "sliced_bytes") if k in stats})
     return c
 
@@ -362,17 +440,18 @@ def _config(cfg, n, stats):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--config", type=int, default=3)
     ap.add_argument("--strategy", type=int, default=-1)
-    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline / parity leg")
     ap.add_argument("--mode", default=None, choices=["sample", "tree"],
                     help="sample sharding (default; C1-C4) or tree sharding (default for C5)")
     ap.add_argument("--rows", type=int, default=None, help="override the config's row count")
     ap.add_argument("--weak", action="store_true",
-                    help="tree mode: duplicate the rows once per GPU (weak scaling, P:2450-2456)")
+                    help="weak scaling: every GPU gets the config's full row count (sample mode: its "
+                         "own rows; tree mode: the rows duplicated once per GPU, P:2450-2456)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help=argparse.SUPPRESS)   # gloo: N>1 code path on one GPU (tests only)
     ap.add_argument("--reduce", default="fused", choices=["fused", "nccl"],
@@ -404,17 +483,21 @@ def main():
     T.load(build_if_missing=(rank == 0 and world == 1))
     args.warmup = max(args.warmup, 3)
     n = cfg.n_samples
-    f, X = build_workload(cfg, rank, n)
+    lo, hi = rank_rows(cfg, n, rank, world, args.weak)
+    n_local = hi - lo
+    n_total = n * world if args.weak else n
+    f = gen.make_forest(cfg, leaf_mode="normal")
+    X = gen.make_rows(cfg, n_local, row0=lo)
     t0 = time.perf_counter()
     F = T.Forest(f, device=local)
     F.layout(gen.make_calibration(cfg))
     layout_s = time.perf_counter() - t0
     stats = F.stats()
-    strategy = args.strategy if args.strategy >= 0 else F.select_strategy(n, cfg.n_features)
+    strategy = args.strategy if args.strategy >= 0 else F.select_strategy(n_local, cfg.n_features)
     Xd = torch.from_numpy(X).to(dev)
     coll_dev = dev if args.dist_backend == "nccl" else torch.device("cpu")
-    out = torch.empty((n, F.n_out), dtype=torch.float32, device=dev)
-    cls = torch.empty(n, dtype=torch.int32, device=dev)
+    out = torch.empty((n_local, F.n_out), dtype=torch.float32, device=dev)
+    cls = torch.empty(n_local, dtype=torch.int32, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
@@ -453,17 +536,20 @@ def main():
         dist.barrier()
     step_ms = [e[0].elapsed_time(e[1]) for e in ev]
     kern_ms = [e[2].elapsed_time(e[3]) for e in ev]
-    tot = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=coll_dev)
+    tot = torch.tensor([sum(step_ms), sum(kern_ms), statistics.median(step_ms), min(step_ms)],
+                       dtype=torch.float64, device=coll_dev)
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
     ms_per_step = float(tot[0]) / args.steps
     kern_avg_ms = float(tot[1]) / args.steps
-    value = world * n / (ms_per_step / 1000.0)
+    value = n_total / (ms_per_step / 1000.0)
+    out_h = out.cpu().numpy()
+    cls_h = cls.cpu().numpy()
 
     # ---- end to end through the public API with HOST buffers (pinned), copies inside
     Xh = torch.from_numpy(X).pin_memory()
-    oh = torch.empty((n, F.n_out), dtype=torch.float32).pin_memory()
-    ch = torch.empty(n, dtype=torch.int32).pin_memory()
+    oh = torch.empty((n_local, F.n_out), dtype=torch.float32).pin_memory()
+    ch = torch.empty(n_local, dtype=torch.int32).pin_memory()
     for _ in range(2):
         F.predict_host(Xh, oh, ch)
     torch.cuda.synchronize()
@@ -478,7 +564,9 @@ def main():
     e2e_t = torch.tensor([statistics.mean(e2e_ms)], dtype=torch.float64, device=coll_dev)
     if world > 1:
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
-    e2e_value = world * n / (float(e2e_t[0]) / 1000.0)
+    e2e_value = n_total / (float(e2e_t[0]) / 1000.0)
+    e2e_same = bool(np.array_equal(oh.numpy(), out_h) and np.array_equal(ch.numpy(), cls_h))
+    del Xh
 
     if rank != 0:
         if world > 1:
@@ -488,23 +576,39 @@ def main():
 
     peaks = _peaks()
     # algorithmic bytes (HBM roofline the metric asks for): sample row read + outputs written
-    hbm_bytes = n * (cfg.n_features * 4 + F.n_out * 4 + 4)
+    hbm_bytes = n_local * (cfg.n_features * 4 + F.n_out * 4 + 4)
     hbm_gbs = hbm_bytes / (ms_per_step / 1000.0) / 1e9
-    # dominant kernel roofline: shared-memory LSU pipe: per node visit
-    # 8 B node + 4 B attribute, per leaf 8 B; peak 128 B/clk/SM x SMs x max SM clock
     cpu = None
+    parity = None
     visits = stats["expected_visits_per_sample"]
+    visits_src = "calibration estimate"
     if not args.no_cpu and world == 1:
-        rate, rows, secs, vis = oracle_rate(f, X, 12.0, 1_000_000)
         import oracle
+        rate, rows, secs, vis, idx, ref = oracle_rate(f, X, 12.0, 1_000_000)
+        r1, m1 = oracle_single_core(f, X)
         cpu = dict(value=rate, unit=UNIT, cores=oracle.n_threads(), kind="oracle",
-                   sample=f"{rows} seeded rows of this workload ({secs:.1f} s of oracle work)")
-        visits = vis
-    smem_bytes_per_sample = visits * 12.0 + cfg.n_trees * 8.0
-    n_sms = stats["num_sms"]
-    smem_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
-    achieved = n * smem_bytes_per_sample / (kern_avg_ms / 1000.0) / 1e9
-    kname = {1: "k_sliced", 2: "k_sliced_codes8" if stats.get("code8") else "k_sliced_codes"}.get(strategy, "k_direct")
+                   sample=f"{rows} seeded rows of this workload ({secs:.1f} s of oracle work)",
+                   single_core=dict(value=r1, unit=UNIT, cores=1, sample=f"first {m1} rows"))
+        parity = parity_record(f, out_h[idx], cls_h[idx], ref)
+        parity["e2e_outputs_equal_device_outputs"] = e2e_same
+        visits, visits_src = vis, f"oracle, mean over the {rows} sampled rows"
+    # dominant kernel roofline: the walk is bound by the shared-memory LSU pipe; its
+    # unit is a node read (internal visit or leaf read), V_int + T per sample; the peak is the
+    # node-read rate of the same walk on ideal data, measured live (tahoe_measure_visit_rate)
+    code8 = bool(stats.get("code8"))
+    kname = {1: "k_sliced", 2: "k_sliced_codes8" if code8 else "k_sliced_codes"}.get(strategy, "k_direct")
+    reads_per_sample = visits + cfg.n_trees
+    achieved = n_local * reads_per_sample / (kern_avg_ms / 1000.0) / 1e9
+    vp = visit_peak(local, 1 if code8 else 0) if strategy == T.STRATEGY_SLICED_CODED else None
+    if vp and "node_reads_per_s" in vp:
+        peak, peak_src = vp["node_reads_per_s"] / 1e9, (
+            "measured live: tahoe_measure_visit_rate variant %d (the production coded walk on ideal "
+            "data: conflict-free, perfect lockstep, 32 warps/SM on every SM)" % vp["variant"])
+    else:
+        n_sms = stats["num_sms"]
+        peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 12.0 / 1e9
+        peak_src = (f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz / 12 B per "
+                    f"node read (no microbenchmark for this strategy)")
     traffic = None
     sector_eff = None
     path_sector_eff = None   # every LSU global load of the step (pre-pass + walk), same capture
@@ -513,7 +617,7 @@ def main():
         try:
             rec = json.load(open(tp)).get(f"C{cfg.cid}", {})
             # only a capture of the kernel this run times (e.g. "k_sliced_codes<0>")
-            if rec.get("kernel", "").split("<")[0] == kname:
+            if rec.get("kernel", "").split("<")[0] == kname and rec.get("n") in (None, n_local):
                 traffic = rec.get("dram_bytes_per_launch")
                 sector_eff = rec.get("global_ld_sector_efficiency")
                 path_sector_eff = rec.get("path_global_ld_sector_efficiency")
@@ -525,25 +629,29 @@ def main():
         launches_per_step += 1   # the row-coding pre-pass (the flag memset is not a kernel of ours)
     line = dict(
         metric=METRIC, value=value, unit=UNIT, n_gpus=world, steps=args.steps, warmup=args.warmup,
-        ms_per_step=ms_per_step, higher_is_better=True, scaling="weak", vs_baseline=None,
+        ms_per_step=ms_per_step, ms_median=float(tot[2]), ms_min=float(tot[3]),
+        per_gpu=dict(value=value / world, unit=UNIT, n_per_gpu=n_local),
+        higher_is_better=True, scaling="weak" if args.weak else "strong", vs_baseline=None,
         dtype="f32", accum="f64", data="synthetic", impl="ours",
-        config=_config(cfg, n, stats),
+        config=_config(cfg, n, stats, world, args.weak),
         strategy={0: "direct", 1: "sliced", 2: "sliced-coded"}.get(strategy, str(strategy)),
-        roofline=dict(bound="alu", pipe="shared-memory LSU, 128 B/clk/SM (DESIGN.md Roofline)",
-                      kernel=kname,
-                      achieved=achieved, peak=smem_peak, unit="GB/s", frac=achieved / smem_peak,
-                      traffic=traffic, kernel_ms=kern_avg_ms,
+        roofline=dict(bound="alu", pipe="shared-memory LSU data pipe (DESIGN.md §5 Roofline)",
+                      kernel=kname, achieved=achieved, peak=peak, unit="G node reads/s",
+                      frac=achieved / peak, traffic=traffic, kernel_ms=kern_avg_ms,
                       global_ld_sector_efficiency=sector_eff,
                       path_global_ld_sector_efficiency=path_sector_eff,
-                      units_per_launch=f"{n} samples x {smem_bytes_per_sample:.0f} B "
-                                       f"({visits:.0f} visits x 12 B + {cfg.n_trees} leaves x 8 B)",
-                      peak_source=f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz"),
+                      units_per_launch=f"{n_local} samples x {reads_per_sample:.0f} node reads "
+                                       f"({visits:.0f} internal visits ({visits_src}) + "
+                                       f"{cfg.n_trees} leaf reads)",
+                      peak_source=peak_src, microbench=vp,
+                      bytes_view=dict(achieved_gbs=achieved * 12.0, unit="GB/s",
+                                      note="node reads x 12 B (8 B node + 4 B attribute)")),
         hbm=dict(achieved=hbm_gbs, peak=peaks["hbm_gbs"], unit="GB/s",
                  frac=hbm_gbs / peaks["hbm_gbs"], bytes_per_step=hbm_bytes,
                  peak_source=peaks["source"]),
-        cpu_baseline=cpu,
-        e2e=dict(value=e2e_value, unit=UNIT, h2d_bytes_per_step=n * cfg.n_features * 4,
-                 d2h_bytes_per_step=n * (F.n_out * 4 + 4)),
+        cpu_baseline=cpu, parity=parity,
+        e2e=dict(value=e2e_value, unit=UNIT, h2d_bytes_per_step=n_local * cfg.n_features * 4,
+                 d2h_bytes_per_step=n_local * (F.n_out * 4 + 4)),
         gpu_launches=launches_per_step * args.steps,
         clocks=clocks, wall_s=wall, layout_s=layout_s)
     print(json.dumps(line), flush=True)

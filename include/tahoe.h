@@ -196,6 +196,23 @@ tahoe_status tahoe_predict_host(const tahoe_forest* f, const float* X_host, int6
  */
 tahoe_status tahoe_forest_l2_persist(const tahoe_forest* f, tahoe_stream stream, float hit_ratio);
 
+/* ---------------- hardware parameters (Algorithm 1 line 4) ---------------- */
+
+/*
+ * tahoe_measure_visit_rate — "Measure hardware parameters by a microbenchmark" (Algorithm 1 line
+ * 4), re-targeted to the walk's bound (DESIGN.md §5 Roofline): the node-read rate of
+ * the production coded walk on ideal data (every lane walks `steps` internal nodes of its own
+ * column, perfect lockstep, conflict-free code loads, no tile traffic), one 1024-thread CTA per SM
+ * on all SMs of `device`, `reps` walks per lane.  variant 0: u16 codes, two chains per lane (the
+ * walk of the rank-coded slices); variant 1: u8 codes, four chains per lane (the wide codes).
+ * Writes *node_reads_per_s (node reads = visits, leaf reads included, per second); optionally
+ * *smem_bytes_per_clk (NULL to skip): conflict-free 16-byte shared-memory loads measured with
+ * clock64, bytes per SM clock.  E_INVAL on a bad variant / steps < 2 / odd steps / reps < 1;
+ * E_CUDA on launch failure.  Synchronous (own stream).
+ */
+tahoe_status tahoe_measure_visit_rate(int32_t device, int32_t variant, int32_t steps, int32_t reps,
+                                      double* node_reads_per_s, double* smem_bytes_per_clk);
+
 /* ---------------- tree sharding (multi-GPU) ---------------- */
 
 /* Sub-forest of the trees assigned to `rank` of `world` (balanced by expected visits per tree,

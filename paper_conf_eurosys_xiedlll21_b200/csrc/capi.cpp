@@ -739,6 +739,64 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   TAHOE_GUARD_END
 }
 
+__attribute__((visibility("default"))) tahoe_status tahoe_measure_visit_rate(
+    int32_t device, int32_t variant, int32_t steps, int32_t reps, double* node_reads_per_s,
+    double* smem_bytes_per_clk) {
+  TAHOE_GUARD_BEGIN
+  if (variant < 0 || variant > 1 || steps < 2 || (steps & 1) || steps > 600 || reps < 1 || !node_reads_per_s)
+    return fail(TAHOE_E_INVAL, "bad microbenchmark arguments");
+  DeviceGuard g(device);
+  if (!g.ok) return fail(TAHOE_E_CUDA, "cannot select device");
+  int sms = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+  cudaStream_t st;
+  cudaError_t e = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+  if (e != cudaSuccess) return cuda_fail(e, "stream");
+  double* sink = nullptr;
+  unsigned long long* cyc = nullptr;
+  uint32_t* sink2 = nullptr;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  e = cudaMalloc(&sink, (size_t)sms * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&cyc, (size_t)sms * 8);
+  if (e == cudaSuccess) e = cudaMalloc(&sink2, (size_t)sms * 4);
+  int rc = e == cudaSuccess ? 0 : (int)e;
+  float ms = 0.0f;
+  if (!rc) rc = launch_visit_peak(variant, steps, std::max(1, reps / 8), sms, sink, st);   // warm-up
+  if (!rc) {
+    cudaEventRecord(a, st);
+    rc = launch_visit_peak(variant, steps, reps, sms, sink, st);
+    cudaEventRecord(b, st);
+  }
+  if (!rc) rc = (int)cudaStreamSynchronize(st);
+  if (!rc) {
+    cudaEventElapsedTime(&ms, a, b);
+    *node_reads_per_s = (double)sms * 1024.0 * 2.0 * steps * (double)reps / (ms / 1000.0);
+  }
+  if (!rc && smem_bytes_per_clk) {
+    const int iters = 4096;
+    rc = launch_smem_bw(iters, sms, cyc, sink2, st);
+    if (!rc) rc = (int)cudaStreamSynchronize(st);
+    if (!rc) {
+      std::vector<unsigned long long> c((size_t)sms);
+      rc = (int)cudaMemcpy(c.data(), cyc, (size_t)sms * 8, cudaMemcpyDeviceToHost);
+      double mean = 0.0;
+      for (unsigned long long v : c) mean += (double)v / sms;
+      *smem_bytes_per_clk = 1024.0 * 16.0 * 8.0 * iters / mean;
+    }
+  }
+  cudaFree(sink);
+  cudaFree(cyc);
+  cudaFree(sink2);
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaStreamDestroy(st);
+  if (rc) return cuda_fail((cudaError_t)rc, "microbenchmark");
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
 __attribute__((visibility("default"))) tahoe_status tahoe_forest_shard(
     const tahoe_forest* f, int32_t rank, int32_t world, int32_t device, tahoe_forest** shard) {
   TAHOE_GUARD_BEGIN
@@ -854,7 +912,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
           return r; }() << "]"
      << ",\"n_slices\":" << f->sl.n_slices << ",\"slots_max\":" << f->sl.slots_max
      << ",\"slot_budget\":" << f->slot_budget << ",\"sliced_bytes\":" << f->sl.bytes()
-     << ",\"lockstep_eff\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim
+     << ",\"column_balance_expected\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim
      << ",\"trees_per_lane\":" << f->sl.trees_per_lane << ",\"cost_fitted\":"
      << (cost_params().fitted ? "true" : "false")
      << ",\"num_sms\":" << f->num_sms << ",\"max_smem\":" << f->max_smem << "}";

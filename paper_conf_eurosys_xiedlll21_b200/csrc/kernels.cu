@@ -149,7 +149,7 @@ __global__ void __launch_bounds__(256) k_direct(const DirectKArgs a) {
         if (LEAF) {
           const int32_t tree = __ldg(&a.img.tree_orig[t]);
           const uint32_t leaf = nd.y & 0x7fffffffu;
-          a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
+          if (a.o.out_leaf) a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
           fp += mix64(((uint64_t)(uint32_t)tree << 32) | leaf);
         }
         if (++t == a.img.n_slots) break;
@@ -228,7 +228,7 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
         if (LEAF) {
           const int32_t tree = __ldg(&a.img.tree_orig[t]);
           const uint32_t leaf = nd.y & 0x7fffffffu;
-          a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
+          if (a.o.out_leaf) a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
           fp += mix64(((uint64_t)(uint32_t)tree << 32) | leaf);
         }
       }
@@ -245,7 +245,7 @@ __global__ void __launch_bounds__(BLOCK) k_direct_tiled(const DirectKArgs a, int
           if (LEAF) {
             const int32_t tree = __ldg(&a.img.tree_orig[t]);
             const uint32_t leaf = nd.y & 0x7fffffffu;
-            a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
+            if (a.o.out_leaf) a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
             fp += mix64(((uint64_t)(uint32_t)tree << 32) | leaf);
           }
           if (++t == a.img.n_slots) break;
@@ -519,7 +519,7 @@ __device__ __forceinline__ double walk_columns_leaf(uint32_t p, uint32_t pe, uin
     if ((yy & k.amask) == k.amask) {
       const uint32_t slot_word = (lp - sbase) >> 3;
       const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * slot_word]);
-      a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
+      if (a.o.out_leaf) a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
       fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
     }
   }
@@ -549,7 +549,7 @@ __device__ __forceinline__ double walk_columns_global(uint32_t p, uint32_t pe,
       acc += (double)__uint_as_float(x);
       if (LEAF && delta) {
         const int2 m = *reinterpret_cast<const int2*>(&leaf_meta[2 * ((p - sbase) >> 3)]);
-        a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
+        if (a.o.out_leaf) a.o.out_leaf[i * a.o.T_leaf + m.x] = m.y;
         fp += mix64(((uint64_t)(uint32_t)m.x << 32) | (uint32_t)m.y);
       }
     }
@@ -2380,6 +2380,109 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
   }
   if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
   return 0;
+}
+
+// ------------------------------------------------------------------ microbenchmarks
+// "Measure hardware parameters by a microbenchmark" (Algorithm 1 line 4), re-targeted:
+// the walk is bound by the shared-memory (LSU) data pipe, so the peak it is measured against is the
+// node-read rate of the production walk itself on ideal data — every lane walks a column of L
+// internal nodes (the same node words, the same walk_coded2 / walk_coded8_split code) that all
+// go left, the two half-warps on different slot rows (an 8-byte node load of a warp is 2
+// wavefronts, its minimum), the code loads conflict-free, perfect lockstep, no tile traffic.
+// A warp-step is then 2 wavefronts of node + 1 of code.  VAR 0: u16 codes, two chains per lane
+// (k_sliced_codes); VAR 1: u8 codes over 2 KB rows, four chains per lane (k_sliced_codes8).
+template <int VAR>
+__global__ void __launch_bounds__(1024, 1) k_visit_peak(int32_t L, int32_t reps, double* sink) {
+  extern __shared__ __align__(1024) unsigned char smem[];
+  constexpr int C = kSlicedCols;
+  const int lane = threadIdx.x & 31, col = lane & (C - 1), half = lane >> 4;
+  // two synthetic slices of L + 1 slots (one per half-warp), then the code rows
+  const uint32_t slice_bytes = (uint32_t)(L + 1) * kSlotBytes;
+  uint32_t* w = reinterpret_cast<uint32_t*>(smem);
+  const uint32_t F = VAR == 0 ? 5u : 11u;                       // attribute field bits
+  const uint32_t sh = VAR == 0 ? F + 2 : F + 1;                 // offset shift
+  const uint32_t amask = VAR == 0 ? ((1u << F) - 1u) << 1 : (1u << F) - 1u;
+  const uint32_t dlbit = VAR == 0 ? 1u << (F + 1) : 1u << F;
+  const uint32_t shmul = 1u << (32 - sh);
+  for (uint32_t q = threadIdx.x; q < 2 * (uint32_t)(L + 1) * C; q += blockDim.x) {
+    const uint32_t slot = (q / C) % (uint32_t)(L + 1), c = q % C;
+    const bool term = slot == (uint32_t)L;
+    // internal: rank t larger than every code (left, next slot); attribute: column c's own code
+    // (u16: bytes 2c of a 64-byte row; u8: byte 4c); terminal: self-loop, all-ones attribute
+    const uint32_t attr = VAR == 0 ? (c << 1) : (c << 2);
+    w[2 * q] = term ? 0u : (VAR == 0 ? 0x7FFFu : 127u);
+    w[2 * q + 1] = term ? amask : attr;
+  }
+  unsigned char* rows = smem + 2 * slice_bytes;
+  for (uint32_t q = threadIdx.x; q < 8192 / 4; q += blockDim.x) reinterpret_cast<uint32_t*>(rows)[q] = 0u;
+  __syncthreads();
+  const uint32_t sb = smem_u32(smem) + (uint32_t)half * slice_bytes;
+  const uint32_t p0 = sb + (uint32_t)col * 8u;
+  const uint32_t pe = sb + ((uint32_t)L * C + (uint32_t)col) * 8u;
+  const uint32_t rb = smem_u32(rows);
+  double tot = 0.0;
+  for (int r = 0; r < reps; r++) {
+    double accA, accB;
+    if (VAR == 0) {
+      // chain A rows of the two halves share one 128-byte line (rows u and u+16), chain B likewise
+      const uint32_t rowA = rb + (uint32_t)half * 64u, rowB = rb + 128u + (uint32_t)half * 64u;
+      walk_coded2<false, false>(p0, p0, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+    } else {
+      const uint32_t rowA = rb + (uint32_t)half * 64u, rowB = rb + 2048u + (uint32_t)half * 64u;
+      const uint32_t pm = sb + ((uint32_t)(L / 2) * C + (uint32_t)col) * 8u;
+      walk_coded8_split<false>(p0, pm, pm, p0, pm, pm, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+    }
+    double v = accA + accB;
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    tot += v;
+  }
+  if (tot != 0.0) sink[blockIdx.x] = tot;   // never true (internal words add +0); keeps the walk
+}
+
+// Raw shared-memory load bandwidth: every warp issues conflict-free 16-byte loads (a warp = 512 B =
+// 4 wavefronts) in independent chains; bytes per SM clock from clock64 around the loop.
+__global__ void __launch_bounds__(1024, 1) k_smem_bw(int32_t iters, unsigned long long* cycles, uint32_t* sink) {
+  extern __shared__ __align__(1024) unsigned char smem[];
+  uint4* v = reinterpret_cast<uint4*>(smem);
+  for (int q = threadIdx.x; q < 4096; q += blockDim.x) v[q] = make_uint4(q, q + 1, q + 2, q + 3);
+  __syncthreads();
+  const uint32_t base = smem_u32(smem) + (uint32_t)(threadIdx.x & 31) * 16u;
+  uint32_t acc = 0;
+  const unsigned long long t0 = clock64();
+  for (int i = 0; i < iters; i++) {
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+      uint4 r;
+      asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                   : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                   : "r"(base + (uint32_t)(((i * 8 + k) & 63) * 512)));
+      acc ^= r.x ^ r.w;
+    }
+  }
+  __syncthreads();
+  const unsigned long long t1 = clock64();
+  if (threadIdx.x == 0) cycles[blockIdx.x] = t1 - t0;
+  if (acc == 0x12345678u) sink[blockIdx.x] = acc;
+}
+
+int launch_visit_peak(int32_t variant, int32_t L, int32_t reps, int32_t grid, double* sink, void* stream) {
+  const int smem = 2 * (L + 1) * kSlotBytes + 8192;
+  auto kern = variant == 0 ? k_visit_peak<0> : k_visit_peak<1>;
+  // at least 120 KB of dynamic shared memory: one CTA per SM, as the production walk
+  const int dyn = std::max(smem, 120 * 1024);
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+  if (e != cudaSuccess) return (int)e;
+  kern<<<grid, 1024, dyn, static_cast<cudaStream_t>(stream)>>>(L, reps, sink);
+  return (int)cudaGetLastError();
+}
+
+int launch_smem_bw(int32_t iters, int32_t grid, unsigned long long* cycles, uint32_t* sink, void* stream) {
+  const int dyn = 120 * 1024;
+  cudaError_t e = cudaFuncSetAttribute(k_smem_bw, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+  if (e != cudaSuccess) return (int)e;
+  k_smem_bw<<<grid, 1024, dyn, static_cast<cudaStream_t>(stream)>>>(iters, cycles, sink);
+  return (int)cudaGetLastError();
 }
 
 int launch_finalize(const FinalizeArgs& a, void* stream) {

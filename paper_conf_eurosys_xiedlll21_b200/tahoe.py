@@ -55,7 +55,7 @@ SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_
            "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced", "tahoe_count_visits",
            "tahoe_forest_layout_counts", "tahoe_forest_l2_persist", "tahoe_comm_unique_id",
            "tahoe_comm_init", "tahoe_comm_free", "tahoe_reduce_rows", "tahoe_predict_reduce",
-           "tahoe_reduce_partials")
+           "tahoe_reduce_partials", "tahoe_measure_visit_rate")
 
 
 def lib_path() -> str:
@@ -107,6 +107,7 @@ def load(build_if_missing: bool = True):
         "tahoe_reduce_rows": (st, [i64, i32, i32, i32, P, P]),
         "tahoe_predict_reduce": (st, [P, P, P, i64, i32, i32, P, P, P]),
         "tahoe_reduce_partials": (st, [P, P, i32, i32, i32, i64, P, P, P]),
+        "tahoe_measure_visit_rate": (st, [i32, i32, i32, i32, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -281,6 +282,16 @@ def tahoe_reduce_partials(full, partials, world: int, rank: int, mode: int, n: i
         *[p if isinstance(p, int) else p.data_ptr() for p in partials])
     _check(load().tahoe_reduce_partials(full, arr, world, rank, mode, n, _dev_ptr(out),
                                         _dev_ptr(out_class), _stream_ptr(stream)))
+
+
+def tahoe_measure_visit_rate(device: int = 0, variant: int = 0, steps: int = 256,
+                             reps: int = 400, smem_bw: bool = True) -> tuple[float, float | None]:
+    """(node reads per second of the ideal coded walk, shared-memory bytes per SM clock)."""
+    r = ctypes.c_double()
+    b = ctypes.c_double()
+    _check(load().tahoe_measure_visit_rate(device, variant, steps, reps, ctypes.byref(r),
+                                           ctypes.byref(b) if smem_bw else None))
+    return r.value, (b.value if smem_bw else None)
 
 
 def tahoe_forest_n_outputs(h) -> int:

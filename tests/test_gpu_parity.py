@@ -431,3 +431,29 @@ def test_rank_codes_row_widths(d, monkeypatch):
         monkeypatch.setenv("TAHOE_CODE_BANKS", banks)
         _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, oracle.AGG_SUM, True,
                want_leaf=False)
+
+
+def test_fingerprint_without_leaf_array_every_strategy():
+    """out_fingerprint alone (out_leaf NULL) through every strategy, single and multi-slice,
+    direct image chunked or not: fingerprints equal the oracle's."""
+    for cid, nt, chunk in ((2, 300, None), (3, 280, None), (5, 80, "64")):
+        import os
+        if chunk:
+            os.environ["TAHOE_DIRECT_CHUNK_KB"] = chunk
+        try:
+            f = gen.make_forest(cid, n_trees=nt)
+            F = T.Forest(f, device=0).layout(gen.make_calibration(cid, 4096))
+        finally:
+            os.environ.pop("TAHOE_DIRECT_CHUNK_KB", None)
+        X = gen.make_rows(cid, 40_003)
+        ref = oracle.predict(f, X)
+        dev = torch.device("cuda", 0)
+        Xd = torch.from_numpy(X).to(dev)
+        for s in _strats(F):
+            fp = torch.empty(X.shape[0], dtype=torch.int64, device=dev)
+            out = torch.empty((X.shape[0], F.n_out), dtype=torch.float32, device=dev)
+            F.predict(Xd, out=out, out_fingerprint=fp, force_strategy=s)
+            torch.cuda.synchronize()
+            assert np.array_equal(fp.cpu().numpy().view(np.uint64), ref["fp"]), (cid, s)
+            assert np.array_equal(out.cpu().numpy(), ref["out"]), (cid, s)
+        F.close()

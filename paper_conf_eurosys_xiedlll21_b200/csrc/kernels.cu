@@ -70,22 +70,18 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
       "r"(phase), "r"(20000u)
       : "memory");
 }
-// Ring tickets (ring-wrap guard): s_gen[b] holds the CTA-wide sequence number of the tile last
-// issued into ring buffer b.  A warp that claimed a unit of tile sequence `seq` first waits until
-// the buffer's ticket names seq and only then waits on the buffer's mbarrier phase, so it never
-// waits on a parity that matches a phase two fills behind (a unit of tile seq + 2 * ring could
-// otherwise be claimed while tile seq's refill is still pending, and its parity wait would return
-// at once on the old data).
-__device__ __forceinline__ void wait_ticket(const uint32_t* gen, uint32_t seq, int lane) {
-  if (lane == 0)
-    while (*reinterpret_cast<const volatile uint32_t*>(gen) != seq) {
-    }
-  __syncwarp();
-}
-__device__ __forceinline__ void set_ticket(uint32_t* gen, uint32_t seq) {
-  __threadfence_block();
-  *reinterpret_cast<volatile uint32_t*>(gen) = seq;
-}
+// Ring-wrap guard of the dynamically claimed tile rings (k_sliced, k_sliced_codes): a ring of
+// kRing buffers uses 2 * kRing "full" mbarriers, tile sequence number seq on barrier seq % (2 kRing)
+// with parity (seq / (2 kRing)) & 1.  A warp claiming a unit of tile seq therefore waits on a
+// parity two phases of THAT barrier apart only if tile seq - 2 kRing has not arrived; but then tile
+// seq - kRing (same buffer) cannot have been issued, so the 2 x 16 units of those two tiles are
+// claimed by 32 blocked warps and no warp is left to claim seq (a CTA has 32 warps; a tile has 16
+// units).  With one barrier per buffer a warp could claim tile seq + 2 kRing while tile seq was still
+// held by one slow unit, and its parity wait would return at once on the old data.
+constexpr int kRingBars = 2 * kSlicedRing;
+__device__ __forceinline__ uint32_t ring_bar(uint32_t seq) { return seq % (uint32_t)kRingBars; }
+__device__ __forceinline__ uint32_t ring_parity(uint32_t seq) { return (seq / (uint32_t)kRingBars) & 1u; }
+
 // issue a (possibly > 64 KB) bulk copy in 64 KB pieces on one barrier; caller did expect_tx(total)
 __device__ __forceinline__ void bulk_g2s_big(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   const uint32_t kPiece = 65536;
@@ -599,10 +595,12 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   float* s_ring = reinterpret_cast<float*>(smem + a.forest_smem);
   uint64_t* s_full = reinterpret_cast<uint64_t*>(
       smem + a.forest_smem + (ROWS_SMEM ? (size_t)kRing * a.buf_floats * sizeof(float) : 0));
-  uint64_t* s_forest = s_full + kRing;
-  int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
+  // control block (kSlicedBarrierBytes): [kRingBars] full barriers, the slice barrier, the unit
+  // counter at +64 B, the per-buffer release counters at +72 B
+  uint64_t* s_forest = s_full + kRingBars;
   unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
-  uint32_t* s_gen = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(s_full) + 72);  // [kRing] tickets
+  int* s_cnt = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(s_full) + 72);
+  static_assert(8 * (kRingBars + 1) <= 64 && 72 + 4 * kRing <= kSlicedBarrierBytes, "control block");
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int nwarps = blockDim.x >> 5;
@@ -623,7 +621,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   if (threadIdx.x == 0) {
     // full barriers: one arrive.expect_tx per TMA fill, or 32 cp.async arrivals (misaligned X)
     const uint32_t arrivals = (ROWS == kRowsDense && !a.x_aligned) ? 32u : 1u;
-    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], arrivals); s_cnt[b] = 0; s_gen[b] = 0xffffffffu; }
+    for (int b = 0; b < kRingBars; b++) mbar_init(&s_full[b], arrivals);
+    for (int b = 0; b < kRing; b++) s_cnt[b] = 0;
     *s_next = 0ull;
     mbar_init(s_forest, 1);
     fence_mbar_init();
@@ -635,16 +634,17 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
   auto issue_tile = [&](int64_t tile, int b, uint32_t seq) {
     const int64_t r0 = tile * R;
     float* dst = s_ring + (size_t)b * a.buf_floats;
+    uint64_t* bar = &s_full[ring_bar(seq)];
     if (PADDED) {
       // one 2-D tensor copy: box [row_stride][R] at (0, r0); columns >= d and rows >= n are
       // zero-filled by the TMA unit and still counted in the transaction bytes
       if (lane == 0) {
         fence_proxy_async_smem();
-        mbar_expect_tx(&s_full[b], (uint32_t)(R * rs * sizeof(float)));
+        mbar_expect_tx(bar, (uint32_t)(R * rs * sizeof(float)));
         asm volatile(
             "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
             " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_u32(dst)),
-            "l"(reinterpret_cast<uint64_t>(&a.tmap)), "r"(0), "r"((int32_t)r0), "r"(smem_u32(&s_full[b]))
+            "l"(reinterpret_cast<uint64_t>(&a.tmap)), "r"(0), "r"((int32_t)r0), "r"(smem_u32(bar))
             : "memory");
       }
     } else {
@@ -656,8 +656,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
           const uint32_t body = bytes & ~15u;
           for (uint32_t q = body / 4; q < bytes / 4; q++) dst[q] = __ldg(&src[q]);  // <= 3 floats
           fence_proxy_async_smem();
-          mbar_expect_tx(&s_full[b], body);
-          if (body) bulk_g2s_big(dst, src, body, &s_full[b]);
+          mbar_expect_tx(bar, body);
+          if (body) bulk_g2s_big(dst, src, body, bar);
         }
       } else {
         // misaligned X: 4-byte cp.async copies by the warp, each lane's completion counted on the
@@ -666,12 +666,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         for (uint32_t q = lane; q < cnt; q += 32)
           asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst + q)), "l"(src + q)
                        : "memory");
-        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(&s_full[b]))
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar))
                      : "memory");
       }
     }
-    __syncwarp();
-    if (lane == 0) set_ticket(&s_gen[b], seq);
     __syncwarp();
   };
 
@@ -718,10 +716,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
     if (!LEAF) {
       // Dynamic schedule over work units of 4 rows {u, u+16, u+32, u+48} of a 64-row tile: half h
       // of the warp walks rows u+16h (chain A) and u+32+16h (chain B).  Warps grab units from a CTA
-      // counter, so a slow unit delays nobody.  Claims are not bounded by the ring: while one slow
-      // unit holds tile T, other warps may finish T+1, T+2, T+4, T+5 and claim T+6 (buffer and
-      // parity of T), so a claim waits for the buffer's ticket before its mbarrier phase
-      // (wait_ticket).  Rows too wide to stage are read from global memory with the same schedule.
+      // counter, so a slow unit delays nobody (claims may run ahead of the ring: see ring_bar).
+      // Rows too wide to stage are read from global memory with the same schedule.
       constexpr int kUnits = kSlicedTileRows / 4;
       const uint64_t total = (uint64_t)my_tiles * kUnits;
       for (;;) {
@@ -735,10 +731,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         const int b = (int)(gt % kRing);
         const int64_t r0 = (t0 + it * ts) * R;
         const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-        if (ROWS_SMEM) {
-          wait_ticket(&s_gen[b], gt, lane);
-          mbar_wait(&s_full[b], (gt / kRing) & 1u);
-        }
+        if (ROWS_SMEM) mbar_wait(&s_full[ring_bar(gt)], ring_parity(gt));
         if (u < nr) {
           const int rA = u + 16 * half, rB = rA + 32;
           const bool okA = rA < nr, okB = rB < nr;
@@ -784,7 +777,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced(const __grid_constant__ Slic
         const int64_t r0 = tile * R;
         const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
         const float* tbuf = s_ring + (size_t)b * a.buf_floats;
-        if (ROWS_SMEM) mbar_wait(&s_full[b], (g / kRing) & 1u);
+        if (ROWS_SMEM) mbar_wait(&s_full[ring_bar(g)], ring_parity(g));
         for (int r = warp; r < (int)(R / 2); r += nwarps) {
           const int rr = r + 32 * half;
           const bool ok = rr < nr;
@@ -1143,10 +1136,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   extern __shared__ __align__(1024) unsigned char smem[];
   unsigned char* s_ring = smem + a.forest_smem;
   uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)kRing * a.tstride);
-  uint64_t* s_forest = s_full + kRing;
-  int* s_cnt = reinterpret_cast<int*>(s_forest + 1);
+  // control block as k_sliced's (ring_bar: 2 x kRing full barriers)
+  uint64_t* s_forest = s_full + kRingBars;
   unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
-  uint32_t* s_gen = reinterpret_cast<uint32_t*>(reinterpret_cast<unsigned char*>(s_full) + 72);  // [kRing] tickets
+  int* s_cnt = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(s_full) + 72);
   // slice partials of the tiles in the ring, written out coalesced by the warp closing a tile
   double* s_part = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_full) + kSlicedBarrierBytes);
   const int lane = threadIdx.x & 31;
@@ -1164,14 +1157,15 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   const int64_t ntiles = (a.n + R - 1) / R;
 
   if (threadIdx.x == 0) {
-    for (int b = 0; b < kRing; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; s_gen[b] = 0xffffffffu; }
+    for (int b = 0; b < kRingBars; b++) mbar_init(&s_full[b], 1);
+    for (int b = 0; b < kRing; b++) s_cnt[b] = 0;
     *s_next = 0ull;
     mbar_init(s_forest, 1);
     fence_mbar_init();
   }
   __syncthreads();
 
-  // stage tile `tile` (CTA-wide sequence number seq) into buffer b, then publish the ticket
+  // stage tile `tile` (CTA-wide sequence number seq) into buffer b (barrier ring_bar(seq))
   auto issue_tile = [&](int64_t tile, int b, uint32_t seq, int64_t ahead = -1) {
     if (lane == 0) {
       // optional L2 prefetch of this CTA's tile `ahead` (a later tile of its sequence)
@@ -1179,11 +1173,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
                      "r"((uint32_t)a.tstride) : "memory");
       fence_proxy_async_smem();
-      mbar_expect_tx(&s_full[b], (uint32_t)a.tstride);
+      mbar_expect_tx(&s_full[ring_bar(seq)], (uint32_t)a.tstride);
       bulk_g2s(s_ring + (size_t)b * a.tstride,
                reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride,
-               (uint32_t)a.tstride, &s_full[b]);
-      set_ticket(&s_gen[b], seq);
+               (uint32_t)a.tstride, &s_full[ring_bar(seq)]);
     }
     __syncwarp();
   };
@@ -1269,8 +1262,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
       const int64_t tile = t0 + it * ts;
       const int64_t r0 = tile * R;
       const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-      wait_ticket(&s_gen[b], gt, lane);
-      mbar_wait(&s_full[b], (gt / kRing) & 1u);
+      mbar_wait(&s_full[ring_bar(gt)], ring_parity(gt));
       if (u < nr) {
         const int rA = u + 16 * half, rB = rA + 32;
         const bool okA = rA < nr, okB = rB < nr;

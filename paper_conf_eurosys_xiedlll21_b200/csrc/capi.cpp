@@ -76,14 +76,13 @@ static cudaError_t scratch_alloc(void** p, size_t bytes, cudaStream_t st) {
 static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
   const int32_t fb = feature_bits(n_features + 1);
   const bool padded = n_features % 4 == 0;   // predict with d == n_features takes the 2-D TMA path
-  int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb, padded));
-  // forests that can take the u16 rank codes (reading R7) keep room for their code-tile ring and
-  // staged partials too (rows of ~100-127 attributes are too wide for the fp32 ring, which would
-  // otherwise leave the whole of shared memory to the slice)
-  if (fb <= kCodeMaxFbits)
-    ring = std::max<int64_t>(ring, (int64_t)kSlicedRing * code_tile_stride(fb) + (int64_t)kSlicedRing * kSlicedTileRows * 8);
+  int64_t ring = std::max<int64_t>(0, sliced_ring_bytes(n_features, fb, padded)) + kSlicedBarrierBytes;
+  // forests that can take the u16 rank codes (reading R7) keep room for their (minimum, 3-deep)
+  // code-tile ring, control block and staged partials too (rows of ~100-127 attributes are too wide
+  // for the fp32 ring, which would otherwise leave the whole of shared memory to the slice)
+  if (fb <= kCodeMaxFbits) ring = std::max<int64_t>(ring, coded_ring_smem(kSlicedRing, code_tile_stride(fb)));
   // the slice region is rounded up to 1 KB so the ring's row bases stay aligned
-  return (int32_t)std::max<int64_t>(0, ((max_smem - ring - kSlicedBarrierBytes) & ~1023LL) / kSlotBytes);
+  return (int32_t)std::max<int64_t>(0, ((max_smem - ring) & ~1023LL) / kSlotBytes);
 }
 
 static void free_device(tahoe_forest* f) {
@@ -348,7 +347,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   if (strat == TAHOE_STRATEGY_SLICED_CODED && !f->sl.code8) {
     // the code-tile ring (+ trailers and staged partials) must fit next to the slice
     const int64_t need = (((int64_t)f->sl.slots_max * kSlotBytes + 1023) & ~1023LL) +
-                         3LL * code_tile_stride(f->sl.fbits) + kSlicedBarrierBytes + 3LL * kSlicedTileRows * 8;
+                         coded_ring_smem(kSlicedRing, code_tile_stride(f->sl.fbits));
     if (need > f->max_smem) {
       if (forced == TAHOE_STRATEGY_SLICED_CODED)
         return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices: code-tile ring does not fit shared memory");

@@ -1034,8 +1034,17 @@ struct CodedKArgs {
   int32_t cps;           // CTAs per slice (single-pass, no cta_start)
   const int32_t* cta_start;  // or: slice s is worked by CTAs [cta_start[s], cta_start[s+1])
   int32_t prefetch;      // entries of the CTA's tile sequence to prefetch into L2 ahead (0 = none)
+  int32_t ring;          // ring depth (kSlicedRing .. kCodedRingMax): as many tiles as shared memory holds
+  uint32_t ring_m, bars_m;   // ceil(2^32 / ring), ceil(2^32 / (2 ring)): division by multiply-high
   OutArgs o;
 };
+
+// x / d and x % d for a small runtime divisor d (<= 16) and x < 2^24: q = umulhi(x, ceil(2^32 / d))
+// is exact there (error term x (m d - 2^32) / 2^32 < x d / 2^32 < 1 / d)
+__device__ __forceinline__ uint32_t fdiv_small(uint32_t x, uint32_t m) { return __umulhi(x, m); }
+__device__ __forceinline__ uint32_t fmod_small(uint32_t x, uint32_t d, uint32_t m) {
+  return x - __umulhi(x, m) * d;
+}
 
 // One step on a coded slice: node {x = t or leaf value, y}, attribute code at (y & amask) | row,
 // left iff code < t (NaN-aware: or NaN and default-left), right / next root at +(y >> (F+2)).
@@ -1135,13 +1144,17 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
   unsigned char* s_ring = smem + a.forest_smem;
-  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)kRing * a.tstride);
-  // control block as k_sliced's (ring_bar: 2 x kRing full barriers)
-  uint64_t* s_forest = s_full + kRingBars;
-  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_full) + 8;  // +64 B
-  int* s_cnt = reinterpret_cast<int*>(reinterpret_cast<unsigned char*>(s_full) + 72);
+  // ring depth: a.ring buffers, 2 * a.ring full barriers (the ring-wrap guard of ring_bar, with the
+  // depth a runtime value here)
+  const uint32_t ring = (uint32_t)a.ring, nbars = 2u * ring;
+  // control block (kCodedCtlBytes): [2 ring] full barriers, slice barrier, unit counter (u32),
+  // [ring] release counters
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)ring * a.tstride);
+  uint64_t* s_forest = s_full + nbars;
+  unsigned int* s_next = reinterpret_cast<unsigned int*>(s_forest + 1);
+  int* s_cnt = reinterpret_cast<int*>(s_next + 1);
   // slice partials of the tiles in the ring, written out coalesced by the warp closing a tile
-  double* s_part = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_full) + kSlicedBarrierBytes);
+  double* s_part = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_full) + kCodedCtlBytes);
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
   const int col = lane & (C - 1);
@@ -1157,9 +1170,9 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   const int64_t ntiles = (a.n + R - 1) / R;
 
   if (threadIdx.x == 0) {
-    for (int b = 0; b < kRingBars; b++) mbar_init(&s_full[b], 1);
-    for (int b = 0; b < kRing; b++) s_cnt[b] = 0;
-    *s_next = 0ull;
+    for (uint32_t b = 0; b < nbars; b++) mbar_init(&s_full[b], 1);
+    for (uint32_t b = 0; b < ring; b++) s_cnt[b] = 0;
+    *s_next = 0u;
     mbar_init(s_forest, 1);
     fence_mbar_init();
   }
@@ -1173,15 +1186,15 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
                      "r"((uint32_t)a.tstride) : "memory");
       fence_proxy_async_smem();
-      mbar_expect_tx(&s_full[ring_bar(seq)], (uint32_t)a.tstride);
+      mbar_expect_tx(&s_full[fmod_small(seq, nbars, a.bars_m)], (uint32_t)a.tstride);
       bulk_g2s(s_ring + (size_t)b * a.tstride,
                reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride,
-               (uint32_t)a.tstride, &s_full[ring_bar(seq)]);
+               (uint32_t)a.tstride, &s_full[fmod_small(seq, nbars, a.bars_m)]);
     }
     __syncwarp();
   };
   // after one work unit: the warp finishing the tile's last unit writes the tile's 64 slice
-  // partials (two coalesced 256-byte stores) and refills the buffer with the tile kRing ahead
+  // partials (two coalesced 256-byte stores) and refills the buffer with the tile `ring` ahead
   auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts,
                      int sl, int64_t r0, int nr, uint32_t seq) {
     __syncwarp();
@@ -1194,8 +1207,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     last = __shfl_sync(0xffffffffu, last, 0);
     if (!last) return;
     if (FUSED) {
-      if (it + kRing < my_tiles)
-        issue_tile(t0 + (it + kRing) * ts, b, seq + (uint32_t)kRing, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
+      if (it + ring < my_tiles)
+        issue_tile(t0 + (it + ring) * ts, b, seq + ring, a.prefetch ? t0 + (it + ring + a.prefetch) * ts : -1);
       return;
     }
     // take the tile's 64 partials out of shared memory, refill the buffer at once, then store the
@@ -1205,8 +1218,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     const double* sp = s_part + b * kSlicedTileRows;
     const double p0 = lane < nr ? sp[lane] : 0.0, p1 = lane + 32 < nr ? sp[lane + 32] : 0.0;
     __syncwarp();
-    if (it + kRing < my_tiles)
-      issue_tile(t0 + (it + kRing) * ts, b, seq + (uint32_t)kRing, a.prefetch ? t0 + (it + kRing + a.prefetch) * ts : -1);
+    if (it + ring < my_tiles)
+      issue_tile(t0 + (it + ring) * ts, b, seq + ring, a.prefetch ? t0 + (it + ring + a.prefetch) * ts : -1);
     double* dst = a.o.raw + (size_t)sl * a.n + r0;
     if (lane < nr) dst[lane] = p0;
     if (lane + 32 < nr) dst[lane + 32] = p1;
@@ -1237,8 +1250,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         mbar_expect_tx(s_forest, bytes);
         bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
-      for (int64_t q = 0; q < kRing && q < my_tiles; q++)
-        issue_tile(t0 + q * ts, (int)((g + q) % kRing), g + (uint32_t)q);
+      for (int64_t q = 0; q < (int64_t)ring && q < my_tiles; q++)
+        issue_tile(t0 + q * ts, (int)fmod_small(g + (uint32_t)q, ring, a.ring_m), g + (uint32_t)q);
     }
     const uint32_t sbase = smem_u32(smem);
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
@@ -1251,18 +1264,18 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     constexpr int kUnits = kSlicedTileRows / 4;
     const uint64_t total = (uint64_t)my_tiles * kUnits;
     for (;;) {
-      unsigned long long q = 0;
-      if (lane == 0) q = atomicAdd(s_next, 1ull);
+      uint32_t q = 0;
+      if (lane == 0) q = atomicAdd(s_next, 1u);   // 32-bit: a native ATOMS.ADD (64-bit was a CAS loop)
       q = __shfl_sync(0xffffffffu, q, 0);
-      if (q >= total) break;
+      if ((uint64_t)q >= total) break;
       const int64_t it = (int64_t)(q / kUnits);
       const int u = (int)(q % kUnits);
       const uint32_t gt = g + (uint32_t)it;
-      const int b = (int)(gt % kRing);
+      const int b = (int)fmod_small(gt, ring, a.ring_m);
       const int64_t tile = t0 + it * ts;
       const int64_t r0 = tile * R;
       const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-      mbar_wait(&s_full[ring_bar(gt)], ring_parity(gt));
+      mbar_wait(&s_full[fmod_small(gt, nbars, a.bars_m)], fdiv_small(gt, a.bars_m) & 1u);
       if (u < nr) {
         const int rA = u + 16 * half, rB = rA + 32;
         const bool okA = rA < nr, okB = rB < nr;
@@ -1313,7 +1326,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     }
     g += (uint32_t)my_tiles;
     __syncthreads();
-    if (threadIdx.x == 0) *s_next = 0ull;
+    if (threadIdx.x == 0) *s_next = 0u;
     __syncthreads();
   }
 }
@@ -1725,8 +1738,14 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   a.cta_start = plan.cta_start;
   a.prefetch = std::getenv("TAHOE_CODES_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODES_PREFETCH")) : 0;
   a.o = o;
-  const int smem = plan.forest_smem + kRing * tstride + kSlicedBarrierBytes +
-                   kRing * kSlicedTileRows * (int)sizeof(double);
+  // ring depth: every tile the shared memory next to the slice holds (3 .. kCodedRingMax); a deeper
+  // ring lets the warps that claimed the next tile's units work instead of sleeping on its copy
+  a.ring = coded_ring_depth(plan.forest_smem, tstride);
+  if (const char* e = std::getenv("TAHOE_CODES_RING"))   // experiments (capped by what fits)
+    a.ring = std::max(kSlicedRing, std::min(a.ring, std::atoi(e)));
+  a.ring_m = (uint32_t)((0x100000000ULL + a.ring - 1) / a.ring);
+  a.bars_m = (uint32_t)((0x100000000ULL + 2 * a.ring - 1) / (2 * a.ring));
+  const int smem = plan.forest_smem + coded_ring_smem(a.ring, tstride);
   // rows of >= 128 bytes are stored swizzled (code_slot_swz); the others keep the plain walk;
   // leaf ids / fingerprints take the LEAF instantiation of the same walk
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;

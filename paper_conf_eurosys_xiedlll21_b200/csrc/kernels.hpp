@@ -159,6 +159,18 @@ constexpr int32_t kSlotBytes = kSlicedCols * 8;  // one slot row: 16 columns x 8
 constexpr int32_t kSlicedRing = 3;          // sample-tile ring depth of k_sliced
 constexpr int32_t kSlicedTileRows = 64;     // rows per tile (two per warp of a 1024-thread CTA)
 constexpr int32_t kSlicedBarrierBytes = 128;
+// rank-coded slices (k_sliced_codes): ring of `ring` code tiles (3 .. kCodedRingMax, as many as fit),
+// a control block, `ring` x 64 staged fp64 partials
+constexpr int32_t kCodedRingMax = 8;
+constexpr int32_t kCodedCtlBytes = 256;
+inline int32_t coded_ring_smem(int32_t ring, int32_t tstride) {
+  return ring * tstride + kCodedCtlBytes + ring * kSlicedTileRows * 8;
+}
+inline int32_t coded_ring_depth(int32_t forest_smem, int32_t tstride) {
+  int32_t r = kCodedRingMax;
+  while (r > kSlicedRing && forest_smem + coded_ring_smem(r, tstride) > kMaxSmemOptin) r--;
+  return r;
+}
 
 // PADDED staging: rows at a stride that is a multiple of 2^fbits floats (>= d, >= 4), so that row
 // bases are aligned to the attribute byte-offset field and a leaf's all-ones attribute stays

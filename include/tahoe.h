@@ -57,19 +57,26 @@ typedef enum {
   TAHOE_STRATEGY_SLICED = 1,  /* lane = tree; forest slices resident in shared memory, sample
                                  tiles staged by TMA ("shared forest" / "splitting shared
                                  forest")                                        */
-  TAHOE_STRATEGY_SLICED_CODED = 2  /* SLICED over exact rank codes of the attributes (DESIGN.md
+  TAHOE_STRATEGY_SLICED_CODED = 2, /* SLICED over exact rank codes of the attributes (DESIGN.md
                                  reading R7; same results bit for bit): a pre-pass turns each
                                  row into u16 codes, the slices compare codes with threshold
                                  ranks.  AUTO takes it instead of SLICED when the forest
                                  qualifies (<= 127 attributes, <= 32000 distinct thresholds per
-                                 attribute, no subnormal leaf value) and no leaf ids or
-                                 fingerprints are requested; forcing it otherwise returns
-                                 E_UNSUPPORTED.  Forests over more than 127 attributes get the
+                                 attribute, no subnormal leaf value); leaf ids and fingerprints
+                                 come from the same walk's diagnostic instantiation; forcing it
+                                 on a forest that does not qualify returns E_UNSUPPORTED.
+                                 Forests over more than 127 attributes get the
                                  WIDE codes instead (reading R8): u8 codes over virtual
                                  attributes (<= 127 thresholds each), 2^V-byte code rows staged
                                  in shared memory next to slices packed for that room; they
                                  qualify while the used attributes need <= 4 KB rows and every
                                  tree fits the smaller lane column                            */
+  TAHOE_STRATEGY_ROWS = 3     /* small batches (the paper's batch-100 workload
+                                 P:1714-1717): one CTA per sample, lane = tree over the direct
+                                 image, fixed-order block reduction and finalize in the same
+                                 kernel (one launch, no scratch: CUDA-graph capturable).  Needs
+                                 4 d + 4 n_trees + 512 bytes of shared memory (E_UNSUPPORTED
+                                 when forced beyond that)                                     */
 } tahoe_strategy;
 
 /*

@@ -93,6 +93,7 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->dd.cls);
   cudaFree((void*)f->dd.tree_orig);
   cudaFree((void*)f->dd.slot_orig);
+  cudaFree((void*)f->dd.cls_seg);
   cudaFree((void*)f->ds.nodes);
   cudaFree((void*)f->ds.col_len);
   cudaFree((void*)f->ds.slots);
@@ -176,6 +177,7 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
   if ((st = upload(f->di.cls, &f->dd.cls)) != TAHOE_OK) return st;
   if ((st = upload(f->di.tree_orig, &f->dd.tree_orig)) != TAHOE_OK) return st;
   if ((st = upload(f->di.slot_orig, &f->dd.slot_orig)) != TAHOE_OK) return st;
+  if ((st = upload(f->di.cls_seg, &f->dd.cls_seg)) != TAHOE_OK) return st;
   f->dd.n_slots = (int32_t)f->di.root.size();
   f->dd.fbits = f->di.fbits;
   f->dd.n_nodes = (int64_t)f->di.nodes.size() / 2;
@@ -288,6 +290,10 @@ static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   st.sliced_eff = f->sl.eff_sim;
   st.n_slices = f->sl.n_slices;
   st.num_sms = f->num_sms;
+  st.n_trees = (int32_t)f->di.root.size();
+  const int64_t rs = rows_smem_bytes(d, st.n_trees);
+  st.rows_ok = rs <= (int64_t)f->max_smem - 1024;
+  st.rows_per_sm = (int32_t)std::max<int64_t>(1, std::min<int64_t>(4, 232448 / (rs + 1024)));
   return st;
 }
 
@@ -297,6 +303,7 @@ static int32_t choose(const tahoe_forest* f, int64_t n, int32_t d, int32_t force
     if (env && *env) forced = std::atoi(env);
   }
   if (forced == TAHOE_STRATEGY_DIRECT) return TAHOE_STRATEGY_DIRECT;
+  if (forced == TAHOE_STRATEGY_ROWS) return plan_stats(f, d).rows_ok ? TAHOE_STRATEGY_ROWS : -4;
   if (forced == TAHOE_STRATEGY_SLICED) return f->sl.valid ? TAHOE_STRATEGY_SLICED : -2;
   if (forced == TAHOE_STRATEGY_SLICED_CODED)
     return !f->sl.valid ? -2 : (f->ds.cnodes ? TAHOE_STRATEGY_SLICED_CODED : -3);
@@ -344,6 +351,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   int32_t strat = choose(f, n, d, forced);
   if (strat == -2) return fail(TAHOE_E_UNSUPPORTED, "sliced strategy unavailable: " + f->sl.why_invalid);
   if (strat == -3) return fail(TAHOE_E_UNSUPPORTED, "rank-coded slices unavailable: " + f->sl.code_why);
+  if (strat == -4) return fail(TAHOE_E_UNSUPPORTED, "rows strategy: row + per-tree values exceed shared memory");
   if (strat == TAHOE_STRATEGY_SLICED_CODED && !f->sl.code8) {
     // the code-tile ring (+ trailers and staged partials) must fit next to the slice
     const int64_t need = (((int64_t)f->sl.slots_max * kSlotBytes + 1023) & ~1023LL) +
@@ -376,6 +384,14 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
   fa.out_class = out_class;
   fa.raw_out = raw_user;
   const bool scalar = C == 1 && H.agg != TAHOE_AGG_VOTE;
+  if (strat == TAHOE_STRATEGY_ROWS) {   // one launch: walk + combine + finalize (or raw sums)
+    o.raw = raw_user;
+    if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
+    const int rc = launch_rows(f->dd, X, n, d, o, f->num_sms, st);
+    if (ev_e) cudaEventRecord(static_cast<cudaEvent_t>(ev_e), st);
+    if (rc) return cuda_fail((cudaError_t)rc, "rows kernel");
+    return TAHOE_OK;
+  }
   if (strat == TAHOE_STRATEGY_DIRECT) {
     const size_t nchunks = f->direct_chunks.size() - 1;
     if (scalar && !raw_user && nchunks == 1) {
@@ -914,6 +930,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"column_balance_expected\":" << f->sl.eff << ",\"lockstep_eff_sim\":" << f->sl.eff_sim
      << ",\"trees_per_lane\":" << f->sl.trees_per_lane << ",\"cost_fitted\":"
      << (cost_params().fitted ? "true" : "false")
+     << ",\"rows_ok\":" << (plan_stats(f).rows_ok ? "true" : "false")
      << ",\"num_sms\":" << f->num_sms << ",\"max_smem\":" << f->max_smem << "}";
   std::string s = js.str();
   if ((int64_t)s.size() + 1 > len) return fail(TAHOE_E_INVAL, "buffer too small");

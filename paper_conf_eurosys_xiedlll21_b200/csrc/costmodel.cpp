@@ -1,5 +1,5 @@
 // costmodel.cpp — per-batch strategy choice (Algorithm 1 lines 8-13; Eq. 1-7
-// reconstructed in SURVEY Appendix A), re-targeted to the two B200 strategies.
+// reconstructed in SURVEY Appendix A), re-targeted to the B200 strategies.
 //
 // Eq. 1 (T = T_SMEM + T_GMEM + T_B_REDU + T_G_REDU) becomes, per batch of n rows:
 //   sliced : T = a_s + b_s * U_s * (rows in global memory ? g_s : 1),
@@ -11,7 +11,10 @@
 //            L1/L2-throughput-bound above it (T_GMEM);
 //   coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs
 //            the rank-coded slices (reading R7): the same busiest-CTA node reads at a cheaper
-//            per-read cost b_c, plus the row-coding pre-pass (passes of 32 attributes per row).
+//            per-read cost b_c, plus the row-coding pre-pass (passes of 32 attributes per row);
+//   rows   : T = a_r + b_r * waves * ceil(T_trees / 512) * V / T_trees
+//            one CTA per sample (small batches): waves of one-row CTAs, each as long as the
+//            longest chain of dependent node reads of one thread (L2 latency per read).
 // V = expected node reads per sample (calibrated E[path] + 1 leaf read, summed over trees,
 // reading Z16).  The constants are fitted on the chip by scripts/fit_costmodel.py and read from
 // costmodel_b200.json next to libtahoe.so (or $TAHOE_COSTMODEL); defaults are round-1 B200
@@ -74,6 +77,8 @@ const CostParams& cost_params() {
     if (read_key(js, "a_w", &v)) c.a_w = v;
     if (read_key(js, "b_w", &v)) c.b_w = v;
     if (read_key(js, "e_w", &v)) c.e_w = v;
+    if (read_key(js, "a_r", &v)) c.a_r = v;
+    if (read_key(js, "b_r", &v)) c.b_r = v;
     c.fitted = all;
     return c;
   }();
@@ -99,15 +104,27 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
     return c.a_s + c.b_s * U * (st.rows_global ? c.g_s : 1.0);
   }
   const double sms = st.num_sms > 0 ? st.num_sms : 148;
+  if (strategy == TAHOE_STRATEGY_ROWS) {
+    // rows: waves of one-row CTAs; a wave lasts the longest tree chain of a thread:
+    // ceil(T / 512) trees of mean path V / T dependent node reads each (L2 latency b_r)
+    if (!st.rows_ok) return INFINITY;
+    const double waves = std::ceil((double)n / (sms * std::max(1, st.rows_per_sm)));
+    const double chain = std::ceil((double)st.n_trees / kRowsThreads) * st.V / std::max(1, st.n_trees);
+    return c.a_r + c.b_r * waves * chain;
+  }
   const double g = st.wide_rows ? c.g_d : 1.0;
   return c.a_d + g * std::max(c.l_d * st.V, c.b_d * st.V * (double)n / sms);
 }
 
 int32_t select_strategy(const PlanStats& st, int64_t n, int32_t d, int32_t agg) {
   (void)d;
-  if (agg == TAHOE_AGG_VOTE || !st.sliced_ok) return TAHOE_STRATEGY_DIRECT;
   int32_t best = TAHOE_STRATEGY_DIRECT;
   double tb = predict_us(st, TAHOE_STRATEGY_DIRECT, n);
+  {
+    const double t = predict_us(st, TAHOE_STRATEGY_ROWS, n);
+    if (t < tb) { tb = t; best = TAHOE_STRATEGY_ROWS; }
+  }
+  if (agg == TAHOE_AGG_VOTE || !st.sliced_ok) return best;
   for (int32_t s : {TAHOE_STRATEGY_SLICED, TAHOE_STRATEGY_SLICED_CODED}) {
     const double t = predict_us(st, s, n);
     if (t < tb) { tb = t; best = s; }

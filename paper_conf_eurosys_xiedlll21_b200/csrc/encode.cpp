@@ -69,6 +69,10 @@ tahoe_status encode_direct(const Forest& F, DirectImage& D) {
     }
     base += (int64_t)pre.size();
   }
+  // trees are class-major (F.order), so each class's tree slots are one contiguous range
+  D.cls_seg.assign(F.n_classes + 1, 0);
+  for (int32_t c : D.cls) D.cls_seg[c + 1]++;
+  for (int32_t c = 0; c < F.n_classes; c++) D.cls_seg[c + 1] += D.cls_seg[c];
   return TAHOE_OK;
 }
 

@@ -126,6 +126,7 @@ struct DirectImage {
   std::vector<uint32_t> nodes;        // [N*2]
   std::vector<int32_t> root, cls, tree_orig;
   std::vector<int32_t> slot_orig;     // caller node id per node slot
+  std::vector<int32_t> cls_seg;       // [n_classes + 1]: tree slots of class c are [cls_seg[c], cls_seg[c+1])
   int64_t bytes() const { return (int64_t)nodes.size() * 4; }
 };
 
@@ -147,6 +148,9 @@ struct PlanStats {
   bool coded_ok = false;     // rank-coded twin available and enabled (reading R7)
   int32_t code_passes = 1;   // row-coding passes of 32 attributes
   bool code8 = false;        // the coded twin is the wide-code one (reading R8)
+  bool rows_ok = false;      // the ROWS strategy fits shared memory (row + per-tree values)
+  int32_t rows_per_sm = 1;   // resident ROWS CTAs per SM
+  int32_t n_trees = 1;
 };
 // Fitted per-platform constants (costmodel_b200.json, scripts/fit_costmodel.py), microseconds.
 struct CostParams {
@@ -156,6 +160,7 @@ struct CostParams {
   double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
   double a_c = 30.0, b_c = 6.6e-5, e_c = 1.6e-5; // coded: launches; per unit; per row-pass per SM
   double a_w = 40.0, b_w = 1.5e-4, e_w = 1.6e-5; // wide codes (reading R8): the same three terms
+  double a_r = 8.0, b_r = 0.7;                    // rows (f1): launch; per dependent node read of a wave
   bool fitted = false;
 };
 const CostParams& cost_params();

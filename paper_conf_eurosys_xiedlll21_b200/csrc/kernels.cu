@@ -2393,6 +2393,131 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
   return 0;
 }
 
+// ------------------------------------------------------------------ ROWS strategy (f1)
+// Small batches (the paper's low-parallelism workload, batch 100): the sliced
+// strategies stage a ~200 KB slice per CTA and need a finalize launch, which dominates a 100-row
+// batch.  Here a CTA takes one sample: it stages the row in shared memory, each thread walks trees
+// j = tid, tid + B, ... of the DIRECT image (hot child next; kept L2-resident across
+// calls by tahoe_forest_l2_persist) and parks the tree's leaf value in shared memory; then every
+// class's fp64 sum is formed by a fixed-order block reduction (each thread a contiguous chunk of the
+// class's tree slots, then a fixed butterfly), and the block finalises the row (reading Z14/Z17).
+// One launch, no scratch: CUDA-graph capturable.
+__device__ __forceinline__ double block_sum_fixed(double v, double* red) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = blockDim.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  __syncthreads();
+  if (lane == 0) red[warp] = v;
+  __syncthreads();
+  double t = lane < W ? red[lane] : 0.0;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+  return t;   // every lane of every warp: the same bits
+}
+
+template <bool LEAF>
+__global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  float* s_row = reinterpret_cast<float*>(smem);
+  float* s_val = reinterpret_cast<float*>(smem + ((size_t)a.d * 4 + 15) / 16 * 16);
+  double* s_red = reinterpret_cast<double*>(s_val + a.img.n_slots);
+  __shared__ unsigned long long s_fp[kRowsThreads / 32];
+  const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(a.img.nodes);
+  const int fbits = a.img.fbits;
+  const uint32_t fmask = (1u << fbits) - 1u;
+  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const int32_t T = a.img.n_slots, C = a.o.n_classes, B = blockDim.x;
+  const bool vote = a.o.agg == TAHOE_AGG_VOTE;
+  for (int64_t i = blockIdx.x; i < a.n; i += gridDim.x) {
+    __syncthreads();   // the previous row's values and reductions are consumed
+    const float* __restrict__ x = a.X + i * a.d;
+    for (int c = threadIdx.x; c < a.d; c += B) s_row[c] = __ldg(&x[c]);
+    __syncthreads();
+    uint64_t fp = 0;
+    for (int32_t j = threadIdx.x; j < T; j += B) {
+      uint32_t k = (uint32_t)__ldg(&a.img.root[j]);
+      uint2 nd = __ldg(&nodes[k]);
+      while ((int32_t)nd.y >= 0) {   // internal: "x_j < b_i", NaN -> default
+        k += step(nd.x, nd.y, s_row[nd.y & fmask], fbits, offmask);
+        nd = __ldg(&nodes[k]);
+      }
+      s_val[j] = __uint_as_float(nd.x);
+      if (LEAF) {
+        const int32_t tree = __ldg(&a.img.tree_orig[j]);
+        const uint32_t leaf = nd.y & 0x7fffffffu;
+        if (a.o.out_leaf) a.o.out_leaf[i * a.o.T_leaf + tree] = (int32_t)leaf;
+        fp += mix64(((uint64_t)(uint32_t)tree << 32) | leaf);
+      }
+    }
+    __syncthreads();
+    // a9 combine: per class, a fixed-order fp64 sum of its tree slots (VOTE: exact counts)
+    int best = 0;
+    double bv = 0.0;
+    for (int32_t c = 0; c < C; c++) {
+      const int32_t s0 = vote ? 0 : __ldg(&a.img.cls_seg[c]), s1 = vote ? T : __ldg(&a.img.cls_seg[c + 1]);
+      const int32_t len = s1 - s0, chunk = (len + B - 1) / B;
+      const int32_t q0 = s0 + threadIdx.x * chunk, q1 = min(s1, q0 + chunk);
+      double part = 0.0;
+      for (int32_t q = q0; q < q1; q++)
+        part += vote ? (s_val[q] == (float)c ? 1.0 : 0.0) : (double)s_val[q];
+      const double sum = block_sum_fixed(part, s_red);
+      if (threadIdx.x == 0) {
+        if (a.o.raw) {
+          a.o.raw[i * C + c] = sum;
+        } else {
+          // a10 finalize (as finalize_row / write_scalar)
+          double v;
+          if (vote) v = sum;
+          else if (a.o.agg == TAHOE_AGG_AVERAGE) v = sum / (double)a.o.n_trees_full + (double)a.o.base;
+          else v = sum + (double)a.o.base;
+          a.o.out[i * C + c] = (float)v;
+          if (c == 0 || v > bv) { best = c; bv = v; }
+        }
+      }
+    }
+    if (threadIdx.x == 0 && !a.o.raw && a.o.out_class) {
+      if (a.o.agg == TAHOE_AGG_BINARY) a.o.out_class[i] = bv > 0.0 ? 1 : 0;
+      else if (a.o.agg == TAHOE_AGG_CLASS_SUM || vote) a.o.out_class[i] = best;
+      else a.o.out_class[i] = 0;
+    }
+    if (LEAF && a.o.out_fp) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) fp += __shfl_xor_sync(0xffffffffu, fp, o);
+      if ((threadIdx.x & 31) == 0) s_fp[threadIdx.x >> 5] = fp;
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        unsigned long long t = 0;
+        for (int w = 0; w < (B >> 5); w++) t += s_fp[w];
+        a.o.out_fp[i] += t;   // the launcher zeroed out_fp; chunked images add per launch
+      }
+    }
+  }
+}
+
+int launch_rows(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
+                int32_t num_sms, void* stream) {
+  const int64_t smem = rows_smem_bytes(d, img.n_slots);
+  if (smem > kMaxSmemOptin - 1024) return (int)cudaErrorInvalidValue;
+  DirectKArgs a{img, X, n, d, o};
+  const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
+  auto kern = leaf ? k_rows<true> : k_rows<false>;
+  static std::atomic<int> configured[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev >= 0 && dev < 64 && configured[dev].load() < smem) {
+    cudaError_t e = cudaFuncSetAttribute(k_rows<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(k_rows<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
+    if (e != cudaSuccess) return (int)e;
+    configured[dev].store(kMaxSmemOptin);
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kRowsThreads, (size_t)smem);
+  if (per_sm < 1) per_sm = 1;
+  const int grid = (int)std::min<int64_t>(n, (int64_t)num_sms * per_sm);
+  kern<<<grid, kRowsThreads, (size_t)smem, static_cast<cudaStream_t>(stream)>>>(a);
+  return (int)cudaGetLastError();
+}
+
 // ------------------------------------------------------------------ microbenchmarks
 // "Measure hardware parameters by a microbenchmark" (Algorithm 1 line 4), re-targeted:
 // the walk is bound by the shared-memory (LSU) data pipe, so the peak it is measured against is the

@@ -25,6 +25,7 @@ struct DevDirect {
   const int32_t* cls = nullptr;      // per tree slot
   const int32_t* tree_orig = nullptr;
   const int32_t* slot_orig = nullptr; // caller node id of every node slot (visit counting)
+  const int32_t* cls_seg = nullptr;   // [n_classes + 1] tree-slot range of each class (class-major)
   int32_t n_slots = 0;
   int32_t fbits = 0;
   int64_t n_nodes = 0;
@@ -216,6 +217,15 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
                          int32_t d, uint8_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
                          void* stream, void* ev_b, void* ev_e);
 int launch_finalize(const FinalizeArgs& a, void* stream);
+// ROWS strategy (small batches): one CTA per sample, lane = tree over the direct
+// image, fixed-order block reduction and in-kernel finalize; one launch, no scratch.  Returns
+// cudaErrorInvalidValue when the row + per-tree values exceed the shared memory it may use.
+constexpr int32_t kRowsThreads = 512;
+inline int64_t rows_smem_bytes(int32_t d, int32_t n_slots) {
+  return ((int64_t)d * 4 + 15) / 16 * 16 + (int64_t)n_slots * 4 + 64 * 8;
+}
+int launch_rows(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
+                int32_t num_sms, void* stream);
 int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t d,
                         uint32_t* counts, int32_t num_sms, void* stream);
 int set_sliced_smem_limit(int32_t bytes);

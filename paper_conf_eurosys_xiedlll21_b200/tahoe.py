@@ -22,7 +22,7 @@ _lib = None
 
 TAHOE_OK, TAHOE_E_INVAL, TAHOE_E_NOMEM, TAHOE_E_CUDA, TAHOE_E_UNSUPPORTED, TAHOE_E_STATE = range(6)
 AGG_SUM, AGG_AVERAGE, AGG_BINARY, AGG_CLASS_SUM, AGG_VOTE = range(5)
-STRATEGY_AUTO, STRATEGY_DIRECT, STRATEGY_SLICED, STRATEGY_SLICED_CODED = -1, 0, 1, 2
+STRATEGY_AUTO, STRATEGY_DIRECT, STRATEGY_SLICED, STRATEGY_SLICED_CODED, STRATEGY_ROWS = -1, 0, 1, 2, 3
 REDUCE_SCATTER, REDUCE_ALL = 0, 1
 COMM_ID_BYTES = 128
 

@@ -19,11 +19,13 @@ pytestmark = pytest.mark.gpu
 
 from paper_conf_eurosys_xiedlll21_b200 import tahoe as T  # noqa: E402
 
-STRATS = [T.STRATEGY_DIRECT, T.STRATEGY_SLICED, T.STRATEGY_SLICED_CODED]
+STRATS = [T.STRATEGY_DIRECT, T.STRATEGY_SLICED, T.STRATEGY_SLICED_CODED, T.STRATEGY_ROWS]
 
 
 def _usable(F, s):
     st = F.stats()
+    if s == T.STRATEGY_ROWS:
+        return st["rows_ok"]
     if s == T.STRATEGY_SLICED:
         return st["sliced_valid"]
     if s == T.STRATEGY_SLICED_CODED:
@@ -338,7 +340,7 @@ def test_rank_codes_threshold_ties_signed_zero_inf_nan():
         r = _gpu_run(F, X, s)
         _check(r, ref, f["agg"], True)
         outs.append(r["out"])
-    assert len(outs) == 3 and all(np.array_equal(o, outs[0]) for o in outs)
+    assert len(outs) == 4 and all(np.array_equal(o, outs[0]) for o in outs)
 
 
 def test_rank_codes_eligibility_and_auto_choice():

@@ -12,9 +12,9 @@
 //   coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs
 //            the rank-coded slices (reading R7): the same busiest-CTA node reads at a cheaper
 //            per-read cost b_c, plus the row-coding pre-pass (passes of 32 attributes per row);
-//   rows   : T = a_r + b_r * waves * ceil(T_trees / 512) * V / T_trees
-//            one CTA per sample (small batches): waves of one-row CTAs, each as long as the
-//            longest chain of dependent node reads of one thread (L2 latency per read).
+//   rows   : T = a_r + max(b_r * ceil(T_trees / 512) * V / T_trees, c_r * n * V / SMs)
+//            one CTA per sample (small batches): the chain of dependent node reads of one thread
+//            (L2 latency per read) while the GPU is not full, the node-read throughput beyond.
 // V = expected node reads per sample (calibrated E[path] + 1 leaf read, summed over trees,
 // reading Z16).  The constants are fitted on the chip by scripts/fit_costmodel.py and read from
 // costmodel_b200.json next to libtahoe.so (or $TAHOE_COSTMODEL); defaults are round-1 B200
@@ -79,6 +79,7 @@ const CostParams& cost_params() {
     if (read_key(js, "e_w", &v)) c.e_w = v;
     if (read_key(js, "a_r", &v)) c.a_r = v;
     if (read_key(js, "b_r", &v)) c.b_r = v;
+    if (read_key(js, "c_r", &v)) c.c_r = v;
     c.fitted = all;
     return c;
   }();
@@ -105,12 +106,12 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
   }
   const double sms = st.num_sms > 0 ? st.num_sms : 148;
   if (strategy == TAHOE_STRATEGY_ROWS) {
-    // rows: waves of one-row CTAs; a wave lasts the longest tree chain of a thread:
-    // ceil(T / 512) trees of mean path V / T dependent node reads each (L2 latency b_r)
+    // rows: latency-bound while the batch leaves the GPU idle (a thread's chain of ceil(T / 512)
+    // trees of mean path V / T dependent node reads, b_r per read), throughput-bound beyond
+    // (c_r per node read per SM)
     if (!st.rows_ok) return INFINITY;
-    const double waves = std::ceil((double)n / (sms * std::max(1, st.rows_per_sm)));
     const double chain = std::ceil((double)st.n_trees / kRowsThreads) * st.V / std::max(1, st.n_trees);
-    return c.a_r + c.b_r * waves * chain;
+    return c.a_r + std::max(c.b_r * chain, c.c_r * (double)n * st.V / sms);
   }
   const double g = st.wide_rows ? c.g_d : 1.0;
   return c.a_d + g * std::max(c.l_d * st.V, c.b_d * st.V * (double)n / sms);

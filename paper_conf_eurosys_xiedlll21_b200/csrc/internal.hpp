@@ -160,7 +160,9 @@ struct CostParams {
   double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
   double a_c = 30.0, b_c = 6.6e-5, e_c = 1.6e-5; // coded: launches; per unit; per row-pass per SM
   double a_w = 40.0, b_w = 1.5e-4, e_w = 1.6e-5; // wide codes (reading R8): the same three terms
-  double a_r = 8.0, b_r = 0.7;                    // rows (f1): launch; per dependent node read of a wave
+  // rows (f1): launch; per dependent node read (latency); per node read per SM (throughput) —
+  // fitted on the B200 latency sweep (profiles/r02_latency.md)
+  double a_r = 2.0, b_r = 0.9, c_r = 8.1e-4;
   bool fitted = false;
 };
 const CostParams& cost_params();

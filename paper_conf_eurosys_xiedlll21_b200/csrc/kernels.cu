@@ -2420,7 +2420,8 @@ __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   float* s_row = reinterpret_cast<float*>(smem);
   float* s_val = reinterpret_cast<float*>(smem + ((size_t)a.d * 4 + 15) / 16 * 16);
-  double* s_red = reinterpret_cast<double*>(s_val + a.img.n_slots);
+  double* s_red = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_val) +
+                                            ((size_t)a.img.n_slots * 4 + 15) / 16 * 16);
   __shared__ unsigned long long s_fp[kRowsThreads / 32];
   const uint2* __restrict__ nodes = reinterpret_cast<const uint2*>(a.img.nodes);
   const int fbits = a.img.fbits;
@@ -2428,6 +2429,10 @@ __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
   const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
   const int32_t T = a.img.n_slots, C = a.o.n_classes, B = blockDim.x;
   const bool vote = a.o.agg == TAHOE_AGG_VOTE;
+  // the first tree's root node is fetched before the row is staged (two dependent L2 reads that
+  // overlap the staging); it is the same for every row of this CTA
+  const uint32_t k0 = threadIdx.x < T ? (uint32_t)__ldg(&a.img.root[threadIdx.x]) : 0u;
+  const uint2 nd0 = threadIdx.x < T ? __ldg(&nodes[k0]) : make_uint2(0u, 0u);
   for (int64_t i = blockIdx.x; i < a.n; i += gridDim.x) {
     __syncthreads();   // the previous row's values and reductions are consumed
     const float* __restrict__ x = a.X + i * a.d;
@@ -2435,8 +2440,8 @@ __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
     __syncthreads();
     uint64_t fp = 0;
     for (int32_t j = threadIdx.x; j < T; j += B) {
-      uint32_t k = (uint32_t)__ldg(&a.img.root[j]);
-      uint2 nd = __ldg(&nodes[k]);
+      uint32_t k = j == (int32_t)threadIdx.x ? k0 : (uint32_t)__ldg(&a.img.root[j]);
+      uint2 nd = j == (int32_t)threadIdx.x ? nd0 : __ldg(&nodes[k]);
       while ((int32_t)nd.y >= 0) {   // internal: "x_j < b_i", NaN -> default
         k += step(nd.x, nd.y, s_row[nd.y & fmask], fbits, offmask);
         nd = __ldg(&nodes[k]);

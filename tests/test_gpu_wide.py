@@ -71,7 +71,7 @@ def test_wide_codes_piece_boundaries_ties_signed_zero_inf_nan():
         r = _gpu_run(F, X, s)          # leaf ids + fingerprints (LEAF instantiations)
         _check(r, ref, oracle.AGG_SUM, True)
         outs.append(r["out"])
-    assert len(outs) == 3 and all(np.array_equal(o, outs[0]) for o in outs)
+    assert len(outs) == len(_strats(F)) >= 3 and all(np.array_equal(o, outs[0]) for o in outs)
 
 
 @pytest.mark.parametrize("d", [130, 255, 600, 1500])

@@ -85,9 +85,37 @@ static int32_t slot_budget_for(int32_t max_smem, int32_t n_features) {
   return (int32_t)std::max<int64_t>(0, ((max_smem - ring) & ~1023LL) / kSlotBytes);
 }
 
+static void free_host_pipe(tahoe_forest* f) {
+  auto& h = f->hp;
+  if (!h.ready) return;
+  cudaStreamDestroy(h.s_in);
+  cudaStreamDestroy(h.s_cmp);
+  cudaStreamDestroy(h.s_out);
+  cudaEventDestroy(h.ev_start);
+  for (int b = 0; b < 3; b++) { cudaEventDestroy(h.ev_in[b]); cudaEventDestroy(h.ev_cmp[b]); cudaEventDestroy(h.ev_out[b]); }
+  h = tahoe_forest::HostPipe();
+}
+
+static cudaError_t init_host_pipe(tahoe_forest* f) {
+  auto& h = f->hp;
+  if (h.ready) return cudaSuccess;
+  cudaError_t e = cudaStreamCreateWithFlags(&h.s_in, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h.s_cmp, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h.s_out, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h.ev_start, cudaEventDisableTiming);
+  for (int b = 0; b < 3 && e == cudaSuccess; b++) {
+    e = cudaEventCreateWithFlags(&h.ev_in[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h.ev_cmp[b], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h.ev_out[b], cudaEventDisableTiming);
+  }
+  h.ready = e == cudaSuccess;
+  return e;
+}
+
 static void free_device(tahoe_forest* f) {
   if (f->device < 0) return;
   DeviceGuard g(f->device);
+  free_host_pipe(f);
   cudaFree((void*)f->dd.nodes);
   cudaFree((void*)f->dd.root);
   cudaFree((void*)f->dd.cls);
@@ -693,17 +721,14 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   cuts.push_back(n);
   const int64_t nchunks = (int64_t)cuts.size() - 1;
   constexpr int NB = 3;
-  cudaStream_t s_in, s_cmp, s_out;
-  cudaStreamCreateWithFlags(&s_in, cudaStreamNonBlocking);
-  cudaStreamCreateWithFlags(&s_cmp, cudaStreamNonBlocking);
-  cudaStreamCreateWithFlags(&s_out, cudaStreamNonBlocking);
-  cudaEvent_t ev_start, ev_in[NB], ev_cmp[NB], ev_out[NB];
-  cudaEventCreateWithFlags(&ev_start, cudaEventDisableTiming);
-  for (int b = 0; b < NB; b++) {
-    cudaEventCreateWithFlags(&ev_in[b], cudaEventDisableTiming);
-    cudaEventCreateWithFlags(&ev_cmp[b], cudaEventDisableTiming);
-    cudaEventCreateWithFlags(&ev_out[b], cudaEventDisableTiming);
-  }
+  tahoe_forest* fm = const_cast<tahoe_forest*>(f);   // the pipe is handle-owned scratch state
+  std::lock_guard<std::mutex> lock(fm->host_mu);
+  if (cudaError_t ie = init_host_pipe(fm)) return cuda_fail(ie, "tahoe_predict_host streams");
+  cudaStream_t s_in = fm->hp.s_in, s_cmp = fm->hp.s_cmp, s_out = fm->hp.s_out;
+  cudaEvent_t ev_start = fm->hp.ev_start;
+  cudaEvent_t* ev_in = fm->hp.ev_in;
+  cudaEvent_t* ev_cmp = fm->hp.ev_cmp;
+  cudaEvent_t* ev_out = fm->hp.ev_out;
   const int64_t nbuf = std::min<int64_t>(NB, nchunks);
   float* dX = nullptr;
   float* dO = nullptr;
@@ -743,11 +768,6 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   if (dX) cudaFreeAsync(dX, user);
   if (dO) cudaFreeAsync(dO, user);
   if (dC) cudaFreeAsync(dC, user);
-  cudaEventDestroy(ev_start);
-  for (int b = 0; b < NB; b++) { cudaEventDestroy(ev_in[b]); cudaEventDestroy(ev_cmp[b]); cudaEventDestroy(ev_out[b]); }
-  cudaStreamDestroy(s_in);
-  cudaStreamDestroy(s_cmp);
-  cudaStreamDestroy(s_out);
   if (st != TAHOE_OK) return st;
   if (e != cudaSuccess) return cuda_fail(e, "tahoe_predict_host");
   return TAHOE_OK;

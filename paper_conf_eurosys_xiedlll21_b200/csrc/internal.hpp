@@ -2,6 +2,8 @@
 // Everything here is product code (libtahoe.so); nothing is shared with oracle/.
 #pragma once
 #include <cstdint>
+#include <mutex>
+#include <cuda_runtime.h>
 #include <string>
 #include <vector>
 
@@ -193,4 +195,13 @@ struct tahoe_forest {
   std::vector<int32_t> cta_start;
   int32_t* d_cta_start = nullptr;
   int32_t* d_class_parts = nullptr;
+  // tahoe_predict_host's copy / compute / copy-back streams and their events, created on first use
+  // and kept for the handle's lifetime (not per call); host_mu serialises concurrent host calls on
+  // one handle (they share these streams)
+  struct HostPipe {
+    bool ready = false;
+    cudaStream_t s_in = nullptr, s_cmp = nullptr, s_out = nullptr;
+    cudaEvent_t ev_start = nullptr, ev_in[3] = {}, ev_cmp[3] = {}, ev_out[3] = {};
+  } hp;
+  std::mutex host_mu;
 };

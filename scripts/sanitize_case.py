@@ -29,13 +29,42 @@ for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
         F.predict(Xd, out=out, out_class=cls, force_strategy=s)
         F.predict(Xd, out=out, out_class=cls, out_leaf=leaf, out_fingerprint=fp, force_strategy=s)
     os.environ.pop("TAHOE_DIRECT_VARIANT")
-    # rank-coded slices (reading R7): both row-coding pre-passes
+    # large-batch direct kernels (staged rows, P threads per row): C2 / C3 only (d <= 256)
+    if X.shape[1] <= 256:
+        big = torch.from_numpy(gen.make_rows(cid, 33_001)).to(dev)
+        for variant in ("5", "3", "2"):
+            os.environ["TAHOE_DIRECT_VARIANT"] = variant
+            F.predict(big, force_strategy=0)
+        os.environ.pop("TAHOE_DIRECT_VARIANT")
+        del big
+    # rank-coded slices (reading R7 u16 rows, swizzled rows of >= 128 bytes for C3; reading R8
+    # wide codes for C4): both row-coding pre-passes, production and LEAF instantiations, a
+    # multi-tile batch so the ring wraps, and the minimum ring depth
     if F.stats()["coded_valid"]:
+        big = torch.from_numpy(gen.make_rows(cid, 20_011)).to(dev)
+        big[::13, 2] = float("nan")
         for banks in ("1", "0"):
             os.environ["TAHOE_CODE_BANKS"] = banks
-            out = torch.empty((n, F.n_out), device=dev)
-            F.predict(Xd, out=out, force_strategy=2)
+            for Xs in (Xd, big):
+                m = Xs.shape[0]
+                out = torch.empty((m, F.n_out), device=dev)
+                F.predict(Xs, out=out, force_strategy=2)
+                F.predict(Xs, out=out, out_leaf=torch.empty((m, F.n_trees), dtype=torch.int32, device=dev),
+                          out_fingerprint=torch.empty(m, dtype=torch.int64, device=dev), force_strategy=2)
         os.environ.pop("TAHOE_CODE_BANKS")
+        os.environ["TAHOE_CODES_RING"] = "3"
+        F.predict(big, force_strategy=2)
+        os.environ.pop("TAHOE_CODES_RING")
+        del big
+    # ROWS strategy (f1), with and without leaf diagnostics, and its raw partial path
+    if F.stats()["rows_ok"]:
+        out = torch.empty((n, F.n_out), device=dev)
+        F.predict(Xd, out=out, out_class=torch.empty(n, dtype=torch.int32, device=dev), force_strategy=3)
+        F.predict(Xd, out=out, out_leaf=torch.empty((n, F.n_trees), dtype=torch.int32, device=dev),
+                  out_fingerprint=torch.empty(n, dtype=torch.int64, device=dev), force_strategy=3)
+        os.environ["TAHOE_FORCE_STRATEGY"] = "3"
+        F.predict_partial(Xd)
+        os.environ.pop("TAHOE_FORCE_STRATEGY")
     # misaligned X -> warp-copy staging path
     buf = torch.empty(X.size + 1, device=dev)
     buf[1:] = Xd.reshape(-1)
@@ -56,5 +85,8 @@ for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
         S1.predict_reduce(comm, Xd)
         torch.cuda.synchronize()
         comm.close()
+# microbenchmarks (Algorithm 1 line 4): both walk variants and the raw shared-memory load kernel
+T.tahoe_measure_visit_rate(0, 0, 16, 2)
+T.tahoe_measure_visit_rate(0, 1, 16, 2)
 torch.cuda.synchronize()
 print("sanitize case done")

@@ -220,6 +220,21 @@ tahoe_status tahoe_forest_l2_persist(const tahoe_forest* f, tahoe_stream stream,
 tahoe_status tahoe_measure_visit_rate(int32_t device, int32_t variant, int32_t steps, int32_t reps,
                                       double* node_reads_per_s, double* smem_bytes_per_clk);
 
+/*
+ * tahoe_profile_walk — load-balance measurement (Table 3 "A.C.V.", the
+ * coefficient of variation of execution time across threads, Fig. 2(c)):
+ * predicts X (device, n x d) with the u16 rank-coded slices through an instrumented copy of their
+ * walk that reads the SM clock every iteration, writing out (device, n x n_out) as tahoe_predict
+ * does and stats[8] (HOST doubles):
+ *   stats[0] / stats[2]  mean over work units of the CV of the 32 lanes' walk spans,
+ *   stats[1] / stats[2]  mean over work units of mean/max lane span (lockstep efficiency),
+ *   stats[3] / stats[2]  mean lane span in SM cycles,
+ *   stats[4] / stats[5]  mean over warps of the CV of the lanes' total spans over the launch.
+ * E_UNSUPPORTED unless the forest has the u16 coded slices; synchronous (waits on `stream`).
+ */
+tahoe_status tahoe_profile_walk(const tahoe_forest* f, const float* X, int64_t n, int32_t d,
+                                float* out, double* stats, tahoe_stream stream);
+
 /* ---------------- tree sharding (multi-GPU) ---------------- */
 
 /* Sub-forest of the trees assigned to `rank` of `world` (balanced by expected visits per tree,

@@ -373,7 +373,8 @@ static SlicedPlan sliced_plan(const tahoe_forest* f, const float* X, int64_t n, 
 // One batch on the device.  mode 0: final outputs; mode 1: raw fp64 partial [n x n_out].
 static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_t d, float* out,
                         int32_t* out_class, int32_t* out_leaf, uint64_t* out_fp, double* raw_user,
-                        int32_t forced, cudaStream_t st, void* ev_b = nullptr, void* ev_e = nullptr) {
+                        int32_t forced, cudaStream_t st, void* ev_b = nullptr, void* ev_e = nullptr,
+                        double* prof = nullptr) {
   const Forest& H = f->host;
   const int32_t C = H.n_out();
   int32_t strat = choose(f, n, d, forced);
@@ -506,7 +507,7 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
       cp.cta_start = f->d_cta_start;
     }
     rc = launch_sliced_codes(f->ds, cp, X, n, d, static_cast<uint16_t*>(cbuf), o, fused,
-                             f->num_sms, st, ev_b, ev_e);
+                             f->num_sms, st, ev_b, ev_e, prof);
     cudaFreeAsync(cbuf, st);
   } else {
     if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
@@ -693,6 +694,34 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_ex(
   if (opts) o = *opts;
   return run(f, X, n, d, out, o.out_class, o.out_leaf, o.out_fingerprint, nullptr, o.force_strategy,
              reinterpret_cast<cudaStream_t>(stream), o.ev_main_begin, o.ev_main_end);
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_profile_walk(
+    const tahoe_forest* f, const float* X, int64_t n, int32_t d, float* out, double* stats,
+    tahoe_stream stream) {
+  TAHOE_GUARD_BEGIN
+  tahoe_status st = check_predict(f, X, n, d, out);
+  if (st != TAHOE_OK || n == 0) return st;
+  if (!stats) return fail(TAHOE_E_INVAL, "NULL stats");
+  if (!f->sl.valid || !f->ds.cnodes || f->sl.code8)
+    return fail(TAHOE_E_UNSUPPORTED, "walk profiling needs the u16 rank-coded slices");
+  DeviceGuard g(f->device);
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  double* dev = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&dev, 8 * sizeof(double), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(dev, 0, 8 * sizeof(double), s);
+  if (e != cudaSuccess) return cuda_fail(e, "profile buffer");
+  st = run(f, X, n, d, out, nullptr, nullptr, nullptr, nullptr, TAHOE_STRATEGY_SLICED_CODED, s,
+           nullptr, nullptr, dev);
+  if (st == TAHOE_OK) {
+    e = cudaMemcpyAsync(stats, dev, 8 * sizeof(double), cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  }
+  cudaFreeAsync(dev, s);
+  if (st != TAHOE_OK) return st;
+  if (e != cudaSuccess) return cuda_fail(e, "profile readback");
+  return TAHOE_OK;
   TAHOE_GUARD_END
 }
 

@@ -1036,6 +1036,7 @@ struct CodedKArgs {
   int32_t prefetch;      // entries of the CTA's tile sequence to prefetch into L2 ahead (0 = none)
   int32_t ring;          // ring depth (kSlicedRing .. kCodedRingMax): as many tiles as shared memory holds
   uint32_t ring_m, bars_m;   // ceil(2^32 / ring), ceil(2^32 / (2 ring)): division by multiply-high
+  double* prof;          // PROF instantiation: load-balance statistics (prof_unit), else null
   OutArgs o;
 };
 
@@ -1134,13 +1135,75 @@ __device__ __forceinline__ void walk_coded2_leaf(uint32_t pA, uint32_t pB, uint3
   }
 }
 
+// walk_coded2 with per-lane timing (load-balance measurement, Table 3 analog): the
+// same steps; each iteration records the SM clock, so `span` = cycles from the walk's start to the
+// start of the lane's last iteration (a lane leaves the loop when both its chains are done).
+template <bool NAN_AWARE, bool SWZ>
+__device__ __forceinline__ void walk_coded2_prof(uint32_t pA, uint32_t pB, uint32_t pe, uint32_t rowA,
+                                                 uint32_t rowB, uint32_t amask, uint32_t dlbit,
+                                                 uint32_t shmul, double& accA, double& accB,
+                                                 uint32_t& span) {
+  accA = 0.0;
+  accB = 0.0;
+  const uint32_t t0 = (uint32_t)clock();
+  uint32_t tl = t0;
+  while ((pA != pe) | (pB != pe)) {
+    tl = (uint32_t)clock();
+    const float a1 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+    const float b1 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+    const float a2 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+    const float b2 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+    add_pair_ftz(accA, a1, a2);
+    add_pair_ftz(accB, b1, b2);
+  }
+  span = tl - t0;
+}
+
+// Per-unit and per-lane load-balance statistics of a profiled walk (prof[8], device doubles):
+// [0] sum over units of the CV of lane spans, [1] sum of mean/max lane span (lockstep efficiency),
+// [2] units, [3] sum of mean lane span (cycles), [4] sum over warps of the CV of the lanes' total
+// spans over the whole launch, [5] warps.
+__device__ __forceinline__ void prof_unit(double* prof, uint32_t span) {
+  const double x = (double)span;
+  double s = x, q = x * x, m = x;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    s += __shfl_xor_sync(0xffffffffu, s, o);
+    q += __shfl_xor_sync(0xffffffffu, q, o);
+    m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+  }
+  if ((threadIdx.x & 31) == 0 && m > 0.0) {
+    const double mean = s / 32.0, var = fmax(0.0, q / 32.0 - mean * mean);
+    atomicAdd(&prof[0], sqrt(var) / mean);
+    atomicAdd(&prof[1], mean / m);
+    atomicAdd(&prof[2], 1.0);
+    atomicAdd(&prof[3], mean);
+  }
+}
+__device__ __forceinline__ void prof_lanes(double* prof, double total) {
+  double s = total, q = total * total;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    s += __shfl_xor_sync(0xffffffffu, s, o);
+    q += __shfl_xor_sync(0xffffffffu, q, o);
+  }
+  if ((threadIdx.x & 31) == 0 && s > 0.0) {
+    const double mean = s / 32.0, var = fmax(0.0, q / 32.0 - mean * mean);
+    atomicAdd(&prof[4], sqrt(var) / mean);
+    atomicAdd(&prof[5], 1.0);
+  }
+}
+
 // k_sliced_codes: k_sliced's persistent slice-stationary schedule (slice in shared memory, 3-deep
 // ring of 64-row tiles refilled by the warp that finishes a tile, dynamic 4-row work units, one
 // half-warp per row, two chains per lane) over code tiles (one 1-D bulk copy per tile).
 // LEAF: the same schedule and walk, also writing per-(sample, tree) caller leaf ids (out_leaf, may
 // be null) and accumulating fingerprints (out_fp, u64 atomic adds per slice).
-template <bool FUSED, bool SWZ, bool LEAF>
+// MODE 0: production; 1: LEAF (leaf ids / fingerprints); 2: PROF (per-lane spans, prof_unit)
+template <bool FUSED, bool SWZ, int MODE>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant__ CodedKArgs a) {
+  constexpr bool LEAF = MODE == 1, PROF = MODE == 2;
+  double lane_total = 0.0;   // PROF: this lane's spans over the launch
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
   unsigned char* s_ring = smem + a.forest_smem;
@@ -1298,6 +1361,12 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
             walk_coded2_leaf<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
           else
             walk_coded2_leaf<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+        } else if (PROF) {
+          uint32_t span;
+          if (nan_flag) walk_coded2_prof<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, span);
+          else walk_coded2_prof<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, span);
+          prof_unit(a.prof, span);
+          lane_total += (double)span;
         } else if (nan_flag) {
           walk_coded2<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
         } else {
@@ -1329,6 +1398,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     if (threadIdx.x == 0) *s_next = 0u;
     __syncthreads();
   }
+  if (PROF) prof_lanes(a.prof, lane_total);
 }
 
 static int grid_for(int64_t n, int block, int num_sms, int per_sm);
@@ -1651,7 +1721,7 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
 
 int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                         int32_t d, uint16_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
-                        void* stream, void* ev_b, void* ev_e) {
+                        void* stream, void* ev_b, void* ev_e, double* prof) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
   const int32_t tstride = code_tile_stride(img.fbits);
@@ -1749,22 +1819,29 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   // rows of >= 128 bytes are stored swizzled (code_slot_swz); the others keep the plain walk;
   // leaf ids / fingerprints take the LEAF instantiation of the same walk
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
-  auto kern = leaf ? (a.rb >= 128 ? (fused ? k_sliced_codes<true, true, true> : k_sliced_codes<false, true, true>)
-                                  : (fused ? k_sliced_codes<true, false, true> : k_sliced_codes<false, false, true>))
-                   : (a.rb >= 128 ? (fused ? k_sliced_codes<true, true, false> : k_sliced_codes<false, true, false>)
-                                  : (fused ? k_sliced_codes<true, false, false> : k_sliced_codes<false, false, false>));
+  a.prof = prof;
+  using KFn = void (*)(CodedKArgs);
+  // [mode][swz][fused]
+  static const KFn table[3][2][2] = {
+      {{k_sliced_codes<false, false, 0>, k_sliced_codes<true, false, 0>},
+       {k_sliced_codes<false, true, 0>, k_sliced_codes<true, true, 0>}},
+      {{k_sliced_codes<false, false, 1>, k_sliced_codes<true, false, 1>},
+       {k_sliced_codes<false, true, 1>, k_sliced_codes<true, true, 1>}},
+      {{k_sliced_codes<false, false, 2>, k_sliced_codes<true, false, 2>},
+       {k_sliced_codes<false, true, 2>, k_sliced_codes<true, true, 2>}}};
+  const int mode = prof ? 2 : (leaf ? 1 : 0);
+  auto kern = table[mode][a.rb >= 128 ? 1 : 0][fused ? 1 : 0];
   {
     static std::atomic<int> configured[64];
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
-      for (auto k : {k_sliced_codes<true, false, false>, k_sliced_codes<false, false, false>,
-                     k_sliced_codes<true, true, false>, k_sliced_codes<false, true, false>,
-                     k_sliced_codes<true, false, true>, k_sliced_codes<false, false, true>,
-                     k_sliced_codes<true, true, true>, k_sliced_codes<false, true, true>}) {
-        e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
-        if (e != cudaSuccess) return (int)e;
-      }
+      for (const auto& m : table)
+        for (const auto& w : m)
+          for (KFn k : w) {
+            e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
+            if (e != cudaSuccess) return (int)e;
+          }
       configured[dev].store(1);
     }
   }

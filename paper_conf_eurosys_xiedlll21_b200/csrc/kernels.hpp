@@ -207,9 +207,10 @@ int launch_sliced(const DevSliced& img, const SlicedPlan& plan, const float* X, 
                   int32_t d, const OutArgs& o, bool fused, void* stream);
 // rank-coded sliced strategy: encode X into code tiles (codes: device scratch of
 // ntiles * code_tile_stride bytes), then walk the coded slices
+// prof != nullptr: the PROF instantiation (per-lane walk spans -> prof[6], load-balance statistics)
 int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const float* X, int64_t n,
                         int32_t d, uint16_t* codes, const OutArgs& o, bool fused, int32_t num_sms,
-                        void* stream, void* ev_b, void* ev_e);
+                        void* stream, void* ev_b, void* ev_e, double* prof = nullptr);
 // wide rank codes (reading R8): per chunk of code8_chunk_rows rows, u8 code tiles (codes: scratch
 // of ctiles * code8_tile_bytes + ctiles * 16 bytes of NaN flags + n_slices * 8 bytes of counters,
 // ctiles = the chunk's tiles), then the coded slices over them

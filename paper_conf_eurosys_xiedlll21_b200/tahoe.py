@@ -55,7 +55,7 @@ SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_
            "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced", "tahoe_count_visits",
            "tahoe_forest_layout_counts", "tahoe_forest_l2_persist", "tahoe_comm_unique_id",
            "tahoe_comm_init", "tahoe_comm_free", "tahoe_reduce_rows", "tahoe_predict_reduce",
-           "tahoe_reduce_partials", "tahoe_measure_visit_rate")
+           "tahoe_reduce_partials", "tahoe_measure_visit_rate", "tahoe_profile_walk")
 
 
 def lib_path() -> str:
@@ -108,6 +108,7 @@ def load(build_if_missing: bool = True):
         "tahoe_predict_reduce": (st, [P, P, P, i64, i32, i32, P, P, P]),
         "tahoe_reduce_partials": (st, [P, P, i32, i32, i32, i64, P, P, P]),
         "tahoe_measure_visit_rate": (st, [i32, i32, i32, i32, P, P]),
+        "tahoe_profile_walk": (st, [P, P, i64, i32, P, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -292,6 +293,16 @@ def tahoe_measure_visit_rate(device: int = 0, variant: int = 0, steps: int = 256
     _check(load().tahoe_measure_visit_rate(device, variant, steps, reps, ctypes.byref(r),
                                            ctypes.byref(b) if smem_bw else None))
     return r.value, (b.value if smem_bw else None)
+
+
+def tahoe_profile_walk(h, X, n: int, d: int, out, stream=None) -> dict:
+    """Instrumented coded walk (per-lane SM-clock spans): load-balance statistics of the launch."""
+    st = np.zeros(8, np.float64)
+    _check(load().tahoe_profile_walk(h, _dev_ptr(X), n, d, _dev_ptr(out), _np_ptr(st),
+                                     _stream_ptr(stream)))
+    u, w = max(st[2], 1.0), max(st[5], 1.0)
+    return dict(unit_cv=st[0] / u, unit_lockstep=st[1] / u, mean_span_cycles=st[3] / u,
+                lane_total_cv=st[4] / w, units=int(st[2]), warps=int(st[5]))
 
 
 def tahoe_forest_n_outputs(h) -> int:

@@ -78,13 +78,19 @@ for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
     parts = [F.shard(r, 2).predict_partial(Xd) for r in range(2)]
     for r in range(2):
         for mode in (T.REDUCE_SCATTER, T.REDUCE_ALL):
-            F.reduce_partials(parts, r, mode=mode, out_class=torch.empty(n, dtype=torch.int32, device=dev))
+            lo, hi = T.tahoe_reduce_rows(n, 2, r, mode)
+            F.reduce_partials(parts, r, mode=mode, out_class=torch.empty(hi - lo, dtype=torch.int32, device=dev))
     if cid == 2:
         comm = T.Comm(T.tahoe_comm_unique_id(), 1, 0, 0)
         S1 = F.shard(0, 1)
         S1.predict_reduce(comm, Xd)
         torch.cuda.synchronize()
         comm.close()
+# instrumented walk (tahoe_profile_walk, f3) on a C2 forest
+fp2 = gen.make_forest(2, n_trees=64)
+Fp = T.Forest(fp2, device=0).layout(gen.make_calibration(2, 2048))
+Xp = torch.from_numpy(gen.make_rows(2, 9001)).to(dev)
+T.tahoe_profile_walk(Fp.handle, Xp, 9001, Xp.shape[1], torch.empty((9001, 1), device=dev))
 # microbenchmarks (Algorithm 1 line 4): both walk variants and the raw shared-memory load kernel
 T.tahoe_measure_visit_rate(0, 0, 16, 2)
 T.tahoe_measure_visit_rate(0, 1, 16, 2)

@@ -1207,19 +1207,28 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
   unsigned char* s_ring = smem + a.forest_smem;
-  // ring depth: a.ring buffers, 2 * a.ring full barriers (the ring-wrap guard of ring_bar, with the
-  // depth a runtime value here)
+  // Producer / consumer ring (mbarrier hand-off only): warp PW (the last) stages the slice and
+  // every code tile of the CTA's sequence, refilling buffer b once the kUnits units of its previous
+  // tile have all arrived on empty[b] (and writing that tile's slice partials out first); the other
+  // 31 warps claim 4-row work units from a CTA counter, wait on the tile's full barrier, walk, and
+  // arrive on empty[b].  Tile seq uses buffer seq % ring, full barrier seq % (2 ring) with parity
+  // (seq / (2 ring)) & 1: a consumer claiming seq could only see a stale phase if tile
+  // seq - 2 ring had not arrived, but then seq - ring is not issued either, and the 2 x 16 units
+  // of those two tiles would hold 32 blocked consumers — there are 31 (the ring-wrap guard of
+  // ring_bar, with a runtime depth).
   const uint32_t ring = (uint32_t)a.ring, nbars = 2u * ring;
-  // control block (kCodedCtlBytes): [2 ring] full barriers, slice barrier, unit counter (u32),
-  // [ring] release counters
+  constexpr int kUnits = kSlicedTileRows / 4;
+  // control block (kCodedCtlBytes): [2 ring] full barriers, [ring] empty barriers, slice barrier,
+  // unit counter (u32)
   uint64_t* s_full = reinterpret_cast<uint64_t*>(s_ring + (size_t)ring * a.tstride);
-  uint64_t* s_forest = s_full + nbars;
+  uint64_t* s_empty = s_full + nbars;
+  uint64_t* s_forest = s_empty + ring;
   unsigned int* s_next = reinterpret_cast<unsigned int*>(s_forest + 1);
-  int* s_cnt = reinterpret_cast<int*>(s_next + 1);
-  // slice partials of the tiles in the ring, written out coalesced by the warp closing a tile
+  // slice partials of the tiles in the ring (consumers write, the producer stores them coalesced)
   double* s_part = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_full) + kCodedCtlBytes);
   const int lane = threadIdx.x & 31;
   const int warp = threadIdx.x >> 5;
+  const int PW = (int)(blockDim.x >> 5) - 1;   // producer warp
   const int col = lane & (C - 1);
   const int half = lane >> 4;
   const uint32_t F = (uint32_t)a.img.fbits;
@@ -1234,60 +1243,12 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
 
   if (threadIdx.x == 0) {
     for (uint32_t b = 0; b < nbars; b++) mbar_init(&s_full[b], 1);
-    for (uint32_t b = 0; b < ring; b++) s_cnt[b] = 0;
+    for (uint32_t b = 0; b < ring; b++) mbar_init(&s_empty[b], kUnits);
     *s_next = 0u;
     mbar_init(s_forest, 1);
     fence_mbar_init();
   }
   __syncthreads();
-
-  // stage tile `tile` (CTA-wide sequence number seq) into buffer b (barrier ring_bar(seq))
-  auto issue_tile = [&](int64_t tile, int b, uint32_t seq, int64_t ahead = -1) {
-    if (lane == 0) {
-      // optional L2 prefetch of this CTA's tile `ahead` (a later tile of its sequence)
-      if (ahead >= 0 && ahead < ntiles)
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
-                     "r"((uint32_t)a.tstride) : "memory");
-      fence_proxy_async_smem();
-      mbar_expect_tx(&s_full[fmod_small(seq, nbars, a.bars_m)], (uint32_t)a.tstride);
-      bulk_g2s(s_ring + (size_t)b * a.tstride,
-               reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride,
-               (uint32_t)a.tstride, &s_full[fmod_small(seq, nbars, a.bars_m)]);
-    }
-    __syncwarp();
-  };
-  // after one work unit: the warp finishing the tile's last unit writes the tile's 64 slice
-  // partials (two coalesced 256-byte stores) and refills the buffer with the tile `ring` ahead
-  auto release = [&](int b, int units, int64_t it, int64_t my_tiles, int64_t t0, int64_t ts,
-                     int sl, int64_t r0, int nr, uint32_t seq) {
-    __syncwarp();
-    int last = 0;
-    if (lane == 0) {
-      __threadfence_block();
-      last = atomicAdd(&s_cnt[b], 1) == units - 1;
-      if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
-    }
-    last = __shfl_sync(0xffffffffu, last, 0);
-    if (!last) return;
-    if (FUSED) {
-      if (it + ring < my_tiles)
-        issue_tile(t0 + (it + ring) * ts, b, seq + ring, a.prefetch ? t0 + (it + ring + a.prefetch) * ts : -1);
-      return;
-    }
-    // take the tile's 64 partials out of shared memory, refill the buffer at once, then store the
-    // partials (two coalesced 256-byte stores).  (Finalizing in-kernel by the CTA that closes a
-    // tile's last slice needs a global fence per tile; measured slower than k_finalize: C2
-    // 1.689 -> 1.730 ms, C3 4.75 -> 4.95 ms per step.)
-    const double* sp = s_part + b * kSlicedTileRows;
-    const double p0 = lane < nr ? sp[lane] : 0.0, p1 = lane + 32 < nr ? sp[lane + 32] : 0.0;
-    __syncwarp();
-    if (it + ring < my_tiles)
-      issue_tile(t0 + (it + ring) * ts, b, seq + ring, a.prefetch ? t0 + (it + ring + a.prefetch) * ts : -1);
-    double* dst = a.o.raw + (size_t)sl * a.n + r0;
-    if (lane < nr) dst[lane] = p0;
-    if (lane + 32 < nr) dst[lane + 32] = p1;
-    __syncwarp();
-  };
 
   uint32_t g = 0;
   uint32_t ph_forest = 0;
@@ -1306,25 +1267,57 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
     const int64_t t0 = multipass ? 0 : t0s;
     const int64_t ts = multipass ? 1 : tss;
     const int64_t my_tiles = t0 < ntiles ? (ntiles - t0 + ts - 1) / ts : 0;
-    if (warp == 0) {
-      if (lane == 0) {
+    const uint32_t sbase = smem_u32(smem);
+    if (warp == PW) {
+      // ---- producer
+      if (lane == 0) {   // a7: the slice, one bulk copy of slots x 128 bytes
         const uint32_t bytes = (uint32_t)a.img.slots[sl] * (uint32_t)kSlotBytes;
         fence_proxy_async_smem();
         mbar_expect_tx(s_forest, bytes);
         bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
-      for (int64_t q = 0; q < (int64_t)ring && q < my_tiles; q++)
-        issue_tile(t0 + q * ts, (int)fmod_small(g + (uint32_t)q, ring, a.ring_m), g + (uint32_t)q);
-    }
-    const uint32_t sbase = smem_u32(smem);
+      // tile `it` of this slice consumed: store its 64 slice partials (two coalesced 256-byte
+      // stores; non-fused launches)
+      auto drain = [&](int64_t it) {
+        const uint32_t seq = g + (uint32_t)it;
+        const uint32_t b = fmod_small(seq, ring, a.ring_m);
+        mbar_wait(&s_empty[b], fdiv_small(seq, a.ring_m) & 1u);
+        if (!FUSED) {
+          const int64_t r0 = (t0 + it * ts) * R;
+          const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+          const double* sp = s_part + b * kSlicedTileRows;
+          double* dst = a.o.raw + (size_t)sl * a.n + r0;
+          if (lane < nr) dst[lane] = sp[lane];
+          if (lane + 32 < nr) dst[lane + 32] = sp[lane + 32];
+        }
+        __syncwarp();
+      };
+      for (int64_t it = 0; it < my_tiles; it++) {
+        const uint32_t seq = g + (uint32_t)it;
+        if (it >= (int64_t)ring) drain(it - ring);   // buffer seq % ring is free again
+        if (lane == 0) {
+          const int64_t tile = t0 + it * ts;
+          const int64_t ahead = a.prefetch ? t0 + (it + a.prefetch) * ts : -1;
+          if (ahead >= 0 && ahead < ntiles)   // optional L2 prefetch of a later tile
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
+                         "r"((uint32_t)a.tstride) : "memory");
+          uint64_t* bar = &s_full[fmod_small(seq, nbars, a.bars_m)];
+          fence_proxy_async_smem();
+          mbar_expect_tx(bar, (uint32_t)a.tstride);
+          bulk_g2s(s_ring + (size_t)fmod_small(seq, ring, a.ring_m) * a.tstride,
+                   reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride, (uint32_t)a.tstride, bar);
+        }
+        __syncwarp();
+      }
+      for (int64_t it = my_tiles > (int64_t)ring ? my_tiles - ring : 0; it < my_tiles; it++) drain(it);
+    } else {
+    // ---- consumers
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
     const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
     const int2* __restrict__ meta =
         LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
     mbar_wait(s_forest, ph_forest);
-    ph_forest ^= 1u;
 
-    constexpr int kUnits = kSlicedTileRows / 4;
     const uint64_t total = (uint64_t)my_tiles * kUnits;
     for (;;) {
       uint32_t q = 0;
@@ -1391,14 +1384,18 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
             atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[r0 + rr]), (unsigned long long)fv);
         }
       }
-      release(b, kUnits, it, my_tiles, t0, ts, sl, r0, nr, gt);
+      // the unit is done with buffer b (its partials are in s_part): release-arrive on empty[b]
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[b])) : "memory");
     }
+    }
+    ph_forest ^= 1u;
     g += (uint32_t)my_tiles;
     __syncthreads();
     if (threadIdx.x == 0) *s_next = 0u;
     __syncthreads();
   }
-  if (PROF) prof_lanes(a.prof, lane_total);
+  if (PROF && warp != PW) prof_lanes(a.prof, lane_total);
 }
 
 static int grid_for(int64_t n, int block, int num_sms, int per_sm);

@@ -287,7 +287,8 @@ def run_tree_sharded(args, cfg):
     n = cfg.n_samples * reps
     f = gen.make_forest(cfg, leaf_mode="normal")
     t0 = time.perf_counter()
-    full = T.Forest(f, device=-1).layout(gen.make_calibration(cfg))
+    # rank 0 lays the full forest out once; the other ranks apply its layout state (dist.shared_layout)
+    full = D.shared_layout(T.Forest(f, device=-1), gen.make_calibration(cfg) if rank == 0 else None)
     S = full.shard(rank, world, device=local)
     layout_s = time.perf_counter() - t0
     Xh = gen.make_rows(cfg, cfg.n_samples)

@@ -203,6 +203,18 @@ tahoe_status tahoe_predict_host(const tahoe_forest* f, const float* X_host, int6
  */
 tahoe_status tahoe_forest_l2_persist(const tahoe_forest* f, tahoe_stream stream, float hit_ratio);
 
+/*
+ * tahoe_forest_layout_export / _import — the layout state of a handle (calibration counts, hot
+ * children, expected reads, tree order, the kept simulation rows, the options) as an opaque byte
+ * blob, so one rank lays a forest out (Algorithm 1 lines 5-7) and the others apply the result to
+ * their own build of the same node arrays (e.g. before tahoe_forest_shard) instead of repeating
+ * it.  export: *size = blob bytes; buf may be NULL (size query), else cap >= *size (E_INVAL
+ * otherwise).  import: E_INVAL unless the blob came from a forest with the same trees and nodes;
+ * then re-encodes and re-uploads the images (must not overlap predictions on the handle).
+ */
+tahoe_status tahoe_forest_layout_export(const tahoe_forest* f, void* buf, int64_t cap, int64_t* size);
+tahoe_status tahoe_forest_layout_import(tahoe_forest* f, const void* buf, int64_t size);
+
 /* ---------------- hardware parameters (Algorithm 1 line 4) ---------------- */
 
 /*

@@ -547,6 +547,33 @@ using namespace tahoe;
   catch (const std::exception& ex) { return fail(TAHOE_E_INVAL, ex.what()); }  \
   catch (...) { return fail(TAHOE_E_INVAL, "unknown exception"); }
 
+// ---- layout state export / import (ship a laid-out forest to other ranks without re-running
+// calibration, similarity detection and balancing; SURVEY §8(e) tree sharding)
+namespace {
+struct BlobW {
+  std::vector<uint8_t> b;
+  template <class T> void put(const T& v) { const uint8_t* p = reinterpret_cast<const uint8_t*>(&v); b.insert(b.end(), p, p + sizeof(T)); }
+  template <class T> void vec(const std::vector<T>& v) {
+    put<int64_t>((int64_t)v.size());
+    const uint8_t* p = reinterpret_cast<const uint8_t*>(v.data());
+    b.insert(b.end(), p, p + v.size() * sizeof(T));
+  }
+};
+struct BlobR {
+  const uint8_t* p; int64_t n, o = 0;
+  template <class T> bool get(T& v) { if (o + (int64_t)sizeof(T) > n) return false; std::memcpy(&v, p + o, sizeof(T)); o += sizeof(T); return true; }
+  template <class T> bool vec(std::vector<T>& v) {
+    int64_t k;
+    if (!get(k) || k < 0 || o + k * (int64_t)sizeof(T) > n) return false;
+    v.resize((size_t)k);
+    std::memcpy(v.data(), p + o, (size_t)k * sizeof(T));
+    o += k * (int64_t)sizeof(T);
+    return true;
+  }
+};
+constexpr uint32_t kLayoutMagic = 0x59414c54u;   // "TLAY"
+}  // namespace
+
 extern "C" {
 
 __attribute__((visibility("default"))) const char* tahoe_last_error(void) { return g_err.c_str(); }
@@ -611,6 +638,67 @@ static tahoe_status layout_opts_fill(const tahoe_layout_opts* opts, tahoe_layout
   if (o->m_chunks <= 0) o->m_chunks = 64;
   if (o->m_chunks > o->l_hash) return fail(TAHOE_E_INVAL, "m_chunks > l_hash");
   return TAHOE_OK;
+}
+
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_layout_export(
+    const tahoe_forest* f, void* buf, int64_t cap, int64_t* size) {
+  TAHOE_GUARD_BEGIN
+  if (!f || !size) return fail(TAHOE_E_INVAL, "NULL argument");
+  const Forest& F = f->host;
+  BlobW w;
+  w.put<uint32_t>(kLayoutMagic);
+  w.put<int32_t>(1);                                     // version
+  w.put<int32_t>(F.n_trees);
+  w.put<int64_t>((int64_t)F.feat.size());
+  w.put(F.opts);
+  w.put<int32_t>(F.calibrated ? 1 : 0);
+  w.put<int64_t>(F.n_cal);
+  w.put<int32_t>(F.dsim);
+  w.vec(F.count);
+  w.vec(F.hot_left);
+  w.vec(F.exp_reads);
+  w.vec(F.order);
+  w.vec(F.Xsim);
+  *size = (int64_t)w.b.size();
+  if (!buf) return TAHOE_OK;
+  if (cap < *size) return fail(TAHOE_E_INVAL, "buffer too small");
+  std::memcpy(buf, w.b.data(), w.b.size());
+  return TAHOE_OK;
+  TAHOE_GUARD_END
+}
+
+__attribute__((visibility("default"))) tahoe_status tahoe_forest_layout_import(
+    tahoe_forest* f, const void* buf, int64_t size) {
+  TAHOE_GUARD_BEGIN
+  if (!f || !buf || size <= 0) return fail(TAHOE_E_INVAL, "bad argument");
+  Forest& F = f->host;
+  BlobR r{static_cast<const uint8_t*>(buf), size};
+  uint32_t magic = 0;
+  int32_t ver = 0, T = 0, cal = 0, dsim = 0;
+  int64_t N = 0, ncal = 0;
+  tahoe_layout_opts opts{};
+  Forest G = F;   // applied only when the whole blob parses and matches this forest
+  bool ok = r.get(magic) && magic == kLayoutMagic && r.get(ver) && ver == 1 && r.get(T) &&
+            r.get(N) && r.get(opts) && r.get(cal) && r.get(ncal) && r.get(dsim) &&
+            r.vec(G.count) && r.vec(G.hot_left) && r.vec(G.exp_reads) && r.vec(G.order) &&
+            r.vec(G.Xsim) && r.o == size;
+  if (!ok) return fail(TAHOE_E_INVAL, "not a layout state blob");
+  if (T != F.n_trees || N != (int64_t)F.feat.size() || (int64_t)G.count.size() != N ||
+      (int64_t)G.hot_left.size() != N || (int64_t)G.exp_reads.size() != T || (int64_t)G.order.size() != T ||
+      (dsim > 0 && (int64_t)G.Xsim.size() % dsim != 0))
+    return fail(TAHOE_E_INVAL, "layout state does not match this forest");
+  std::vector<int32_t> seen((size_t)T, 0);
+  for (int32_t t : G.order) {
+    if (t < 0 || t >= T || seen[t]++) return fail(TAHOE_E_INVAL, "layout state: bad tree order");
+  }
+  G.opts = opts;
+  G.calibrated = cal != 0;
+  G.n_cal = ncal;
+  G.dsim = dsim;
+  F = std::move(G);
+  return encode_and_upload(f);
+  TAHOE_GUARD_END
 }
 
 __attribute__((visibility("default"))) tahoe_status tahoe_count_visits(

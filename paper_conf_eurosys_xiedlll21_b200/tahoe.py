@@ -55,7 +55,8 @@ SYMBOLS = ("tahoe_forest_build", "tahoe_forest_layout", "tahoe_predict", "tahoe_
            "tahoe_lsh_order", "tahoe_sha1", "tahoe_forest_export_sliced", "tahoe_count_visits",
            "tahoe_forest_layout_counts", "tahoe_forest_l2_persist", "tahoe_comm_unique_id",
            "tahoe_comm_init", "tahoe_comm_free", "tahoe_reduce_rows", "tahoe_predict_reduce",
-           "tahoe_reduce_partials", "tahoe_measure_visit_rate", "tahoe_profile_walk")
+           "tahoe_reduce_partials", "tahoe_measure_visit_rate", "tahoe_profile_walk",
+           "tahoe_forest_layout_export", "tahoe_forest_layout_import")
 
 
 def lib_path() -> str:
@@ -109,6 +110,8 @@ def load(build_if_missing: bool = True):
         "tahoe_reduce_partials": (st, [P, P, i32, i32, i32, i64, P, P, P]),
         "tahoe_measure_visit_rate": (st, [i32, i32, i32, i32, P, P]),
         "tahoe_profile_walk": (st, [P, P, i64, i32, P, P, P]),
+        "tahoe_forest_layout_export": (st, [P, P, i64, P]),
+        "tahoe_forest_layout_import": (st, [P, P, i64]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -169,6 +172,19 @@ def tahoe_forest_layout(h, X_calib: np.ndarray, opts: LayoutOpts | None = None):
     X = np.ascontiguousarray(X_calib, dtype=np.float32)
     _check(load().tahoe_forest_layout(h, _np_ptr(X), X.shape[0], X.shape[1],
                                       None if opts is None else ctypes.byref(opts)))
+
+
+def tahoe_forest_layout_export(h) -> bytes:
+    n = ctypes.c_int64()
+    _check(load().tahoe_forest_layout_export(h, None, 0, ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(max(1, n.value))
+    _check(load().tahoe_forest_layout_export(h, buf, n.value, ctypes.byref(n)))
+    return buf.raw[: n.value]
+
+
+def tahoe_forest_layout_import(h, blob: bytes):
+    buf = ctypes.create_string_buffer(blob, len(blob))
+    _check(load().tahoe_forest_layout_import(h, buf, len(blob)))
 
 
 def tahoe_forest_l2_persist(h, stream=None, hit_ratio: float = 1.0):
@@ -473,6 +489,15 @@ class Forest:
                               kw.get("node_reorder", 1), kw.get("tree_group", 1), 0,
                               kw.get("seed", 0))
         tahoe_forest_layout(self.handle, X_calib, opts)
+        return self
+
+    def layout_state(self) -> bytes:
+        """The handle's layout state (tahoe_forest_layout_export) — ship it to other ranks."""
+        return tahoe_forest_layout_export(self.handle)
+
+    def apply_layout_state(self, blob: bytes):
+        """Apply another handle's layout of the same forest (tahoe_forest_layout_import)."""
+        tahoe_forest_layout_import(self.handle, blob)
         return self
 
     def layout_gpu(self, X_calib_dev, **kw):

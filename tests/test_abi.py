@@ -350,3 +350,30 @@ def test_wide_code_layout_host():
     leaf, _ = decode_sliced(img, X, len(f["root"]), f["n_classes"])
     assert np.array_equal(leaf, oracle.predict(f, X, want_leaf=True)["leaf"])
     T.tahoe_forest_free(h)
+
+
+def test_layout_state_export_import_roundtrip():
+    """tahoe_forest_layout_export / _import: a second build of the same arrays that imports the
+    first handle's layout state has the same counts, hot children, expected reads, tree order and
+    the same encoded sliced image; blobs from another forest or garbage are refused (E_INVAL)."""
+    import gen
+    from paper_conf_eurosys_xiedlll21_b200 import tahoe as T
+    f = gen.make_forest(3, n_trees=60)
+    a = T.Forest(f, device=-1).layout(gen.make_calibration(3, 3000))
+    blob = a.layout_state()
+    b = T.Forest(f, device=-1).apply_layout_state(blob)
+    ia = T.tahoe_forest_layout_info(a.handle, len(f["feature"]), a.n_trees)
+    ib = T.tahoe_forest_layout_info(b.handle, len(f["feature"]), b.n_trees)
+    for k in ("count", "hot_left", "exp_reads", "order"):
+        assert np.array_equal(ia[k], ib[k]), k
+    ea, eb = a.export_sliced(), b.export_sliced()
+    for k in ("nodes", "leaf_meta", "col_len", "slice_info"):
+        assert np.array_equal(ea[k], eb[k]), k
+    assert a.stats()["lockstep_eff_sim"] == b.stats()["lockstep_eff_sim"]
+    other = T.Forest(gen.make_forest(3, n_trees=61), device=-1)
+    with pytest.raises(T.TahoeError):
+        other.apply_layout_state(blob)
+    with pytest.raises(T.TahoeError):
+        b.apply_layout_state(b"not a layout blob at all")
+    with pytest.raises(T.TahoeError):
+        b.apply_layout_state(blob[:-3])

@@ -101,6 +101,14 @@ def _worker(rank, world, port, q):
         ref = oracle.predict(f, X, agg=oracle.AGG_CLASS_SUM)
         assert np.array_equal(s.numpy(), ref["raw"][lo:hi])
 
+        # one rank lays the forest out, every rank applies the same layout (dist.shared_layout)
+        g = T.Forest(f, device=-1)
+        D.shared_layout(g, gen.make_calibration(3, 1000) if rank == 0 else None)
+        order = T.tahoe_forest_layout_info(g.handle, len(f["feature"]), g.n_trees)["order"]
+        orders = [None] * world
+        dist.all_gather_object(orders, order.tolist())
+        ref_order = T.tahoe_forest_layout_info(full, len(f["feature"]), 56)["order"]
+        assert all(o == ref_order.tolist() for o in orders), "every rank has rank 0's layout"
         m = D.max_over_ranks(float(rank) + 0.5)
         assert m == world - 0.5
         T.tahoe_forest_free(sh)

@@ -319,7 +319,9 @@ static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   st.n_slices = f->sl.n_slices;
   st.num_sms = f->num_sms;
   st.n_trees = (int32_t)f->di.root.size();
-  const int64_t rs = rows_smem_bytes(d, st.n_trees);
+  st.d = d;
+  st.n_out = f->host.n_out();
+  const int64_t rs = rows_smem_bytes(d, st.n_trees, f->host.n_out());
   st.rows_ok = rs <= (int64_t)f->max_smem - 1024;
   st.rows_per_sm = (int32_t)std::max<int64_t>(1, std::min<int64_t>(4, 232448 / (rs + 1024)));
   return st;
@@ -1068,6 +1070,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"trees_per_lane\":" << f->sl.trees_per_lane << ",\"cost_fitted\":"
      << (cost_params().fitted ? "true" : "false")
      << ",\"rows_ok\":" << (plan_stats(f).rows_ok ? "true" : "false")
+     << ",\"sliced_rows_global\":" << (plan_stats(f).rows_global ? "true" : "false")
      << ",\"num_sms\":" << f->num_sms << ",\"max_smem\":" << f->max_smem << "}";
   std::string s = js.str();
   if ((int64_t)s.size() + 1 > len) return fail(TAHOE_E_INVAL, "buffer too small");

@@ -12,9 +12,10 @@
 //   coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs
 //            the rank-coded slices (reading R7): the same busiest-CTA node reads at a cheaper
 //            per-read cost b_c, plus the row-coding pre-pass (passes of 32 attributes per row);
-//   rows   : T = a_r + max(b_r * ceil(T_trees / 512) * V / T_trees, c_r * n * V / SMs)
+//   rows   : T = a_r + max(b_r * ceil(T_trees / 512) * V / T_trees, n * (c_r V + k_r C + w_r d) / SMs)
 //            one CTA per sample (small batches): the chain of dependent node reads of one thread
-//            (L2 latency per read) while the GPU is not full, the node-read throughput beyond.
+//            (L2 latency per read) while the GPU is not full, the per-row throughput beyond (node
+//            reads, the block reduction per output class, the row staging per attribute).
 // V = expected node reads per sample (calibrated E[path] + 1 leaf read, summed over trees,
 // reading Z16).  The constants are fitted on the chip by scripts/fit_costmodel.py and read from
 // costmodel_b200.json next to libtahoe.so (or $TAHOE_COSTMODEL); defaults are round-1 B200
@@ -80,6 +81,8 @@ const CostParams& cost_params() {
     if (read_key(js, "a_r", &v)) c.a_r = v;
     if (read_key(js, "b_r", &v)) c.b_r = v;
     if (read_key(js, "c_r", &v)) c.c_r = v;
+    if (read_key(js, "k_r", &v)) c.k_r = v;
+    if (read_key(js, "w_r", &v)) c.w_r = v;
     c.fitted = all;
     return c;
   }();
@@ -111,7 +114,8 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
     // (c_r per node read per SM)
     if (!st.rows_ok) return INFINITY;
     const double chain = std::ceil((double)st.n_trees / kRowsThreads) * st.V / std::max(1, st.n_trees);
-    return c.a_r + std::max(c.b_r * chain, c.c_r * (double)n * st.V / sms);
+    const double per_row = c.c_r * st.V + c.k_r * st.n_out + c.w_r * st.d;
+    return c.a_r + std::max(c.b_r * chain, (double)n * per_row / sms);
   }
   const double g = st.wide_rows ? c.g_d : 1.0;
   return c.a_d + g * std::max(c.l_d * st.V, c.b_d * st.V * (double)n / sms);

@@ -153,6 +153,8 @@ struct PlanStats {
   bool rows_ok = false;      // the ROWS strategy fits shared memory (row + per-tree values)
   int32_t rows_per_sm = 1;   // resident ROWS CTAs per SM
   int32_t n_trees = 1;
+  int32_t d = 0;             // attributes per row of the batch
+  int32_t n_out = 1;         // output groups (classes)
 };
 // Fitted per-platform constants (costmodel_b200.json, scripts/fit_costmodel.py), microseconds.
 struct CostParams {
@@ -162,9 +164,9 @@ struct CostParams {
   double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
   double a_c = 30.0, b_c = 6.6e-5, e_c = 1.6e-5; // coded: launches; per unit; per row-pass per SM
   double a_w = 40.0, b_w = 1.5e-4, e_w = 1.6e-5; // wide codes (reading R8): the same three terms
-  // rows (f1): launch; per dependent node read (latency); per node read per SM (throughput) —
-  // fitted on the B200 latency sweep (profiles/r02_latency.md)
-  double a_r = 2.0, b_r = 0.9, c_r = 8.1e-4;
+  // rows (f1): launch; per dependent node read (latency); per row and SM (throughput): per node
+  // read, per output class (the block reduction), per attribute (row staging)
+  double a_r = 2.0, b_r = 0.9, c_r = 3.3e-4, k_r = 0.2, w_r = 2.4e-4;
   bool fitted = false;
 };
 const CostParams& cost_params();

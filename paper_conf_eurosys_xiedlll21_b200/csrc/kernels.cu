@@ -2476,19 +2476,6 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
 // class's fp64 sum is formed by a fixed-order block reduction (each thread a contiguous chunk of the
 // class's tree slots, then a fixed butterfly), and the block finalises the row (reading Z14/Z17).
 // One launch, no scratch: CUDA-graph capturable.
-__device__ __forceinline__ double block_sum_fixed(double v, double* red) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = blockDim.x >> 5;
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-  __syncthreads();
-  if (lane == 0) red[warp] = v;
-  __syncthreads();
-  double t = lane < W ? red[lane] : 0.0;
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
-  return t;   // every lane of every warp: the same bits
-}
-
 template <bool LEAF>
 __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -2529,35 +2516,51 @@ __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
       }
     }
     __syncthreads();
-    // a9 combine: per class, a fixed-order fp64 sum of its tree slots (VOTE: exact counts)
-    int best = 0;
-    double bv = 0.0;
+    // a9 combine: per class a fixed-order fp64 sum of its tree slots (VOTE: exact counts) — each
+    // thread a contiguous chunk, a warp butterfly, the warps' values summed in warp order; all
+    // classes share the two block barriers
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = B >> 5;
     for (int32_t c = 0; c < C; c++) {
       const int32_t s0 = vote ? 0 : __ldg(&a.img.cls_seg[c]), s1 = vote ? T : __ldg(&a.img.cls_seg[c + 1]);
-      const int32_t len = s1 - s0, chunk = (len + B - 1) / B;
+      const int32_t chunk = (s1 - s0 + B - 1) / B;
       const int32_t q0 = s0 + threadIdx.x * chunk, q1 = min(s1, q0 + chunk);
       double part = 0.0;
       for (int32_t q = q0; q < q1; q++)
         part += vote ? (s_val[q] == (float)c ? 1.0 : 0.0) : (double)s_val[q];
-      const double sum = block_sum_fixed(part, s_red);
-      if (threadIdx.x == 0) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+      if (lane == 0) s_red[c * W + warp] = part;
+    }
+    __syncthreads();
+    double* s_cls = s_red + (size_t)C * W;
+    for (int32_t c = threadIdx.x; c < C; c += B) {
+      double sum = 0.0;
+      for (int w = 0; w < W; w++) sum += s_red[c * W + w];
+      s_cls[c] = sum;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int best = 0;
+      double bv = 0.0;
+      for (int32_t c = 0; c < C; c++) {
+        const double sum = s_cls[c];
         if (a.o.raw) {
           a.o.raw[i * C + c] = sum;
-        } else {
-          // a10 finalize (as finalize_row / write_scalar)
-          double v;
-          if (vote) v = sum;
-          else if (a.o.agg == TAHOE_AGG_AVERAGE) v = sum / (double)a.o.n_trees_full + (double)a.o.base;
-          else v = sum + (double)a.o.base;
-          a.o.out[i * C + c] = (float)v;
-          if (c == 0 || v > bv) { best = c; bv = v; }
+          continue;
         }
+        // a10 finalize (as finalize_row / write_scalar)
+        double v;
+        if (vote) v = sum;
+        else if (a.o.agg == TAHOE_AGG_AVERAGE) v = sum / (double)a.o.n_trees_full + (double)a.o.base;
+        else v = sum + (double)a.o.base;
+        a.o.out[i * C + c] = (float)v;
+        if (c == 0 || v > bv) { best = c; bv = v; }
       }
-    }
-    if (threadIdx.x == 0 && !a.o.raw && a.o.out_class) {
-      if (a.o.agg == TAHOE_AGG_BINARY) a.o.out_class[i] = bv > 0.0 ? 1 : 0;
-      else if (a.o.agg == TAHOE_AGG_CLASS_SUM || vote) a.o.out_class[i] = best;
-      else a.o.out_class[i] = 0;
+      if (!a.o.raw && a.o.out_class) {
+        if (a.o.agg == TAHOE_AGG_BINARY) a.o.out_class[i] = bv > 0.0 ? 1 : 0;
+        else if (a.o.agg == TAHOE_AGG_CLASS_SUM || vote) a.o.out_class[i] = best;
+        else a.o.out_class[i] = 0;
+      }
     }
     if (LEAF && a.o.out_fp) {
 #pragma unroll
@@ -2575,7 +2578,7 @@ __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
 
 int launch_rows(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                 int32_t num_sms, void* stream) {
-  const int64_t smem = rows_smem_bytes(d, img.n_slots);
+  const int64_t smem = rows_smem_bytes(d, img.n_slots, o.n_classes);
   if (smem > kMaxSmemOptin - 1024) return (int)cudaErrorInvalidValue;
   DirectKArgs a{img, X, n, d, o};
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;

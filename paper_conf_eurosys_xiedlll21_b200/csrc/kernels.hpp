@@ -222,8 +222,10 @@ int launch_finalize(const FinalizeArgs& a, void* stream);
 // image, fixed-order block reduction and in-kernel finalize; one launch, no scratch.  Returns
 // cudaErrorInvalidValue when the row + per-tree values exceed the shared memory it may use.
 constexpr int32_t kRowsThreads = 512;
-inline int64_t rows_smem_bytes(int32_t d, int32_t n_slots) {   // row | per-tree values | reduction
-  return ((int64_t)d * 4 + 15) / 16 * 16 + ((int64_t)n_slots * 4 + 15) / 16 * 16 + 64 * 8;
+// row | per-tree values | per-(class, warp) partials + per-class sums
+inline int64_t rows_smem_bytes(int32_t d, int32_t n_slots, int32_t n_out = 1) {
+  return ((int64_t)d * 4 + 15) / 16 * 16 + ((int64_t)n_slots * 4 + 15) / 16 * 16 +
+         (int64_t)n_out * (kRowsThreads / 32 + 1) * 8;
 }
 int launch_rows(const DevDirect& img, const float* X, int64_t n, int32_t d, const OutArgs& o,
                 int32_t num_sms, void* stream);

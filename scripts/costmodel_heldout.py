@@ -58,7 +58,8 @@ def predict(p, r, s):
         if not r["rows_ok"]:
             return math.inf
         chain = math.ceil(r["n_trees"] / 512) * r["V"] / max(1, r["n_trees"])
-        return p["a_r"] + max(p["b_r"] * chain, p["c_r"] * r["n"] * r["V"] / sms)
+        per_row = p["c_r"] * r["V"] + p["k_r"] * r["n_out"] + p["w_r"] * r["d"]
+        return p["a_r"] + max(p["b_r"] * chain, r["n"] * per_row / sms)
     g = p["g_d"] if r["wide_rows"] else 1.0
     return p["a_d"] + g * max(p["l_d"] * r["V"], p["b_d"] * r["V"] * r["n"] / sms)
 
@@ -83,7 +84,7 @@ def fit(rows, base):
     fit_keys(["a_s", "b_s", "g_s"], "sliced", rows, [p["a_s"], p["b_s"], p["g_s"]])
     fit_keys(["a_c", "b_c", "e_c"], "coded", [r for r in rows if not r["code8"]], [p["a_c"], p["b_c"], p["e_c"]])
     fit_keys(["a_w", "b_w", "e_w"], "coded", [r for r in rows if r["code8"]], [p["a_w"], p["b_w"], p["e_w"]])
-    fit_keys(["a_r", "b_r", "c_r"], "rows", rows, [p["a_r"], p["b_r"], p["c_r"]])
+    fit_keys(["a_r", "b_r", "c_r", "k_r", "w_r"], "rows", rows, [p["a_r"], p["b_r"], p["c_r"], p["k_r"], p["w_r"]])
     return p
 
 
@@ -134,7 +135,8 @@ def measure():
                      sliced_ok=st["sliced_valid"], coded_ok=st["sliced_valid"] and st["coded_valid"],
                      code8=bool(st["code8"]), rows_ok=st["rows_ok"], n_trees=st["n_trees"],
                      code_passes=max(1, (1 << (st["code8_vfbits"] if st["code8"] else st["sliced_fbits"])) // 32),
-                     rows_global=False, wide_rows=X.shape[1] > 256)
+                     rows_global=bool(st["sliced_rows_global"]), wide_rows=X.shape[1] > 256,
+                     d=X.shape[1], n_out=F.n_out)
             # the library's own predictions with the shipped constants (checks the restatement)
             r["lib_pred_us"] = {s: F.predict_cost_us(ids[s], n) for s in STRATS}
             for s in STRATS:
@@ -150,7 +152,8 @@ def measure():
 def main():
     shipped = json.load(open(os.path.join(ROOT, "paper_conf_eurosys_xiedlll21_b200", "costmodel_b200.json")))
     base = dict(a_s=22.3, b_s=9.5e-5, g_s=4.0, a_d=11.8, l_d=0.34, b_d=6.3e-4, g_d=4.0, a_c=30.0,
-                b_c=6.6e-5, e_c=1.6e-5, a_w=40.0, b_w=1.5e-4, e_w=1.6e-5, a_r=2.0, b_r=0.9, c_r=8.1e-4)
+                b_c=6.6e-5, e_c=1.6e-5, a_w=40.0, b_w=1.5e-4, e_w=1.6e-5, a_r=2.0, b_r=0.9, c_r=3.3e-4,
+                k_r=0.2, w_r=2.4e-4)
     base.update({k: v for k, v in shipped.items() if k in base})
     if "--refit" in sys.argv:
         rows = json.load(open(sys.argv[sys.argv.index("--refit") + 1]))["rows"]

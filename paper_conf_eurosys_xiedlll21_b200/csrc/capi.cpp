@@ -321,6 +321,7 @@ static PlanStats plan_stats(const tahoe_forest* f, int32_t d = -1) {
   st.n_trees = (int32_t)f->di.root.size();
   st.d = d;
   st.n_out = f->host.n_out();
+  st.scalar = st.n_out == 1 && f->host.agg != TAHOE_AGG_VOTE;
   const int64_t rs = rows_smem_bytes(d, st.n_trees, f->host.n_out());
   st.rows_ok = rs <= (int64_t)f->max_smem - 1024;
   st.rows_per_sm = (int32_t)std::max<int64_t>(1, std::min<int64_t>(4, 232448 / (rs + 1024)));

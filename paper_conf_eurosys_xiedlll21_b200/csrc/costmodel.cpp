@@ -6,9 +6,10 @@
 //            U_s = ceil(tiles / cps) * 64 * V / (slices * eff)
 //            the node reads of the busiest CTA (T_SMEM at the simulated lockstep efficiency eff);
 //            a_s absorbs launch, slice staging and the fixed-order slice reduction (T_G_REDU);
-//   direct : T = a_d + (d > 256 ? g_d : 1) * max(l_d * V, b_d * V * n / SMs)
+//   direct : T = a_d + (d > 256 ? g_d : 1) * max(l_d * V, (tlp ? b_t : b_d) * V * n / SMs)
 //            one thread per sample: latency-bound below a full GPU of threads (l_d per visit),
-//            L1/L2-throughput-bound above it (T_GMEM);
+//            L1/L2-throughput-bound above it (T_GMEM); tlp = the staged-row kernel with eight
+//            threads per row that launch_direct takes for >= 32K rows of scalar outputs;
 //   coded  : T = a_c + b_c * U_s + e_c * ceil(n / 64) * 64 * passes / SMs
 //            the rank-coded slices (reading R7): the same busiest-CTA node reads at a cheaper
 //            per-read cost b_c, plus the row-coding pre-pass (passes of 32 attributes per row);
@@ -82,6 +83,7 @@ const CostParams& cost_params() {
     if (read_key(js, "b_r", &v)) c.b_r = v;
     if (read_key(js, "c_r", &v)) c.c_r = v;
     if (read_key(js, "k_r", &v)) c.k_r = v;
+    if (read_key(js, "b_t", &v)) c.b_t = v;
     if (read_key(js, "w_r", &v)) c.w_r = v;
     c.fitted = all;
     return c;
@@ -118,7 +120,10 @@ double predict_us(const PlanStats& st, int32_t strategy, int64_t n) {
     return c.a_r + std::max(c.b_r * chain, (double)n * per_row / sms);
   }
   const double g = st.wide_rows ? c.g_d : 1.0;
-  return c.a_d + g * std::max(c.l_d * st.V, c.b_d * st.V * (double)n / sms);
+  // >= 32K rows with one output and rows of <= 256 attributes: the staged-row kernel with eight
+  // threads per row (launch_direct's default), a cheaper per-read throughput b_t
+  const bool tlp = n >= 32768 && st.scalar && !st.wide_rows;
+  return c.a_d + g * std::max(c.l_d * st.V, (tlp ? c.b_t : c.b_d) * st.V * (double)n / sms);
 }
 
 int32_t select_strategy(const PlanStats& st, int64_t n, int32_t d, int32_t agg) {

@@ -155,12 +155,14 @@ struct PlanStats {
   int32_t n_trees = 1;
   int32_t d = 0;             // attributes per row of the batch
   int32_t n_out = 1;         // output groups (classes)
+  bool scalar = true;        // one output, not VOTE (the direct large-batch kernel applies)
 };
 // Fitted per-platform constants (costmodel_b200.json, scripts/fit_costmodel.py), microseconds.
 struct CostParams {
   double a_s = 22.3, b_s = 9.5e-5;           // sliced: launch + slice staging; per work unit
   double g_s = 4.0;                          // sliced: slowdown when rows stay in global memory
   double a_d = 11.8, l_d = 0.34, b_d = 6.3e-4; // direct: launch; per-visit latency; per unit
+  double b_t = 2.0e-4;                         // direct, >= 32K rows, scalar: staged rows, 8 threads per row
   double g_d = 4.0;                            // direct: slowdown for wide rows (d > 256)
   double a_c = 30.0, b_c = 6.6e-5, e_c = 1.6e-5; // coded: launches; per unit; per row-pass per SM
   double a_w = 40.0, b_w = 1.5e-4, e_w = 1.6e-5; // wide codes (reading R8): the same three terms

@@ -2,18 +2,27 @@
 //
 // Every (sample, tree) pair walks root -> leaf on "x_j < b_i"; NaN takes the node's
 // default path; leaf values are combined per sample in fp64 (reading Z17) and rounded
-// once to fp32.  Two strategies (Algorithm 1 line 15, re-targeted):
+// once to fp32.  Strategies (Algorithm 1 line 15, re-targeted):
 //
-//  k_direct  — the paper's "direct method": one thread per sample walks every tree
-//              of a forest image that stays in HBM / L2; no shared memory, no reduction.
-//  k_sliced  — the paper's "shared forest" / "splitting shared forest" re-designed:
-//              a persistent CTA keeps one forest SLICE resident in shared memory (cp.async.bulk +
-//              mbarrier), streams sample tiles into shared memory with double-buffered TMA bulk
-//              copies, and a warp evaluates one sample with its 32 lanes walking 32 lane columns
-//              of trees (conflict-free 8-byte node loads, one-row feature loads), then reduces the
-//              32 fp64 lane sums with a shuffle butterfly.  Slices write fp64 partials that a
-//              fixed-order finalize kernel combines; a single-slice forest finalizes in-kernel.
-//  k_finalize — fixed-order fp64 sum of parts per class, base / average / argmax, RN to fp32.
+//  k_direct*        — the paper's "direct method": threads walk trees of a forest
+//                     image that stays in HBM / L2 (one thread per sample, or eight per sample over
+//                     rows staged in shared memory for large batches); images over 64 MB are walked
+//                     in L2-sized chunks of trees (reading R4).
+//  k_sliced         — "shared forest" / "splitting shared forest" re-designed: a
+//                     persistent CTA keeps one forest SLICE (16 lane columns of trees) resident in
+//                     shared memory, streams 64-row sample tiles through a 3-deep TMA ring, and a
+//                     half-warp walks one sample (lane = lane column), two samples per lane.
+//  k_sliced_codes   — the same walk over exact u16 rank codes of the rows (reading R7), produced by
+//                     a pre-pass (k_encode_rows_banks); a producer warp stages the slice and the
+//                     code tiles (cp.async.bulk into a ring of up to 8 tiles, full / empty mbarriers),
+//                     31 consumer warps claim 4-row work units; LEAF / PROF instantiations add leaf
+//                     ids + fingerprints / per-lane timing.
+//  k_sliced_codes8  — wide rows (reading R8): u8 codes over virtual attributes, dynamic tile claiming
+//                     across ~30 slices, four chains per lane.
+//  k_rows           — small batches (f1): one CTA per sample, lane = tree over the direct image,
+//                     fixed-order block reduction and finalize in one launch.
+//  k_finalize       — fixed-order fp64 sum of parts per class, base / average / argmax, RN to fp32.
+//  k_visit_peak / k_smem_bw — the microbenchmarks of Algorithm 1 line 4 (the roofline peak).
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <algorithm>
@@ -1242,8 +1251,11 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   const int64_t ntiles = (a.n + R - 1) / R;
 
   if (threadIdx.x == 0) {
-    for (uint32_t b = 0; b < nbars; b++) mbar_init(&s_full[b], 1);
-    for (uint32_t b = 0; b < ring; b++) mbar_init(&s_empty[b], kUnits);
+    // every lane of the producer arrives on a full barrier (lane 0 with the transaction bytes) and
+    // every consumer lane on an empty barrier: each lane's own shared-memory accesses are released
+    // by its own arrival
+    for (uint32_t b = 0; b < nbars; b++) mbar_init(&s_full[b], 32);
+    for (uint32_t b = 0; b < ring; b++) mbar_init(&s_empty[b], kUnits * 32);
     *s_next = 0u;
     mbar_init(s_forest, 1);
     fence_mbar_init();
@@ -1295,19 +1307,20 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
       for (int64_t it = 0; it < my_tiles; it++) {
         const uint32_t seq = g + (uint32_t)it;
         if (it >= (int64_t)ring) drain(it - ring);   // buffer seq % ring is free again
+        uint64_t* bar = &s_full[fmod_small(seq, nbars, a.bars_m)];
         if (lane == 0) {
           const int64_t tile = t0 + it * ts;
           const int64_t ahead = a.prefetch ? t0 + (it + a.prefetch) * ts : -1;
           if (ahead >= 0 && ahead < ntiles)   // optional L2 prefetch of a later tile
             asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
                          "r"((uint32_t)a.tstride) : "memory");
-          uint64_t* bar = &s_full[fmod_small(seq, nbars, a.bars_m)];
           fence_proxy_async_smem();
           mbar_expect_tx(bar, (uint32_t)a.tstride);
           bulk_g2s(s_ring + (size_t)fmod_small(seq, ring, a.ring_m) * a.tstride,
                    reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride, (uint32_t)a.tstride, bar);
+        } else {
+          asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
         }
-        __syncwarp();
       }
       for (int64_t it = my_tiles > (int64_t)ring ? my_tiles - ring : 0; it < my_tiles; it++) drain(it);
     } else {
@@ -1384,9 +1397,11 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
             atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[r0 + rr]), (unsigned long long)fv);
         }
       }
-      // the unit is done with buffer b (its partials are in s_part): release-arrive on empty[b]
-      __syncwarp();
-      if (lane == 0) asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[b])) : "memory");
+      // the unit is done with buffer b (its partials are in s_part): every lane release-arrives on
+      // empty[b], so each lane's own reads of the tile and writes of s_part are ordered before the
+      // producer's refill (one arrival per lane rather than one per warp after __syncwarp: the same
+      // ordering, and the form compute-sanitizer racecheck tracks)
+      asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[b])) : "memory");
     }
     }
     ph_forest ^= 1u;

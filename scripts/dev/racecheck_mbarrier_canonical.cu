@@ -2,6 +2,9 @@
 // synchronization?  Two canonical hand-offs, each correct under the PTX memory model:
 //   A: warp 0 writes shared memory, arrives (release) on an mbarrier; warp 1 waits (acquire), reads.
 //   B: the same with a __syncthreads() instead of the mbarrier (control).
+//   C: as A, but after __syncwarp() only lane 0 arrives (count 1) for the whole warp — equally
+//      ordered by the PTX memory model (bar.warp.sync orders the lanes' writes before lane 0's
+//      release).
 // nvcc -gencode arch=compute_100a,code=sm_100a -o /tmp/rc racecheck_mbarrier_canonical.cu
 // compute-sanitizer --tool racecheck /tmp/rc A   |   ... /tmp/rc B
 #include <cstdio>
@@ -15,14 +18,16 @@ __global__ void k(int mode, int* out) {
   __shared__ int buf[32];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   if (threadIdx.x == 0) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sa(&bar)), "r"(32) : "memory");
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sa(&bar)), "r"(mode == 2 ? 1 : 32) : "memory");
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (mode == 0) {
+  if (mode == 0 || mode == 2) {
     if (warp == 0) {
       buf[lane] = lane * 3;
-      asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(sa(&bar)) : "memory");
+      if (mode == 2) __syncwarp();
+      if (mode == 0 || lane == 0)
+        asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(sa(&bar)) : "memory");
     } else {
       asm volatile("{\n\t.reg .pred p;\nW:\n\tmbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%0], 0;\n\t@!p bra W;\n}" ::"r"(sa(&bar)) : "memory");
       out[lane] = buf[31 - lane];
@@ -35,12 +40,12 @@ __global__ void k(int mode, int* out) {
 }
 
 int main(int argc, char** argv) {
-  const int mode = (argc > 1 && !strcmp(argv[1], "B")) ? 1 : 0;
+  const int mode = (argc > 1 && !strcmp(argv[1], "B")) ? 1 : (argc > 1 && !strcmp(argv[1], "C")) ? 2 : 0;
   int* d;
   cudaMalloc(&d, 128);
   k<<<1, 64>>>(mode, d);
   int h[32];
   cudaMemcpy(h, d, 128, cudaMemcpyDeviceToHost);
-  printf("mode %s: out[0] = %d (expect 93)\n", mode ? "B (syncthreads)" : "A (mbarrier)", h[0]);
+  printf("mode %s: out[0] = %d (expect 93)\n", mode == 1 ? "B (syncthreads)" : mode == 2 ? "C (lane-0 arrive)" : "A (mbarrier)", h[0]);
   return h[0] == 93 ? 0 : 1;
 }

@@ -1999,7 +1999,6 @@ struct Coded8KArgs {
   int64_t n_all;         // rows of the whole batch (row stride of the raw partials)
   int32_t switch_slices; // 1: a CTA whose slice is exhausted moves to another (0: experiments)
   int32_t prefetch;      // tiles ahead of a claim to prefetch into L2 (0 = none)
-  uint32_t sleep_ns;     // back-off between ticket polls
   int32_t split;         // 1: four chains per lane (each column walked as two halves)
   OutArgs o;
 };
@@ -2135,29 +2134,33 @@ __device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA
 }
 
 // k_sliced_codes8: k_sliced_codes' walk (slice resident in shared memory, dynamic 4-row work
-// units, half-warp per row, two chains per lane, ring refilled by the warp closing a tile) over
-// 16-row tiles of u8 code rows; unit u of a tile: half h walks rows u + 4h (chain A) and
-// u + 8 + 4h (chain B).  Tiles are claimed dynamically from a per-slice global counter, in
-// increasing order (so the ~30 slices sweep the code rows together and each tile is read from
-// HBM about once); a CTA whose slice runs out of tiles moves to the slice with the most remaining
-// work per CTA (re-staging that slice), so no SM idles while another slice still has tiles.
-// Ring entries are numbered by a CTA-wide sequence; entry e uses buffer e % 3 and that buffer's
-// mbarrier phase e / 3, and the warp releasing the last unit of entry e issues entry e + 3.  The
-// ring holds 12 units, fewer than the CTA's warps, so a warp may grab a unit of an entry not
-// issued yet: it waits until the buffer's ticket names its entry (set by the issuing warp), and
-// only then on the mbarrier phase, which is then the current one.  Once the slice's tiles are
-// all claimed, entries are issued EMPTY (tile -1, the phase completes without data) and released
-// like the others, so the chain of tickets never stalls; a warp leaves the slice when it meets an
-// empty entry and every valid entry issued so far has been released.
-constexpr int kCode8Threads = 384;
-// R rows per walked tile (a multiple of the pre-pass tile, whose NaN flags it carries), kR8 tiles
-// in the ring (R * kR8 rows in shared memory).
+// units, half-warp per row, two / four chains per lane) over 8-row tiles of u8 code rows; unit u of
+// a tile: half h walks rows u + 2h (chain A) and u + 4 + 2h (chain B).  Tiles are claimed
+// dynamically from a per-slice global counter (so the ~30 slices sweep the code rows together); a
+// CTA whose slice runs out of tiles moves to the slice with the most remaining work per CTA
+// (re-staging it), so no SM idles while another slice still has tiles.
+// Ring hand-off with mbarriers only: entry e of a slice lives in buffer e % kR8 and completes full
+// barrier e % kFull8 (parity (e / kFull8) & 1); every lane that worked on a unit of entry e arrives
+// on the buffer's empty barrier, and the warp that releases the entry's LAST unit (elected by a
+// per-buffer counter) waits on that empty phase, stores the entry's partials and issues entry
+// e + kR8 into the buffer (all its lanes arrive on the new entry's full barrier, lane 0 with the
+// transaction bytes) — the refill follows the release at once, with no producer warp to wake.  A
+// consumer could wait on a stale full phase only if entry e - kFull8 had not arrived; then the
+// kFull8 / kR8 later entries of that buffer are not issued and their units would hold every other
+// consumer (static_assert below).  Past the slice's last tile an issue is a terminator (tile -1,
+// no data); a buffer that issued one issues only terminators; consumers keep releasing entries
+// and leave once every buffer has issued a terminator and every valid entry has been drained.  The
+// barriers are re-initialised for the next slice.
+constexpr int kCode8Threads = 384;            // 12 warps
+constexpr int kFull8 = 36;                    // full barriers (6 per ring buffer)
 template <bool FUSED, int R, int kR8, bool LEAF>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {
   constexpr int C = kSlicedCols;
   constexpr int FS = R / kCode8TileRows;   // pre-pass tiles (NaN flags) per walked tile
   static_assert(R % kCode8TileRows == 0 && R * kR8 == kCode8TileRows * kCode8Ring, "ring rows");
   constexpr int kUnits = R / 4;
+  constexpr int kWarps = kCode8Threads / 32;
+  static_assert(kFull8 % kR8 == 0 && (kFull8 / kR8) * kUnits >= kWarps, "ring-wrap guard");
   extern __shared__ __align__(1024) unsigned char smem[];
   const uint32_t V = (uint32_t)a.img.vfbits;
   const uint32_t RB = 1u << V;
@@ -2167,18 +2170,18 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
   unsigned char* s_ring = smem + ring_off;
   uint32_t* s_flag = reinterpret_cast<uint32_t*>(s_ring + (size_t)kR8 * tile_bytes);
   double* s_part = reinterpret_cast<double*>(s_flag + kR8 * FS * 4);
-  // control block (kCode8Ctl bytes): mbarriers, unit counter, per-buffer counters, CTA state
-  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_part + kR8 * R);      // [ring] tile arrived
-  uint64_t* s_forest = s_full + kR8;                                       // slice staged
-  unsigned long long* s_next = reinterpret_cast<unsigned long long*>(s_forest + 1);  // unit counter
-  int* s_cnt = reinterpret_cast<int*>(s_next + 1);                         // [ring] units released
-  uint32_t* s_gen = reinterpret_cast<uint32_t*>(s_cnt + kR8);              // [ring] ticket: entry issued
-  int32_t* s_tile = reinterpret_cast<int32_t*>(s_gen + kR8);               // [ring] tile of the entry
-  uint32_t* s_vis = reinterpret_cast<uint32_t*>(s_tile + kR8);            // valid entries issued
-  uint32_t* s_vdone = s_vis + 1;                                           // valid entries released
-  int32_t* s_slice = reinterpret_cast<int32_t*>(s_vis + 2);
-  uint32_t* s_issued = s_vis + 3;                                          // entries issued
-  static_assert(8 * (kR8 + 2) + 12 * kR8 + 16 <= kCode8Ctl, "control block");
+  // control block (kCode8Ctl bytes): barriers, counters, tiles of the ring entries, slice
+  uint64_t* s_full = reinterpret_cast<uint64_t*>(s_part + kR8 * R);   // [kFull8] entry arrived
+  uint64_t* s_empty = s_full + kFull8;                                  // [kR8] entry released
+  uint64_t* s_forest = s_empty + kR8;                                   // slice staged
+  unsigned int* s_next = reinterpret_cast<unsigned int*>(s_forest + 1); // unit counter
+  int32_t* s_cnt = reinterpret_cast<int32_t*>(s_next + 1);              // [kR8] units released
+  int32_t* s_tile = s_cnt + kR8;                                        // [kR8] tile of the entry
+  int32_t* s_vis = s_tile + kR8;                                        // valid entries issued
+  int32_t* s_vdone = s_vis + 1;                                         // valid entries drained
+  int32_t* s_dead = s_vis + 2;                                          // buffers that issued a terminator
+  int32_t* s_slice = s_vis + 3;
+  static_assert(8 * (kFull8 + kR8 + 1) + 4 * (1 + 2 * kR8 + 4) <= kCode8Ctl, "control block");
   const int lane = threadIdx.x & 31;
   const int col = lane & (C - 1);
   const int half = lane >> 4;
@@ -2189,9 +2192,6 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
   const int32_t ntiles = (int32_t)((a.n + R - 1) / R);
 
   if (threadIdx.x == 0) {
-    for (int b = 0; b < kR8; b++) { mbar_init(&s_full[b], 1); s_cnt[b] = 0; s_gen[b] = 0xffffffffu; }
-    mbar_init(s_forest, 1);
-    fence_mbar_init();
     int32_t sl = (int32_t)blockIdx.x % ns;
     if (a.cta_start) {
       sl = 0;
@@ -2200,175 +2200,172 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
     *s_slice = sl;
     atomicAdd(&a.cta_on[sl], 1);
   }
-  __syncthreads();
-
-  uint32_t g = 0;   // sequence number of this slice's first ring entry
-  uint32_t ph_forest = 0;
-  // claim the slice's next tile for entry e (buffer e % 3) and issue its copies; past the slice's
-  // last tile the entry is marked empty (its mbarrier phase completes without data)
-  auto issue = [&](int sl, uint32_t e) {
+  // issue entry e of slice sl into buffer e % kR8 (one whole warp); prev_dead: the buffer already
+  // issued a terminator (then this is one too, without claiming)
+  auto issue = [&](int sl, uint32_t e, bool prev_dead) {
+    const int b = (int)(e % kR8);
+    uint64_t* bar = &s_full[e % kFull8];
     if (lane == 0) {
-      const int b = (int)(e % kR8);
-      const int32_t tile = atomicAdd(&a.tile_next[sl], 1);
-      const bool ok = tile < ntiles;
-      s_tile[b] = ok ? tile : -1;
-      __threadfence_block();   // the buffer's previous partials were read before this point
-      *reinterpret_cast<volatile uint32_t*>(&s_gen[b]) = e;
-      if (!ok) {
-        mbar_expect_tx(&s_full[b], 0u);
-      } else {
-        atomicAdd(s_vis, 1u);
-        // warm L2 with the tile this slice's CTAs will claim a few claims from now (the tiles
-        // are mostly not in L2: the slices drift apart over the batch)
+      int32_t tile = -1;
+      if (!prev_dead) {
+        tile = atomicAdd(&a.tile_next[sl], 1);
+        if (tile >= ntiles) tile = -1;
+      }
+      s_tile[b] = tile;
+      if (tile >= 0) {
+        atomicAdd(s_vis, 1);
+        // warm L2 with the tile this slice's CTAs will claim a few claims from now
         if (a.prefetch > 0 && tile + a.prefetch < ntiles)
           asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a.codes + (int64_t)(tile + a.prefetch) * tile_bytes),
                        "r"(tile_bytes) : "memory");
         fence_proxy_async_smem();
-        mbar_expect_tx(&s_full[b], tile_bytes + 16u * FS);
-        bulk_g2s(s_ring + (size_t)b * tile_bytes, a.codes + (int64_t)tile * tile_bytes, tile_bytes, &s_full[b]);
-        bulk_g2s(s_flag + b * FS * 4, a.flags + (int64_t)tile * FS * 4, 16u * FS, &s_full[b]);
+        mbar_expect_tx(bar, tile_bytes + 16u * FS);
+        bulk_g2s(s_ring + (size_t)b * tile_bytes, a.codes + (int64_t)tile * tile_bytes, tile_bytes, bar);
+        bulk_g2s(s_flag + b * FS * 4, a.flags + (int64_t)tile * FS * 4, 16u * FS, bar);
+      } else {
+        if (!prev_dead) atomicAdd(s_dead, 1);
+        asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
       }
-      atomicAdd(s_issued, 1u);
+    } else {
+      asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
     }
-    __syncwarp();
   };
 
-  for (;;) {
-    const int32_t sl = *s_slice;
-    if (sl < 0) break;
+  for (bool first = true;; first = false) {
+    // (re)initialise the barriers and counters for this slice: every wait of the previous slice
+    // has returned
     if (threadIdx.x == 0) {
-      *s_next = 0ull;
-      *s_vis = 0u;
-      *s_vdone = 0u;
-      *s_issued = 0u;
-      // the last slice's trailing (empty) entries may have been released only partly
+      for (int b = 0; b < kFull8 + kR8 + 1; b++) {
+        if (!first) asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(&s_full[b])) : "memory");
+        mbar_init(&s_full[b], b < kFull8 ? 32u : (b < kFull8 + kR8 ? (uint32_t)(kUnits * 32) : 1u));
+      }
+      *s_next = 0u;
       for (int b = 0; b < kR8; b++) s_cnt[b] = 0;
+      *s_vis = 0;
+      *s_vdone = 0;
+      *s_dead = 0;
+      fence_mbar_init();
     }
     __syncthreads();
+    const int32_t sl = *s_slice;
+    if (sl < 0) break;
     if (threadIdx.x < 32) {
-      if (lane == 0) {
+      if (lane == 0) {   // a7: the slice
         const uint32_t bytes = (uint32_t)a.img.slots[sl] * (uint32_t)kSlotBytes;
         fence_proxy_async_smem();
         mbar_expect_tx(s_forest, bytes);
         bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
-      for (uint32_t q = 0; q < (uint32_t)kR8; q++) issue(sl, g + q);
+      for (uint32_t q = 0; q < (uint32_t)kR8; q++) issue(sl, q, false);
     }
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
     const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
     const int2* __restrict__ meta =
         LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
-    mbar_wait(s_forest, ph_forest);
-    ph_forest ^= 1u;
+    mbar_wait(s_forest, 0u);
     for (;;) {
-      unsigned long long q = 0;
-      if (lane == 0) q = atomicAdd(s_next, 1ull);
+      uint32_t q = 0;
+      if (lane == 0) q = atomicAdd(s_next, 1u);
       q = __shfl_sync(0xffffffffu, q, 0);
-      const uint32_t it = (uint32_t)(q / kUnits);
+      const uint32_t e = q / kUnits;
       const int u = (int)(q % kUnits);
-      const uint32_t e = g + it;
       const int b = (int)(e % kR8);
-      if (lane == 0)
-        while (*reinterpret_cast<volatile uint32_t*>(&s_gen[b]) != e) {
-          if (a.sleep_ns) __nanosleep(a.sleep_ns);
-        }
-      __syncwarp();
-      mbar_wait(&s_full[b], (e / kR8) & 1u);
-      const int32_t tile = *reinterpret_cast<volatile int32_t*>(&s_tile[b]);
-      const int64_t r0 = (int64_t)tile * R;
-      const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-      if (tile >= 0 && u < nr) {
-        const int rA = u + (R / 4) * half, rB = rA + R / 2;
-        const bool okA = rA < nr, okB = rB < nr;
-        const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
-        const uint32_t tb = sbase + ring_off + (uint32_t)b * tile_bytes;
-        const uint32_t rowA = tb + ((uint32_t)(okA ? rA : u) << V);
-        const uint32_t rowB = tb + ((uint32_t)(okB ? rB : u) << V);
-        uint32_t nan_flag = 0;
+      mbar_wait(&s_full[e % kFull8], (e / kFull8) & 1u);
+      const int32_t tile = s_tile[b];
+      if (tile >= 0) {
+        const int64_t r0 = (int64_t)tile * R;
+        const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+        if (u < nr) {
+          const int rA = u + (R / 4) * half, rB = rA + R / 2;
+          const bool okA = rA < nr, okB = rB < nr;
+          const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
+          const uint32_t tb = sbase + ring_off + (uint32_t)b * tile_bytes;
+          const uint32_t rowA = tb + ((uint32_t)(okA ? rA : u) << V);
+          const uint32_t rowB = tb + ((uint32_t)(okB ? rB : u) << V);
+          uint32_t nan_flag = 0;
 #pragma unroll
-        for (int k = 0; k < FS; k++) {
-          uint32_t fk;
-          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(fk) : "r"(smem_u32(s_flag + (b * FS + k) * 4)));
-          nan_flag |= fk;
-        }
-        double accA, accB;
-        uint64_t fpA = 0, fpB = 0;
-        int32_t* oA = nullptr;
-        int32_t* oB = nullptr;
-        if (LEAF && a.o.out_leaf) {
-          if (okA) oA = a.o.out_leaf + (a.row0 + r0 + rA) * (int64_t)a.o.T_leaf;
-          if (okB) oB = a.o.out_leaf + (a.row0 + r0 + rB) * (int64_t)a.o.T_leaf;
-        }
-        if (a.split) {
-          const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
-          const uint32_t mA = okA ? pm : pe, mB = okB ? pm : pe;
-          if (LEAF) {
-            if (nan_flag) walk_coded8_split_leaf<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
-            else walk_coded8_split_leaf<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
-          } else {
-            if (nan_flag) walk_coded8_split<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-            else walk_coded8_split<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          for (int k = 0; k < FS; k++) {
+            uint32_t fk;
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(fk) : "r"(smem_u32(s_flag + (b * FS + k) * 4)));
+            nan_flag |= fk;
           }
-        } else if (LEAF) {
-          if (nan_flag) walk_coded8_leaf<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
-          else walk_coded8_leaf<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
-        } else if (nan_flag) {
-          walk_coded8<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-        } else {
-          walk_coded8<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-        }
-        // butterfly over the 16 lane columns: after the xor-8 exchange lanes with bit 3 clear
-        // hold chain A, set hold chain B (lanes 0, 8, 16, 24 own rows rA(h=0), rB(h=0), rA(h=1),
-        // rB(h=1))
-        const bool b3 = lane & 8;
-        double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
+          double accA, accB;
+          uint64_t fpA = 0, fpB = 0;
+          int32_t* oA = nullptr;
+          int32_t* oB = nullptr;
+          if (LEAF && a.o.out_leaf) {
+            if (okA) oA = a.o.out_leaf + (a.row0 + r0 + rA) * (int64_t)a.o.T_leaf;
+            if (okB) oB = a.o.out_leaf + (a.row0 + r0 + rB) * (int64_t)a.o.T_leaf;
+          }
+          if (a.split) {
+            const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
+            const uint32_t mA = okA ? pm : pe, mB = okB ? pm : pe;
+            if (LEAF) {
+              if (nan_flag) walk_coded8_split_leaf<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+              else walk_coded8_split_leaf<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+            } else {
+              if (nan_flag) walk_coded8_split<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+              else walk_coded8_split<false>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+            }
+          } else if (LEAF) {
+            if (nan_flag) walk_coded8_leaf<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+            else walk_coded8_leaf<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+          } else if (nan_flag) {
+            walk_coded8<true>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          } else {
+            walk_coded8<false>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          }
+          // butterfly over the 16 lane columns: after the xor-8 exchange lanes with bit 3 clear
+          // hold chain A, set hold chain B (lanes 0, 8, 16, 24 own rows rA(h=0), rB(h=0), rA(h=1),
+          // rB(h=1))
+          const bool b3 = lane & 8;
+          double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
 #pragma unroll
-        for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        uint64_t fv = 0;
-        if (LEAF) {
-          fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
+          for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+          uint64_t fv = 0;
+          if (LEAF) {
+            fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
 #pragma unroll
-          for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
+            for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
+          }
+          const int rr = b3 ? rB : rA;
+          if ((lane & 7) == 0 && (b3 ? okB : okA)) {
+            if (FUSED) write_scalar(a.o, a.row0 + r0 + rr, v);
+            else s_part[b * R + rr] = v;
+            if (LEAF && a.o.out_fp)
+              atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[a.row0 + r0 + rr]), (unsigned long long)fv);
+          }
         }
-        const int rr = b3 ? rB : rA;
-        if ((lane & 7) == 0 && (b3 ? okB : okA)) {
-          if (FUSED) write_scalar(a.o, a.row0 + r0 + rr, v);
-          else s_part[b * R + rr] = v;
-          if (LEAF && a.o.out_fp)
-            atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[a.row0 + r0 + rr]), (unsigned long long)fv);
-        }
-      }
-      // release the unit; the warp closing the entry writes its partials and issues entry e + 3
-      __syncwarp();
+    }
+      // release the unit: every lane arrives on the buffer's empty barrier; the warp releasing the
+      // entry's last unit waits for the whole entry, stores its partials and issues entry e + kR8
+      asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[b])) : "memory");
       int last = 0;
       if (lane == 0) {
-        __threadfence_block();
         last = atomicAdd(&s_cnt[b], 1) == kUnits - 1;
-        if (last) { atomicExch(&s_cnt[b], 0); __threadfence_block(); }
+        if (last) atomicExch(&s_cnt[b], 0);
       }
       last = __shfl_sync(0xffffffffu, last, 0);
       if (last) {
-        if (FUSED || tile < 0) {
-          issue(sl, e + kR8);
-        } else {
-          const double p = lane < nr ? s_part[b * R + lane] : 0.0;
-          __syncwarp();
-          issue(sl, e + kR8);
-          if (lane < nr) a.o.raw[(size_t)sl * a.n_all + a.row0 + r0 + lane] = p;
+        mbar_wait(&s_empty[b], (e / kR8) & 1u);
+        if (tile >= 0 && !FUSED) {
+          const int64_t r0 = (int64_t)tile * R;
+          const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+          if (lane < nr) a.o.raw[(size_t)sl * a.n_all + a.row0 + r0 + lane] = s_part[b * R + lane];
         }
-        if (tile >= 0 && lane == 0) atomicAdd(s_vdone, 1u);
+        __syncwarp();
+        issue(sl, e + kR8, tile < 0);
+        if (tile >= 0 && lane == 0) atomicAdd(s_vdone, 1);
       }
       if (tile < 0) {
         int done = 0;
         if (lane == 0)
-          done = *reinterpret_cast<volatile uint32_t*>(s_vdone) == *reinterpret_cast<volatile uint32_t*>(s_vis);
+          done = *reinterpret_cast<volatile int32_t*>(s_dead) == kR8 &&
+                 *reinterpret_cast<volatile int32_t*>(s_vdone) == *reinterpret_cast<volatile int32_t*>(s_vis);
         if (__shfl_sync(0xffffffffu, done, 0)) break;
       }
     }
-    __syncthreads();   // every entry of this slice is consumed or empty
-    const uint32_t issued = *s_issued;
-    g += issued;
-    // the forest barrier completed one phase this slice: re-init for the next one
+    __syncthreads();   // every valid entry of this slice is consumed and drained
     if (threadIdx.x == 0) {
       atomicSub(&a.cta_on[sl], 1);
       // next slice: the most remaining work per CTA already on it
@@ -2456,10 +2453,6 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     // L2 prefetch 8 tiles ahead of each claim (C4 walk 7.27 -> 6.88 ms; 24 and 64 the same within
     // 1 %); $TAHOE_CODE8_PREFETCH overrides (experiments)
     a.prefetch = std::getenv("TAHOE_CODE8_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODE8_PREFETCH")) : 8;
-    // ticket polls spin without back-off: the walk issues at ~33 %, so the polls cost little,
-    // while a 32 / 128 / 512 ns back-off delays the waiting warps (C4 walk 6.39 / 6.80 / 6.88 /
-    // 11.46 ms); $TAHOE_CODE8_SLEEP overrides (experiments)
-    a.sleep_ns = std::getenv("TAHOE_CODE8_SLEEP") ? (uint32_t)std::atoi(std::getenv("TAHOE_CODE8_SLEEP")) : 0u;
     // four chains per lane (C4 walk 6.43 -> 6.22 ms); $TAHOE_CODE8_SPLIT=0: two (experiments)
     a.split = img.col_mid ? (std::getenv("TAHOE_CODE8_SPLIT") ? std::atoi(std::getenv("TAHOE_CODE8_SPLIT")) : 1) : 0;
     // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
@@ -2493,7 +2486,7 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
 // One launch, no scratch: CUDA-graph capturable.
 template <bool LEAF>
 __global__ void __launch_bounds__(kRowsThreads) k_rows(const DirectKArgs a) {
-  extern __shared__ __align__(16) unsigned char smem[];
+  extern __shared__ __align__(1024) unsigned char smem[];
   float* s_row = reinterpret_cast<float*>(smem);
   float* s_val = reinterpret_cast<float*>(smem + ((size_t)a.d * 4 + 15) / 16 * 16);
   double* s_red = reinterpret_cast<double*>(reinterpret_cast<unsigned char*>(s_val) +

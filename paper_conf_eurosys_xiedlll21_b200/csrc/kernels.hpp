@@ -116,7 +116,7 @@ inline int64_t code8_chunk_rows(int32_t vfbits, int64_t n) {
   if (c < kCode8TileRows) c = kCode8TileRows;
   return n < c ? n : c;
 }
-constexpr int32_t kCode8Ctl = 256;               // mbarriers, counters, tickets
+constexpr int32_t kCode8Ctl = 512;               // mbarriers (36 full, 6 empty, slice), counters, entry tiles
 // shared memory next to the slice: the ring (aligned to the row size), the flags, staged partials,
 // the control block
 inline int64_t code8_ring_smem(int32_t vfbits) {

@@ -69,7 +69,9 @@ def load(build_if_missing: bool = True):
     if _lib is not None:
         return _lib
     path = _build.LIB
-    if build_if_missing:
+    if os.environ.get("TAHOE_LIB_AB"):   # same-box A/B experiments: another in-tree build
+        path = os.path.join(os.path.dirname(_build.LIB), os.environ["TAHOE_LIB_AB"])
+    elif build_if_missing:
         path = _build.build()
     if not os.path.exists(path):
         raise ImportError(f"libtahoe.so not found at {path}: run __graft_entry__.build()")

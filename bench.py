@@ -369,21 +369,29 @@ def run_tree_sharded(args, cfg):
                 oh_dev = out.cpu().numpy()
                 parity = parity_record(f, oh_dev[idx], np.zeros(len(idx), np.int32), ref)
         # roofline of the traversal (k_direct_tlp over the L2-sized chunks of the shard's image):
-        # algorithmic bytes per sample = node visits x (8 B node + 4 B attribute) + leaves x 8 B,
-        # against the L1 / shared-memory data pipe the node and attribute loads go through
-        # (128 B/clk/SM, the same unit and peak as the sliced kernels' roofline); the time is the
-        # whole step (traversal launches + the reduce/finalize kernel, < 1 % of it)
-        peaks = _peaks()
+        # node reads per sample (internal visits + one leaf read per tree) against the node-read
+        # rate of the same direct walk when every node read hits L1 (tahoe_measure_visit_rate
+        # variant 2, measured live); the time is the whole step (traversal launches + the
+        # reduce/finalize kernel, < 1 % of it)
         n_sms = st["num_sms"]
-        pipe_peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 1e9
-        bytes_per_sample = visits * 12.0 + st["n_trees"] * 8.0
-        achieved = n * bytes_per_sample / (ms / 1000.0) / 1e9
-        roofline = dict(bound="alu", pipe="L1/shared-memory LSU data pipe, 128 B/clk/SM (DESIGN.md Roofline)",
-                        kernel="k_direct_tlp", achieved=achieved, peak=pipe_peak, unit="GB/s",
-                        frac=achieved / pipe_peak, traffic=None, kernel_ms=ms,
-                        units_per_launch=f"{n} samples x {bytes_per_sample:.0f} B ({visits:.0f} visits x 12 B"
-                                         f" + {st['n_trees']} leaves x 8 B) per step",
-                        peak_source=f"derived: 128 B/clk x {n_sms} SMs x {peaks['sm_max_mhz']:.0f} MHz")
+        reads_per_sample = visits + st["n_trees"]
+        achieved = n * reads_per_sample / (ms / 1000.0) / 1e9
+        vp = visit_peak(local, 2)
+        if vp and "node_reads_per_s" in vp:
+            peak, peak_src = vp["node_reads_per_s"] / 1e9, (
+                "measured live: tahoe_measure_visit_rate variant 2 (the direct walk, every node read "
+                "an L1 hit: 8 threads per row over staged rows, 4 CTAs of 512 threads per SM)")
+        else:
+            peaks = _peaks()
+            peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 12.0 / 1e9
+            peak_src = "derived: 128 B/clk/SM / 12 B per node read (microbenchmark unavailable)"
+        roofline = dict(bound="alu", pipe="L1/TEX data pipe (node loads) (DESIGN.md §5 Roofline)",
+                        kernel="k_direct_tlp", achieved=achieved, peak=peak, unit="G node reads/s",
+                        frac=achieved / peak, traffic=None, kernel_ms=ms,
+                        units_per_launch=f"{n} samples x {reads_per_sample:.0f} node reads ({visits:.0f} visits"
+                                         f" + {st['n_trees']} leaf reads) per step",
+                        peak_source=peak_src, microbench=vp)
+        peaks = _peaks()
         hbm_bytes = n * (cfg.n_features * 4) + (hi - lo if fused else n) * 4
         hbm = dict(achieved=hbm_bytes / (ms / 1000.0) / 1e9, peak=peaks["hbm_gbs"], unit="GB/s",
                    frac=hbm_bytes / (ms / 1000.0) / 1e9 / peaks["hbm_gbs"], bytes_per_step=hbm_bytes,
@@ -597,14 +605,20 @@ def main():
     # unit is a node read (internal visit or leaf read), V_int + T per sample; the peak is the
     # node-read rate of the same walk on ideal data, measured live (tahoe_measure_visit_rate)
     code8 = bool(stats.get("code8"))
-    kname = {1: "k_sliced", 2: "k_sliced_codes8" if code8 else "k_sliced_codes"}.get(strategy, "k_direct")
+    kname = {1: "k_sliced", 2: "k_sliced_codes8" if code8 else "k_sliced_codes",
+             3: "k_rows"}.get(strategy, "k_direct")
     reads_per_sample = visits + cfg.n_trees
     achieved = n_local * reads_per_sample / (kern_avg_ms / 1000.0) / 1e9
-    vp = visit_peak(local, 1 if code8 else 0) if strategy == T.STRATEGY_SLICED_CODED else None
+    # peak: the microbenchmark of the walk this strategy runs (0: u16 coded slices, also the
+    # closest for the fp32 slices; 1: wide codes; 2: the direct walk through L1, also for ROWS)
+    variant = {2: 1 if code8 else 0, 1: 0}.get(strategy, 2)
+    vp = visit_peak(local, variant)
     if vp and "node_reads_per_s" in vp:
+        what = {0: "the production coded walk on ideal data: conflict-free, perfect lockstep, 32 "
+                   "warps/SM on every SM", 1: "the wide-code walk on ideal data, four chains per lane",
+                2: "the direct walk with every node read an L1 hit"}[variant]
         peak, peak_src = vp["node_reads_per_s"] / 1e9, (
-            "measured live: tahoe_measure_visit_rate variant %d (the production coded walk on ideal "
-            "data: conflict-free, perfect lockstep, 32 warps/SM on every SM)" % vp["variant"])
+            "measured live: tahoe_measure_visit_rate variant %d (%s)" % (variant, what))
     else:
         n_sms = stats["num_sms"]
         peak = 128.0 * n_sms * peaks["sm_max_mhz"] * 1e6 / 12.0 / 1e9
@@ -635,7 +649,7 @@ def main():
         higher_is_better=True, scaling="weak" if args.weak else "strong", vs_baseline=None,
         dtype="f32", accum="f64", data="synthetic", impl="ours",
         config=_config(cfg, n, stats, world, args.weak),
-        strategy={0: "direct", 1: "sliced", 2: "sliced-coded"}.get(strategy, str(strategy)),
+        strategy={0: "direct", 1: "sliced", 2: "sliced-coded", 3: "rows"}.get(strategy, str(strategy)),
         roofline=dict(bound="alu", pipe="shared-memory LSU data pipe (DESIGN.md §5 Roofline)",
                       kernel=kname, achieved=achieved, peak=peak, unit="G node reads/s",
                       frac=achieved / peak, traffic=traffic, kernel_ms=kern_avg_ms,

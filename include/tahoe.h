@@ -223,7 +223,10 @@ tahoe_status tahoe_forest_layout_import(tahoe_forest* f, const void* buf, int64_
  * the production coded walk on ideal data (every lane walks `steps` internal nodes of its own
  * column, perfect lockstep, conflict-free code loads, no tile traffic), one 1024-thread CTA per SM
  * on all SMs of `device`, `reps` walks per lane.  variant 0: u16 codes, two chains per lane (the
- * walk of the rank-coded slices); variant 1: u8 codes, four chains per lane (the wide codes).
+ * walk of the rank-coded slices); variant 1: u8 codes, four chains per lane (the wide codes);
+ * variant 2: the direct walk (8-byte nodes through L1 by __ldg, attributes from staged rows, hot
+ * child next, eight threads per row, 4 CTAs of 512 threads per SM) over a 32 KB node array that
+ * stays L1-resident: steps x reps node reads per thread.
  * Writes *node_reads_per_s (node reads = visits, leaf reads included, per second); optionally
  * *smem_bytes_per_clk (NULL to skip): conflict-free 16-byte shared-memory loads measured with
  * clock64, bytes per SM clock.  E_INVAL on a bad variant / steps < 2 / odd steps / reps < 1;

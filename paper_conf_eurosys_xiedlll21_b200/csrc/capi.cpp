@@ -898,7 +898,7 @@ __attribute__((visibility("default"))) tahoe_status tahoe_measure_visit_rate(
     int32_t device, int32_t variant, int32_t steps, int32_t reps, double* node_reads_per_s,
     double* smem_bytes_per_clk) {
   TAHOE_GUARD_BEGIN
-  if (variant < 0 || variant > 1 || steps < 2 || (steps & 1) || steps > 600 || reps < 1 || !node_reads_per_s)
+  if (variant < 0 || variant > 2 || steps < 2 || (steps & 1) || steps > 600 || reps < 1 || !node_reads_per_s)
     return fail(TAHOE_E_INVAL, "bad microbenchmark arguments");
   DeviceGuard g(device);
   if (!g.ok) return fail(TAHOE_E_CUDA, "cannot select device");
@@ -918,16 +918,42 @@ __attribute__((visibility("default"))) tahoe_status tahoe_measure_visit_rate(
   if (e == cudaSuccess) e = cudaMalloc(&sink2, (size_t)sms * 4);
   int rc = e == cudaSuccess ? 0 : (int)e;
   float ms = 0.0f;
-  if (!rc) rc = launch_visit_peak(variant, steps, std::max(1, reps / 8), sms, sink, st);   // warm-up
-  if (!rc) {
-    cudaEventRecord(a, st);
-    rc = launch_visit_peak(variant, steps, reps, sms, sink, st);
-    cudaEventRecord(b, st);
-  }
-  if (!rc) rc = (int)cudaStreamSynchronize(st);
-  if (!rc) {
-    cudaEventElapsedTime(&ms, a, b);
-    *node_reads_per_s = (double)sms * 1024.0 * 2.0 * steps * (double)reps / (ms / 1000.0);
+  if (variant == 2) {
+    // the direct walk: 4096 internal nodes whose hot child is the next one (attribute = slot % 100,
+    // threshold +inf so "x < b" holds, hot = left), 4 CTAs of 512 threads per SM
+    std::vector<uint32_t> h(2 * 4096);
+    for (uint32_t q = 0; q < 4096; q++) {
+      h[2 * q] = 0x7f800000u;
+      h[2 * q + 1] = kHotLeftBit | (1u << 7) | (q % 100u);
+    }
+    void* nodes = nullptr;
+    if (!rc) rc = (int)cudaMalloc(&nodes, h.size() * 4);
+    if (!rc) rc = (int)cudaMemcpy(nodes, h.data(), h.size() * 4, cudaMemcpyHostToDevice);
+    const int grid = sms * 4, total = steps * reps;
+    if (!rc) rc = launch_visit_peak_direct(nodes, total / 8, grid, sink, st);   // warm-up
+    if (!rc) {
+      cudaEventRecord(a, st);
+      rc = launch_visit_peak_direct(nodes, total, grid, sink, st);
+      cudaEventRecord(b, st);
+    }
+    if (!rc) rc = (int)cudaStreamSynchronize(st);
+    if (!rc) {
+      cudaEventElapsedTime(&ms, a, b);
+      *node_reads_per_s = (double)grid * 512.0 * (double)total / (ms / 1000.0);
+    }
+    cudaFree(nodes);
+  } else {
+    if (!rc) rc = launch_visit_peak(variant, steps, std::max(1, reps / 8), sms, sink, st);   // warm-up
+    if (!rc) {
+      cudaEventRecord(a, st);
+      rc = launch_visit_peak(variant, steps, reps, sms, sink, st);
+      cudaEventRecord(b, st);
+    }
+    if (!rc) rc = (int)cudaStreamSynchronize(st);
+    if (!rc) {
+      cudaEventElapsedTime(&ms, a, b);
+      *node_reads_per_s = (double)sms * 1024.0 * 2.0 * steps * (double)reps / (ms / 1000.0);
+    }
   }
   if (!rc && smem_bytes_per_clk) {
     const int iters = 4096;

@@ -2666,6 +2666,30 @@ __global__ void __launch_bounds__(1024, 1) k_visit_peak(int32_t L, int32_t reps,
   if (tot != 0.0) sink[blockIdx.x] = tot;   // never true (internal words add +0); keeps the walk
 }
 
+// VAR 2: the direct walk's peak (k_direct_tlp's step: an 8-byte node through L1 with __ldg, the
+// attribute from a row staged in shared memory, the hot child next): every thread walks a chain of
+// internal nodes that all go to their hot child, in a node array small enough to stay L1-resident
+// (`nodes`, 4096 nodes = 32 KB), eight threads per row over 64 staged rows per CTA as the
+// production kernel — i.e. the node-read rate when every node read hits L1.
+__global__ void __launch_bounds__(512) k_visit_peak_direct(const uint2* __restrict__ nodes, int32_t steps,
+                                                           double* sink) {
+  __shared__ float s_rows[64 * 101];
+  for (int q = threadIdx.x; q < 64 * 101; q += blockDim.x) s_rows[q] = (float)(q % 7);
+  __syncthreads();
+  const int fbits = 7;
+  const uint32_t fmask = (1u << fbits) - 1u;
+  const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
+  const float* row = s_rows + (threadIdx.x >> 3) * 101;
+  uint32_t k = (threadIdx.x * 37u) & 4095u;
+  double acc = 0.0;
+  for (int i = 0; i < steps; i++) {
+    const uint2 nd = __ldg(&nodes[k]);
+    k = (k + step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask)) & 4095u;
+    acc += (double)(k == 0xFFFFFFFFu);   // never; keeps the chain live
+  }
+  if (acc != 0.0) sink[blockIdx.x] = acc;
+}
+
 // Raw shared-memory load bandwidth: every warp issues conflict-free 16-byte loads (a warp = 512 B =
 // 4 wavefronts) in independent chains; bytes per SM clock from clock64 around the loop.
 __global__ void __launch_bounds__(1024, 1) k_smem_bw(int32_t iters, unsigned long long* cycles, uint32_t* sink) {
@@ -2700,6 +2724,11 @@ int launch_visit_peak(int32_t variant, int32_t L, int32_t reps, int32_t grid, do
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
   if (e != cudaSuccess) return (int)e;
   kern<<<grid, 1024, dyn, static_cast<cudaStream_t>(stream)>>>(L, reps, sink);
+  return (int)cudaGetLastError();
+}
+
+int launch_visit_peak_direct(const void* nodes, int32_t steps, int32_t grid, double* sink, void* stream) {
+  k_visit_peak_direct<<<grid, 512, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<const uint2*>(nodes), steps, sink);
   return (int)cudaGetLastError();
 }
 

@@ -235,5 +235,6 @@ int set_sliced_smem_limit(int32_t bytes);
 // microbenchmarks (Algorithm 1 line 4): the coded walk on ideal data; raw shared-memory loads
 int launch_visit_peak(int32_t variant, int32_t L, int32_t reps, int32_t grid, double* sink, void* stream);
 int launch_smem_bw(int32_t iters, int32_t grid, unsigned long long* cycles, uint32_t* sink, void* stream);
+int launch_visit_peak_direct(const void* nodes, int32_t steps, int32_t grid, double* sink, void* stream);
 
 }  // namespace tahoe

@@ -2672,7 +2672,7 @@ __global__ void __launch_bounds__(1024, 1) k_visit_peak(int32_t L, int32_t reps,
 // (`nodes`, 4096 nodes = 32 KB), eight threads per row over 64 staged rows per CTA as the
 // production kernel — i.e. the node-read rate when every node read hits L1.
 __global__ void __launch_bounds__(512) k_visit_peak_direct(const uint2* __restrict__ nodes, int32_t steps,
-                                                           double* sink) {
+                                                           uint32_t mask, double* sink) {
   __shared__ float s_rows[64 * 101];
   for (int q = threadIdx.x; q < 64 * 101; q += blockDim.x) s_rows[q] = (float)(q % 7);
   __syncthreads();
@@ -2680,14 +2680,12 @@ __global__ void __launch_bounds__(512) k_visit_peak_direct(const uint2* __restri
   const uint32_t fmask = (1u << fbits) - 1u;
   const uint32_t offmask = (1u << (kOffsetTop - fbits)) - 1u;
   const float* row = s_rows + (threadIdx.x >> 3) * 101;
-  uint32_t k = (threadIdx.x * 37u) & 4095u;
-  double acc = 0.0;
+  uint32_t k = (threadIdx.x * 37u) & mask;   // mask (4095) is a kernel argument: the chain is live
   for (int i = 0; i < steps; i++) {
     const uint2 nd = __ldg(&nodes[k]);
-    k = (k + step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask)) & 4095u;
-    acc += (double)(k == 0xFFFFFFFFu);   // never; keeps the chain live
+    k = (k + step(nd.x, nd.y, row[nd.y & fmask], fbits, offmask)) & mask;
   }
-  if (acc != 0.0) sink[blockIdx.x] = acc;
+  if (k == 0xFFFFFFFFu) sink[blockIdx.x] = (double)k;   // never (mask < 2^32 - 1)
 }
 
 // Raw shared-memory load bandwidth: every warp issues conflict-free 16-byte loads (a warp = 512 B =
@@ -2728,7 +2726,7 @@ int launch_visit_peak(int32_t variant, int32_t L, int32_t reps, int32_t grid, do
 }
 
 int launch_visit_peak_direct(const void* nodes, int32_t steps, int32_t grid, double* sink, void* stream) {
-  k_visit_peak_direct<<<grid, 512, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<const uint2*>(nodes), steps, sink);
+  k_visit_peak_direct<<<grid, 512, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<const uint2*>(nodes), steps, 4095u, sink);
   return (int)cudaGetLastError();
 }
 

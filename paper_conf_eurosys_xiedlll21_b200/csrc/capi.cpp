@@ -272,10 +272,12 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
         f->ds.c8_bands = f->sl.c8_bands;
         f->ds.vfbits = f->sl.vfbits;
         f->ds.code8 = 1;
-        std::vector<float> w(f->sl.slice_work.begin(), f->sl.slice_work.end());
-        if ((st = upload(w, &f->ds.slice_w)) != TAHOE_OK) return st;
         if ((st = upload(f->sl.col_mid, &f->ds.col_mid)) != TAHOE_OK) return st;
       }
+      // slice weights for the coded kernels' slice switching (simulated lane-steps per row)
+      std::vector<float> w(f->sl.slice_work.begin(), f->sl.slice_work.end());
+      if (w.size() != (size_t)f->sl.n_slices) w.assign((size_t)f->sl.n_slices, 1.0f);
+      if ((st = upload(w, &f->ds.slice_w)) != TAHOE_OK) return st;
     }
   }
   return TAHOE_OK;
@@ -496,7 +498,8 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
     cudaFreeAsync(cbuf, st);
   } else if (strat == TAHOE_STRATEGY_SLICED_CODED) {
     const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
-    const size_t cbytes = (size_t)ntiles * code_tile_stride(f->sl.fbits);
+    // code tiles, then per-slice tile / CTA counters (dynamic tile claiming, slice switching)
+    const size_t cbytes = (size_t)ntiles * code_tile_stride(f->sl.fbits) + (size_t)f->sl.n_slices * 8;
     void* cbuf = nullptr;
     if ((e = scratch_alloc(&cbuf, cbytes, st)) != cudaSuccess) {
       if (part) cudaFreeAsync(part, st);

@@ -1046,6 +1046,9 @@ struct CodedKArgs {
   int32_t ring;          // ring depth (kSlicedRing .. kCodedRingMax): as many tiles as shared memory holds
   uint32_t ring_m, bars_m;   // ceil(2^32 / ring), ceil(2^32 / (2 ring)): division by multiply-high
   double* prof;          // PROF instantiation: load-balance statistics (prof_unit), else null
+  int32_t* tile_next;    // [ns] next unclaimed tile of each slice (zeroed per launch)
+  int32_t* cta_on;       // [ns] CTAs currently on each slice (zeroed per launch)
+  const float* work;     // [ns] simulated lane-steps per row of each slice (slice choice weights)
   OutArgs o;
 };
 
@@ -1216,15 +1219,19 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   constexpr int C = kSlicedCols;
   extern __shared__ __align__(1024) unsigned char smem[];
   unsigned char* s_ring = smem + a.forest_smem;
-  // Producer / consumer ring (mbarrier hand-off only): warp PW (the last) stages the slice and
-  // every code tile of the CTA's sequence, refilling buffer b once the kUnits units of its previous
-  // tile have all arrived on empty[b] (and writing that tile's slice partials out first); the other
-  // 31 warps claim 4-row work units from a CTA counter, wait on the tile's full barrier, walk, and
-  // arrive on empty[b].  Tile seq uses buffer seq % ring, full barrier seq % (2 ring) with parity
-  // (seq / (2 ring)) & 1: a consumer claiming seq could only see a stale phase if tile
-  // seq - 2 ring had not arrived, but then seq - ring is not issued either, and the 2 x 16 units
-  // of those two tiles would hold 32 blocked consumers — there are 31 (the ring-wrap guard of
-  // ring_bar, with a runtime depth).
+  // Producer / consumer ring (mbarrier hand-off only): warp PW (the last) stages the slice, claims
+  // the slice's tiles from its global counter (so every CTA on a slice finishes with the slice) and
+  // issues them into the ring, refilling buffer b once the kUnits units of its previous tile have
+  // all arrived on empty[b] (and writing that tile's slice partials out first); the other 31 warps
+  // claim 4-row work units from a CTA counter, wait on the tile's full barrier, walk, and arrive on
+  // empty[b].  Entry e (of the CTA's stay on a slice) uses buffer e % ring and full barrier
+  // e % (2 ring) with parity (e / (2 ring)) & 1: a consumer claiming e could only see a stale phase
+  // if entry e - 2 ring had not arrived, but then e - ring is not issued either, and the 2 x 16
+  // units of those two entries would hold 32 blocked consumers — there are 31 (the ring-wrap guard
+  // of ring_bar, with a runtime depth).  Past the slice's last tile the producer issues kTerm
+  // terminator entries (tile -1, no data: 2 x 16 units reach all 31 consumers' next claims); the
+  // CTA then moves to the slice with the most remaining work per CTA (re-staging it), and the
+  // barriers are re-initialised.
   const uint32_t ring = (uint32_t)a.ring, nbars = 2u * ring;
   constexpr int kUnits = kSlicedTileRows / 4;
   // control block (kCodedCtlBytes): [2 ring] full barriers, [ring] empty barriers, slice barrier,
@@ -1250,36 +1257,41 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
   const int64_t R = kSlicedTileRows;
   const int64_t ntiles = (a.n + R - 1) / R;
 
-  if (threadIdx.x == 0) {
-    // every lane of the producer arrives on a full barrier (lane 0 with the transaction bytes) and
-    // every consumer lane on an empty barrier: each lane's own shared-memory accesses are released
-    // by its own arrival
-    for (uint32_t b = 0; b < nbars; b++) mbar_init(&s_full[b], 32);
-    for (uint32_t b = 0; b < ring; b++) mbar_init(&s_empty[b], kUnits * 32);
-    *s_next = 0u;
-    mbar_init(s_forest, 1);
-    fence_mbar_init();
-  }
-  __syncthreads();
-
-  uint32_t g = 0;
+  constexpr uint32_t kTerm = 2;
+  static_assert(kTerm * kUnits >= 31 && kTerm <= kSlicedRing, "terminators reach every consumer");
   uint32_t ph_forest = 0;
   const uint32_t ring0 = smem_u32(s_ring);
-  // single pass: this CTA's slice and its place among the slice's CTAs (weighted map, or
-  // round-robin); it takes every ts-th tile starting at t0
-  int32_t sl0 = (int32_t)blockIdx.x % ns;
-  int64_t t0s = blockIdx.x / ns, tss = a.cps;
-  if (!multipass && a.cta_start) {
-    sl0 = 0;
-    while (sl0 + 1 < ns && __ldg(&a.cta_start[sl0 + 1]) <= (int32_t)blockIdx.x) sl0++;
-    t0s = blockIdx.x - __ldg(&a.cta_start[sl0]);
-    tss = __ldg(&a.cta_start[sl0 + 1]) - __ldg(&a.cta_start[sl0]);
+  const uint32_t sbase = smem_u32(smem);
+  int32_t* s_slice = reinterpret_cast<int32_t*>(s_next + 1);
+  int32_t* s_tile = s_slice + 1;   // [ring] tile of the entry in each buffer (-1: terminator)
+  if (threadIdx.x == 0) {
+    // first slice: the weighted CTA map (or round-robin; CTA b of a multi-pass launch takes slice b)
+    int32_t sl = (int32_t)blockIdx.x % ns;
+    if (!multipass && a.cta_start) {
+      sl = 0;
+      while (sl + 1 < ns && __ldg(&a.cta_start[sl + 1]) <= (int32_t)blockIdx.x) sl++;
+    } else if (multipass) {
+      sl = (int32_t)blockIdx.x;
+    }
+    *s_slice = sl;
+    atomicAdd(&a.cta_on[sl], 1);
   }
-  for (int32_t sl = multipass ? (int32_t)blockIdx.x : sl0; sl < ns; sl += multipass ? G : ns) {
-    const int64_t t0 = multipass ? 0 : t0s;
-    const int64_t ts = multipass ? 1 : tss;
-    const int64_t my_tiles = t0 < ntiles ? (ntiles - t0 + ts - 1) / ts : 0;
-    const uint32_t sbase = smem_u32(smem);
+  for (bool first = true;; first = false) {
+    // (re)initialise the barriers for this slice: every wait of the previous slice has returned.
+    // Every lane of the producer arrives on a full barrier (lane 0 with the transaction bytes)
+    // and every consumer lane on an empty barrier: each lane's own shared-memory accesses are
+    // released by its own arrival.
+    if (threadIdx.x == 0) {
+      for (uint32_t b = 0; b < nbars + ring + 1; b++) {
+        if (!first) asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(&s_full[b])) : "memory");
+        mbar_init(&s_full[b], b < nbars ? 32u : (b < nbars + ring ? (uint32_t)(kUnits * 32) : 1u));
+      }
+      *s_next = 0u;
+      fence_mbar_init();
+    }
+    __syncthreads();
+    const int32_t sl = *s_slice;
+    if (sl < 0) break;
     if (warp == PW) {
       // ---- producer
       if (lane == 0) {   // a7: the slice, one bulk copy of slots x 128 bytes
@@ -1288,14 +1300,13 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         mbar_expect_tx(s_forest, bytes);
         bulk_g2s_big(smem, a.img.cnodes + (size_t)sl * a.img.slots_max * C * 2, bytes, s_forest);
       }
-      // tile `it` of this slice consumed: store its 64 slice partials (two coalesced 256-byte
-      // stores; non-fused launches)
-      auto drain = [&](int64_t it) {
-        const uint32_t seq = g + (uint32_t)it;
-        const uint32_t b = fmod_small(seq, ring, a.ring_m);
-        mbar_wait(&s_empty[b], fdiv_small(seq, a.ring_m) & 1u);
+      // entry x (valid) consumed: store its 64 slice partials (two coalesced 256-byte stores;
+      // non-fused launches)
+      auto drain = [&](uint32_t x) {
+        const uint32_t b = fmod_small(x, ring, a.ring_m);
+        mbar_wait(&s_empty[b], fdiv_small(x, a.ring_m) & 1u);
         if (!FUSED) {
-          const int64_t r0 = (t0 + it * ts) * R;
+          const int64_t r0 = (int64_t)s_tile[b] * R;
           const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
           const double* sp = s_part + b * kSlicedTileRows;
           double* dst = a.o.raw + (size_t)sl * a.n + r0;
@@ -1304,110 +1315,140 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
         }
         __syncwarp();
       };
-      for (int64_t it = 0; it < my_tiles; it++) {
-        const uint32_t seq = g + (uint32_t)it;
-        if (it >= (int64_t)ring) drain(it - ring);   // buffer seq % ring is free again
-        uint64_t* bar = &s_full[fmod_small(seq, nbars, a.bars_m)];
+      // tiles are claimed one at a time from the slice's counter, the next claim issued before
+      // this one is used (its latency overlaps the drain and the issue)
+      int32_t next = 0;
+      if (lane == 0) next = atomicAdd(&a.tile_next[sl], 1);
+      uint32_t e = 0, n_valid = 0, terms = 0;
+      while (terms < kTerm) {
+        if (e >= ring && e - ring < n_valid) drain(e - ring);   // buffer e % ring is free again
+        int32_t tile = -1;
+        if (terms == 0) {
+          tile = __shfl_sync(0xffffffffu, next, 0);
+          if (tile >= (int32_t)ntiles) tile = -1;
+          else if (lane == 0) next = atomicAdd(&a.tile_next[sl], 1);
+        }
+        const uint32_t b = fmod_small(e, ring, a.ring_m);
+        uint64_t* bar = &s_full[fmod_small(e, nbars, a.bars_m)];
         if (lane == 0) {
-          const int64_t tile = t0 + it * ts;
-          const int64_t ahead = a.prefetch ? t0 + (it + a.prefetch) * ts : -1;
-          if (ahead >= 0 && ahead < ntiles)   // optional L2 prefetch of a later tile
-            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
-                         "r"((uint32_t)a.tstride) : "memory");
-          fence_proxy_async_smem();
-          mbar_expect_tx(bar, (uint32_t)a.tstride);
-          bulk_g2s(s_ring + (size_t)fmod_small(seq, ring, a.ring_m) * a.tstride,
-                   reinterpret_cast<const unsigned char*>(a.codes) + tile * a.tstride, (uint32_t)a.tstride, bar);
+          s_tile[b] = tile;
+          if (tile >= 0) {
+            const int64_t ahead = a.prefetch ? (int64_t)tile + a.prefetch : -1;
+            if (ahead >= 0 && ahead < ntiles)   // optional L2 prefetch of a later tile
+              asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const unsigned char*>(a.codes) + ahead * a.tstride),
+                           "r"((uint32_t)a.tstride) : "memory");
+            fence_proxy_async_smem();
+            mbar_expect_tx(bar, (uint32_t)a.tstride);
+            bulk_g2s(s_ring + (size_t)b * a.tstride,
+                     reinterpret_cast<const unsigned char*>(a.codes) + (int64_t)tile * a.tstride, (uint32_t)a.tstride, bar);
+          } else {
+            asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+          }
         } else {
           asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
         }
+        if (tile >= 0) n_valid++;
+        else terms++;
+        e++;
       }
-      for (int64_t it = my_tiles > (int64_t)ring ? my_tiles - ring : 0; it < my_tiles; it++) drain(it);
+      // the valid entries not yet drained (the last ring - kTerm of them at most)
+      for (uint32_t x = e > ring ? e - ring : 0; x < n_valid; x++) drain(x);
     } else {
-    // ---- consumers
-    const uint32_t p0 = sbase + (uint32_t)col * 8u;
-    const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
-    const int2* __restrict__ meta =
-        LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
-    mbar_wait(s_forest, ph_forest);
-
-    const uint64_t total = (uint64_t)my_tiles * kUnits;
-    for (;;) {
-      uint32_t q = 0;
-      if (lane == 0) q = atomicAdd(s_next, 1u);   // 32-bit: a native ATOMS.ADD (64-bit was a CAS loop)
-      q = __shfl_sync(0xffffffffu, q, 0);
-      if ((uint64_t)q >= total) break;
-      const int64_t it = (int64_t)(q / kUnits);
-      const int u = (int)(q % kUnits);
-      const uint32_t gt = g + (uint32_t)it;
-      const int b = (int)fmod_small(gt, ring, a.ring_m);
-      const int64_t tile = t0 + it * ts;
-      const int64_t r0 = tile * R;
-      const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
-      mbar_wait(&s_full[fmod_small(gt, nbars, a.bars_m)], fdiv_small(gt, a.bars_m) & 1u);
-      if (u < nr) {
-        const int rA = u + 16 * half, rB = rA + 32;
-        const bool okA = rA < nr, okB = rB < nr;
-        const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
-        const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tstride;
-        // row base | swizzle (code_slot_swz in bytes): the attribute offset is XORed into it
-        const int qA = okA ? rA : u, qB = okB ? rB : u;
-        const uint32_t rowA = SWZ ? (tb + code_row_off(qA, a.rb)) | (code_slot_swz(qA, a.rb) << 1)
-                                  : tb + code_row_off(qA, a.rb);
-        const uint32_t rowB = SWZ ? (tb + code_row_off(qB, a.rb)) | (code_slot_swz(qB, a.rb) << 1)
-                                  : tb + code_row_off(qB, a.rb);
-        uint32_t nan_flag;
-        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(tb + (uint32_t)a.tile_bytes));
-        double accA, accB;
-        uint64_t fpA = 0, fpB = 0;
-        if (LEAF) {
-          int32_t* oA = (a.o.out_leaf && okA) ? a.o.out_leaf + (r0 + rA) * (int64_t)a.o.T_leaf : nullptr;
-          int32_t* oB = (a.o.out_leaf && okB) ? a.o.out_leaf + (r0 + rB) * (int64_t)a.o.T_leaf : nullptr;
-          if (nan_flag)
-            walk_coded2_leaf<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
-          else
-            walk_coded2_leaf<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
-        } else if (PROF) {
-          uint32_t span;
-          if (nan_flag) walk_coded2_prof<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, span);
-          else walk_coded2_prof<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, span);
-          prof_unit(a.prof, span);
-          lane_total += (double)span;
-        } else if (nan_flag) {
-          walk_coded2<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-        } else {
-          walk_coded2<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
-        }
-        // a9: the k_sliced butterfly (lanes 0, 8, 16, 24 own rows u, u+32, u+16, u+48)
-        const bool b3 = lane & 8;
-        double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
+      // ---- consumers
+      const uint32_t p0 = sbase + (uint32_t)col * 8u;
+      const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+      const int2* __restrict__ meta =
+          LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
+      mbar_wait(s_forest, 0u);
+      for (;;) {
+        uint32_t q = 0;
+        if (lane == 0) q = atomicAdd(s_next, 1u);   // 32-bit: a native ATOMS.ADD (64-bit was a CAS loop)
+        q = __shfl_sync(0xffffffffu, q, 0);
+        const uint32_t gt = q / kUnits;
+        const int u = (int)(q % kUnits);
+        const int b = (int)fmod_small(gt, ring, a.ring_m);
+        mbar_wait(&s_full[fmod_small(gt, nbars, a.bars_m)], fdiv_small(gt, a.bars_m) & 1u);
+        const int32_t tile = s_tile[b];
+        if (tile < 0) break;   // terminator: the slice's tiles are exhausted
+        const int64_t r0 = (int64_t)tile * R;
+        const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
+        if (u < nr) {
+          const int rA = u + 16 * half, rB = rA + 32;
+          const bool okA = rA < nr, okB = rB < nr;
+          const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
+          const uint32_t tb = ring0 + (uint32_t)b * (uint32_t)a.tstride;
+          // row base | swizzle (code_slot_swz in bytes): the attribute offset is XORed into it
+          const int qA = okA ? rA : u, qB = okB ? rB : u;
+          const uint32_t rowA = SWZ ? (tb + code_row_off(qA, a.rb)) | (code_slot_swz(qA, a.rb) << 1)
+                                    : tb + code_row_off(qA, a.rb);
+          const uint32_t rowB = SWZ ? (tb + code_row_off(qB, a.rb)) | (code_slot_swz(qB, a.rb) << 1)
+                                    : tb + code_row_off(qB, a.rb);
+          uint32_t nan_flag;
+          asm volatile("ld.shared.u32 %0, [%1];" : "=r"(nan_flag) : "r"(tb + (uint32_t)a.tile_bytes));
+          double accA, accB;
+          uint64_t fpA = 0, fpB = 0;
+          if (LEAF) {
+            int32_t* oA = (a.o.out_leaf && okA) ? a.o.out_leaf + (r0 + rA) * (int64_t)a.o.T_leaf : nullptr;
+            int32_t* oB = (a.o.out_leaf && okB) ? a.o.out_leaf + (r0 + rB) * (int64_t)a.o.T_leaf : nullptr;
+            if (nan_flag)
+              walk_coded2_leaf<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+            else
+              walk_coded2_leaf<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);
+          } else if (PROF) {
+            uint32_t span;
+            if (nan_flag) walk_coded2_prof<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, span);
+            else walk_coded2_prof<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, span);
+            prof_unit(a.prof, span);
+            lane_total += (double)span;
+          } else if (nan_flag) {
+            walk_coded2<true, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          } else {
+            walk_coded2<false, SWZ>(pA, pB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+          }
+          // a9: the k_sliced butterfly (lanes 0, 8, 16, 24 own rows u, u+32, u+16, u+48)
+          const bool b3 = lane & 8;
+          double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
 #pragma unroll
-        for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        uint64_t fv = 0;
-        if (LEAF) {
-          fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
+          for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+          uint64_t fv = 0;
+          if (LEAF) {
+            fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
 #pragma unroll
-          for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
+            for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
+          }
+          const int rr = b3 ? rB : rA;
+          if ((lane & 7) == 0 && (b3 ? okB : okA)) {
+            if (FUSED) write_scalar(a.o, r0 + rr, v);
+            else s_part[b * kSlicedTileRows + rr] = v;
+            if (LEAF && a.o.out_fp)
+              atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[r0 + rr]), (unsigned long long)fv);
+          }
         }
-        const int rr = b3 ? rB : rA;
-        if ((lane & 7) == 0 && (b3 ? okB : okA)) {
-          if (FUSED) write_scalar(a.o, r0 + rr, v);
-          else s_part[b * kSlicedTileRows + rr] = v;
-          if (LEAF && a.o.out_fp)
-            atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[r0 + rr]), (unsigned long long)fv);
-        }
+        // the unit is done with buffer b (its partials are in s_part): every lane release-arrives on
+        // empty[b], so each lane's own reads of the tile and writes of s_part are ordered before the
+        // producer's refill (one arrival per lane rather than one per warp after __syncwarp: the same
+        // ordering, and the form compute-sanitizer racecheck tracks)
+        asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[b])) : "memory");
       }
-      // the unit is done with buffer b (its partials are in s_part): every lane release-arrives on
-      // empty[b], so each lane's own reads of the tile and writes of s_part are ordered before the
-      // producer's refill (one arrival per lane rather than one per warp after __syncwarp: the same
-      // ordering, and the form compute-sanitizer racecheck tracks)
-      asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[b])) : "memory");
     }
+    (void)ph_forest;
+    __syncthreads();   // every valid entry of this slice is consumed and drained
+    if (threadIdx.x == 0) {
+      atomicSub(&a.cta_on[sl], 1);
+      // next slice: the most remaining work per CTA already on it (a slice nobody works on is
+      // always taken while it has tiles)
+      int32_t best = -1;
+      float bw = 0.0f;
+      for (int32_t s2 = 0; s2 < ns; s2++) {
+        const int32_t rem = (int32_t)ntiles - *reinterpret_cast<volatile int32_t*>(&a.tile_next[s2]);
+        const int32_t on = *reinterpret_cast<volatile int32_t*>(&a.cta_on[s2]);
+        if (rem < 1 || (on > 0 && rem < 2)) continue;
+        const float w = (float)rem * __ldg(&a.work[s2]) / (float)(1 + on);
+        if (w > bw) { bw = w; best = s2; }
+      }
+      if (best >= 0) atomicAdd(&a.cta_on[best], 1);
+      *s_slice = best;
     }
-    ph_forest ^= 1u;
-    g += (uint32_t)my_tiles;
-    __syncthreads();
-    if (threadIdx.x == 0) *s_next = 0u;
     __syncthreads();
   }
   if (PROF && warp != PW) prof_lanes(a.prof, lane_total);
@@ -1738,9 +1779,13 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   const int64_t ntiles = (n + kSlicedTileRows - 1) / kSlicedTileRows;
   const int32_t tstride = code_tile_stride(img.fbits);
   const int32_t tbytes = code_tile_bytes(img.fbits);
-  // zero every tile's NaN flag (the trailer word after its rows)
+  // zero every tile's NaN flag (the trailer word after its rows) and the per-slice tile / CTA
+  // counters after the tiles
   cudaError_t e = cudaMemset2DAsync(reinterpret_cast<char*>(codes) + tbytes, (size_t)tstride, 0, 4,
                                     (size_t)ntiles, st);
+  if (e != cudaSuccess) return (int)e;
+  int32_t* counters = reinterpret_cast<int32_t*>(reinterpret_cast<char*>(codes) + ntiles * tstride);
+  e = cudaMemsetAsync(counters, 0, (size_t)img.n_slices * 8, st);
   if (e != cudaSuccess) return (int)e;
   EncodeRowsArgs ea;
   ea.X = X;
@@ -1832,6 +1877,9 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   // leaf ids / fingerprints take the LEAF instantiation of the same walk
   const bool leaf = o.out_leaf != nullptr || o.out_fp != nullptr;
   a.prof = prof;
+  a.tile_next = counters;
+  a.cta_on = counters + img.n_slices;
+  a.work = img.slice_w;
   using KFn = void (*)(CodedKArgs);
   // [mode][swz][fused]
   static const KFn table[3][2][2] = {

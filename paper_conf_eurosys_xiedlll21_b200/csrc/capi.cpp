@@ -838,9 +838,31 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   // launch / tail cost + per-row cost) stays below its H2D; 16 equal chunks, and 8 chunks followed
   // by halving tail chunks, measured slower (more fixed per-chunk cost).  Three buffers, so a copy
   // never waits for the compute of the chunk before the previous one.
-  const int64_t chunk = std::min<int64_t>(n, std::max<int64_t>(65536, (n + 7) / 8));
+  int64_t chunk = std::min<int64_t>(n, std::max<int64_t>(65536, (n + 7) / 8));
   std::vector<int64_t> cuts;
-  for (int64_t r = 0; r < n; r += chunk) cuts.push_back(r);
+  // ramp ($TAHOE_HOST_RAMP, default on for >= 2M rows): the pipeline's fill (H2D of the first
+  // chunk) and drain (compute of the last) are what the overlap cannot hide, so the first and last
+  // chunks are small (n/64, n/32, ... doubling up to n/16 in the middle): a few more launches,
+  // each worth its fixed cost only when the batch is large
+  static const int ramp_env = std::getenv("TAHOE_HOST_RAMP") ? std::atoi(std::getenv("TAHOE_HOST_RAMP")) : -1;
+  const bool ramp = ramp_env >= 0 ? ramp_env != 0 : n >= 2000000;
+  if (ramp) {
+    chunk = std::max<int64_t>(65536, (n + 15) / 16);
+    std::vector<int64_t> head, tail;
+    int64_t left = n;
+    for (int64_t s = std::max<int64_t>(65536, n / 64); s < chunk && left > 4 * s; s *= 2) {
+      head.push_back(s);
+      tail.push_back(s);
+      left -= 2 * s;
+    }
+    std::vector<int64_t> sizes(head);
+    for (; left > 0; left -= std::min(left, chunk)) sizes.push_back(std::min(left, chunk));
+    sizes.insert(sizes.end(), tail.rbegin(), tail.rend());
+    int64_t r = 0;
+    for (int64_t z : sizes) { cuts.push_back(r); r += z; }
+  } else {
+    for (int64_t r = 0; r < n; r += chunk) cuts.push_back(r);
+  }
   cuts.push_back(n);
   const int64_t nchunks = (int64_t)cuts.size() - 1;
   constexpr int NB = 3;

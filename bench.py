@@ -152,18 +152,27 @@ def rank_rows(cfg, n: int, rank: int, world: int, weak: bool) -> tuple[int, int]
     return (n * rank) // world, (n * (rank + 1)) // world
 
 
+def host_cores() -> int:
+    """The box's host cores available to this process (torchrun sets OMP_NUM_THREADS=1 per rank,
+    so the oracle is given its thread count explicitly)."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
 def oracle_rate(f, X, target_s: float, max_rows: int):
     """Oracle (as it stands) on a bounded seeded sample of X, all host cores.  Returns (rows/s,
     rows, seconds, mean visits, sample indices, oracle result)."""
     import oracle
     probe = min(2000, X.shape[0])
     t = time.perf_counter()
-    oracle.predict(f, X[:probe])
+    oracle.predict(f, X[:probe], nthreads=host_cores())
     dt = max(time.perf_counter() - t, 1e-6)
     rows = int(min(max_rows, X.shape[0], max(probe, probe / dt * target_s)))
     idx = gen.subsample(4242, X.shape[0], rows)
     t = time.perf_counter()
-    r = oracle.predict(f, X, rows=idx)
+    r = oracle.predict(f, X, rows=idx, nthreads=host_cores())
     dt = time.perf_counter() - t
     return rows / dt, rows, dt, float(r["visits"].mean()), idx, r
 
@@ -234,16 +243,16 @@ def run_reference(args, cfg):
     n = cfg.n_samples
     f = gen.make_forest(cfg, leaf_mode="normal")
     X = gen.make_rows(cfg, min(n, 200_000))
-    cores = oracle.n_threads()
+    cores = host_cores()
     rate0 = oracle_rate(f, X, 1.0, 20000)[0]
     rows = int(min(X.shape[0], max(1000, rate0 * 4.0)))   # ~4 s of oracle work per step
     idx = gen.subsample(99, X.shape[0], rows)
     for _ in range(args.warmup):
-        oracle.predict(f, X, rows=idx[: max(1, rows // 8)])
+        oracle.predict(f, X, rows=idx[: max(1, rows // 8)], nthreads=cores)
     times = []
     for _ in range(args.steps):
         t = time.perf_counter()
-        oracle.predict(f, X, rows=idx)
+        oracle.predict(f, X, rows=idx, nthreads=cores)
         times.append(time.perf_counter() - t)
     ms = 1000.0 * statistics.mean(times)
     value = rows / (ms / 1000.0)
@@ -360,7 +369,7 @@ def run_tree_sharded(args, cfg):
             import oracle
             rate, rows, secs, vis, idx, ref = oracle_rate(f, Xh, 12.0, 200_000)
             r1, m1 = oracle_single_core(f, Xh, 500)
-            cpu = dict(value=rate, unit=UNIT, cores=oracle.n_threads(), kind="oracle",
+            cpu = dict(value=rate, unit=UNIT, cores=host_cores(), kind="oracle",
                        sample=f"{rows} seeded rows of this workload, full {cfg.n_trees}-tree forest "
                               f"({secs:.1f} s of oracle work)",
                        single_core=dict(value=r1, unit=UNIT, cores=1, sample=f"first {m1} rows"))
@@ -595,7 +604,7 @@ def main():
         import oracle
         rate, rows, secs, vis, idx, ref = oracle_rate(f, X, 12.0, 1_000_000)
         r1, m1 = oracle_single_core(f, X)
-        cpu = dict(value=rate, unit=UNIT, cores=oracle.n_threads(), kind="oracle",
+        cpu = dict(value=rate, unit=UNIT, cores=host_cores(), kind="oracle",
                    sample=f"{rows} seeded rows of this workload ({secs:.1f} s of oracle work)",
                    single_core=dict(value=r1, unit=UNIT, cores=1, sample=f"first {m1} rows"))
         parity = parity_record(f, out_h[idx], cls_h[idx], ref)

@@ -2199,7 +2199,13 @@ __device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA
 // no data); a buffer that issued one issues only terminators; consumers keep releasing entries
 // and leave once every buffer has issued a terminator and every valid entry has been drained.  The
 // barriers are re-initialised for the next slice.
-constexpr int kCode8Threads = 384;            // 12 warps
+// 10 warps: the ring holds 6 x 2 four-row units, so two units are loading while ten are walked
+// (same-box C4 walk: 8 warps 6.42 ms, 10 warps 5.88 ms, 12 warps 6.11 ms — with 12, every refill's
+// latency sat in front of a waiting warp); -DTAHOE_CODE8_THREADS for experiments
+#ifndef TAHOE_CODE8_THREADS
+#define TAHOE_CODE8_THREADS 320
+#endif
+constexpr int kCode8Threads = TAHOE_CODE8_THREADS;
 constexpr int kFull8 = 36;                    // full barriers (6 per ring buffer)
 template <bool FUSED, int R, int kR8, bool LEAF>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {

@@ -21,13 +21,15 @@ for seed in range(s0, s1):
     ref = oracle.predict(f, X, agg=agg, n_classes=nc, base_score=base, want_leaf=True)
     msg = []
     for s in _strats(F) + [-1]:
-        r = _gpu_run(F, X, s, want_leaf=(s in (0, 1)))
+        r = _gpu_run(F, X, s, want_leaf=(s >= 0))   # every strategy has leaf ids (round 2)
         if not np.array_equal(r["out"], ref["out"]):
             msg.append(f"out s={s} ({int((r['out'] != ref['out']).sum())})")
         if agg != oracle.AGG_SUM and agg != oracle.AGG_AVERAGE and not np.array_equal(r["cls"], ref["cls"]):
             msg.append(f"cls s={s}")
         if "leaf" in r and not np.array_equal(r["leaf"], ref["leaf"]):
             msg.append(f"leaf s={s}")
+        if "fp" in r and not np.array_equal(r["fp"], ref["fp"]):
+            msg.append(f"fp s={s}")
     if agg != oracle.AGG_VOTE:   # raw sums: no base, no average
         rsum = oracle.predict(f, X, agg=oracle.AGG_SUM if nc == 1 else oracle.AGG_CLASS_SUM, n_classes=nc)["raw"]
         part = F.predict_partial(torch.from_numpy(X).cuda())

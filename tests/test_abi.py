@@ -377,3 +377,18 @@ def test_layout_state_export_import_roundtrip():
         b.apply_layout_state(b"not a layout blob at all")
     with pytest.raises(T.TahoeError):
         b.apply_layout_state(blob[:-3])
+
+
+def test_microbenchmark_and_profile_walk_argument_checks():
+    """tahoe_measure_visit_rate refuses bad variants / step counts before touching a device;
+    tahoe_profile_walk on a host-only handle is E_STATE (no CPU prediction path)."""
+    r = ctypes.c_double()
+    L = T.load()
+    for variant, steps, reps in ((3, 256, 10), (-1, 256, 10), (0, 1, 10), (0, 255, 10), (0, 256, 0),
+                                 (2, 10_000, 1)):
+        assert L.tahoe_measure_visit_rate(0, variant, steps, reps, ctypes.byref(r), None) == T.TAHOE_E_INVAL
+    h = _build(_stump_arrays())
+    st = np.zeros(8, np.float64)
+    rc = L.tahoe_profile_walk(h, ctypes.c_void_p(1), 4, 1, ctypes.c_void_p(1), st.ctypes.data, None)
+    assert rc == T.TAHOE_E_STATE
+    T.tahoe_forest_free(h)

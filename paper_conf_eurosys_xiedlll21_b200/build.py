@@ -44,13 +44,17 @@ def _stale() -> bool:
     return any(os.path.getmtime(p) > t for p in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None,
+          defines: list[str] | None = None) -> str:
+    """out / defines: another in-tree build with extra -D flags (same-box A/B experiments,
+    selected at run time by $TAHOE_LIB_AB)."""
+    if out is None and not force and not _stale():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
+    dst = out or LIB
+    tmp = dst + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-lineinfo", "-O3", "-std=c++17", "-shared", "-cudart", "static",
            "-Xcompiler", "-fPIC,-fvisibility=hidden,-O3", "-I", nccl_include(), "-I", INCLUDE, "-I", CSRC,
-           "-o", tmp, *sources(), "-lpthread", "-ldl"]
+           *[f"-D{d}" for d in (defines or [])], "-o", tmp, *sources(), "-lpthread", "-ldl"]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -59,10 +63,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed building libtahoe.so")
     if verbose:
         sys.stderr.write(r.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, dst)
+    return dst
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="--verbose" in sys.argv)
-    print(LIB)
+    # --out NAME -DX=Y ...: an A/B variant next to libtahoe.so
+    args = sys.argv[1:]
+    out = os.path.join(PKG, args[args.index("--out") + 1]) if "--out" in args else None
+    print(build(force="--force" in args, verbose="--verbose" in args, out=out,
+                defines=[a[2:] for a in args if a.startswith("-D")]))

@@ -2048,6 +2048,7 @@ struct Coded8KArgs {
   int32_t switch_slices; // 1: a CTA whose slice is exhausted moves to another (0: experiments)
   int32_t prefetch;      // tiles ahead of a claim to prefetch into L2 (0 = none)
   int32_t split;         // 1: four chains per lane (each column walked as two halves)
+  int32_t claim;         // tiles one ring buffer claims per global atomic (>= 1)
   OutArgs o;
 };
 
@@ -2206,7 +2207,7 @@ __device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA
 #define TAHOE_CODE8_THREADS 320
 #endif
 constexpr int kCode8Threads = TAHOE_CODE8_THREADS;
-constexpr int kFull8 = 36;                    // full barriers (6 per ring buffer)
+constexpr int kFull8 = 6 * kCode8Ring;         // full barriers (6 per ring buffer)
 template <bool FUSED, int R, int kR8, bool LEAF>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant__ Coded8KArgs a) {
   constexpr int C = kSlicedCols;
@@ -2235,7 +2236,9 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
   int32_t* s_vdone = s_vis + 1;                                         // valid entries drained
   int32_t* s_dead = s_vis + 2;                                          // buffers that issued a terminator
   int32_t* s_slice = s_vis + 3;
-  static_assert(8 * (kFull8 + kR8 + 1) + 4 * (1 + 2 * kR8 + 4) <= kCode8Ctl, "control block");
+  int32_t* s_cnext = s_vis + 4;                                         // [kR8] buffer's next claimed tile
+  int32_t* s_cleft = s_cnext + kR8;                                     // [kR8] claimed tiles left
+  static_assert(8 * (kFull8 + kR8 + 1) + 4 * (1 + 4 * kR8 + 4) <= kCode8Ctl, "control block");
   const int lane = threadIdx.x & 31;
   const int col = lane & (C - 1);
   const int half = lane >> 4;
@@ -2260,9 +2263,18 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
     const int b = (int)(e % kR8);
     uint64_t* bar = &s_full[e % kFull8];
     if (lane == 0) {
+      // a buffer claims a.claim consecutive tiles per global atomic and issues them one by one
+      // (its issues are serialised by the ring, so the pair s_cnext / s_cleft needs no lock); a
+      // chunk is used up before the buffer claims again, so a CTA leaving the slice (every buffer
+      // past the last tile) holds no unprocessed claimed tile
       int32_t tile = -1;
       if (!prev_dead) {
-        tile = atomicAdd(&a.tile_next[sl], 1);
+        if (s_cleft[b] == 0) {
+          s_cnext[b] = atomicAdd(&a.tile_next[sl], a.claim);
+          s_cleft[b] = a.claim;
+        }
+        tile = s_cnext[b]++;
+        s_cleft[b]--;
         if (tile >= ntiles) tile = -1;
       }
       s_tile[b] = tile;
@@ -2294,7 +2306,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
         mbar_init(&s_full[b], b < kFull8 ? 32u : (b < kFull8 + kR8 ? (uint32_t)(kUnits * 32) : 1u));
       }
       *s_next = 0u;
-      for (int b = 0; b < kR8; b++) s_cnt[b] = 0;
+      for (int b = 0; b < kR8; b++) s_cnt[b] = s_cleft[b] = 0;
       *s_vis = 0;
       *s_vdone = 0;
       *s_dead = 0;
@@ -2504,11 +2516,16 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     a.n_all = n;
     a.forest_smem = plan.forest_smem;
     a.switch_slices = !(std::getenv("TAHOE_CODE8_SWITCH") && std::atoi(std::getenv("TAHOE_CODE8_SWITCH")) == 0);
-    // L2 prefetch 8 tiles ahead of each claim (C4 walk 7.27 -> 6.88 ms; 24 and 64 the same within
-    // 1 %); $TAHOE_CODE8_PREFETCH overrides (experiments)
-    a.prefetch = std::getenv("TAHOE_CODE8_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODE8_PREFETCH")) : 8;
+    // L2 prefetch 32 tiles ahead of each issued tile (round 1, one tile per claim: 8 ahead, C4 walk
+    // 7.27 -> 6.88 ms); $TAHOE_CODE8_PREFETCH overrides (experiments)
+    a.prefetch = std::getenv("TAHOE_CODE8_PREFETCH") ? std::atoi(std::getenv("TAHOE_CODE8_PREFETCH")) : 32;
     // four chains per lane (C4 walk 6.43 -> 6.22 ms); $TAHOE_CODE8_SPLIT=0: two (experiments)
     a.split = img.col_mid ? (std::getenv("TAHOE_CODE8_SPLIT") ? std::atoi(std::getenv("TAHOE_CODE8_SPLIT")) : 1) : 0;
+    // 8 tiles per claim: the global atomic's round trip sat in front of every refill (ncu: 4 % of
+    // warp samples on its result, 19 % on the full barrier of entries it delayed).  Same-box C4
+    // walk, tiles per claim 1 / 2 / 4 / 8 / 16 / 32: 5.95 / 5.71 / 5.59 / 5.53 / 5.56 / 5.61 ms
+    // (prefetch 32; 8 per claim with prefetch 8 / 0: 5.55 / 5.62)
+    a.claim = std::getenv("TAHOE_CODE8_CLAIM") ? std::max(1, std::atoi(std::getenv("TAHOE_CODE8_CLAIM"))) : 8;
     // a full GPU of CTAs (shared out among the slices by simulated work) once the chunk gives
     // every CTA a few tiles, else the plan's grid
     const bool full = plan.cta_start && ntiles >= 4LL * num_sms;

@@ -101,7 +101,10 @@ inline int32_t code_tile_stride(int32_t fbits) {
 constexpr int32_t kCode8MaxRank = 127;
 constexpr int32_t kCode8MaxFbits = 12;           // rows of <= 4 KB
 constexpr int32_t kCode8TileRows = 8;
-constexpr int32_t kCode8Ring = 6;
+#ifndef TAHOE_CODE8_RING
+#define TAHOE_CODE8_RING 6   // -DTAHOE_CODE8_RING for experiments
+#endif
+constexpr int32_t kCode8Ring = TAHOE_CODE8_RING;
 constexpr int32_t kCode8BandBudget = 200 * 1024; // pre-pass tables per CTA
 constexpr int8_t kCode8Nan = -2;
 constexpr int8_t kCode8Pad = -1;
@@ -116,7 +119,8 @@ inline int64_t code8_chunk_rows(int32_t vfbits, int64_t n) {
   if (c < kCode8TileRows) c = kCode8TileRows;
   return n < c ? n : c;
 }
-constexpr int32_t kCode8Ctl = 512;               // mbarriers (36 full, 6 empty, slice), counters, entry tiles
+// mbarriers (6 full per buffer, one empty per buffer, slice), counters, entry tiles and claims
+constexpr int32_t kCode8Ctl = kCode8Ring <= 6 ? 512 : 1024;
 // shared memory next to the slice: the ring (aligned to the row size), the flags, staged partials,
 // the control block
 inline int64_t code8_ring_smem(int32_t vfbits) {

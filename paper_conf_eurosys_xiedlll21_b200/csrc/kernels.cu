@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 #include <algorithm>
 #include <atomic>
+#include <numeric>
 #include <cstdlib>
 #include <cstdint>
 
@@ -1032,6 +1033,35 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
   }
 }
 
+// One row: fixed-order fp64 sum of the row's parts per class, then base / average / argmax and one
+// round to fp32 (Z14, Z17).  Parts are read through L2 (they may have been written by other SMs).
+__device__ __forceinline__ void finalize_row(const FinalizeArgs& a, int64_t i) {
+  const int32_t C = a.n_classes;
+  int best = 0;
+  double bv = 0.0;
+  for (int32_t c = 0; c < C; c++) {
+    double s = 0.0;
+    if (a.class_ptr) {
+      for (int32_t p = a.class_ptr[c]; p < a.class_ptr[c + 1]; p++)
+        s += __ldcg(&a.partial[(int64_t)a.class_parts[p] * a.part_stride + i * a.row_stride]);
+    } else {
+      s = __ldcg(&a.partial[(int64_t)c * a.part_stride + i * a.row_stride]);
+    }
+    if (a.raw_out) { a.raw_out[i * C + c] = s; continue; }
+    double v;
+    if (a.agg == TAHOE_AGG_VOTE) v = s;
+    else if (a.agg == TAHOE_AGG_AVERAGE) v = s / (double)a.n_trees_full + (double)a.base;
+    else v = s + (double)a.base;
+    a.out[i * C + c] = (float)v;
+    if (c == 0 || v > bv) { best = c; bv = v; }
+  }
+  if (!a.raw_out && a.out_class) {
+    if (a.agg == TAHOE_AGG_BINARY) a.out_class[i] = bv > 0.0 ? 1 : 0;
+    else if (a.agg == TAHOE_AGG_CLASS_SUM || a.agg == TAHOE_AGG_VOTE) a.out_class[i] = best;
+    else a.out_class[i] = 0;
+  }
+}
+
 struct CodedKArgs {
   DevSliced img;
   const uint16_t* codes;
@@ -1500,35 +1530,6 @@ int launch_count_visits(const DevDirect& img, const float* X, int64_t n, int32_t
 }
 
 // ------------------------------------------------------------------ finalize
-// One row: fixed-order fp64 sum of the row's parts per class, then base / average / argmax and one
-// round to fp32 (Z14, Z17).  Parts are read through L2 (they may have been written by other SMs).
-__device__ __forceinline__ void finalize_row(const FinalizeArgs& a, int64_t i) {
-  const int32_t C = a.n_classes;
-  int best = 0;
-  double bv = 0.0;
-  for (int32_t c = 0; c < C; c++) {
-    double s = 0.0;
-    if (a.class_ptr) {
-      for (int32_t p = a.class_ptr[c]; p < a.class_ptr[c + 1]; p++)
-        s += __ldcg(&a.partial[(int64_t)a.class_parts[p] * a.part_stride + i * a.row_stride]);
-    } else {
-      s = __ldcg(&a.partial[(int64_t)c * a.part_stride + i * a.row_stride]);
-    }
-    if (a.raw_out) { a.raw_out[i * C + c] = s; continue; }
-    double v;
-    if (a.agg == TAHOE_AGG_VOTE) v = s;
-    else if (a.agg == TAHOE_AGG_AVERAGE) v = s / (double)a.n_trees_full + (double)a.base;
-    else v = s + (double)a.base;
-    a.out[i * C + c] = (float)v;
-    if (c == 0 || v > bv) { best = c; bv = v; }
-  }
-  if (!a.raw_out && a.out_class) {
-    if (a.agg == TAHOE_AGG_BINARY) a.out_class[i] = bv > 0.0 ? 1 : 0;
-    else if (a.agg == TAHOE_AGG_CLASS_SUM || a.agg == TAHOE_AGG_VOTE) a.out_class[i] = best;
-    else a.out_class[i] = 0;
-  }
-}
-
 __global__ void __launch_bounds__(256) k_finalize(const FinalizeArgs a) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -1972,64 +1973,89 @@ __global__ void __launch_bounds__(THREADS, 1) k_encode_rows8(const Encode8Args a
   extern __shared__ __align__(1024) float s_img[];
   __shared__ uint64_t s_bar;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = blockDim.x >> 5;
-  const int b = blockIdx.x % a.bands;
-  const int64_t chunk = blockIdx.x / a.bands;
-  const int4 bd = __ldg(&a.band[b]);
   if (threadIdx.x == 0) {
     mbar_init(&s_bar, 1);
     fence_mbar_init();
   }
   __syncthreads();
-  if (bd.y > 0) {
-    if (threadIdx.x == 0) {
-      fence_proxy_async_smem();
-      mbar_expect_tx(&s_bar, (uint32_t)bd.y);
-      bulk_g2s_big(s_img, reinterpret_cast<const unsigned char*>(a.img) + bd.x, (uint32_t)bd.y, &s_bar);
-    }
-    mbar_wait(&s_bar, 0);
-  }
-  static_assert(kCode8TileRows % kR == 0, "a row group stays inside one tile");
-  // this chunk's rows, in whole groups of kR
-  const int64_t groups = (a.n + kR - 1) / kR;
-  const int64_t per = (groups + a.chunks - 1) / a.chunks;
-  const int64_t r_lo = chunk * per * kR;
-  const int64_t r_hi = min(a.n, (chunk + 1) * per * kR);
-  const uint32_t V = (uint32_t)a.vfbits;
-  const int64_t tile_bytes = (int64_t)kCode8TileRows << V;
-  const uint32_t sbase = smem_u32(s_img) + (uint32_t)lane * 4u;
-  for (int64_t r0 = r_lo + (int64_t)warp * kR; r0 < r_hi; r0 += (int64_t)W * kR) {
-    const int nq = (int)min((int64_t)kR, r_hi - r0);   // rows of this group (the tail is ragged)
-    bool nan_any = false;
-    uint8_t* row0 = a.codes + (r0 / kCode8TileRows) * tile_bytes + ((r0 % kCode8TileRows) << V);
-    // the next group's attribute values are loaded before this group is searched (rows past the
-    // tail re-read the last row; their codes are not stored)
-    auto load_x = [&](int g, float* x, int& src) {
-      src = g < bd.w ? __ldg(&a.v_src[g * 32 + lane]) : -1;
-      const float* xs = a.X + (src >= 0 ? src : 0);
-#pragma unroll
-      for (int q = 0; q < kR; q++) x[q] = __ldg(xs + (r0 + (q < nq ? q : nq - 1)) * a.d);
-    };
-    float xn[kR];
-    int srcn;
-    load_x(bd.z, xn, srcn);
-    for (int g = bd.z; g < bd.w; g++) {
-      const int v = g * 32 + lane;
-      const int src = srcn;
-      float x[kR];
-#pragma unroll
-      for (int q = 0; q < kR; q++) x[q] = xn[q];
-      load_x(g + 1, xn, srcn);
-      uint32_t pos[kR];
-      bisect8<7, kR>(sbase + (uint32_t)__ldg(&a.grp[g]).x * 4u, x, pos);
-#pragma unroll
-      for (int q = 0; q < kR; q++) {
-        const bool isnan_q = src >= 0 && x[q] != x[q];
-        nan_any |= isnan_q && q < nq;
-        const int8_t c = src < 0 ? kCode8Pad : (isnan_q ? kCode8Nan : (int8_t)pos[q]);
-        if (q < nq) row0[((uint32_t)q << V) + (uint32_t)v] = (uint8_t)c;
+  // persistent CTAs over (band, chunk) items, band-major: the launcher makes the item count a
+  // multiple of the grid, so every CTA codes the same number of equal row chunks
+  const int items = a.bands * a.chunks;
+  uint32_t phase = 0;
+  for (int item = blockIdx.x; item < items; item += gridDim.x) {
+    const int b = item / a.chunks;
+    const int64_t chunk = item % a.chunks;
+    const int4 bd = __ldg(&a.band[b]);
+    __syncthreads();   // every warp is done with the previous item's table
+    if (bd.y > 0) {
+      if (threadIdx.x == 0) {
+        fence_proxy_async_smem();
+        mbar_expect_tx(&s_bar, (uint32_t)bd.y);
+        bulk_g2s_big(s_img, reinterpret_cast<const unsigned char*>(a.img) + bd.x, (uint32_t)bd.y, &s_bar);
       }
+      mbar_wait(&s_bar, phase);
+      phase ^= 1u;
     }
-    if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 / kCode8TileRows) * 4] = 1u;
+    static_assert(kCode8TileRows % kR == 0, "a row group stays inside one tile");
+    // this chunk's rows, in whole groups of kR
+    const int64_t groups = (a.n + kR - 1) / kR;
+    const int64_t per = (groups + a.chunks - 1) / a.chunks;
+    const int64_t r_lo = chunk * per * kR;
+    const int64_t r_hi = min(a.n, (chunk + 1) * per * kR);
+    const uint32_t V = (uint32_t)a.vfbits;
+    const int64_t tile_bytes = (int64_t)kCode8TileRows << V;
+    const uint32_t sbase = smem_u32(s_img) + (uint32_t)lane * 4u;
+    static_assert(kR == 4, "the quad byte transpose below stores 4 rows");
+    const int quad = lane & 3;   // after the transpose: this lane stores row `quad` ...
+    const uint32_t qoff = (uint32_t)(lane >> 2) * 4u;   // ... bytes qoff .. qoff + 3 of the group
+    for (int64_t r0 = r_lo + (int64_t)warp * kR; r0 < r_hi; r0 += (int64_t)W * kR) {
+      const int nq = (int)min((int64_t)kR, r_hi - r0);   // rows of this group (the tail is ragged)
+      bool nan_any = false;
+      uint8_t* row0 = a.codes + (r0 / kCode8TileRows) * tile_bytes + ((r0 % kCode8TileRows) << V);
+      // the group's rows as 32-bit offsets from one 64-bit base (rows past the tail re-read the
+      // last row; their codes are not stored)
+      const float* xb = a.X + r0 * a.d;
+      uint32_t roff[kR];
+#pragma unroll
+      for (int q = 0; q < kR; q++) roff[q] = (uint32_t)(q < nq ? q : nq - 1) * (uint32_t)a.d;
+      // the next group's attribute values are loaded before this group is searched
+      auto load_x = [&](int g, float* x, int& src) {
+        src = g < bd.w ? __ldg(&a.v_src[g * 32 + lane]) : -1;
+        const uint32_t so = src >= 0 ? (uint32_t)src : 0u;
+#pragma unroll
+        for (int q = 0; q < kR; q++) x[q] = __ldg(xb + (roff[q] + so));
+      };
+      float xn[kR];
+      int srcn;
+      load_x(bd.z, xn, srcn);
+      for (int g = bd.z; g < bd.w; g++) {
+        const int src = srcn;
+        float x[kR];
+#pragma unroll
+        for (int q = 0; q < kR; q++) x[q] = xn[q];
+        load_x(g + 1, xn, srcn);
+        uint32_t pos[kR];
+        bisect8<7, kR>(sbase + (uint32_t)__ldg(&a.grp[g]).x * 4u, x, pos);
+        // this lane's codes of rows 0..3 as the bytes of one word, then a 4 x 4 byte transpose
+        // inside each quad of lanes (two exchanges): lane 4j + k ends with row k's codes of the
+        // group's attributes 4j .. 4j + 3, one 32-bit store (four byte stores before)
+        uint32_t w = 0;
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          const bool isnan_q = src >= 0 && x[q] != x[q];
+          nan_any |= isnan_q && q < nq;
+          const int8_t c = src < 0 ? kCode8Pad : (isnan_q ? kCode8Nan : (int8_t)pos[q]);
+          w |= (uint32_t)(uint8_t)c << (8 * q);
+        }
+        uint32_t p = __shfl_xor_sync(0xffffffffu, w, 1);
+        w = (lane & 1) ? __byte_perm(w, p, 0x3715) : __byte_perm(w, p, 0x6240);
+        p = __shfl_xor_sync(0xffffffffu, w, 2);
+        w = (lane & 2) ? __byte_perm(w, p, 0x3276) : __byte_perm(w, p, 0x5410);
+        if (quad < nq)
+          *reinterpret_cast<uint32_t*>(row0 + ((uint32_t)quad << V) + (uint32_t)g * 32u + qoff) = w;
+      }
+      if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 / kCode8TileRows) * 4] = 1u;
+    }
   }
 }
 
@@ -2495,14 +2521,15 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     ea.d = d;
     ea.vfbits = img.vfbits;
     ea.bands = img.c8_bands;
-    ea.chunks = std::max(1, num_sms / std::max(1, img.c8_bands));
+    // lcm(bands, SMs) items of equal rows: one persistent CTA per SM, bands / gcd items each
+    ea.chunks = num_sms / std::gcd(std::max(1, img.c8_bands), num_sms);
     ea.img = img.c8_img;
     ea.grp = reinterpret_cast<const int4*>(img.c8_grp);
     ea.band = reinterpret_cast<const int4*>(img.c8_band);
     ea.v_src = img.v_src;
     ea.codes = codes;
     ea.flags = flags;
-    k_encode_rows8<kEncode8Threads, kEncode8Rows><<<ea.bands * ea.chunks, kEncode8Threads, kCode8BandBudget, st>>>(ea);
+    k_encode_rows8<kEncode8Threads, kEncode8Rows><<<num_sms, kEncode8Threads, kCode8BandBudget, st>>>(ea);
     if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
     Coded8KArgs a{};
     a.img = img;

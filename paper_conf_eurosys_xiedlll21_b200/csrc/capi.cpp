@@ -270,6 +270,19 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
         f->ds.c8_grp = reinterpret_cast<const int4x*>(grp);
         f->ds.c8_band = reinterpret_cast<const int4x*>(band);
         f->ds.c8_bands = f->sl.c8_bands;
+        // the TMA-staged pre-pass: every band at most kCode8BandGroups groups, its tables at most
+        // kCode8TmaTables bytes and its source attributes one kCode8BoxW-float box (an imported layout
+        // may come from another band plan)
+        f->ds.c8_tma = 1;
+        for (int32_t b = 0; b < f->sl.c8_bands; b++) {
+          const int32_t* bd = &f->sl.c8_band[(size_t)b * 4];
+          int32_t lo = INT32_MAX, hi = -1;
+          for (int32_t v = bd[2] * 32; v < bd[3] * 32 && v < (int32_t)f->sl.v_src.size(); v++)
+            if (f->sl.v_src[v] >= 0) { lo = std::min(lo, f->sl.v_src[v]); hi = std::max(hi, f->sl.v_src[v]); }
+          if (bd[3] - bd[2] > kCode8BandGroups || bd[1] > kCode8TmaTables || (hi >= 0 && hi - (lo & ~3) >= kCode8BoxW) ||
+              (hi >= 0 && f->sl.v_src[(size_t)bd[2] * 32] != lo))
+            f->ds.c8_tma = 0;
+        }
         f->ds.vfbits = f->sl.vfbits;
         f->ds.code8 = 1;
         if ((st = upload(f->sl.col_mid, &f->ds.col_mid)) != TAHOE_OK) return st;

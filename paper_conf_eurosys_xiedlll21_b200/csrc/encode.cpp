@@ -407,8 +407,9 @@ static void build_code_banks(const std::vector<std::vector<float>>& tabs, int32_
 // sits at word (row0_g + i) * 32 + a (lane a owns bank a: the 32 probes of a warp never collide);
 // every lane of a group is padded with NaN to 2^k - 1 elements, k = the group's probe count, so
 // the bisection has a uniform trip count ("tab[i] <= x" stays true on a prefix: NaN <= x is
-// false).  Groups are dealt to bands of balanced size <= kCode8BandBudget bytes; a pre-pass CTA
-// stages one band.
+// false).  Groups are dealt to bands of balanced size <= kCode8BandBudget bytes and at most
+// kCode8BandGroups groups (the TMA-staged pre-pass reads a band's attributes as one tensor box
+// per row); a pre-pass CTA stages one band.
 static void build_code8_banks(const std::vector<std::vector<float>>& vt, int32_t vfbits,
                               SlicedImage& S) {
   const int32_t G = (1 << vfbits) / 32;
@@ -426,13 +427,16 @@ static void build_code8_banks(const std::vector<std::vector<float>>& vt, int32_t
   }
   auto gbytes = [&](int32_t g) { return (((int64_t)1 << probes[g]) - 1) * 128; };
   std::vector<int32_t> cut;
-  for (int32_t nb = (int32_t)std::max<int64_t>(1, (total + kCode8BandBudget - 1) / kCode8BandBudget);; nb++) {
+  for (int32_t nb = (int32_t)std::max<int64_t>({(int64_t)1, (total + kCode8BandBudget - 1) / kCode8BandBudget,
+                                                 ((int64_t)G + kCode8BandGroups - 1) / kCode8BandGroups});; nb++) {
     const int64_t target = (total + nb - 1) / nb;
     cut.assign(1, 0);
     int32_t g = 0;
     for (int32_t b = 0; b < nb; b++) {
       int64_t acc = 0;
-      while (g < G && acc + gbytes(g) <= kCode8BandBudget && (acc < target || b == nb - 1)) acc += gbytes(g++);
+      while (g < G && acc + gbytes(g) <= kCode8BandBudget && g - cut.back() < kCode8BandGroups &&
+             (acc < target || b == nb - 1))
+        acc += gbytes(g++);
       cut.push_back(g);
     }
     if (g == G) break;

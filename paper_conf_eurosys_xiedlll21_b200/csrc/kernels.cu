@@ -2059,6 +2059,128 @@ __global__ void __launch_bounds__(THREADS, 1) k_encode_rows8(const Encode8Args a
   }
 }
 
+// k_encode_rows8_tma: k_encode_rows8 with the rows staged by TMA.  ncu of k_encode_rows8 put 35 %
+// of its stall samples on the X loads (the consumer of each group's LDGs); here thread 0 loads
+// 128-row x kCode8BoxW-float boxes of X (the band's source attributes, one 2-D tensor copy per
+// stage) into a two-stage ring, and warp w codes the stage's rows 4w .. 4w + 3 over the band's
+// groups from shared memory.  Codes, stores and NaN flags as k_encode_rows8.
+struct alignas(64) Encode8TmaArgs {
+  CUtensorMap tmap;   // X as a 2-D tensor [n][d] fp32, box [kCode8BoxW][kCode8StageRows]
+  Encode8Args e;
+};
+
+template <int kR>
+__global__ void __launch_bounds__(1024, 1) k_encode_rows8_tma(const __grid_constant__ Encode8TmaArgs ta) {
+  const Encode8Args& a = ta.e;
+  const uint64_t tmap = reinterpret_cast<uint64_t>(&ta.tmap);   // in the parameter space
+  extern __shared__ __align__(1024) float s_img[];
+  float* s_x = s_img + kCode8TmaTables / 4;   // [2][kCode8StageRows][kCode8BoxW]
+  // barriers after the stages: no static shared memory, so the dynamic block starts at the
+  // window's base and the stages keep the 128-byte alignment tensor copies need (a static barrier
+  // in front shifted them: illegal instruction)
+  uint64_t* s_bars = reinterpret_cast<uint64_t*>(s_x + 2 * (kCode8StageBytes / 4));
+  uint64_t& s_tab = s_bars[0];
+  uint64_t* s_full = s_bars + 1;
+  uint64_t* s_empty = s_bars + 3;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, W = blockDim.x >> 5;
+  if (threadIdx.x == 0) {
+    mbar_init(&s_tab, 1);
+    for (int b = 0; b < 2; b++) {
+      mbar_init(&s_full[b], 1);
+      mbar_init(&s_empty[b], (uint32_t)W);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  static_assert(kR == 4 && kCode8StageRows % kCode8TileRows == 0 && kCode8StageRows == 4 * 32,
+                "one 4-row group per warp, whole tiles per stage");
+  const uint32_t V = (uint32_t)a.vfbits;
+  const int64_t tile_bytes = (int64_t)kCode8TileRows << V;
+  const uint32_t sbase = smem_u32(s_img) + (uint32_t)lane * 4u;
+  const int quad = lane & 3;
+  const uint32_t qoff = (uint32_t)(lane >> 2) * 4u;
+  const int items = a.bands * a.chunks;
+  const int64_t groups = (a.n + kR - 1) / kR;
+  const int64_t per = (groups + a.chunks - 1) / a.chunks;
+  uint32_t ph_tab = 0, sc = 0;   // table loads so far; stages issued so far (CTA-uniform)
+  for (int item = blockIdx.x; item < items; item += gridDim.x) {
+    const int b = item / a.chunks;
+    const int64_t chunk = item % a.chunks;
+    const int4 bd = __ldg(&a.band[b]);
+    const int64_t r_lo = chunk * per * kR;
+    const int64_t r_hi = min(a.n, (chunk + 1) * per * kR);
+    const int nst = r_hi > r_lo ? (int)((r_hi - r_lo + kCode8StageRows - 1) / kCode8StageRows) : 0;
+    // the band's first source attribute, rounded down to a 16-byte boundary (the box start)
+    const int32_t s_lo = __ldg(&a.v_src[bd.z * 32]) & ~3;
+    __syncthreads();   // every warp is done with the previous item's table and stages
+    auto issue = [&](uint32_t k, int st) {   // stage st of this item as ring stage k
+      uint64_t* bar = &s_full[k & 1];
+      fence_proxy_async_smem();
+      mbar_expect_tx(bar, (uint32_t)kCode8StageBytes);
+      asm volatile(
+          "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
+          " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_u32(s_x + (size_t)(k & 1) * (kCode8StageBytes / 4))),
+          "l"(tmap), "r"(s_lo), "r"((int32_t)(r_lo + (int64_t)st * kCode8StageRows)),
+          "r"(smem_u32(bar))
+          : "memory");
+    };
+    if (threadIdx.x == 0) {
+      if (bd.y > 0) {
+        fence_proxy_async_smem();
+        mbar_expect_tx(&s_tab, (uint32_t)bd.y);
+        bulk_g2s_big(s_img, reinterpret_cast<const unsigned char*>(a.img) + bd.x, (uint32_t)bd.y, &s_tab);
+      }
+      for (int st = 0; st < nst && st < 2; st++) issue(sc + (uint32_t)st, st);
+    }
+    if (bd.y > 0) {
+      mbar_wait(&s_tab, ph_tab);
+      ph_tab ^= 1u;
+    }
+    for (int st = 0; st < nst; st++, sc++) {
+      const uint32_t k = sc & 1u;
+      mbar_wait(&s_full[k], (sc >> 1) & 1u);
+      const float* sx = s_x + (size_t)k * (kCode8StageBytes / 4);
+      const int64_t rs0 = r_lo + (int64_t)st * kCode8StageRows;
+      const int64_t r0 = rs0 + warp * kR;
+      const int nq = r0 < r_hi ? (int)min((int64_t)kR, r_hi - r0) : 0;
+      bool nan_any = false;
+      uint8_t* row0 = a.codes + (r0 / kCode8TileRows) * tile_bytes + ((r0 % kCode8TileRows) << V);
+      for (int g = bd.z; nq > 0 && g < bd.w; g++) {
+        const int src = __ldg(&a.v_src[g * 32 + lane]);
+        const int col = src >= 0 ? src - s_lo : 0;
+        float x[kR];
+#pragma unroll
+        for (int q = 0; q < kR; q++) x[q] = sx[(warp * kR + q) * kCode8BoxW + col];
+        uint32_t pos[kR];
+        bisect8<7, kR>(sbase + (uint32_t)__ldg(&a.grp[g]).x * 4u, x, pos);
+        uint32_t w = 0;
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          const bool isnan_q = src >= 0 && x[q] != x[q];
+          nan_any |= isnan_q && q < nq;
+          const int8_t c = src < 0 ? kCode8Pad : (isnan_q ? kCode8Nan : (int8_t)pos[q]);
+          w |= (uint32_t)(uint8_t)c << (8 * q);
+        }
+        uint32_t p = __shfl_xor_sync(0xffffffffu, w, 1);
+        w = (lane & 1) ? __byte_perm(w, p, 0x3715) : __byte_perm(w, p, 0x6240);
+        p = __shfl_xor_sync(0xffffffffu, w, 2);
+        w = (lane & 2) ? __byte_perm(w, p, 0x3276) : __byte_perm(w, p, 0x5410);
+        if (quad < nq)
+          *reinterpret_cast<uint32_t*>(row0 + ((uint32_t)quad << V) + (uint32_t)g * 32u + qoff) = w;
+      }
+      if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 / kCode8TileRows) * 4] = 1u;
+      // the warp is done with stage k: one arrival per warp (after its lanes' reads)
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&s_empty[k])) : "memory");
+      // thread 0 refills the stage once every warp has left it
+      if (threadIdx.x == 0 && st + 2 < nst) {
+        mbar_wait(&s_empty[k], (sc >> 1) & 1u);
+        issue(sc + 2, st + 2);
+      }
+    }
+  }
+}
+
 struct Coded8KArgs {
   DevSliced img;
   const uint8_t* codes;
@@ -2494,6 +2616,9 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     if (dev >= 0 && dev < 64 && !configured[dev].load()) {
       e = cudaFuncSetAttribute(k_encode_rows8<kEncode8Threads, kEncode8Rows>,
                                cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin - 1024);
+      if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_encode_rows8_tma<kEncode8Rows>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 kMaxSmemOptin - 1024);
       for (auto k : {k_sliced_codes8<true, kCode8TileRows, kCode8Ring, false>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring, false>,
                      k_sliced_codes8<true, kCode8TileRows, kCode8Ring, true>, k_sliced_codes8<false, kCode8TileRows, kCode8Ring, true>})
         if (e == cudaSuccess) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemOptin);
@@ -2529,7 +2654,26 @@ int launch_sliced_codes8(const DevSliced& img, const SlicedPlan& plan, const flo
     ea.v_src = img.v_src;
     ea.codes = codes;
     ea.flags = flags;
-    k_encode_rows8<kEncode8Threads, kEncode8Rows><<<num_sms, kEncode8Threads, kCode8BandBudget, st>>>(ea);
+    // TMA-staged rows when X is a valid 2-D tensor (16-byte aligned rows) and every band fits one
+    // box; else the rows through L1 ($TAHOE_CODE8_TMA=0 forces that path: experiments, tests)
+    const bool tma_off = std::getenv("TAHOE_CODE8_TMA") && std::atoi(std::getenv("TAHOE_CODE8_TMA")) == 0;
+    EncodeTiledFn enc = encode_tiled_fn();
+    const bool tma = !tma_off && enc && img.c8_tma && (reinterpret_cast<uintptr_t>(X) & 15) == 0 && d % 4 == 0;
+    if (tma) {
+      Encode8TmaArgs ta{};
+      ta.e = ea;
+      const cuuint64_t gdim[2] = {(cuuint64_t)d, (cuuint64_t)cn};   // this chunk's rows
+      const cuuint64_t gstride[1] = {(cuuint64_t)d * 4};
+      const cuuint32_t box[2] = {(cuuint32_t)kCode8BoxW, (cuuint32_t)kCode8StageRows};
+      const cuuint32_t estride[2] = {1, 1};
+      CUresult r = enc(&ta.tmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(X + c0 * d), gdim,
+                       gstride, box, estride, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) return (int)cudaErrorInvalidValue;
+      k_encode_rows8_tma<kEncode8Rows><<<num_sms, kEncode8Threads, kCode8TmaTables + 2 * kCode8StageBytes + 64, st>>>(ta);
+    } else {
+      k_encode_rows8<kEncode8Threads, kEncode8Rows><<<num_sms, kEncode8Threads, kCode8BandBudget, st>>>(ea);
+    }
     if ((e = cudaGetLastError()) != cudaSuccess) return (int)e;
     Coded8KArgs a{};
     a.img = img;

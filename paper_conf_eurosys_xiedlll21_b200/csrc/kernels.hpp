@@ -58,6 +58,7 @@ struct DevSliced {
   const int4x* c8_grp = nullptr;     // [2^vfbits / 32] {word offset in band, probes, band, 0}
   const int4x* c8_band = nullptr;    // [bands] {byte offset, bytes, first group, end group}
   int32_t c8_bands = 0;
+  int32_t c8_tma = 0;                // every band fits k_encode_rows8_tma (<= 8 groups, 256 sources)
   const float* slice_w = nullptr;    // [ns] simulated lane-steps per row (dynamic slice choice)
   const int32_t* col_mid = nullptr;  // [ns][16] split slot of each column (two chains per row)
 };
@@ -106,6 +107,16 @@ constexpr int32_t kCode8TileRows = 8;
 #endif
 constexpr int32_t kCode8Ring = TAHOE_CODE8_RING;
 constexpr int32_t kCode8BandBudget = 200 * 1024; // pre-pass tables per CTA
+// TMA-staged pre-pass (k_encode_rows8_tma): a band is at most 3 groups (96 virtual attributes, so
+// at most 96 source attributes; from the first one rounded down to a 16-byte boundary — a box
+// start off that boundary is an illegal instruction — they fit one 2-D tensor box of 128 floats
+// per row) and its tables at most 3 x 127 x 128 bytes; two 128-row stages of X (one 4-row group
+// per warp of the 1024-thread CTA) follow the tables in shared memory
+constexpr int32_t kCode8BandGroups = 3;
+constexpr int32_t kCode8BoxW = 128;
+constexpr int32_t kCode8StageRows = 128;
+constexpr int32_t kCode8StageBytes = kCode8StageRows * kCode8BoxW * 4;
+constexpr int32_t kCode8TmaTables = kCode8BandGroups * 127 * 128;
 constexpr int8_t kCode8Nan = -2;
 constexpr int8_t kCode8Pad = -1;
 inline int64_t code8_tile_bytes(int32_t vfbits) { return (int64_t)kCode8TileRows << vfbits; }

@@ -74,10 +74,13 @@ def test_wide_codes_piece_boundaries_ties_signed_zero_inf_nan():
     assert len(outs) == len(_strats(F)) >= 3 and all(np.array_equal(o, outs[0]) for o in outs)
 
 
+@pytest.mark.parametrize("tma", ["1", "0"])
 @pytest.mark.parametrize("d", [130, 255, 600, 1500])
-def test_wide_codes_row_geometries(d):
+def test_wide_codes_row_geometries(d, tma, monkeypatch):
     """Code rows of 256 B .. 2 KB (V = 8 .. 11), one or several pre-pass bands, ragged last
-    tile; NaN rows take their default paths."""
+    tile; NaN rows take their default paths.  Both pre-pass kernels: rows staged by TMA (d % 4 ==
+    0) and rows through L1 ($TAHOE_CODE8_TMA=0, and every d % 4 != 0)."""
+    monkeypatch.setenv("TAHOE_CODE8_TMA", tma)
     f, rng = _wide_forest(d, d, 160, 8, 300)
     F = T.Forest(f, n_features=d, n_classes=1, agg=oracle.AGG_SUM, device=0)
     st = F.stats()
@@ -131,3 +134,34 @@ def test_wide_codes_unused_attributes_take_no_bytes_and_fallback():
         ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1)
         for s in _strats(F):
             _check(_gpu_run(F, X, s, want_leaf=False), ref, oracle.AGG_SUM, True, want_leaf=False)
+
+
+def _chunked_case():
+    """Body of test_wide_codes_chunked_launches (run in a child with $TAHOE_CODE8_CHUNK_MB set:
+    the chunk size is read once per process)."""
+    d = 600
+    f, rng = _wide_forest(77, d, 160, 8, 300)
+    F = T.Forest(f, n_features=d, n_classes=1, agg=oracle.AGG_SUM, device=0)
+    assert F.stats()["code8"]
+    X = rng.normal(size=(9001, d)).astype(np.float32)
+    X[::29, 3] = np.nan
+    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
+    _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, oracle.AGG_SUM, True,
+           want_leaf=False)
+    _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED), ref, oracle.AGG_SUM, True)
+
+
+@pytest.mark.parametrize("tma", ["1", "0"])
+def test_wide_codes_chunked_launches(tma):
+    """Batches coded and walked in several launches of whole tiles (1 MB of code rows each: the
+    pre-pass's tensor map starts at each chunk's first row), both pre-pass kernels."""
+    import os
+    import subprocess
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    root = os.path.dirname(here)
+    env = dict(os.environ, TAHOE_CODE8_CHUNK_MB="1", TAHOE_CODE8_TMA=tma,
+               PYTHONPATH=os.pathsep.join([root, here, os.environ.get("PYTHONPATH", "")]))
+    r = subprocess.run([sys.executable, "-c", "import test_gpu_wide as t; t._chunked_case()"],
+                       cwd=here, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]

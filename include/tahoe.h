@@ -229,7 +229,8 @@ tahoe_status tahoe_forest_layout_import(tahoe_forest* f, const void* buf, int64_
  * stays L1-resident: steps x reps node reads per thread.
  * Writes *node_reads_per_s (node reads = visits, leaf reads included, per second); optionally
  * *smem_bytes_per_clk (NULL to skip): conflict-free 16-byte shared-memory loads measured with
- * clock64, bytes per SM clock.  E_INVAL on a bad variant / steps < 2 / odd steps / reps < 1;
+ * clock64, bytes per SM clock.  E_INVAL on a bad variant / steps < 2 / odd steps (variant 0: steps
+ * not a multiple of 4) / reps < 1;
  * E_CUDA on launch failure.  Synchronous (own stream).
  */
 tahoe_status tahoe_measure_visit_rate(int32_t device, int32_t variant, int32_t steps, int32_t reps,
@@ -294,7 +295,11 @@ enum tahoe_reduce_mode {
 tahoe_status tahoe_comm_unique_id(uint8_t id[TAHOE_COMM_ID_BYTES]);
 
 /* Collective over `world` processes, one per GPU: ncclCommInitRank on `device`, plus a device
- * communicator with one LSA barrier per SM.  *comm is owned by the caller (tahoe_comm_free). */
+ * communicator with one LSA barrier per SM.  *comm is owned by the caller (tahoe_comm_free).
+ * Environment TAHOE_REDUCE_NVLS=1 (world > 1): the device communicator also maps the window's
+ * NVLS multicast address and tahoe_predict_reduce sums the ranks' partials in the switch
+ * (multimem.ld_reduce; addition order unspecified, within reading Z17's fp64 bound); where
+ * multicast is unavailable the peer-load kernel (rank-order sum, reading R5) is used. */
 tahoe_status tahoe_comm_init(const uint8_t id[TAHOE_COMM_ID_BYTES], int32_t world, int32_t rank,
                              int32_t device, tahoe_comm** comm);
 void tahoe_comm_free(tahoe_comm* comm);   /* synchronises the device first; NULL is a no-op     */

@@ -90,6 +90,7 @@ static void free_host_pipe(tahoe_forest* f) {
   if (!h.ready) return;
   cudaStreamDestroy(h.s_in);
   cudaStreamDestroy(h.s_cmp);
+  cudaStreamDestroy(h.s_cmp2);
   cudaStreamDestroy(h.s_out);
   cudaEventDestroy(h.ev_start);
   for (int b = 0; b < 3; b++) { cudaEventDestroy(h.ev_in[b]); cudaEventDestroy(h.ev_cmp[b]); cudaEventDestroy(h.ev_out[b]); }
@@ -101,6 +102,7 @@ static cudaError_t init_host_pipe(tahoe_forest* f) {
   if (h.ready) return cudaSuccess;
   cudaError_t e = cudaStreamCreateWithFlags(&h.s_in, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h.s_cmp, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h.s_cmp2, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h.s_out, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h.ev_start, cudaEventDisableTiming);
   for (int b = 0; b < 3 && e == cudaSuccess; b++) {
@@ -131,6 +133,7 @@ static void free_device(tahoe_forest* f) {
   cudaFree((void*)f->ds.thr_off);
   cudaFree((void*)f->ds.cb_img);
   cudaFree((void*)f->ds.cb_desc);
+  cudaFree((void*)f->ds.slot_attr);
   cudaFree((void*)f->ds.v_src);
   cudaFree((void*)f->ds.c8_img);
   cudaFree((void*)f->ds.c8_grp);
@@ -252,6 +255,7 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
       if ((st = upload(f->sl.cnodes, &f->ds.cnodes)) != TAHOE_OK) return st;
       if ((st = upload(f->sl.thr_tab, &f->ds.thr_tab)) != TAHOE_OK) return st;
       if ((st = upload(f->sl.thr_off, &f->ds.thr_off)) != TAHOE_OK) return st;
+      if (!f->sl.code8 && (st = upload(f->sl.slot_attr, &f->ds.slot_attr)) != TAHOE_OK) return st;
       f->ds.n_features = f->host.n_features;
       f->ds.n_thr = f->sl.thr_off.back();
       if (!f->sl.cb_img.empty()) {
@@ -882,7 +886,12 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   tahoe_forest* fm = const_cast<tahoe_forest*>(f);   // the pipe is handle-owned scratch state
   std::lock_guard<std::mutex> lock(fm->host_mu);
   if (cudaError_t ie = init_host_pipe(fm)) return cuda_fail(ie, "tahoe_predict_host streams");
-  cudaStream_t s_in = fm->hp.s_in, s_cmp = fm->hp.s_cmp, s_out = fm->hp.s_out;
+  // chunks alternate between two compute streams, so the next chunk's pre-pass and walk start on
+  // the SMs the previous walk's tail releases (one compute stream: every chunk's tail idled the GPU)
+  cudaStream_t s_in = fm->hp.s_in, s_out = fm->hp.s_out;
+  cudaStream_t s_cmps[2] = {fm->hp.s_cmp, fm->hp.s_cmp2};
+  static const int two_env = std::getenv("TAHOE_HOST_STREAMS") ? std::atoi(std::getenv("TAHOE_HOST_STREAMS")) : 2;
+  const int ncmp = two_env == 1 ? 1 : 2;
   cudaEvent_t ev_start = fm->hp.ev_start;
   cudaEvent_t* ev_in = fm->hp.ev_in;
   cudaEvent_t* ev_cmp = fm->hp.ev_cmp;
@@ -896,10 +905,12 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   if (e == cudaSuccess && class_host) e = scratch_alloc((void**)&dC, (size_t)nbuf * chunk * 4, user);
   cudaEventRecord(ev_start, user);
   cudaStreamWaitEvent(s_in, ev_start, 0);
-  cudaStreamWaitEvent(s_cmp, ev_start, 0);
+  cudaStreamWaitEvent(s_cmps[0], ev_start, 0);
+  cudaStreamWaitEvent(s_cmps[1], ev_start, 0);
   cudaStreamWaitEvent(s_out, ev_start, 0);
   for (int64_t c = 0; c < nchunks && e == cudaSuccess && st == TAHOE_OK; c++) {
     const int b = (int)(c % NB);
+    cudaStream_t s_cmp = s_cmps[c % ncmp];
     const int64_t r0 = cuts[c], nr = cuts[c + 1] - cuts[c];
     float* xb = dX + (size_t)b * chunk * d;
     float* ob = dO + (size_t)b * chunk * C;
@@ -918,10 +929,12 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
     cudaEventRecord(ev_out[b], s_out);
   }
   cudaEventRecord(ev_in[0], s_in);
-  cudaEventRecord(ev_cmp[0], s_cmp);
+  cudaEventRecord(ev_cmp[0], s_cmps[0]);
+  cudaEventRecord(ev_cmp[1], s_cmps[1]);
   cudaEventRecord(ev_out[0], s_out);
   cudaStreamWaitEvent(user, ev_in[0], 0);
   cudaStreamWaitEvent(user, ev_cmp[0], 0);
+  cudaStreamWaitEvent(user, ev_cmp[1], 0);
   cudaStreamWaitEvent(user, ev_out[0], 0);
   if (dX) cudaFreeAsync(dX, user);
   if (dO) cudaFreeAsync(dO, user);
@@ -936,7 +949,9 @@ __attribute__((visibility("default"))) tahoe_status tahoe_measure_visit_rate(
     int32_t device, int32_t variant, int32_t steps, int32_t reps, double* node_reads_per_s,
     double* smem_bytes_per_clk) {
   TAHOE_GUARD_BEGIN
-  if (variant < 0 || variant > 2 || steps < 2 || (steps & 1) || steps > 600 || reps < 1 || !node_reads_per_s)
+  // variant 0 tests its exit every four steps per chain (walk_coded2): steps a multiple of 4
+  if (variant < 0 || variant > 2 || steps < 2 || (steps & 1) || (variant == 0 && (steps & 3)) || steps > 600 ||
+      reps < 1 || !node_reads_per_s)
     return fail(TAHOE_E_INVAL, "bad microbenchmark arguments");
   DeviceGuard g(device);
   if (!g.ok) return fail(TAHOE_E_CUDA, "cannot select device");

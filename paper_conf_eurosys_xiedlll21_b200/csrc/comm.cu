@@ -181,6 +181,44 @@ __global__ void __launch_bounds__(kReduceBlock) k_reduce_lsa(const ReduceArgs a,
   bar.sync(ncclCoopCta(), cuda::memory_order_acq_rel);
 }
 
+// NVLS variant (opt-in, TAHOE_REDUCE_NVLS=1 at tahoe_comm_init, world > 1 on an NVSwitch system
+// with multicast): the per-class sum over ranks is one multimem.ld_reduce of the window's
+// multicast address — the switch adds the G ranks' fp64 partials and returns the sum, so each row
+// costs one NVLink load per class instead of G peer loads.  The switch's addition order is not
+// specified, so reading R5's rank order (bit-reproducible run to run) does not hold; the sum stays
+// within reading Z17's fp64 bound (dyadic forests: exact).
+__global__ void __launch_bounds__(kReduceBlock) k_reduce_nvls(const ReduceArgs a,
+                                                             const __grid_constant__ ncclDevComm dc,
+                                                             ncclWindow_t win) {
+  ncclLsaBarrierSession<ncclCoopCta> bar(ncclCoopCta(), dc, ncclTeamLsa(dc), dc.lsaBarrier, blockIdx.x);
+  bar.sync(ncclCoopCta(), cuda::memory_order_acq_rel);
+  const double* mc = reinterpret_cast<const double*>(ncclGetLsaMultimemPointer(win, 0, dc));
+  const int32_t C = a.C;
+  for (int64_t i = a.lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.hi;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int best = 0;
+    double bv = 0.0;
+    for (int32_t c = 0; c < C; c++) {
+      double s;
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.add.f64 %0, [%1];"
+                   : "=d"(s) : "l"(mc + i * C + c) : "memory");
+      double v;
+      if (a.agg == TAHOE_AGG_VOTE) v = s;
+      else if (a.agg == TAHOE_AGG_AVERAGE) v = s / (double)a.n_trees_full + (double)a.base;
+      else v = s + (double)a.base;
+      a.out[(i - a.lo) * C + c] = (float)v;
+      if (c == 0 || v > bv) { best = c; bv = v; }
+    }
+    if (a.out_class) {
+      int32_t k = 0;
+      if (a.agg == TAHOE_AGG_BINARY) k = bv > 0.0 ? 1 : 0;
+      else if (a.agg == TAHOE_AGG_CLASS_SUM || a.agg == TAHOE_AGG_VOTE) k = best;
+      a.out_class[i - a.lo] = k;
+    }
+  }
+  bar.sync(ncclCoopCta(), cuda::memory_order_acq_rel);
+}
+
 static tahoe_status rows_of(int64_t n, int32_t world, int32_t rank, int32_t mode, int64_t* lo,
                             int64_t* hi) {
   if (n < 0) return fail(TAHOE_E_INVAL, "n < 0");
@@ -222,6 +260,7 @@ struct tahoe_comm {
   ncclComm_t comm = nullptr;
   ncclDevComm dev{};
   bool dev_ok = false;
+  bool nvls = false;              // devComm created with lsaMultimem (k_reduce_nvls)
   int32_t world = 1, rank = 0, device = 0;
   int32_t grid = 0;               // CTAs of k_reduce_lsa == LSA barriers requested
   void* buf = nullptr;            // symmetric window (partials of this rank)
@@ -282,7 +321,17 @@ __attribute__((visibility("default"))) tahoe_status tahoe_comm_init(const uint8_
   ncclDevCommRequirements reqs;
   std::memset(&reqs, 0, sizeof reqs);
   reqs.lsaBarrierCount = c->grid;
-  r = nccl_api().DevCommCreate(c->comm, &reqs, &c->dev);
+  const char* nv = std::getenv("TAHOE_REDUCE_NVLS");
+  if (world > 1 && nv && std::strcmp(nv, "1") == 0) {
+    // multicast (NVLS) team memory; without NVSwitch multicast the creation fails and the
+    // peer-load kernel is used
+    reqs.lsaMultimem = true;
+    r = nccl_api().DevCommCreate(c->comm, &reqs, &c->dev);
+    c->nvls = r == ncclSuccess && c->dev.lsaMultimem.mcBasePtr != nullptr;
+    if (r == ncclSuccess && !c->nvls) nccl_api().DevCommDestroy(c->comm, &c->dev);
+    reqs.lsaMultimem = false;
+  }
+  if (!c->nvls) r = nccl_api().DevCommCreate(c->comm, &reqs, &c->dev);
   if (r != ncclSuccess) {
     nccl_api().CommDestroy(c->comm);
     delete c;
@@ -359,9 +408,10 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_reduce(
   st = tahoe_predict_partial(shard, X, n, d, static_cast<double*>(c->buf), stream);
   if (st != TAHOE_OK) return st;
   ReduceArgs a = reduce_args(shard, c->world, lo, hi, out, out_class);
-  k_reduce_lsa<<<c->grid, kReduceBlock, 0, s>>>(a, c->dev, c->win);
+  if (c->nvls) k_reduce_nvls<<<c->grid, kReduceBlock, 0, s>>>(a, c->dev, c->win);
+  else k_reduce_lsa<<<c->grid, kReduceBlock, 0, s>>>(a, c->dev, c->win);
   cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return cuda_err(e, "k_reduce_lsa launch");
+  if (e != cudaSuccess) return cuda_err(e, c->nvls ? "k_reduce_nvls launch" : "k_reduce_lsa launch");
   return TAHOE_OK;
   TAHOE_COMM_GUARD_END
 }

@@ -295,6 +295,91 @@ static void pack_refine(const Forest& F, const std::vector<int32_t>& reads, int6
   pack_stats(F, P);
 }
 
+// Code-row slot of every attribute (reading R7; R10).  The two half-warps of a coded
+// walk read u16 codes from two different rows; rows of >= 128 bytes keep attribute slot j of the
+// second half's row at slot j ^ 32 (code_slot_swz), so logical words w and w ^ 16 of the two rows
+// share a bank and collide (two wavefronts) whenever one half reads word w while the other reads
+// word w ^ 16 (rows of 256 bytes: also words w and w + 32 of one row).  Which attribute sits in
+// which slot does not change a single decision, so the slots are chosen to make collisions rare:
+// every lane reads the word holding its node's attribute (probability of attribute a = its share
+// of the calibrated internal visits, or of 2^-depth without calibration) or, at a leaf, the pad
+// word of slot 2^F - 1 (probability T / (visits + T)); a deterministic local search (swaps and
+// moves to free slots) minimises the estimated probability that some bank sees two addresses
+// (16 active lanes per half, independent lanes).  Slot 2^F - 1 stays the leaves' pad.  Rows of
+// 64 bytes (F <= 5) put the two rows in the two halves of one bank line: identity.
+static std::vector<int32_t> code_slots(const Forest& F, int32_t fbits) {
+  const int32_t nf = F.n_features;
+  std::vector<int32_t> slot(nf);
+  std::iota(slot.begin(), slot.end(), 0);
+  const int32_t NS = 1 << fbits;
+  if (fbits < 6 || nf <= 0 || nf >= NS) return slot;
+  std::vector<double> wa(nf, 0.0);
+  double visits = 0.0;
+  const bool cal = !F.count.empty() && F.n_cal > 0;
+  for (int32_t t = 0; t < F.n_trees; t++)
+    for (int32_t k = F.node_base[t]; k < F.node_base[t + 1]; k++) {
+      if (F.feat[k] < 0) continue;
+      const double pk = cal ? (double)F.count[k] / (double)F.n_cal : std::ldexp(1.0, -std::min(F.depth[k], 60));
+      wa[F.feat[k]] += pk;
+      visits += pk;
+    }
+  if (!(visits > 0.0)) return slot;
+  const double pl = (double)F.n_trees / (visits + (double)F.n_trees);
+  for (auto& v : wa) v = v / visits * (1.0 - pl);
+  const int32_t NW = NS / 2, leafw = (NS - 1) / 2;
+  constexpr int kLanes = 16;
+  auto cost = [&](const std::vector<int32_t>& sl) {
+    std::vector<double> M(NW, 0.0);
+    for (int32_t a = 0; a < nf; a++) M[sl[a] / 2] += wa[a];
+    M[leafw] += pl;
+    // physical word pw of half h holds logical word pw ^ (16 h); bank = pw % 32
+    double ok = 1.0;
+    for (int32_t b = 0; b < 32; b++) {
+      double none = 1.0, one = 0.0;
+      for (int32_t h = 0; h < 2; h++)
+        for (int32_t pw = b; pw < NW; pw += 32) {
+          const double u = 1.0 - std::pow(1.0 - M[pw ^ (16 * h)], kLanes);   // address used
+          one = one * (1.0 - u) + none * u;
+          none *= 1.0 - u;
+        }
+      ok *= none + one;   // at most one address in bank b
+    }
+    return 1.0 - ok;
+  };
+  std::vector<int32_t> best = slot;
+  double bc = cost(best);
+  std::vector<int32_t> free_slots;
+  {
+    std::vector<uint8_t> used(NS, 0);
+    for (int32_t a = 0; a < nf; a++) used[slot[a]] = 1;
+    for (int32_t j = 0; j < NS - 1; j++)
+      if (!used[j]) free_slots.push_back(j);
+  }
+  uint64_t rs = 0x9E3779B97F4A7C15ull;
+  auto rnd = [&](uint64_t m) {   // xorshift64*, deterministic
+    rs ^= rs >> 12; rs ^= rs << 25; rs ^= rs >> 27;
+    return (rs * 0x2545F4914F6CDD1Dull >> 33) % m;
+  };
+  for (int it = 0; it < 20000; it++) {
+    if (free_slots.empty() || rnd(2) == 0) {
+      const int32_t i = (int32_t)rnd(nf), j = (int32_t)rnd(nf);
+      if (i == j) continue;
+      std::swap(best[i], best[j]);
+      const double c = cost(best);
+      if (c < bc) bc = c;
+      else std::swap(best[i], best[j]);
+    } else {
+      const int32_t i = (int32_t)rnd(nf);
+      const size_t k = (size_t)rnd(free_slots.size());
+      std::swap(best[i], free_slots[k]);
+      const double c = cost(best);
+      if (c < bc) bc = c;
+      else std::swap(best[i], free_slots[k]);
+    }
+  }
+  return best;
+}
+
 // Bank-private threshold tables for k_encode_rows_banks (reading R7).  A warp codes one row per
 // pass: lane l of pass p bisects the sorted thresholds of one attribute, and every attribute of a
 // pass owns its own set of m = 2^sh shared-memory banks {b, b + 32/m, b + 2*32/m, ...}: element i
@@ -306,7 +391,7 @@ static void pack_refine(const Forest& F, const std::vector<int32_t>& reads, int6
 // in decreasing order of threshold count, trying every size of the first pass.  The image is used
 // when it fits kCodeBankBudget bytes of shared memory.
 static void build_code_banks(const std::vector<std::vector<float>>& tabs, int32_t fbits,
-                             SlicedImage& S) {
+                             const std::vector<int32_t>& code_slot, SlicedImage& S) {
   S.cb_img.clear();
   S.cb_desc.clear();
   S.cb_passes = 0;
@@ -362,7 +447,12 @@ static void build_code_banks(const std::vector<std::vector<float>>& tabs, int32_
   S.cb_desc.assign((size_t)P * 32 * 4, -1);
   // pad slots: every code slot that no attribute writes
   std::vector<int32_t> pads;
-  for (int32_t j = nf; j < std::max(slots, 32); j++) pads.push_back(j);
+  {
+    std::vector<uint8_t> used((size_t)std::max(slots, 32), 0);
+    for (int32_t a = 0; a < nf; a++) used[code_slot[a]] = 1;
+    for (int32_t j = 0; j < std::max(slots, 32); j++)
+      if (!used[j]) pads.push_back(j);
+  }
   size_t pad_i = 0;
   int64_t region = 0;
   for (int32_t p = 0; p < P; p++) {
@@ -386,7 +476,7 @@ static void build_code_banks(const std::vector<std::vector<float>>& tabs, int32_
       const auto& v = tabs[a];
       for (size_t i = 0; i < v.size(); i++) S.cb_img[(size_t)region * 32 + b + i * stride] = v[i];
       int32_t* d = &S.cb_desc[((size_t)p * 32 + lane++) * 4];
-      d[0] = a;                                            // code slot written
+      d[0] = code_slot[a];                                 // code slot written
       d[1] = a;                                            // attribute read
       d[2] = (int32_t)((region * 32 + b) * 4);             // byte offset of element 0
       d[3] = ((stride * 4) << 16) | (int32_t)v.size();     // element stride (bytes) | K
@@ -654,7 +744,12 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
     if (S.code_valid) {
       S.thr_tab.reserve(S.thr_off[F.n_features]);
       for (auto& v : tabs) S.thr_tab.insert(S.thr_tab.end(), v.begin(), v.end());
-      build_code_banks(tabs, S.fbits, S);
+      S.code_slot = code_slots(F, S.fbits);
+      build_code_banks(tabs, S.fbits, S.code_slot, S);
+      // the fallback pre-pass (k_encode_rows) writes attribute j at slot j
+      if (S.cb_passes == 0) std::iota(S.code_slot.begin(), S.code_slot.end(), 0);
+      S.slot_attr.assign((size_t)1 << S.fbits, -1);
+      for (int32_t a = 0; a < F.n_features; a++) S.slot_attr[S.code_slot[a]] = a;
     }
   }
   auto index_of = [&](int32_t a, float b) -> uint32_t {   // j: b == tab_a[j]
@@ -666,7 +761,7 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
     return S.code8 ? j % (uint32_t)kCode8MaxRank + 1u : j + 1u;
   };
   auto code_attr = [&](int32_t a, float b) -> uint32_t {   // attribute field of a code word
-    return S.code8 ? (uint32_t)vbase[a] + index_of(a, b) / (uint32_t)kCode8MaxRank : (uint32_t)a << 1;
+    return S.code8 ? (uint32_t)vbase[a] + index_of(a, b) / (uint32_t)kCode8MaxRank : (uint32_t)S.code_slot[a] << 1;
   };
   // code words: R7 off_bytes << (F+2) | dl << (F+1) | attribute << 1;
   //             R8 off_bytes << (V+1) | dl << V | virtual attribute

@@ -101,6 +101,8 @@ struct SlicedImage {
   std::vector<uint32_t> cnodes;                  // [ns*slots_max*16*2]
   std::vector<float> thr_tab;                    // concatenated sorted distinct thresholds
   std::vector<int32_t> thr_off;                  // [n_features + 1]
+  std::vector<int32_t> code_slot;                // [n_features] u16 slot of each attribute in a code row (R10)
+  std::vector<int32_t> slot_attr;                // [2^fbits] its inverse (-1 = pad slot)
   // bank-private threshold tables for the row-coding pre-pass (encode.cpp build_code_banks);
   // empty when they do not fit shared memory (the pre-pass then bisects thr_tab through L2)
   std::vector<float> cb_img;                     // [cb_rows][32] words: the shared-memory image
@@ -204,7 +206,7 @@ struct tahoe_forest {
   // one handle (they share these streams)
   struct HostPipe {
     bool ready = false;
-    cudaStream_t s_in = nullptr, s_cmp = nullptr, s_out = nullptr;
+    cudaStream_t s_in = nullptr, s_cmp = nullptr, s_cmp2 = nullptr, s_out = nullptr;
     cudaEvent_t ev_start = nullptr, ev_in[3] = {}, ev_cmp[3] = {}, ev_out[3] = {};
   } hp;
   std::mutex host_mu;

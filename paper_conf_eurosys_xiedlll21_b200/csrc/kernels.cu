@@ -852,6 +852,7 @@ struct EncodeRowsArgs {
   uint16_t* codes;
   int32_t tstride;   // bytes per code tile (rows + trailer)
   int64_t ntiles;
+  const int32_t* slot_attr;   // [2^fbits] attribute of each code slot, -1 = pad (R10)
 };
 
 __device__ __forceinline__ uint32_t code_row_off(int r, int rb) {
@@ -886,16 +887,17 @@ __global__ void __launch_bounds__(1024) k_encode_rows(const EncodeRowsArgs a) {
   for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
        e += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = e >> a.fbits;
-    const int j = (int)(e & smask);
+    const int j = (int)(e & smask);            // code slot
+    const int att = __ldg(&a.slot_attr[j]);    // attribute coded there
     uint16_t code = kCodePad;
-    if (r < a.n && j < a.nf) {
-      const float x = __ldg(&a.X[r * a.d + j]);
+    if (r < a.n && att >= 0) {
+      const float x = __ldg(&a.X[r * a.d + att]);
       if (x != x) {
         code = kCodeNan;
         *reinterpret_cast<int32_t*>(a.codes + (r >> 6) * tile_u16 + flag_u16) = 1;
       } else {
-        const int32_t b0 = off[j];
-        int32_t lo = b0, len = off[j + 1] - b0;
+        const int32_t b0 = off[att];
+        int32_t lo = b0, len = off[att + 1] - b0;
         while (len > 0) {   // lo := first index with tab[lo] > x
           const int32_t h = len >> 1;
           if (tab[lo + h] <= x) { lo += h + 1; len -= h + 1; }
@@ -942,118 +944,161 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
   const int rb = RB64 ? 64 : a.rb;
   const int64_t tile_u16 = a.tstride >> 1;
   const int32_t flag_u16 = 32 * rb;   // trailer word (after the rows)
-  // a warp codes kR consecutive rows at once (independent bisections interleaved; the next
-  // group's attribute values are loaded before this group is searched)
+  // a warp codes kR consecutive rows at once (independent bisections interleaved).  Work units
+  // are (row group, pass) with the pass fastest: all passes of a row group run back to back, so
+  // the row's X lines are still in L1 / L2 for its later passes and its code row is written whole
+  // (passes outermost read X once per pass from HBM: C3 ncu 2.95 GB of DRAM traffic for 1.4 GB
+  // algorithmic).  The next unit's attribute values are loaded before this unit is searched.
   constexpr int kR = 8;
   static_assert(64 % kR == 0, "a row group stays inside one tile");
   const int64_t wstride = (int64_t)gridDim.x * (blockDim.x >> 5) * kR;
   const int64_t w0 = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * kR;
   const uint32_t d = (uint32_t)a.d;
-  for (int p = 0; p < a.passes; p++) {
-    const int4 dsc = __ldg(&a.desc[p * 32 + lane]);
+  const int P = a.passes;
+  auto load_x = [&](int64_t r0, int feat, float* x) {
+    const float* xr = a.X + (feat >= 0 ? feat : 0) + r0 * a.d;
+    if (feat >= 0 && r0 + kR <= a.n) {
+#pragma unroll
+      for (int q = 0; q < kR; q++) x[q] = __ldg(xr + q * d);
+    } else {
+#pragma unroll
+      for (int q = 0; q < kR; q++) x[q] = (feat >= 0 && r0 + q < a.n) ? __ldg(xr + q * d) : 0.0f;
+    }
+  };
+  float xn[kR];
+  int4 dn = __ldg(&a.desc[lane]);
+  if (w0 < a.nrows) load_x(w0, dn.y, xn);
+  int64_t r0 = w0;
+  int p = 0;
+  while (r0 < a.nrows) {
+    const int4 dsc = dn;
+    float x[kR];
+#pragma unroll
+    for (int q = 0; q < kR; q++) x[q] = xn[q];
+    // next unit: pass p + 1 of this group, or pass 0 of the next group
+    int64_t r1 = r0;
+    int p1 = p + 1;
+    if (p1 == P) { p1 = 0; r1 += wstride; }
+    if (r1 < a.nrows) {
+      dn = __ldg(&a.desc[p1 * 32 + lane]);
+      load_x(r1, dn.y, xn);
+    }
     const int slot = dsc.x, feat = dsc.y;
     const uint32_t base = smem_u32(s_img) + (uint32_t)dsc.z;   // element 0 of this lane's table
     const uint32_t stride = (uint32_t)dsc.w >> 16;               // bytes between elements
     const uint32_t lstride = 31u - __clz(stride | 1u);           // stride is a power of two
     const int K = dsc.w & 0xffff;
     const int top = K > 0 ? 1 << (31 - __clz(K)) : 0;            // largest power of two <= K
-    const float* Xf = a.X + (feat >= 0 ? feat : 0);
-    auto load_x = [&](int64_t r0, float* x) {
-      const float* xr = Xf + r0 * a.d;
-      if (feat >= 0 && r0 + kR <= a.n) {
+    // pos := #{thresholds <= x} by Shar's bisection (uniform trip count for every row of this
+    // lane, every probe in range, no bounds tests): after the first probe at top - 1 the count
+    // lies in [pos, pos + top]; each halving step keeps it in [pos, pos + step]; a last probe
+    // at pos decides between pos and pos + 1.  Positions are byte offsets (pos * stride).
+    uint32_t pos[kR];
 #pragma unroll
-        for (int q = 0; q < kR; q++) x[q] = __ldg(xr + q * d);
-      } else {
+    for (int q = 0; q < kR; q++) pos[q] = 0;
+    if (top > 0) {
+      float v0;
+      asm("ld.shared.f32 %0, [%1];" : "=f"(v0) : "r"(base + (uint32_t)(top - 1) * stride));
+      const uint32_t hi = (uint32_t)(K - top) * stride;
 #pragma unroll
-        for (int q = 0; q < kR; q++) x[q] = (feat >= 0 && r0 + q < a.n) ? __ldg(xr + q * d) : 0.0f;
-      }
-    };
-    float xn[kR];
-    if (w0 < a.nrows) load_x(w0, xn);
-    for (int64_t r0 = w0; r0 < a.nrows; r0 += wstride) {
-      float x[kR];
-#pragma unroll
-      for (int q = 0; q < kR; q++) x[q] = xn[q];
-      if (r0 + wstride < a.nrows) load_x(r0 + wstride, xn);
-      // pos := #{thresholds <= x} by Shar's bisection (uniform trip count for every row of this
-      // lane, every probe in range, no bounds tests): after the first probe at top - 1 the count
-      // lies in [pos, pos + top]; each halving step keeps it in [pos, pos + step]; a last probe
-      // at pos decides between pos and pos + 1.  Positions are byte offsets (pos * stride).
-      uint32_t pos[kR];
-#pragma unroll
-      for (int q = 0; q < kR; q++) pos[q] = 0;
-      if (top > 0) {
-        float v0;
-        asm("ld.shared.f32 %0, [%1];" : "=f"(v0) : "r"(base + (uint32_t)(top - 1) * stride));
-        const uint32_t hi = (uint32_t)(K - top) * stride;
-#pragma unroll
-        for (int q = 0; q < kR; q++) pos[q] = v0 <= x[q] ? hi : 0u;
-        for (uint32_t stepb = ((uint32_t)top >> 1) * stride; stepb >= stride; stepb >>= 1) {
-          const uint32_t as = base + stepb - stride;
-#pragma unroll
-          for (int q = 0; q < kR; q++) {
-            float v;
-            asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(as + pos[q]));
-            pos[q] += v <= x[q] ? stepb : 0u;
-          }
-        }
+      for (int q = 0; q < kR; q++) pos[q] = v0 <= x[q] ? hi : 0u;
+      for (uint32_t stepb = ((uint32_t)top >> 1) * stride; stepb >= stride; stepb >>= 1) {
+        const uint32_t as = base + stepb - stride;
 #pragma unroll
         for (int q = 0; q < kR; q++) {
           float v;
-          asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(base + pos[q]));
-          pos[q] = (pos[q] >> lstride) + (v <= x[q] ? 1u : 0u);
+          asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(as + pos[q]));
+          pos[q] += v <= x[q] ? stepb : 0u;
         }
       }
-      if (slot >= 0) {
-        // the kR rows r0 .. r0+kR-1 of a group (r0 % kR == 0) sit at a constant stride in the
-        // tile: 128 bytes apart in the 64-byte-row layout (same bits 4-5 of r), rb otherwise
-        uint16_t* tb = a.codes + (r0 >> 6) * tile_u16;
-        uint16_t* p0 = tb + (code_row_off((int)(r0 & 63), rb) >> 1) + (slot ^ code_slot_swz((int)(r0 & 63), rb));
-        const int rstride = RB64 ? 64 : (rb >> 1);
-        bool nan = false;
-        if (feat >= 0 && r0 + kR <= a.n) {
 #pragma unroll
-          for (int q = 0; q < kR; q++) {
-            const bool isnan_q = x[q] != x[q];
-            nan |= isnan_q;
-            p0[q * rstride] = isnan_q ? kCodeNan : (uint16_t)pos[q];
-          }
-        } else {
-#pragma unroll
-          for (int q = 0; q < kR; q++) {
-            uint16_t code = (uint16_t)pos[q];
-            if (feat < 0 || r0 + q >= a.n) code = kCodePad;
-            else if (x[q] != x[q]) { code = kCodeNan; nan = true; }
-            p0[q * rstride] = code;
-          }
-        }
-        if (nan) *reinterpret_cast<int32_t*>(tb + flag_u16) = 1;
+      for (int q = 0; q < kR; q++) {
+        float v;
+        asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(base + pos[q]));
+        pos[q] = (pos[q] >> lstride) + (v <= x[q] ? 1u : 0u);
       }
     }
+    if (slot >= 0) {
+      // the kR rows r0 .. r0+kR-1 of a group (r0 % kR == 0) sit at a constant stride in the
+      // tile: 128 bytes apart in the 64-byte-row layout (same bits 4-5 of r), rb otherwise
+      uint16_t* tb = a.codes + (r0 >> 6) * tile_u16;
+      uint16_t* p0 = tb + (code_row_off((int)(r0 & 63), rb) >> 1) + (slot ^ code_slot_swz((int)(r0 & 63), rb));
+      const int rstride = RB64 ? 64 : (rb >> 1);
+      bool nan = false;
+      if (feat >= 0 && r0 + kR <= a.n) {
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          const bool isnan_q = x[q] != x[q];
+          nan |= isnan_q;
+          p0[q * rstride] = isnan_q ? kCodeNan : (uint16_t)pos[q];
+        }
+      } else {
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          uint16_t code = (uint16_t)pos[q];
+          if (feat < 0 || r0 + q >= a.n) code = kCodePad;
+          else if (x[q] != x[q]) { code = kCodeNan; nan = true; }
+          p0[q * rstride] = code;
+        }
+      }
+      if (nan) *reinterpret_cast<int32_t*>(tb + flag_u16) = 1;
+    }
+    r0 = r1;
+    p = p1;
   }
 }
 
 // One row: fixed-order fp64 sum of the row's parts per class, then base / average / argmax and one
 // round to fp32 (Z14, Z17).  Parts are read through L2 (they may have been written by other SMs).
+// The row's parts are walked in CSR order (class by class, each class's parts in slice order) in
+// batches of kFinBatch independent loads issued before any is added, so a thread waits for one
+// memory round trip per batch instead of one per part; the additions keep the same order.
+constexpr int kFinBatch = 8;
 __device__ __forceinline__ void finalize_row(const FinalizeArgs& a, int64_t i) {
   const int32_t C = a.n_classes;
+  const int32_t np = a.class_ptr ? __ldg(&a.class_ptr[C]) : C;
   int best = 0;
   double bv = 0.0;
-  for (int32_t c = 0; c < C; c++) {
-    double s = 0.0;
-    if (a.class_ptr) {
-      for (int32_t p = a.class_ptr[c]; p < a.class_ptr[c + 1]; p++)
-        s += __ldcg(&a.partial[(int64_t)a.class_parts[p] * a.part_stride + i * a.row_stride]);
-    } else {
-      s = __ldcg(&a.partial[(int64_t)c * a.part_stride + i * a.row_stride]);
-    }
-    if (a.raw_out) { a.raw_out[i * C + c] = s; continue; }
+  auto emit = [&](int32_t c, double s) {
+    if (a.raw_out) { a.raw_out[i * C + c] = s; return; }
     double v;
     if (a.agg == TAHOE_AGG_VOTE) v = s;
     else if (a.agg == TAHOE_AGG_AVERAGE) v = s / (double)a.n_trees_full + (double)a.base;
     else v = s + (double)a.base;
     a.out[i * C + c] = (float)v;
     if (c == 0 || v > bv) { best = c; bv = v; }
+  };
+  int32_t c = 0;
+  int32_t cend = a.class_ptr ? __ldg(&a.class_ptr[1]) : 1;   // first part of class c + 1
+  double s = 0.0;
+  for (int32_t p0 = 0; p0 < np; p0 += kFinBatch) {
+    double v[kFinBatch];
+#pragma unroll
+    for (int k = 0; k < kFinBatch; k++) {
+      const int32_t p = p0 + k;
+      v[k] = 0.0;
+      if (p < np) {
+        const int64_t part = a.class_ptr ? (int64_t)__ldg(&a.class_parts[p]) : (int64_t)p;
+        v[k] = __ldcg(&a.partial[part * a.part_stride + i * a.row_stride]);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < kFinBatch; k++) {
+      const int32_t p = p0 + k;
+      if (p < np) {
+        while (p == cend) {   // classes ending before part p (empty classes included)
+          emit(c, s);
+          s = 0.0;
+          c++;
+          cend = a.class_ptr ? __ldg(&a.class_ptr[c + 1]) : c + 1;
+        }
+        s += v[k];
+      }
+    }
+  }
+  for (; c < C; c++) {
+    emit(c, s);
+    s = 0.0;
   }
   if (!a.raw_out && a.out_class) {
     if (a.agg == TAHOE_AGG_BINARY) a.out_class[i] = bv > 0.0 ? 1 : 0;
@@ -1125,6 +1170,8 @@ __device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t p
                                             uint32_t shmul, double& accA, double& accB) {
   accA = 0.0;
   accB = 0.0;
+  // four steps per chain between exit tests (a finished chain idles on its column's self-looping
+  // terminal leaf of value 0): the test costs 3 of ~37 instructions per two-step round
   while ((pA != pe) | (pB != pe)) {
     const float a1 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
     const float b1 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
@@ -1132,6 +1179,12 @@ __device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t p
     const float b2 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
     add_pair_ftz(accA, a1, a2);
     add_pair_ftz(accB, b1, b2);
+    const float a3 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+    const float b3 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+    const float a4 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+    const float b4 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+    add_pair_ftz(accA, a3, a4);
+    add_pair_ftz(accB, b3, b4);
   }
 }
 
@@ -1801,6 +1854,7 @@ int launch_sliced_codes(const DevSliced& img, const SlicedPlan& plan, const floa
   ea.codes = codes;
   ea.tstride = tstride;
   ea.ntiles = ntiles;
+  ea.slot_attr = img.slot_attr;
   const int64_t tab_bytes = (int64_t)img.n_thr * 4 + (int64_t)(img.n_features + 1) * 4;
   const int64_t elems = ntiles * kSlicedTileRows << img.fbits;
   const int blk = 1024;

@@ -49,6 +49,7 @@ struct DevSliced {
   int32_t n_thr = 0;                 // thr_off[n_features]
   const float* cb_img = nullptr;     // bank-private tables (cb_rows x 32 words) or nullptr
   const int32_t* cb_desc = nullptr;  // [cb_passes][32] int4
+  const int32_t* slot_attr = nullptr; // [2^fbits] attribute coded in each u16 slot (-1 = pad; R10)
   int32_t cb_rows = 0, cb_passes = 0;
   // wide rank codes (reading R8): cnodes hold u8-code node words when code8 != 0
   int32_t code8 = 0;
@@ -107,13 +108,15 @@ constexpr int32_t kCode8TileRows = 8;
 #endif
 constexpr int32_t kCode8Ring = TAHOE_CODE8_RING;
 constexpr int32_t kCode8BandBudget = 200 * 1024; // pre-pass tables per CTA
-// TMA-staged pre-pass (k_encode_rows8_tma): a band is at most 3 groups (96 virtual attributes, so
-// at most 96 source attributes; from the first one rounded down to a 16-byte boundary — a box
-// start off that boundary is an illegal instruction — they fit one 2-D tensor box of 128 floats
-// per row) and its tables at most 3 x 127 x 128 bytes; two 128-row stages of X (one 4-row group
-// per warp of the 1024-thread CTA) follow the tables in shared memory
-constexpr int32_t kCode8BandGroups = 3;
-constexpr int32_t kCode8BoxW = 128;
+// TMA-staged pre-pass (k_encode_rows8_tma): a band is at most 4 groups (128 virtual attributes, so
+// at most 128 source attributes; from the first one rounded down to a 16-byte boundary — a box
+// start off that boundary is an illegal instruction — they fit one 2-D tensor box of 132 floats
+// per row, 528 bytes, a multiple of 16) and its tables at most 4 x 127 x 128 bytes; two 128-row
+// stages of X (one 4-row group per warp of the 1024-thread CTA) follow the tables in shared
+// memory (65 + 135 KB).  C4: 16 bands read 2112 floats per 2000-float row (3-group bands of
+// 128-float boxes: 22 bands, 2816 floats, 1.41x the row bytes from HBM)
+constexpr int32_t kCode8BandGroups = 4;
+constexpr int32_t kCode8BoxW = 132;
 constexpr int32_t kCode8StageRows = 128;
 constexpr int32_t kCode8StageBytes = kCode8StageRows * kCode8BoxW * 4;
 constexpr int32_t kCode8TmaTables = kCode8BandGroups * 127 * 128;

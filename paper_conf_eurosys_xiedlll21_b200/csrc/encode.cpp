@@ -625,6 +625,14 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
     int64_t total = 0;
     for (int32_t t : G) total += enc_size(F, t);
     int32_t k = (int32_t)std::max<int64_t>(1, (int64_t)std::ceil((double)total / ((double)kSlicedCols * cap * 0.97)));
+    // experiment ($TAHOE_SLICES_TARGET, single-class forests): at least this many slices, cut by
+    // expected work, so an SM count divisible by the slice count gives every slice the same CTAs
+    static const int32_t k_target = std::getenv("TAHOE_SLICES_TARGET") ? std::atoi(std::getenv("TAHOE_SLICES_TARGET")) : 0;
+    const bool by_work = F.n_classes == 1 && k_target > k && !F.exp_reads.empty();
+    if (by_work) k = k_target;
+    auto weight = [&](int32_t t) -> double { return by_work ? F.exp_reads[t] : (double)enc_size(F, t); };
+    double wtotal = 0;
+    for (int32_t t : G) wtotal += weight(t);
     for (;; k++) {
       if (k > (int32_t)G.size()) { S.why_invalid = "cannot pack trees into slices"; return TAHOE_OK; }
       // k contiguous chunks of balanced node counts (each non-empty)
@@ -632,14 +640,14 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
       cut[k] = G.size();
       {
         size_t pos = 0;
-        int64_t acc = 0;
+        double acc = 0;
         for (int32_t j = 1; j < k; j++) {
-          const int64_t target = total * j / k;
-          while (pos < G.size() && acc < target) acc += enc_size(F, G[pos++]);
+          const double target = wtotal * j / k;
+          while (pos < G.size() && acc < target) acc += weight(G[pos++]);
           cut[j] = std::min(std::max(pos, cut[j - 1] + 1), G.size() - (size_t)(k - j));
           pos = cut[j];
           acc = 0;
-          for (size_t q = 0; q < pos; q++) acc += enc_size(F, G[q]);
+          for (size_t q = 0; q < pos; q++) acc += weight(G[q]);
         }
       }
       std::vector<Pack> ps;

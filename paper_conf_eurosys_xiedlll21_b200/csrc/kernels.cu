@@ -993,6 +993,8 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
     // lane, every probe in range, no bounds tests): after the first probe at top - 1 the count
     // lies in [pos, pos + top]; each halving step keeps it in [pos, pos + step]; a last probe
     // at pos decides between pos and pos + 1.  Positions are byte offsets (pos * stride).
+    // rows kept as absolute probe addresses ad = base + pos; one probe = address add, LDS,
+    // FSETP, predicated add (4 instructions; the select + add the compiler emitted made it 5)
     uint32_t pos[kR];
 #pragma unroll
     for (int q = 0; q < kR; q++) pos[q] = 0;
@@ -1000,22 +1002,25 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows_banks(const EncodeBanks
       float v0;
       asm("ld.shared.f32 %0, [%1];" : "=f"(v0) : "r"(base + (uint32_t)(top - 1) * stride));
       const uint32_t hi = (uint32_t)(K - top) * stride;
+      uint32_t ad[kR];
 #pragma unroll
-      for (int q = 0; q < kR; q++) pos[q] = v0 <= x[q] ? hi : 0u;
+      for (int q = 0; q < kR; q++) ad[q] = base + (v0 <= x[q] ? hi : 0u);
       for (uint32_t stepb = ((uint32_t)top >> 1) * stride; stepb >= stride; stepb >>= 1) {
-        const uint32_t as = base + stepb - stride;
+        const uint32_t off = stepb - stride;
 #pragma unroll
-        for (int q = 0; q < kR; q++) {
-          float v;
-          asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(as + pos[q]));
-          pos[q] += v <= x[q] ? stepb : 0u;
-        }
+        for (int q = 0; q < kR; q++)
+          asm("{\n\t.reg .f32 t;\n\t.reg .pred p;\n\t.reg .u32 a;\n\t"
+              "add.u32 a, %0, %2;\n\t"
+              "ld.shared.f32 t, [a];\n\t"
+              "setp.le.f32 p, t, %1;\n\t"
+              "@p add.u32 %0, %0, %3;\n\t}"
+              : "+r"(ad[q]) : "f"(x[q]), "r"(off), "r"(stepb));
       }
 #pragma unroll
       for (int q = 0; q < kR; q++) {
         float v;
-        asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(base + pos[q]));
-        pos[q] = (pos[q] >> lstride) + (v <= x[q] ? 1u : 0u);
+        asm("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(ad[q]));
+        pos[q] = ((ad[q] - base) >> lstride) + (v <= x[q] ? 1u : 0u);
       }
     }
     if (slot >= 0) {

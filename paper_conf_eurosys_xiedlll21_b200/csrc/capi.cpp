@@ -256,6 +256,7 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
       if ((st = upload(f->sl.thr_tab, &f->ds.thr_tab)) != TAHOE_OK) return st;
       if ((st = upload(f->sl.thr_off, &f->ds.thr_off)) != TAHOE_OK) return st;
       if (!f->sl.code8 && (st = upload(f->sl.slot_attr, &f->ds.slot_attr)) != TAHOE_OK) return st;
+      if ((st = upload(f->sl.col_mid, &f->ds.col_mid)) != TAHOE_OK) return st;
       f->ds.n_features = f->host.n_features;
       f->ds.n_thr = f->sl.thr_off.back();
       if (!f->sl.cb_img.empty()) {
@@ -289,7 +290,6 @@ static tahoe_status encode_and_upload(tahoe_forest* f) {
         }
         f->ds.vfbits = f->sl.vfbits;
         f->ds.code8 = 1;
-        if ((st = upload(f->sl.col_mid, &f->ds.col_mid)) != TAHOE_OK) return st;
       }
       // slice weights for the coded kernels' slice switching (simulated lane-steps per row)
       std::vector<float> w(f->sl.slice_work.begin(), f->sl.slice_work.end());

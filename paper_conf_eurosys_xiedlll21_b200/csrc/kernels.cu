@@ -2195,23 +2195,36 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows8_tma(const __grid_const
       mbar_wait(&s_tab, ph_tab);
       ph_tab ^= 1u;
     }
+    // this lane's source attribute and table base of each of the band's (<= 4) groups, once per
+    // item instead of two global loads per group and stage
+    int g_src[kCode8BandGroups];
+    uint32_t g_tab[kCode8BandGroups];
+#pragma unroll
+    for (int j = 0; j < kCode8BandGroups; j++) {
+      const int g = bd.z + j;
+      g_src[j] = g < bd.w ? __ldg(&a.v_src[g * 32 + lane]) : -1;
+      g_tab[j] = g < bd.w ? sbase + (uint32_t)__ldg(&a.grp[g]).x * 4u : sbase;
+    }
     for (int st = 0; st < nst; st++, sc++) {
       const uint32_t k = sc & 1u;
       mbar_wait(&s_full[k], (sc >> 1) & 1u);
-      const float* sx = s_x + (size_t)k * (kCode8StageBytes / 4);
+      const float* sx = s_x + (size_t)k * (kCode8StageBytes / 4) + warp * kR * kCode8BoxW;
       const int64_t rs0 = r_lo + (int64_t)st * kCode8StageRows;
       const int64_t r0 = rs0 + warp * kR;
       const int nq = r0 < r_hi ? (int)min((int64_t)kR, r_hi - r0) : 0;
       bool nan_any = false;
       uint8_t* row0 = a.codes + (r0 / kCode8TileRows) * tile_bytes + ((r0 % kCode8TileRows) << V);
-      for (int g = bd.z; nq > 0 && g < bd.w; g++) {
-        const int src = __ldg(&a.v_src[g * 32 + lane]);
+#pragma unroll
+      for (int j = 0; j < kCode8BandGroups; j++) {
+        const int g = bd.z + j;
+        if (nq <= 0 || g >= bd.w) break;
+        const int src = g_src[j];
         const int col = src >= 0 ? src - s_lo : 0;
         float x[kR];
 #pragma unroll
-        for (int q = 0; q < kR; q++) x[q] = sx[(warp * kR + q) * kCode8BoxW + col];
+        for (int q = 0; q < kR; q++) x[q] = sx[q * kCode8BoxW + col];
         uint32_t pos[kR];
-        bisect8<7, kR>(sbase + (uint32_t)__ldg(&a.grp[g]).x * 4u, x, pos);
+        bisect8<7, kR>(g_tab[j], x, pos);
         uint32_t w = 0;
 #pragma unroll
         for (int q = 0; q < kR; q++) {

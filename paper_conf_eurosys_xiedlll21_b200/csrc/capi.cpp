@@ -455,7 +455,10 @@ static tahoe_status run(const tahoe_forest* f, const float* X, int64_t n, int32_
     double* raw = raw_user;
     if (!raw && (e = scratch_alloc((void**)&raw, (size_t)n * C * 8, st)) != cudaSuccess)
       return fail(TAHOE_E_NOMEM, "cudaMallocAsync partial");
-    if ((e = cudaMemsetAsync(raw, 0, (size_t)n * C * 8, st)) != cudaSuccess) return cuda_fail(e, "memset");
+    if ((e = cudaMemsetAsync(raw, 0, (size_t)n * C * 8, st)) != cudaSuccess) {
+      if (!raw_user) cudaFreeAsync(raw, st);
+      return cuda_fail(e, "memset");
+    }
     o.raw = raw;
     if (ev_b) cudaEventRecord(static_cast<cudaEvent_t>(ev_b), st);
     int rc = 0;

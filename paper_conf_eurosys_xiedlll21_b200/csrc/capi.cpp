@@ -1142,6 +1142,11 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"code8\":" << (f->sl.code8 ? "true" : "false") << ",\"code8_vfbits\":" << f->sl.vfbits
      << ",\"code8_virtual\":" << f->sl.n_virtual << ",\"code8_bands\":" << f->sl.c8_bands
      << ",\"code_bank_rows\":" << f->sl.cb_rows << ",\"code_bank_passes\":" << f->sl.cb_passes
+     << ",\"code_slot\":[" << [&] {
+          std::string r;
+          if (f->sl.code_valid && !f->sl.code8)
+            for (size_t q = 0; q < f->sl.code_slot.size(); q++) r += (q ? "," : "") + std::to_string(f->sl.code_slot[q]);
+          return r; }() << "]"
      << ",\"sliced_fbits\":" << f->sl.fbits << ",\"cta_split\":[" << [&] {
           std::string r;
           for (size_t q = 0; q + 1 < f->cta_start.size(); q++)

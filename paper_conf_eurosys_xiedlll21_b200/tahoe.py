@@ -332,7 +332,7 @@ def tahoe_forest_n_trees(h) -> int:
 
 
 def tahoe_forest_stats(h) -> dict:
-    buf = ctypes.create_string_buffer(8192)
+    buf = ctypes.create_string_buffer(65536)
     _check(load().tahoe_forest_stats(h, buf, len(buf)))
     return json.loads(buf.value.decode())
 

@@ -65,6 +65,12 @@ for cid, n, ntrees in ((2, 3001, 64), (3, 2003, 70), (4, 301, 40)):
         os.environ["TAHOE_FORCE_STRATEGY"] = "3"
         F.predict_partial(Xd)
         os.environ.pop("TAHOE_FORCE_STRATEGY")
+    # end-to-end host call: chunks alternate between two compute streams (3 chunks of 64K rows)
+    if cid == 3:
+        Xh = torch.from_numpy(gen.make_rows(cid, 150_001)).pin_memory()
+        oh = torch.empty((150_001, F.n_out), dtype=torch.float32).pin_memory()
+        F.predict_host(Xh, oh)
+        torch.cuda.synchronize()
     # misaligned X -> warp-copy staging path
     buf = torch.empty(X.size + 1, device=dev)
     buf[1:] = Xd.reshape(-1)

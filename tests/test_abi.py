@@ -392,3 +392,69 @@ def test_microbenchmark_and_profile_walk_argument_checks():
     rc = L.tahoe_profile_walk(h, ctypes.c_void_p(1), 4, 1, ctypes.c_void_p(1), st.ctypes.data, None)
     assert rc == T.TAHOE_E_STATE
     T.tahoe_forest_free(h)
+
+
+def _slot_collision(f, slot, fbits, cal=None):
+    """Estimated probability that some shared-memory bank sees two code words in one warp-wide code
+    load (reading R10): lanes read the word of their node's attribute (weight: calibrated
+    internal visits, or 2^-depth) or, at a leaf, the pad word of slot 2^F - 1; the second half's row
+    holds slot j at j ^ 32.  Python restatement of the objective, for the test only."""
+    feat = np.asarray(f["feature"])
+    left = np.asarray(f["left"])
+    root = np.asarray(f["root"])
+    nf = f["n_features"]
+    depth = np.full(len(feat), -1)
+    for r in root:
+        st = [(int(r), 0)]
+        while st:
+            k, dep = st.pop()
+            depth[k] = dep
+            if left[k] >= 0:
+                st.append((int(left[k]), dep + 1))
+                st.append((int(f["right"][k]), dep + 1))
+    w = np.zeros(nf)
+    internal = (left >= 0) & (depth >= 0)
+    pk = cal if cal is not None else np.ldexp(1.0, -np.minimum(depth, 60))
+    np.add.at(w, feat[internal], pk[internal])
+    visits = w.sum()
+    pl = len(root) / (visits + len(root))
+    w = w / visits * (1 - pl)
+    nw = (1 << fbits) // 2
+    M = np.zeros(nw)
+    np.add.at(M, np.asarray(slot) // 2, w)
+    M[((1 << fbits) - 1) // 2] += pl
+    ok = 1.0
+    for b in range(32):
+        none, one = 1.0, 0.0
+        for h in range(2):
+            for pw in range(b, nw, 32):
+                u = 1 - (1 - M[pw ^ (16 * h)]) ** 16
+                one = one * (1 - u) + none * u
+                none *= 1 - u
+        ok *= none + one
+    return 1 - ok
+
+
+def test_code_slot_assignment():
+    """Reading R10: the u16 code slots are a bijection of the attributes onto slots below the
+    leaves' pad slot 2^F - 1, deterministic, the identity for 64-byte rows (C2), and for C3's
+    128-byte rows they lower the estimated bank-collision probability below the identity's."""
+    for cid, fbits in ((2, 5), (3, 6)):
+        f = gen.make_forest(cid, n_trees=200)
+        slots = []
+        for _ in range(2):
+            h = T.tahoe_forest_build(f, f["n_features"], f["n_classes"], f["agg"], 0.0, -1)
+            st = T.tahoe_forest_stats(h)
+            assert st["coded_valid"] and st["sliced_fbits"] == fbits, st["coded_why"]
+            slots.append(st["code_slot"])
+            T.tahoe_forest_free(h)
+        s = slots[0]
+        assert s == slots[1], "deterministic"
+        assert len(s) == f["n_features"] and len(set(s)) == len(s)
+        assert all(0 <= j < (1 << fbits) - 1 for j in s)
+        if fbits == 5:
+            assert s == list(range(f["n_features"]))
+        else:
+            ident = _slot_collision(f, list(range(f["n_features"])), fbits)
+            mine = _slot_collision(f, s, fbits)
+            assert mine < ident - 0.05, (mine, ident)

@@ -66,10 +66,10 @@ def predict(p, r, s):
 
 
 # pre-pass cost per row-pass of 32 attributes per SM (microseconds), measured on the B200 (ncu
-# launch lists, profiles/): k_encode_rows_banks 0.118 ms per 1M C2 rows (1 pass), 0.23 ms per 1M C3
-# rows (2 passes); k_encode_rows8 2.12 ms per 500K C4 rows (64 passes)
-E_PREPASS_C = 118.0 / (1_000_000 * 1 / 148)
-E_PREPASS_W = 2120.0 / (500_000 * 64 / 148)
+# launch lists, profiles/r02_*): k_encode_rows_banks 0.109 ms per 1M C2 rows (1 pass), 0.64 ms per
+# 4M C3 rows (2 passes); k_encode_rows8_tma 1.44 ms per 500K C4 rows (64 groups)
+E_PREPASS_C = 109.0 / (1_000_000 * 1 / 148)
+E_PREPASS_W = 1440.0 / (500_000 * 64 / 148)
 
 
 def fit(rows, base):

@@ -2335,6 +2335,28 @@ __device__ __forceinline__ void walk_coded8_split(uint32_t pA1, uint32_t mA, uin
   accB = b1 + b2;
 }
 
+// Two chains per lane over one row (two-row work units, TAHOE_CODE8_UROWS=2): the row's column
+// walked as two halves split at col_mid, four steps per chain between exit tests.
+template <bool NAN_AWARE>
+__device__ __forceinline__ void walk_coded8_split1(uint32_t pA1, uint32_t mA, uint32_t pA2, uint32_t pe,
+                                                   uint32_t rowA, uint32_t amask, uint32_t dlbit,
+                                                   uint32_t shmul, double& accA) {
+  double a1 = 0.0, a2 = 0.0;
+  while ((pA1 != mA) | (pA2 != pe)) {
+#pragma unroll
+    for (int k = 0; k < 2; k++) {
+      uint32_t q;
+      q = pA1; const float x1 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul); pA1 = pA1 == mA ? pA1 : q;
+      const float x3 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul);
+      q = pA1; const float x2 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul); pA1 = pA1 == mA ? pA1 : q;
+      const float x4 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul);
+      add_pair_ftz(a1, x1, x2);
+      add_pair_ftz(a2, x3, x4);
+    }
+  }
+  accA = a1 + a2;
+}
+
 // Leaf-diagnostic twins of the two wide-code walks (same steps, same order, same additions; the
 // node read before each step is checked for a leaf, record_leaf).  A first-half chain frozen at its
 // split slot re-reads a tree root, which is never a leaf.
@@ -2426,6 +2448,12 @@ __device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA
 #ifndef TAHOE_CODE8_THREADS
 #define TAHOE_CODE8_THREADS 320
 #endif
+// rows per work unit: 4 (two per half-warp, four chains per lane) or 2 (one per half-warp, two
+// chains per lane: twice the units per ring, so twice the warps; experiments)
+#ifndef TAHOE_CODE8_UROWS
+#define TAHOE_CODE8_UROWS 4
+#endif
+constexpr int kCode8URows = TAHOE_CODE8_UROWS;
 constexpr int kCode8Threads = TAHOE_CODE8_THREADS;
 constexpr int kFull8 = 6 * kCode8Ring;         // full barriers (6 per ring buffer)
 template <bool FUSED, int R, int kR8, bool LEAF>
@@ -2433,8 +2461,9 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
   constexpr int C = kSlicedCols;
   constexpr int FS = R / kCode8TileRows;   // pre-pass tiles (NaN flags) per walked tile
   static_assert(R % kCode8TileRows == 0 && R * kR8 == kCode8TileRows * kCode8Ring, "ring rows");
-  constexpr int kUnits = R / 4;
+  constexpr int kUnits = R / kCode8URows;
   constexpr int kWarps = kCode8Threads / 32;
+  static_assert(kCode8URows == 4 || kCode8URows == 2, "unit rows");
   static_assert(kFull8 % kR8 == 0 && (kFull8 / kR8) * kUnits >= kWarps, "ring-wrap guard");
   extern __shared__ __align__(1024) unsigned char smem[];
   const uint32_t V = (uint32_t)a.img.vfbits;
@@ -2562,8 +2591,10 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
         const int64_t r0 = (int64_t)tile * R;
         const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
         if (u < nr) {
-          const int rA = u + (R / 4) * half, rB = rA + R / 2;
-          const bool okA = rA < nr, okB = rB < nr;
+          // four-row units: half h walks rows u + R/4 h (chain A) and + R/2 (chain B); two-row
+          // units: half h walks row u + R/2 h only (chain B idle)
+          const int rA = u + (R / kCode8URows) * half, rB = rA + R / 2;
+          const bool okA = rA < nr, okB = kCode8URows == 4 && rB < nr;
           const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
           const uint32_t tb = sbase + ring_off + (uint32_t)b * tile_bytes;
           const uint32_t rowA = tb + ((uint32_t)(okA ? rA : u) << V);
@@ -2583,7 +2614,13 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
             if (okA) oA = a.o.out_leaf + (a.row0 + r0 + rA) * (int64_t)a.o.T_leaf;
             if (okB) oB = a.o.out_leaf + (a.row0 + r0 + rB) * (int64_t)a.o.T_leaf;
           }
-          if (a.split) {
+          if (kCode8URows == 2 && !LEAF && a.split) {
+            const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
+            const uint32_t mA = okA ? pm : pe;
+            accB = 0.0;
+            if (nan_flag) walk_coded8_split1<true>(pA, mA, mA, pe, rowA, amask, dlbit, shmul, accA);
+            else walk_coded8_split1<false>(pA, mA, mA, pe, rowA, amask, dlbit, shmul, accA);
+          } else if (a.split) {
             const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
             const uint32_t mA = okA ? pm : pe, mB = okB ? pm : pe;
             if (LEAF) {
@@ -2604,18 +2641,22 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
           // butterfly over the 16 lane columns: after the xor-8 exchange lanes with bit 3 clear
           // hold chain A, set hold chain B (lanes 0, 8, 16, 24 own rows rA(h=0), rB(h=0), rA(h=1),
           // rB(h=1))
-          const bool b3 = lane & 8;
-          double v = (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8);
+          // (two-row units: chain B is empty, the lanes with bit 3 set add their chain A sums too,
+          // in the same xor-8 first order; lanes 0 and 16 own the two rows)
+          const bool b3 = kCode8URows == 4 && (lane & 8);
+          double v = kCode8URows == 4 ? (b3 ? accB : accA) + __shfl_xor_sync(0xffffffffu, b3 ? accA : accB, 8)
+                                      : accA + __shfl_xor_sync(0xffffffffu, accA, 8);
 #pragma unroll
           for (int o = 4; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
           uint64_t fv = 0;
           if (LEAF) {
-            fv = (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8);
+            fv = kCode8URows == 4 ? (b3 ? fpB : fpA) + __shfl_xor_sync(0xffffffffu, b3 ? fpA : fpB, 8)
+                                  : fpA + __shfl_xor_sync(0xffffffffu, fpA, 8);
 #pragma unroll
             for (int o = 4; o > 0; o >>= 1) fv += __shfl_xor_sync(0xffffffffu, fv, o);
           }
           const int rr = b3 ? rB : rA;
-          if ((lane & 7) == 0 && (b3 ? okB : okA)) {
+          if ((lane & (kCode8URows == 4 ? 7 : 15)) == 0 && (b3 ? okB : okA)) {
             if (FUSED) write_scalar(a.o, a.row0 + r0 + rr, v);
             else s_part[b * R + rr] = v;
             if (LEAF && a.o.out_fp)

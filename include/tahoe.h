@@ -230,7 +230,7 @@ tahoe_status tahoe_forest_layout_import(tahoe_forest* f, const void* buf, int64_
  * Writes *node_reads_per_s (node reads = visits, leaf reads included, per second); optionally
  * *smem_bytes_per_clk (NULL to skip): conflict-free 16-byte shared-memory loads measured with
  * clock64, bytes per SM clock.  E_INVAL on a bad variant / steps < 2 / odd steps (variant 0: steps
- * not a multiple of 4) / reps < 1;
+ * not a multiple of 4; variant 1: of 8) / reps < 1;
  * E_CUDA on launch failure.  Synchronous (own stream).
  */
 tahoe_status tahoe_measure_visit_rate(int32_t device, int32_t variant, int32_t steps, int32_t reps,

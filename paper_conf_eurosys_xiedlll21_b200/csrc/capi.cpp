@@ -952,8 +952,10 @@ __attribute__((visibility("default"))) tahoe_status tahoe_measure_visit_rate(
     int32_t device, int32_t variant, int32_t steps, int32_t reps, double* node_reads_per_s,
     double* smem_bytes_per_clk) {
   TAHOE_GUARD_BEGIN
-  // variant 0 tests its exit every four steps per chain (walk_coded2): steps a multiple of 4
-  if (variant < 0 || variant > 2 || steps < 2 || (steps & 1) || (variant == 0 && (steps & 3)) || steps > 600 ||
+  // variant 0 tests its exit every four steps per chain (walk_coded2): steps a multiple of 4;
+  // variant 1 walks each half column (steps / 2 slots) four steps per exit test: a multiple of 8
+  if (variant < 0 || variant > 2 || steps < 2 || (steps & 1) || (variant == 0 && (steps & 3)) ||
+      (variant == 1 && (steps & 7)) || steps > 600 ||
       reps < 1 || !node_reads_per_s)
     return fail(TAHOE_E_INVAL, "bad microbenchmark arguments");
   DeviceGuard g(device);

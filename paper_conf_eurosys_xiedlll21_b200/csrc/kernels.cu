@@ -2442,16 +2442,18 @@ __device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA
 // no data); a buffer that issued one issues only terminators; consumers keep releasing entries
 // and leave once every buffer has issued a terminator and every valid entry has been drained.  The
 // barriers are re-initialised for the next slice.
-// 10 warps: the ring holds 6 x 2 four-row units, so two units are loading while ten are walked
-// (same-box C4 walk: 8 warps 6.42 ms, 10 warps 5.88 ms, 12 warps 6.11 ms — with 12, every refill's
-// latency sat in front of a waiting warp); -DTAHOE_CODE8_THREADS for experiments
+// Work units of 2 rows (one per half-warp, the row's column walked as two halves: two chains per
+// lane) and 20 warps: the ring holds 6 x 4 two-row units, so four units are loading while twenty
+// are walked, and a warp's loop waits for the slowest of 64 half-column walks instead of 128.
+// Same-box C4 walk: four-row units (four chains per lane) with 10 warps 5.52 ms, two-row units
+// with 20 warps 5.38 ms, with 16 warps 5.56 ms (round 2; before, four-row units: 8 warps 6.42 ms,
+// 10 warps 5.88 ms, 12 warps 6.11 ms).  -DTAHOE_CODE8_UROWS=4 -DTAHOE_CODE8_THREADS=320 restores
+// the four-row units (experiments).
 #ifndef TAHOE_CODE8_THREADS
-#define TAHOE_CODE8_THREADS 320
+#define TAHOE_CODE8_THREADS 640
 #endif
-// rows per work unit: 4 (two per half-warp, four chains per lane) or 2 (one per half-warp, two
-// chains per lane: twice the units per ring, so twice the warps; experiments)
 #ifndef TAHOE_CODE8_UROWS
-#define TAHOE_CODE8_UROWS 4
+#define TAHOE_CODE8_UROWS 2
 #endif
 constexpr int kCode8URows = TAHOE_CODE8_UROWS;
 constexpr int kCode8Threads = TAHOE_CODE8_THREADS;
@@ -3011,7 +3013,12 @@ __global__ void __launch_bounds__(1024, 1) k_visit_peak(int32_t L, int32_t reps,
     } else {
       const uint32_t rowA = rb + (uint32_t)half * 64u, rowB = rb + 2048u + (uint32_t)half * 64u;
       const uint32_t pm = sb + ((uint32_t)(L / 2) * C + (uint32_t)col) * 8u;
-      walk_coded8_split<false>(p0, pm, pm, p0, pm, pm, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+      if (kCode8URows == 2) {   // the production walk: one row per half-warp, two chains per lane
+        walk_coded8_split1<false>(p0, pm, pm, pe, rowA, amask, dlbit, shmul, accA);
+        walk_coded8_split1<false>(p0, pm, pm, pe, rowB, amask, dlbit, shmul, accB);
+      } else {
+        walk_coded8_split<false>(p0, pm, pm, p0, pm, pm, pe, rowA, rowB, amask, dlbit, shmul, accA, accB);
+      }
     }
     double v = accA + accB;
 #pragma unroll

@@ -99,6 +99,6 @@ Xp = torch.from_numpy(gen.make_rows(2, 9001)).to(dev)
 T.tahoe_profile_walk(Fp.handle, Xp, 9001, Xp.shape[1], torch.empty((9001, 1), device=dev))
 # microbenchmarks (Algorithm 1 line 4): both walk variants and the raw shared-memory load kernel
 T.tahoe_measure_visit_rate(0, 0, 16, 2)
-T.tahoe_measure_visit_rate(0, 1, 16, 2)
+T.tahoe_measure_visit_rate(0, 1, 16, 2)   # steps: a multiple of 8
 torch.cuda.synchronize()
 print("sanitize case done")

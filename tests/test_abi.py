@@ -384,7 +384,7 @@ def test_microbenchmark_and_profile_walk_argument_checks():
     tahoe_profile_walk on a host-only handle is E_STATE (no CPU prediction path)."""
     r = ctypes.c_double()
     L = T.load()
-    for variant, steps, reps in ((3, 256, 10), (-1, 256, 10), (0, 1, 10), (0, 255, 10), (0, 258, 10),
+    for variant, steps, reps in ((3, 256, 10), (-1, 256, 10), (0, 1, 10), (0, 255, 10), (0, 258, 10), (1, 260, 10),
                                  (0, 256, 0), (2, 10_000, 1)):
         assert L.tahoe_measure_visit_rate(0, variant, steps, reps, ctypes.byref(r), None) == T.TAHOE_E_INVAL
     h = _build(_stump_arrays())

@@ -1144,6 +1144,10 @@ __attribute__((visibility("default"))) tahoe_status tahoe_forest_stats(const tah
      << ",\"code8\":" << (f->sl.code8 ? "true" : "false") << ",\"code8_vfbits\":" << f->sl.vfbits
      << ",\"code8_virtual\":" << f->sl.n_virtual << ",\"code8_bands\":" << f->sl.c8_bands
      << ",\"code_bank_rows\":" << f->sl.cb_rows << ",\"code_bank_passes\":" << f->sl.cb_passes
+     << ",\"code_bank_desc\":[" << [&] {
+          std::string r;
+          for (size_t q = 0; q < f->sl.cb_desc.size(); q++) r += (q ? "," : "") + std::to_string(f->sl.cb_desc[q]);
+          return r; }() << "]"
      << ",\"code_slot\":[" << [&] {
           std::string r;
           if (f->sl.code_valid && !f->sl.code8)

@@ -458,3 +458,37 @@ def test_code_slot_assignment():
             ident = _slot_collision(f, list(range(f["n_features"])), fbits)
             mine = _slot_collision(f, s, fbits)
             assert mine < ident - 0.05, (mine, ident)
+
+
+def test_prepass_lane_plan_covers_every_slot_once():
+    """The row-coding pre-pass plan (encode.cpp build_code_banks, kernels.cu k_encode_rows_banks):
+    replaying the kernel's assignment from the exported lane descriptors ({slot, attribute, table
+    offset, stride | K}, slot < 0: idle lane; every lane codes all rows), every code slot of every
+    row is written exactly once — by a lane of the slot's attribute, or with the pad code for the
+    slots no attribute owns — for C1, C2, C3 and random forests of 3-127 attributes."""
+    from test_oracle_pins import random_forest
+    forests = [gen.make_forest(cid) for cid in (1, 2, 3)]
+    for d, grid in ((3, None), (40, None), (54, 7), (100, None), (127, 41)):
+        rng = np.random.default_rng(d)
+        thr_grid = None if grid is None else np.linspace(-2.0, 2.0, grid)
+        forests.append(dict(random_forest(rng, 60, 7, d, thr_grid=thr_grid), n_features=d))
+    for f in forests:
+        cid = f.get("config", f["n_features"])
+        h = T.tahoe_forest_build(f, f["n_features"], f["n_classes"], f["agg"], 0.0, -1)
+        st = T.tahoe_forest_stats(h)
+        T.tahoe_forest_free(h)
+        assert st["coded_valid"] and st["code_bank_passes"] > 0
+        desc = np.array(st["code_bank_desc"], np.int64).reshape(-1, 4)
+        nslots = max(32, 1 << st["sliced_fbits"])
+        owner = {s: a for a, s in enumerate(st["code_slot"])}
+        writes = np.zeros((32, nslots), np.int64)
+        for dx, feat, _base, _w in desc:
+            if dx < 0:
+                continue                                     # idle lane
+            slot, ph, r = dx & 255, (dx >> 8) & 15, 1 << ((dx >> 12) & 3)
+            assert ph < r
+            assert (feat == -1 and slot not in owner) or owner.get(slot) == feat, (slot, feat)
+            for s in range(4 // r):
+                for q in range(8):
+                    writes[ph + r * (8 * s + q), slot] += 1
+        assert (writes == 1).all(), (cid, np.argwhere(writes != 1)[:5])

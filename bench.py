@@ -572,7 +572,7 @@ def main():
         F.predict_host(Xh, oh, ch)
     torch.cuda.synchronize()
     e2e_ms = []
-    for _ in range(max(3, min(args.steps, 10))):
+    for _ in range(max(3, min(args.steps, 20))):
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         F.predict_host(Xh, oh, ch)

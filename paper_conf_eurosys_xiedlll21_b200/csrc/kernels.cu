@@ -1169,27 +1169,28 @@ __device__ __forceinline__ void add_pair_ftz(double& acc, float v1, float v2) {
   acc += dv;
 }
 
+#ifndef TAHOE_CODED_EXIT
+#define TAHOE_CODED_EXIT 4   // steps per chain between exit tests of walk_coded2 (even)
+#endif
+constexpr int kCodedExit = TAHOE_CODED_EXIT;
 template <bool NAN_AWARE, bool SWZ>
 __device__ __forceinline__ void walk_coded2(uint32_t pA, uint32_t pB, uint32_t pe, uint32_t rowA,
                                             uint32_t rowB, uint32_t amask, uint32_t dlbit,
                                             uint32_t shmul, double& accA, double& accB) {
   accA = 0.0;
   accB = 0.0;
-  // four steps per chain between exit tests (a finished chain idles on its column's self-looping
-  // terminal leaf of value 0): the test costs 3 of ~37 instructions per two-step round
+  // kCodedExit steps per chain between exit tests (a finished chain idles on its column's
+  // self-looping terminal leaf of value 0): the test costs 3 of ~37 instructions per two-step round
   while ((pA != pe) | (pB != pe)) {
-    const float a1 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
-    const float b1 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
-    const float a2 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
-    const float b2 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
-    add_pair_ftz(accA, a1, a2);
-    add_pair_ftz(accB, b1, b2);
-    const float a3 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
-    const float b3 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
-    const float a4 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
-    const float b4 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
-    add_pair_ftz(accA, a3, a4);
-    add_pair_ftz(accB, b3, b4);
+#pragma unroll
+    for (int k = 0; k < kCodedExit / 2; k++) {
+      const float a1 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+      const float b1 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+      const float a2 = coded_step<NAN_AWARE, SWZ>(pA, rowA, amask, dlbit, shmul);
+      const float b2 = coded_step<NAN_AWARE, SWZ>(pB, rowB, amask, dlbit, shmul);
+      add_pair_ftz(accA, a1, a2);
+      add_pair_ftz(accB, b1, b2);
+    }
   }
 }
 

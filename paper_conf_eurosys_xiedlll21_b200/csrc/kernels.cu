@@ -2337,7 +2337,11 @@ __device__ __forceinline__ void walk_coded8_split(uint32_t pA1, uint32_t mA, uin
 }
 
 // Two chains per lane over one row (two-row work units, TAHOE_CODE8_UROWS=2): the row's column
-// walked as two halves split at col_mid, four steps per chain between exit tests.
+// walked as two halves split at col_mid, kCode8Exit steps per chain between exit tests.
+#ifndef TAHOE_CODE8_EXIT
+#define TAHOE_CODE8_EXIT 4
+#endif
+constexpr int kCode8Exit = TAHOE_CODE8_EXIT;
 template <bool NAN_AWARE>
 __device__ __forceinline__ void walk_coded8_split1(uint32_t pA1, uint32_t mA, uint32_t pA2, uint32_t pe,
                                                    uint32_t rowA, uint32_t amask, uint32_t dlbit,
@@ -2345,7 +2349,7 @@ __device__ __forceinline__ void walk_coded8_split1(uint32_t pA1, uint32_t mA, ui
   double a1 = 0.0, a2 = 0.0;
   while ((pA1 != mA) | (pA2 != pe)) {
 #pragma unroll
-    for (int k = 0; k < 2; k++) {
+    for (int k = 0; k < kCode8Exit / 2; k++) {
       uint32_t q;
       q = pA1; const float x1 = coded8_step<NAN_AWARE>(q, rowA, amask, dlbit, shmul); pA1 = pA1 == mA ? pA1 : q;
       const float x3 = coded8_step<NAN_AWARE>(pA2, rowA, amask, dlbit, shmul);

@@ -127,3 +127,23 @@ def test_predict_reduce_nccl_world1_equals_predict():
             F.close()
     finally:
         comm.close()
+
+
+def test_predict_reduce_nvls_request_falls_back_at_world1(monkeypatch):
+    """TAHOE_REDUCE_NVLS=1 asks for the multicast (NVLS) reduce; a one-rank communicator has no
+    multicast team, so tahoe_comm_init keeps the peer-load kernel and the results stay exact."""
+    monkeypatch.setenv("TAHOE_REDUCE_NVLS", "1")
+    comm = _comm_or_skip()
+    try:
+        f = gen.make_forest(2, n_trees=64)
+        F = T.Forest(f, device=0).layout(gen.make_calibration(2, 2048))
+        S = F.shard(0, 1)
+        X = torch.from_numpy(gen.make_rows(2, 5001)).cuda()
+        ref = F.predict(X)
+        out = S.predict_reduce(comm, X)
+        torch.cuda.synchronize()
+        assert torch.equal(out, ref)
+        S.close()
+        F.close()
+    finally:
+        comm.close()

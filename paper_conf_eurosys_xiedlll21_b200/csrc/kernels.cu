@@ -1301,14 +1301,6 @@ __device__ __forceinline__ void prof_lanes(double* prof, double total) {
 // LEAF: the same schedule and walk, also writing per-(sample, tree) caller leaf ids (out_leaf, may
 // be null) and accumulating fingerprints (out_fp, u64 atomic adds per slice).
 // MODE 0: production; 1: LEAF (leaf ids / fingerprints); 2: PROF (per-lane spans, prof_unit)
-// Staged slice partial of tile row r: rows u, u+16, u+32, u+48 (the four rows one warp finishes
-// at once, stored by lanes 0, 8, 16, 24) sit in four different bank pairs (plain indexing put
-// them in one: 4-way store conflicts, ncu 60 M of the walk's wavefronts)
-#ifndef TAHOE_PART_SWZ
-#define TAHOE_PART_SWZ 1
-#endif
-__device__ __forceinline__ int part_slot(int r) { return TAHOE_PART_SWZ ? r ^ ((r >> 4) & 3) : r; }
-
 template <bool FUSED, bool SWZ, int MODE>
 __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant__ CodedKArgs a) {
   constexpr bool LEAF = MODE == 1, PROF = MODE == 2;
@@ -1407,8 +1399,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
           const int nr = (int)((a.n - r0) < R ? (a.n - r0) : R);
           const double* sp = s_part + b * kSlicedTileRows;
           double* dst = a.o.raw + (size_t)sl * a.n + r0;
-          if (lane < nr) dst[lane] = sp[part_slot(lane)];
-          if (lane + 32 < nr) dst[lane + 32] = sp[part_slot(lane + 32)];
+          if (lane < nr) dst[lane] = sp[lane];
+          if (lane + 32 < nr) dst[lane + 32] = sp[lane + 32];
         }
         __syncwarp();
       };
@@ -1516,7 +1508,7 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes(const __grid_constant_
           const int rr = b3 ? rB : rA;
           if ((lane & 7) == 0 && (b3 ? okB : okA)) {
             if (FUSED) write_scalar(a.o, r0 + rr, v);
-            else s_part[b * kSlicedTileRows + part_slot(rr)] = v;
+            else s_part[b * kSlicedTileRows + rr] = v;
             if (LEAF && a.o.out_fp)
               atomicAdd(reinterpret_cast<unsigned long long*>(&a.o.out_fp[r0 + rr]), (unsigned long long)fv);
           }

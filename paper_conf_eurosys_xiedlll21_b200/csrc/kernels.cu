@@ -2001,6 +2001,21 @@ struct Encode8Args {
 // predicated add.
 // one bisection level of bisect8 (probe offset and step are immediates: LDS [ad + imm]; FSETP;
 // predicated IADD: three instructions per probe), then the next level
+#ifndef TAHOE_CODE8_UROWS
+#define TAHOE_CODE8_UROWS 2
+#endif
+constexpr int kCode8URows = TAHOE_CODE8_UROWS;
+// Wide-code rows walked by the second half-warp (tile row bit kCode8SwzBit set: rows u + 4 with
+// two-row units, u + 2 and u + 6 with four-row units) keep code byte v at v ^ s, s = 64 (16 banks
+// over; rows of 2^V < 128 bytes: half the row, which keeps it inside the row):
+// the two half-warps walk the same lane columns, so at the top of every tree and at every leaf
+// (the pad byte) they read the same byte offset of two different rows — one bank, two addresses.
+// The walk XORs the attribute offset into the row base (`(y & amask) ^ row`, one LOP3 as before).
+constexpr uint32_t kCode8SwzBit = kCode8URows == 2 ? 4u : 2u;
+__device__ __forceinline__ uint32_t code8_swz(uint32_t r, uint32_t V) {
+  return (r & kCode8SwzBit) ? min(64u, (1u << V) >> 1) : 0u;
+}
+
 template <int ST, int kR>
 __device__ __forceinline__ void probe8(uint32_t* ad, const float* x) {
 #pragma unroll
@@ -2112,7 +2127,7 @@ __global__ void __launch_bounds__(THREADS, 1) k_encode_rows8(const Encode8Args a
         p = __shfl_xor_sync(0xffffffffu, w, 2);
         w = (lane & 2) ? __byte_perm(w, p, 0x3276) : __byte_perm(w, p, 0x5410);
         if (quad < nq)
-          *reinterpret_cast<uint32_t*>(row0 + ((uint32_t)quad << V) + (uint32_t)g * 32u + qoff) = w;
+          *reinterpret_cast<uint32_t*>(row0 + ((uint32_t)quad << V) + (((uint32_t)g * 32u + qoff) ^ code8_swz((uint32_t)(r0 + quad), V))) = w;
       }
       if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 / kCode8TileRows) * 4] = 1u;
     }
@@ -2239,7 +2254,7 @@ __global__ void __launch_bounds__(1024, 1) k_encode_rows8_tma(const __grid_const
         p = __shfl_xor_sync(0xffffffffu, w, 2);
         w = (lane & 2) ? __byte_perm(w, p, 0x3276) : __byte_perm(w, p, 0x5410);
         if (quad < nq)
-          *reinterpret_cast<uint32_t*>(row0 + ((uint32_t)quad << V) + (uint32_t)g * 32u + qoff) = w;
+          *reinterpret_cast<uint32_t*>(row0 + ((uint32_t)quad << V) + (((uint32_t)g * 32u + qoff) ^ code8_swz((uint32_t)(r0 + quad), V))) = w;
       }
       if (__any_sync(0xffffffffu, nan_any) && lane == 0) a.flags[(r0 / kCode8TileRows) * 4] = 1u;
       // the warp is done with stage k: one arrival per warp (after its lanes' reads)
@@ -2283,7 +2298,7 @@ __device__ __forceinline__ float coded8_step(uint32_t& p, uint32_t rowaddr, uint
   int32_t c;
   asm("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(x), "=r"(y) : "r"(p));
   if (yout) *yout = y;
-  asm("ld.shared.s8 %0, [%1];" : "=r"(c) : "r"((y & amask) | rowaddr));
+  asm("ld.shared.s8 %0, [%1];" : "=r"(c) : "r"((y & amask) ^ rowaddr));
   bool go_left = (uint32_t)c < x;
   if (NAN_AWARE) go_left = go_left || ((c == (int32_t)kCode8Nan) && (y & dlbit));
   p += go_left ? (uint32_t)kSlotBytes : __umulhi(y, shmul);
@@ -2457,10 +2472,6 @@ __device__ __forceinline__ void walk_coded8_split_leaf(uint32_t pA1, uint32_t mA
 #ifndef TAHOE_CODE8_THREADS
 #define TAHOE_CODE8_THREADS 640
 #endif
-#ifndef TAHOE_CODE8_UROWS
-#define TAHOE_CODE8_UROWS 2
-#endif
-constexpr int kCode8URows = TAHOE_CODE8_UROWS;
 constexpr int kCode8Threads = TAHOE_CODE8_THREADS;
 constexpr int kFull8 = 6 * kCode8Ring;         // full barriers (6 per ring buffer)
 template <bool FUSED, int R, int kR8, bool LEAF>
@@ -2604,8 +2615,9 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
           const bool okA = rA < nr, okB = kCode8URows == 4 && rB < nr;
           const uint32_t pA = okA ? p0 : pe, pB = okB ? p0 : pe;
           const uint32_t tb = sbase + ring_off + (uint32_t)b * tile_bytes;
-          const uint32_t rowA = tb + ((uint32_t)(okA ? rA : u) << V);
-          const uint32_t rowB = tb + ((uint32_t)(okB ? rB : u) << V);
+          const uint32_t qA = (uint32_t)(okA ? rA : u), qB = (uint32_t)(okB ? rB : u);
+          const uint32_t rowA = (tb + (qA << V)) | code8_swz(qA, V);   // XORed with the byte offset
+          const uint32_t rowB = (tb + (qB << V)) | code8_swz(qB, V);
           uint32_t nan_flag = 0;
 #pragma unroll
           for (int k = 0; k < FS; k++) {

@@ -2030,10 +2030,14 @@ __device__ __forceinline__ void probe8(uint32_t* ad, const float* x) {
 
 template <int K, int kR>
 __device__ __forceinline__ void bisect8(uint32_t base, const float* x, uint32_t* pos) {
+  // the first level probes the same element for every row: one load for the kR rows
+  constexpr uint32_t kMid = ((1u << (K - 1)) - 1u) << 7, kStep = (1u << (K - 1)) << 7;
+  float v0;
+  asm("ld.shared.f32 %0, [%1+%2];" : "=f"(v0) : "r"(base), "n"(kMid));
   uint32_t ad[kR];
 #pragma unroll
-  for (int q = 0; q < kR; q++) ad[q] = base;
-  probe8<K - 1, kR>(ad, x);
+  for (int q = 0; q < kR; q++) ad[q] = base + (v0 <= x[q] ? kStep : 0u);
+  if constexpr (K > 1) probe8<K - 2, kR>(ad, x);
 #pragma unroll
   for (int q = 0; q < kR; q++) pos[q] = (ad[q] - base) >> 7;
 }
@@ -2593,6 +2597,8 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
     }
     const uint32_t p0 = sbase + (uint32_t)col * 8u;
     const uint32_t pe = sbase + ((uint32_t)a.img.col_len[sl * C + col] * C + (uint32_t)col) * 8u;
+    // the column's split slot (first tree of its second half), once per slice
+    const uint32_t pm_sl = a.split ? sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u : pe;
     const int2* __restrict__ meta =
         LEAF ? reinterpret_cast<const int2*>(a.img.leaf_meta) + (size_t)sl * a.img.slots_max * C : nullptr;
     mbar_wait(s_forest, 0u);
@@ -2634,13 +2640,13 @@ __global__ void __launch_bounds__(1024, 1) k_sliced_codes8(const __grid_constant
             if (okB) oB = a.o.out_leaf + (a.row0 + r0 + rB) * (int64_t)a.o.T_leaf;
           }
           if (kCode8URows == 2 && !LEAF && a.split) {
-            const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
+            const uint32_t pm = pm_sl;
             const uint32_t mA = okA ? pm : pe;
             accB = 0.0;
             if (nan_flag) walk_coded8_split1<true>(pA, mA, mA, pe, rowA, amask, dlbit, shmul, accA);
             else walk_coded8_split1<false>(pA, mA, mA, pe, rowA, amask, dlbit, shmul, accA);
           } else if (a.split) {
-            const uint32_t pm = sbase + ((uint32_t)__ldg(&a.img.col_mid[sl * C + col]) * C + (uint32_t)col) * 8u;
+            const uint32_t pm = pm_sl;
             const uint32_t mA = okA ? pm : pe, mB = okB ? pm : pe;
             if (LEAF) {
               if (nan_flag) walk_coded8_split_leaf<true>(pA, mA, mA, pB, mB, mB, pe, rowA, rowB, amask, dlbit, shmul, accA, accB, sbase, meta, oA, oB, fpA, fpB);

@@ -2030,14 +2030,10 @@ __device__ __forceinline__ void probe8(uint32_t* ad, const float* x) {
 
 template <int K, int kR>
 __device__ __forceinline__ void bisect8(uint32_t base, const float* x, uint32_t* pos) {
-  // the first level probes the same element for every row: one load for the kR rows
-  constexpr uint32_t kMid = ((1u << (K - 1)) - 1u) << 7, kStep = (1u << (K - 1)) << 7;
-  float v0;
-  asm("ld.shared.f32 %0, [%1+%2];" : "=f"(v0) : "r"(base), "n"(kMid));
   uint32_t ad[kR];
 #pragma unroll
-  for (int q = 0; q < kR; q++) ad[q] = base + (v0 <= x[q] ? kStep : 0u);
-  if constexpr (K > 1) probe8<K - 2, kR>(ad, x);
+  for (int q = 0; q < kR; q++) ad[q] = base;
+  probe8<K - 1, kR>(ad, x);
 #pragma unroll
   for (int q = 0; q < kR; q++) pos[q] = (ad[q] - base) >> 7;
 }

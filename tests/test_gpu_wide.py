@@ -165,3 +165,23 @@ def test_wide_codes_chunked_launches(tma):
     r = subprocess.run([sys.executable, "-c", "import test_gpu_wide as t; t._chunked_case()"],
                        cwd=here, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
+@pytest.mark.parametrize("n_trees,depth", [(1, 3), (1, 6), (3, 6), (5, 6)])
+def test_wide_codes_small_rows_half_warp_swizzle(n_trees, depth):
+    """Wide codes whose used attributes fit rows of 32 .. 256 bytes (V = 5 .. 8; few trees over 1000
+    attributes): the second half-warp's rows keep byte v at v ^ min(64, row / 2) — the swizzle
+    must stay inside the row (a first version XORed 64 into 32-byte rows).  Leaf ids, scores and
+    fingerprints bit-exact against the oracle, NaN rows and a ragged last tile included."""
+    d = 1000
+    f, rng = _wide_forest(7 + n_trees + depth, d, n_trees, depth, 300)
+    F = T.Forest(f, n_features=d, n_classes=1, agg=oracle.AGG_SUM, device=0)
+    st = F.stats()
+    assert st["coded_valid"] and st["code8"], st["coded_why"]
+    assert st["code8_vfbits"] <= 8, st["code8_vfbits"]
+    X = rng.normal(size=(3003, d)).astype(np.float32)
+    X[::17, :] = np.nan
+    ref = oracle.predict(f, X, agg=oracle.AGG_SUM, n_classes=1, want_leaf=True)
+    _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED), ref, oracle.AGG_SUM, True)
+    _check(_gpu_run(F, X, T.STRATEGY_SLICED_CODED, want_leaf=False), ref, oracle.AGG_SUM, True,
+           want_leaf=False)

@@ -860,12 +860,13 @@ __attribute__((visibility("default"))) tahoe_status tahoe_predict_host(
   // never waits for the compute of the chunk before the previous one.
   int64_t chunk = std::min<int64_t>(n, std::max<int64_t>(65536, (n + 7) / 8));
   std::vector<int64_t> cuts;
-  // ramp ($TAHOE_HOST_RAMP, default on for >= 2M rows): the pipeline's fill (H2D of the first
+  // ramp ($TAHOE_HOST_RAMP, default on for >= 1M rows; C2's 1M rows: 365-368 -> 374-391 M samples/s
+  // same box): the pipeline's fill (H2D of the first
   // chunk) and drain (compute of the last) are what the overlap cannot hide, so the first and last
   // chunks are small (n/64, n/32, ... doubling up to n/16 in the middle): a few more launches,
   // each worth its fixed cost only when the batch is large
   static const int ramp_env = std::getenv("TAHOE_HOST_RAMP") ? std::atoi(std::getenv("TAHOE_HOST_RAMP")) : -1;
-  const bool ramp = ramp_env >= 0 ? ramp_env != 0 : n >= 2000000;
+  const bool ramp = ramp_env >= 0 ? ramp_env != 0 : n >= 1000000;
   if (ramp) {
     chunk = std::max<int64_t>(65536, (n + 15) / 16);
     std::vector<int64_t> head, tail;

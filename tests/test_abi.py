@@ -492,3 +492,20 @@ def test_prepass_lane_plan_covers_every_slot_once():
                 for q in range(8):
                     writes[ph + r * (8 * s + q), slot] += 1
         assert (writes == 1).all(), (cid, np.argwhere(writes != 1)[:5])
+
+
+def test_cost_model_picks_for_the_bench_workloads():
+    """The shipped cost-model constants (costmodel_b200.json, fitted on the B200) pick the measured
+    fastest strategy for the bench's launch configurations (profiles/r02_costmodel.md): the
+    rank-coded slices for C2 (1M rows), C3 (4M) and C4 (500K), ROWS for a C2 batch of 100."""
+    picks = {}
+    for cid, n in ((2, 1_000_000), (3, 4_000_000), (4, 500_000), (2, 100)):
+        f = gen.make_forest(cid)
+        h = T.tahoe_forest_build(f, f["n_features"], f["n_classes"], f["agg"], 0.0, -1)
+        T.tahoe_forest_layout(h, gen.make_calibration(cid, 4096))
+        picks[(cid, n)] = T.tahoe_select_strategy(h, n, f["n_features"])
+        T.tahoe_forest_free(h)
+    assert picks[(2, 1_000_000)] == T.STRATEGY_SLICED_CODED, picks
+    assert picks[(3, 4_000_000)] == T.STRATEGY_SLICED_CODED, picks
+    assert picks[(4, 500_000)] == T.STRATEGY_SLICED_CODED, picks
+    assert picks[(2, 100)] == T.STRATEGY_ROWS, picks

@@ -47,12 +47,25 @@ def main():
                 rec = dict(config=cid, n=ROWS[cid], node_reorder=nr, tree_group=tg,
                            direct_ms=kernel_ms(F, X, T.STRATEGY_DIRECT),
                            sliced_ms=kernel_ms(F, X, T.STRATEGY_SLICED) if st["sliced_valid"] else None,
+                           coded_ms=kernel_ms(F, X, T.STRATEGY_SLICED_CODED) if st["coded_valid"] and st["sliced_valid"] else None,
                            n_slices=st["n_slices"], eff_sim=st["lockstep_eff_sim"])
                 res.append(rec)
                 print(json.dumps(rec), flush=True)
         F.close()
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     json.dump(res, open(os.path.join(ROOT, "gpurun_out", "ablation.json"), "w"), indent=1)
+    out = ["# Round 2 layout ablation (SURVEY §8(f) f3; the paper's Fig. 8, P:1732-1739)", "",
+           "`python scripts/ablation.py 2 3 4 5` on one B200 (round-2 final kernels): kernel time (CUDA events, "
+           "median of 5) of every strategy with probability-based node rearrangement (node_reorder, P:616-628) and "
+           "similarity-based tree rearrangement (tree_group, P:773-806) switched off/on; C5 uses one 500-tree shard "
+           "(the sliced strategies do not apply: its trees exceed a lane column).", "",
+           "| config | rows | node_reorder | tree_group | direct ms | fp32 sliced ms | rank-coded ms | slices | simulated lockstep eff. |",
+           "|---|---|---|---|---|---|---|---|---|"]
+    f3 = lambda v: "–" if v is None else f"{v:.3f}"
+    for r in res:
+        out.append(f"| C{r['config']} | {r['n']} | {r['node_reorder']} | {r['tree_group']} | {f3(r['direct_ms'])} | "
+                   f"{f3(r['sliced_ms'])} | {f3(r.get('coded_ms'))} | {r['n_slices']} | {r['eff_sim']:.3f} |")
+    open(os.path.join(ROOT, "gpurun_out", "ablation.md"), "w").write("\n".join(out) + "\n")
 
 
 if __name__ == "__main__":

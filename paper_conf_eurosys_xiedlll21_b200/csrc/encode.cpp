@@ -652,16 +652,29 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
       }
       std::vector<Pack> ps;
       bool ok = true;
+      // chunks left to right; a chunk that does not pack hands up to kRecut of its last trees to the
+      // next chunk before k is raised (a similarity order can cluster large trees at a cut): C4
+      // (the bench's calibration) 33 -> 30 slices, simulated lockstep 0.638 -> 0.681, walk
+      // 5.18 -> 5.09 ms
+      constexpr size_t kRecut = 64;
+      size_t start = 0;
       for (int32_t j = 0; j < k && ok; j++) {
-        std::vector<int32_t> chunk(G.begin() + cut[j], G.begin() + cut[j + 1]);
+        const size_t end0 = j == k - 1 ? G.size() : std::max(cut[j + 1], start + 1);
+        if (end0 > G.size() || G.size() - end0 < (size_t)(k - 1 - j)) { ok = false; break; }
         Pack P;
-        if (!pack_best(F, chunk, cap, P)) ok = false;
-        else {
-          if (refine) pack_refine(F, reads, m, cap, P);
-          ps.push_back(P);
-          S.cls.push_back(c);
-          S.ntrees.push_back((int32_t)chunk.size());
+        bool packed = false;
+        size_t end = end0;
+        for (; end > start; end--) {
+          std::vector<int32_t> chunk(G.begin() + start, G.begin() + end);
+          if (pack_best(F, chunk, cap, P)) { packed = true; break; }
+          if (j == k - 1 || end0 - end >= kRecut) break;   // the last chunk cannot hand trees on
         }
+        if (!packed) { ok = false; break; }
+        if (refine) pack_refine(F, reads, m, cap, P);
+        ps.push_back(P);
+        S.cls.push_back(c);
+        S.ntrees.push_back((int32_t)(end - start));
+        start = end;
       }
       if (ok) { packs.insert(packs.end(), ps.begin(), ps.end()); break; }
       S.cls.resize(packs.size());

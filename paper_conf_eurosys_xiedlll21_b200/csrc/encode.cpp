@@ -659,7 +659,18 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
       constexpr size_t kRecut = 64;
       size_t start = 0;
       for (int32_t j = 0; j < k && ok; j++) {
-        const size_t end0 = j == k - 1 ? G.size() : std::max(cut[j + 1], start + 1);
+        // this chunk's share of what is left (the cuts of the initial plan, re-balanced after a
+        // chunk handed trees on)
+        size_t end0 = G.size();
+        if (j < k - 1) {
+          double rest = 0.0;
+          for (size_t q = start; q < G.size(); q++) rest += weight(G[q]);
+          const double target = rest / (double)(k - j);
+          double acc = 0.0;
+          end0 = start;
+          while (end0 < G.size() && acc < target) acc += weight(G[end0++]);
+          end0 = std::max(end0, start + 1);
+        }
         if (end0 > G.size() || G.size() - end0 < (size_t)(k - 1 - j)) { ok = false; break; }
         Pack P;
         bool packed = false;

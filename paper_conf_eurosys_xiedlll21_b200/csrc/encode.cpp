@@ -657,35 +657,53 @@ tahoe_status encode_sliced(const Forest& F, int32_t cap, SlicedImage& S, int32_t
       // (the bench's calibration) 33 -> 30 slices, simulated lockstep 0.638 -> 0.681, walk
       // 5.18 -> 5.09 ms
       constexpr size_t kRecut = 64;
-      size_t start = 0;
-      for (int32_t j = 0; j < k && ok; j++) {
-        // this chunk's share of what is left (the cuts of the initial plan, re-balanced after a
-        // chunk handed trees on)
-        size_t end0 = G.size();
-        if (j < k - 1) {
-          double rest = 0.0;
-          for (size_t q = start; q < G.size(); q++) rest += weight(G[q]);
-          const double target = rest / (double)(k - j);
-          double acc = 0.0;
-          end0 = start;
-          while (end0 < G.size() && acc < target) acc += weight(G[end0++]);
-          end0 = std::max(end0, start + 1);
+      // one left-to-right pass over `order`; refinement only once a whole pass packs
+      auto pass = [&](const std::vector<int32_t>& order, std::vector<Pack>& out,
+                      std::vector<int32_t>& nt) -> bool {
+        out.clear();
+        nt.clear();
+        size_t start = 0;
+        for (int32_t j = 0; j < k; j++) {
+          // this chunk's share of what is left (re-balanced after a chunk handed trees on)
+          size_t end0 = order.size();
+          if (j < k - 1) {
+            double rest = 0.0;
+            for (size_t q = start; q < order.size(); q++) rest += weight(order[q]);
+            const double target = rest / (double)(k - j);
+            double acc = 0.0;
+            end0 = start;
+            while (end0 < order.size() && acc < target) acc += weight(order[end0++]);
+            end0 = std::max(end0, start + 1);
+          }
+          if (end0 > order.size() || order.size() - end0 < (size_t)(k - 1 - j)) return false;
+          Pack P;
+          bool packed = false;
+          size_t end = end0;
+          for (; end > start; end--) {
+            std::vector<int32_t> chunk(order.begin() + start, order.begin() + end);
+            if (pack_best(F, chunk, cap, P)) { packed = true; break; }
+            if (j == k - 1 || end0 - end >= kRecut) break;   // the last chunk cannot hand trees on
+          }
+          if (!packed) return false;
+          out.push_back(P);
+          nt.push_back((int32_t)(end - start));
+          start = end;
         }
-        if (end0 > G.size() || G.size() - end0 < (size_t)(k - 1 - j)) { ok = false; break; }
-        Pack P;
-        bool packed = false;
-        size_t end = end0;
-        for (; end > start; end--) {
-          std::vector<int32_t> chunk(G.begin() + start, G.begin() + end);
-          if (pack_best(F, chunk, cap, P)) { packed = true; break; }
-          if (j == k - 1 || end0 - end >= kRecut) break;   // the last chunk cannot hand trees on
+        return true;
+      };
+      // left to right, then (a failing cut may sit at the other end) right to left
+      std::vector<int32_t> nt;
+      ok = pass(G, ps, nt);
+      if (!ok) {
+        std::vector<int32_t> R(G.rbegin(), G.rend());
+        ok = pass(R, ps, nt);
+      }
+      if (ok) {
+        for (size_t q = 0; q < ps.size(); q++) {
+          if (refine) pack_refine(F, reads, m, cap, ps[q]);
+          S.cls.push_back(c);
+          S.ntrees.push_back(nt[q]);
         }
-        if (!packed) { ok = false; break; }
-        if (refine) pack_refine(F, reads, m, cap, P);
-        ps.push_back(P);
-        S.cls.push_back(c);
-        S.ntrees.push_back((int32_t)(end - start));
-        start = end;
       }
       if (ok) { packs.insert(packs.end(), ps.begin(), ps.end()); break; }
       S.cls.resize(packs.size());
